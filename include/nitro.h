@@ -1,0 +1,284 @@
+/* nitro.h — C ABI of the B200-native Nitro SpMV code-variant hot path.
+ *
+ * The paper (Muralidharan et al., "Nitro: A Framework for Adaptive Code
+ * Variant Tuning", IPDPS 2014) is cited as P:L<n> = line n of its text
+ * (/root/reference/PAPER.md on the build box; the citations are restated in
+ * DESIGN.md so the GPU box never needs the file).
+ *
+ * Two layers:
+ *  1. the generic Nitro layer (Fig. 2): a context, code variants
+ *     with cost-returning variant functions, feature functions, constraints,
+ *     training inputs, offline training (exhaustive search + RBF-SVM)
+ *     and selection;
+ *  2. the SpMV layer (the hot path, BASELINE north_star): a matrix handle over
+ *     a borrowed device CSR, the GPU feature pass, the CSR->ELL/DIA/HYB
+ *     converters, the five SpMV variants, timing, and a registration helper
+ *     that plugs the five variants + features + constraints into layer 1.
+ *  3. the multi-GPU row-partitioned SpMV (x all-gathered with NCCL).
+ *
+ * Conventions (all functions):
+ *  - extern "C"; return nitro_status_t (NITRO_OK = 0); never throw or abort.
+ *    nitro_last_error() returns a thread-local message for the last failure.
+ *  - Handles are opaque.  Device arrays passed in are BORROWED: the caller
+ *    keeps them alive while the handle uses them.  Formats produced by
+ *    conversion are OWNED by the handle and freed by *_destroy.
+ *  - `stream` arguments are cudaStream_t passed as void*; NULL = legacy default.
+ *    GPU work is enqueued on the handle's stream.  Only calls that return host
+ *    results (features, allowed, time, select, call, train, export) synchronise it.
+ *  - Sizes are int64_t element counts unless named *_bytes.
+ */
+#ifndef NITRO_H
+#define NITRO_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef int nitro_status_t;
+enum {
+  NITRO_OK = 0,
+  NITRO_E_INVALID_ARG = 1, /* null pointer, bad enum, size mismatch */
+  NITRO_E_BAD_MATRIX = 2,  /* non-canonical CSR (see nitro_spmv_feat) */
+  NITRO_E_STATE = 3,       /* select before train/load, mutation after train */
+  NITRO_E_CONSTRAINT = 4,  /* explicit run of a variant its constraint rules out */
+  NITRO_E_OOM = 5,         /* device or host allocation failed */
+  NITRO_E_CUDA = 6,        /* CUDA runtime error (message has the CUDA string) */
+  NITRO_E_NCCL = 7,        /* NCCL error */
+  NITRO_E_IO = 8,          /* model file read/write */
+  NITRO_E_UNSUPPORTED = 9  /* configuration outside what this build handles */
+};
+
+const char *nitro_last_error(void);
+const char *nitro_version(void);
+
+/* ========================================================================
+ * 1. Generic Nitro layer (Fig. 2 L71-124; autotuner P:L136-190)
+ * ======================================================================== */
+typedef struct nitro_context nitro_context; /* global state shared by variants */
+typedef struct nitro_cv nitro_cv;           /* code_variant<Policy, ArgTuple> */
+
+/* Variant body: runs the variant on `input`, returns its
+ * cost (default: elapsed seconds; +INFINITY = failed).  Lower is better. */
+typedef double (*nitro_variant_fn)(void *input, void *user);
+/* Feature function: same argument as the variant, returns a double. */
+typedef double (*nitro_feature_fn)(const void *input, void *user);
+/* Fused feature group: fills out[0..n) in one pass (replaces n feature calls;
+ * on the GPU one kernel computes every SpMV feature).  Returns 0 on success. */
+typedef int (*nitro_feature_group_fn)(const void *input, double *out, int n, void *user);
+/* Constraint: nonzero = the variant may run on this input. */
+typedef int (*nitro_constraint_fn)(const void *input, void *user);
+
+nitro_status_t nitro_context_create(nitro_context **out);
+void nitro_context_destroy(nitro_context *ctx);
+
+/* name: copied.  The cv keeps a pointer to ctx (must outlive it). */
+nitro_status_t nitro_cv_create(nitro_context *ctx, const char *name, nitro_cv **out);
+void nitro_cv_destroy(nitro_cv *cv);
+
+/* add_variant: label = insertion index 0..|V|-1. */
+nitro_status_t nitro_cv_add_variant(nitro_cv *cv, const char *name, nitro_variant_fn fn, void *user, int *out_id);
+/* set_default: fallback when a predicted variant is ruled out. */
+nitro_status_t nitro_cv_set_default(nitro_cv *cv, int variant_id);
+/* add_input_feature: appended to the feature table. */
+nitro_status_t nitro_cv_add_feature(nitro_cv *cv, const char *name, nitro_feature_fn fn, void *user, int *out_id);
+/* n features filled by one call (names copied). */
+nitro_status_t nitro_cv_add_feature_group(nitro_cv *cv, const char *const *names, int n,
+                                          nitro_feature_group_fn fn, void *user);
+/* add_constraint(&variant, &constraint).  Several may be
+ * added per variant; all must hold. */
+nitro_status_t nitro_cv_add_constraint(nitro_cv *cv, int variant_id, nitro_constraint_fn fn, void *user);
+/* set_training_args.  `input` is borrowed until train returns. */
+nitro_status_t nitro_cv_add_training_input(nitro_cv *cv, void *input);
+
+/* Training options (Table II of the paper is absent from the text; these are
+ * the readings of DESIGN.md "Readings" R10-R12). */
+typedef struct {
+  int folds;                      /* CV folds (default 5) */
+  uint64_t seed;                  /* fold shuffling seed (default 0) */
+  double tol;                     /* SMO stopping tolerance (default 1e-6) */
+  int log2c_lo, log2c_hi, log2c_step; /* default -5, 15, 2   (libSVM grid.py) */
+  int log2g_lo, log2g_hi, log2g_step; /* default -15, 3, 2 */
+  int verbose;                    /* 0 = silent */
+} nitro_train_opts;
+void nitro_train_opts_default(nitro_train_opts *o);
+
+/* Offline training: for every training input evaluate features,
+ * run every variant (constraint false => cost +INF), label = argmin
+ * (ties -> lowest id); scale features to [-1,1]; CV grid over (C, gamma);
+ * fit the RBF C-SVC (one-vs-one) on all inputs.  Freezes the cv (later
+ * add_* calls return NITRO_E_STATE). */
+nitro_status_t nitro_cv_train(nitro_cv *cv, const nitro_train_opts *opts);
+/* Fit from an externally measured table (same steps after labelling).
+ * feat[n_in * n_feat], cost[n_in * n_var] (row-major). */
+nitro_status_t nitro_cv_train_from_table(nitro_cv *cv, int n_in, const double *feat, const double *cost,
+                                         const nitro_train_opts *opts);
+/* Copies out the training table; any pointer may be NULL.  Sizes: cost
+ * [n_in*n_var], feat [n_in*n_feat], label [n_in]. */
+nitro_status_t nitro_cv_training_table(const nitro_cv *cv, int *n_in, double *cost, double *feat, int *label);
+/* Model facts: chosen C, gamma, CV accuracy, #support vectors. */
+nitro_status_t nitro_cv_model_info(const nitro_cv *cv, double *C, double *gamma, double *cv_acc, int *n_sv);
+nitro_status_t nitro_cv_save_model(const nitro_cv *cv, const char *path);
+nitro_status_t nitro_cv_load_model(nitro_cv *cv, const char *path);
+nitro_status_t nitro_cv_num_features(const nitro_cv *cv, int *n);
+nitro_status_t nitro_cv_num_variants(const nitro_cv *cv, int *n);
+
+/* Deployment: evaluate features, predict, check the
+ * predicted variant's constraints (fail => default).  select does not run the
+ * variant; call runs it and returns its cost.  out_feat (nullable) receives
+ * the raw feature vector. */
+nitro_status_t nitro_cv_select(nitro_cv *cv, const void *input, int *out_variant, double *out_feat);
+nitro_status_t nitro_cv_call(nitro_cv *cv, void *input, int *out_variant, double *out_cost);
+/* Select from an already-computed raw feature vector and allowed mask. */
+nitro_status_t nitro_cv_predict(nitro_cv *cv, const double *feat, const int *allowed /*nullable*/, int *out_variant);
+
+/* Host SVM primitives (the learning step of P:L61-62, L179), exposed so the
+ * host logic can be checked against libSVM without a GPU.
+ * X row-major [n*d] (already scaled), y labels >= 0. */
+typedef struct nitro_svm nitro_svm;
+nitro_status_t nitro_svm_fit(int n, int d, const double *X, const int *y, double C, double gamma, double tol,
+                             nitro_svm **out);
+nitro_status_t nitro_svm_predict(const nitro_svm *m, int n, const double *X, int *out_labels);
+/* one-vs-one decision values, pairs (i<j) in ascending class order [n * n_pairs] */
+nitro_status_t nitro_svm_decision(const nitro_svm *m, int n, const double *X, double *out, int *n_pairs);
+/* dual coefficients y_i*alpha_i of pair p for training sample ids (dense [n_train]) and rho */
+nitro_status_t nitro_svm_pair_dual(const nitro_svm *m, int p, double *coef_dense, double *rho);
+void nitro_svm_destroy(nitro_svm *m);
+/* deterministic stratified folds (R12) */
+nitro_status_t nitro_svm_fold_assign(int n, const int *y, int k, uint64_t seed, int *out_fold);
+nitro_status_t nitro_svm_cv_accuracy(int n, int d, const double *X, const int *y, double C, double gamma,
+                                     double tol, int folds, uint64_t seed, double *out_acc);
+
+/* ========================================================================
+ * 2. SpMV layer — the hot path (BASELINE north_star)
+ * ======================================================================== */
+typedef enum {
+  NITRO_CSR_SCALAR = 0, /* thread per row */
+  NITRO_CSR_VECTOR = 1, /* V lanes (2..32) per row, "a warp to each row" P:L209 */
+  NITRO_ELL = 2,        /* column-major padded ELL */
+  NITRO_DIA = 3,        /* padded diagonals */
+  NITRO_HYB = 4,        /* ELL(K) + atomic-free COO tail */
+  NITRO_NUM_VARIANTS = 5
+} nitro_spmv_variant;
+
+/* Features (P:L97-101 nnz, num_rows; P:L200, L209 AvgNZPerRow, RL-SD,
+ * MaxDeviation, DIA-Fill, ELL-Fillin).  Integer moments are exact; the
+ * doubles follow DESIGN.md R4's finishing expression bit for bit. */
+typedef struct {
+  int64_t rows, cols, nnz;
+  uint64_t sum_len, sum_len2; /* sum L_i, sum L_i^2 */
+  int64_t max_row, ndiag;     /* Lmax, number of occupied diagonals */
+  int32_t canonical, pad_;
+  double mean, sd, max_dev, dia_fill, ell_fill;
+} nitro_spmv_feat;
+
+/* Format facts after prepare. */
+typedef struct {
+  int64_t ld;         /* padded row pitch of ELL/DIA/HYB-ELL (multiple of 32) */
+  int64_t width;      /* ELL: K = Lmax; DIA: ndiag; HYB: K_hyb; CSR-vector: lanes per row */
+  int64_t tail;       /* HYB: COO tail entries; CSR-vector: number of long rows */
+  int64_t bytes;      /* device bytes owned for this format */
+  double compulsory_bytes; /* algorithmic bytes of one multiply */
+} nitro_format_info;
+
+typedef struct nitro_spmv nitro_spmv;
+
+/* Borrow a device CSR (rowptr int32 or int64 [rows+1], colidx int32 [nnz],
+ * vals fp32 or fp64 [nnz]).  Columns must be < 2^31.  Structure is checked in
+ * the feature pass, not here. */
+nitro_status_t nitro_spmv_create(int device, void *stream, int64_t rows, int64_t cols, int64_t nnz,
+                                 const void *d_rowptr, int rowptr_is_64, const int32_t *d_colidx,
+                                 const void *d_vals, int is_fp64, nitro_spmv **out);
+nitro_status_t nitro_spmv_set_stream(nitro_spmv *A, void *stream);
+/* GPU feature pass (one pass over rowptr + colidx) + host finishing.  Syncs.
+ * A non-canonical matrix (rowptr not monotone from 0 to nnz, columns not
+ * strictly increasing in a row, or out of [0, cols)) returns
+ * NITRO_E_BAD_MATRIX with out->canonical = 0.  Cached. */
+nitro_status_t nitro_spmv_features(nitro_spmv *A, nitro_spmv_feat *out);
+/* fix_inputs analogue: enqueue the feature pass now, on the
+ * handle's stream, without waiting; the next features/allowed/select waits. */
+nitro_status_t nitro_spmv_features_async(nitro_spmv *A);
+/* Constraints (R9): DIA needs dia_fill <= 3 and
+ * its padded bytes <= budget; ELL likewise with ell_fill; others always. */
+nitro_status_t nitro_spmv_allowed(nitro_spmv *A, int variant, int *out_allowed);
+/* budget for padded formats in bytes (default: 40% of free HBM at first use) */
+nitro_status_t nitro_spmv_set_budget(nitro_spmv *A, double bytes);
+/* Build the variant's format (cached; conversions are amortised). */
+nitro_status_t nitro_spmv_prepare(nitro_spmv *A, int variant);
+nitro_status_t nitro_spmv_format_info(nitro_spmv *A, int variant, nitro_format_info *out);
+/* y[rows] = A * x[cols] (overwrite), async on the handle's stream.  Prepares
+ * the format if needed (which may sync).  d_x and d_y must not alias. */
+nitro_status_t nitro_spmv_run(nitro_spmv *A, int variant, const void *d_x, void *d_y);
+/* End-to-end call with HOST buffers: copies x in, multiplies, copies y out,
+ * synchronises.  h_x / h_y should be pinned for full speed. */
+nitro_status_t nitro_spmv_run_host(nitro_spmv *A, int variant, const void *h_x, void *h_y);
+/* Timing (a variant's cost is its elapsed time): warmup runs, then
+ * `reps` runs each preceded (if flush_l2) by an L2-evicting write, CUDA events
+ * around the SpMV kernels only; returns the median in seconds.  out_all
+ * (nullable) receives all reps. */
+nitro_status_t nitro_spmv_time(nitro_spmv *A, int variant, const void *d_x, void *d_y, int warmup, int reps,
+                               int flush_l2, double *out_median_s, double *out_all);
+/* Write >= 2x L2 bytes to a scratch buffer on the handle's stream. */
+nitro_status_t nitro_spmv_flush_l2(nitro_spmv *A);
+/* Number of kernel launches one nitro_spmv_run of `variant` issues. */
+nitro_status_t nitro_spmv_launches(nitro_spmv *A, int variant, int *out);
+
+/* Export converted arrays to host (bit-exact tests).  part:
+ *  0 ELL col (int32 [K*ld]), 1 ELL val ([K*ld]),
+ *  2 DIA offsets (int32 [D]), 3 DIA val ([D*ld]),
+ *  4 HYB ELL col, 5 HYB ELL val, 6 HYB tail row (int32 [Zt]), 7 tail col, 8 tail val,
+ *  9 diagonal offsets from the feature pass (int32 [ndiag], ascending).
+ * needed receives the byte size; copies only if cap >= needed.  Syncs. */
+nitro_status_t nitro_spmv_export(nitro_spmv *A, int part, void *host_buf, size_t cap, size_t *needed);
+/* Free one variant's format (variant = -1: all). */
+nitro_status_t nitro_spmv_release(nitro_spmv *A, int variant);
+void nitro_spmv_destroy(nitro_spmv *A);
+
+/* Input record consumed by the registered SpMV variants of a nitro_cv. */
+typedef struct {
+  nitro_spmv *A;
+  const void *d_x;
+  void *d_y;
+  int warmup, reps, flush_l2; /* timing protocol for the variant cost */
+} nitro_spmv_input;
+
+/* Register on a fresh cv: the 5 variants (ids = nitro_spmv_variant), the fused
+ * feature group {nnz, rows, mean, sd, max_dev, dia_fill, ell_fill}, the DIA and
+ * ELL constraints, and default = CSR-vector (Fig. 2).  Inputs passed to
+ * train/select/call are nitro_spmv_input*. */
+nitro_status_t nitro_spmv_register(nitro_cv *cv);
+
+/* ========================================================================
+ * 3. Multi-GPU row-partitioned SpMV (north_star; one process per GPU)
+ * ======================================================================== */
+typedef struct nitro_dist nitro_dist;
+/* 128-byte NCCL unique id, created on rank 0 and broadcast by the caller. */
+nitro_status_t nitro_dist_unique_id(void *out128);
+nitro_status_t nitro_dist_init(const void *id128, int rank, int nranks, int device, nitro_dist **out);
+void nitro_dist_destroy(nitro_dist *D);
+/* nnz-balanced contiguous partition: rank r owns rows [bounds[r], bounds[r+1]),
+ * bounds[r] = first row i with rowptr[i] >= ceil(r*nnz/P) (host rowptr). */
+nitro_status_t nitro_dist_partition(int64_t rows, const int64_t *h_rowptr, int nranks, int64_t *bounds);
+/* Per-rank matrix: this rank's row block of the global matrix, with GLOBAL
+ * column ids, borrowed like nitro_spmv_create.  bounds[nranks+1] is the global
+ * row partition (x is distributed the same way).  Splits interior rows (all
+ * columns owned locally) from boundary rows and remaps columns into the
+ * gathered-x layout (block r at r*B, B = max block rows). */
+nitro_status_t nitro_dist_spmv_create(nitro_dist *D, int64_t global_rows, const int64_t *bounds,
+                                      int64_t local_nnz, const void *d_rowptr, int rowptr_is_64,
+                                      const int32_t *d_colidx, const void *d_vals, int is_fp64,
+                                      nitro_spmv **out_local);
+/* y_local = A_local * x (x all-gathered from every rank's x_local with NCCL on
+ * a side stream; interior rows overlap the gather, boundary rows follow). */
+nitro_status_t nitro_dist_spmv_run(nitro_dist *D, nitro_spmv *A_local, int variant, const void *d_x_local,
+                                   void *d_y_local);
+/* Global features from per-rank feature passes (sum / max all-reduce and a
+ * union of diagonal offsets): identical to the single-GPU features. */
+nitro_status_t nitro_dist_features(nitro_dist *D, nitro_spmv *A_local, nitro_spmv_feat *out);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* NITRO_H */

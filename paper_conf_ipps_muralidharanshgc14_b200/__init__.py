@@ -1,0 +1,530 @@
+"""paper_conf_ipps_muralidharanshgc14_b200 — B200-native Nitro SpMV code-variant hot path.
+
+Thin Python binding of libnitro.so (include/nitro.h): argument marshalling
+only.  Every step of the path — feature pass, conversions, the five SpMV
+variants, timing — runs in the library's sm_100a kernels; the SVM training and
+selection run in the library's C++ host code.  PyTorch only provides device
+memory and streams.  There is no CPU fallback: if libnitro.so is missing the
+import fails loudly.
+"""
+from __future__ import annotations
+
+import ctypes
+import math
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libnitro.so")
+
+CSR_SCALAR, CSR_VECTOR, ELL, DIA, HYB = range(5)
+NUM_VARIANTS = 5
+VARIANT_NAMES = ("csr_scalar", "csr_vector", "ell", "dia", "hyb")
+FEATURE_NAMES = ("nnz", "rows", "mean", "sd", "max_dev", "dia_fill", "ell_fill")
+
+# export parts (nitro_spmv_export)
+PART_ELL_COL, PART_ELL_VAL, PART_DIA_OFF, PART_DIA_VAL = 0, 1, 2, 3
+PART_HYB_COL, PART_HYB_VAL, PART_HYB_TROW, PART_HYB_TCOL, PART_HYB_TVAL = 4, 5, 6, 7, 8
+PART_OFFSETS = 9
+
+STATUS = {0: "OK", 1: "INVALID_ARG", 2: "BAD_MATRIX", 3: "STATE", 4: "CONSTRAINT", 5: "OOM", 6: "CUDA",
+          7: "NCCL", 8: "IO", 9: "UNSUPPORTED"}
+
+
+class NitroError(RuntimeError):
+    def __init__(self, code, msg):
+        super().__init__(f"nitro {STATUS.get(code, code)}: {msg}")
+        self.code = code
+
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"{LIB_PATH} is not built; run `python __graft_entry__.py` (build()) first")
+
+_L = ctypes.CDLL(LIB_PATH)
+
+
+class Feat(ctypes.Structure):
+    _fields_ = [("rows", ctypes.c_int64), ("cols", ctypes.c_int64), ("nnz", ctypes.c_int64),
+                ("sum_len", ctypes.c_uint64), ("sum_len2", ctypes.c_uint64),
+                ("max_row", ctypes.c_int64), ("ndiag", ctypes.c_int64),
+                ("canonical", ctypes.c_int32), ("pad_", ctypes.c_int32),
+                ("mean", ctypes.c_double), ("sd", ctypes.c_double), ("max_dev", ctypes.c_double),
+                ("dia_fill", ctypes.c_double), ("ell_fill", ctypes.c_double)]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_ if k != "pad_"}
+
+
+class FormatInfo(ctypes.Structure):
+    _fields_ = [("ld", ctypes.c_int64), ("width", ctypes.c_int64), ("tail", ctypes.c_int64),
+                ("bytes", ctypes.c_int64), ("compulsory_bytes", ctypes.c_double)]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+class TrainOpts(ctypes.Structure):
+    _fields_ = [("folds", ctypes.c_int), ("seed", ctypes.c_uint64), ("tol", ctypes.c_double),
+                ("log2c_lo", ctypes.c_int), ("log2c_hi", ctypes.c_int), ("log2c_step", ctypes.c_int),
+                ("log2g_lo", ctypes.c_int), ("log2g_hi", ctypes.c_int), ("log2g_step", ctypes.c_int),
+                ("verbose", ctypes.c_int)]
+
+
+class SpmvInput(ctypes.Structure):
+    _fields_ = [("A", ctypes.c_void_p), ("d_x", ctypes.c_void_p), ("d_y", ctypes.c_void_p),
+                ("warmup", ctypes.c_int), ("reps", ctypes.c_int), ("flush_l2", ctypes.c_int)]
+
+
+VARIANT_FN = ctypes.CFUNCTYPE(ctypes.c_double, ctypes.c_void_p, ctypes.c_void_p)
+FEATURE_FN = ctypes.CFUNCTYPE(ctypes.c_double, ctypes.c_void_p, ctypes.c_void_p)
+GROUP_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.POINTER(ctypes.c_double), ctypes.c_int,
+                            ctypes.c_void_p)
+CONSTRAINT_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p)
+
+_vp, _i64, _int, _dbl, _u64 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int, ctypes.c_double, ctypes.c_uint64
+_P = ctypes.POINTER
+_SIGS = {
+    "nitro_last_error": ([], ctypes.c_char_p),
+    "nitro_version": ([], ctypes.c_char_p),
+    # generic layer
+    "nitro_context_create": ([_P(_vp)], _int),
+    "nitro_context_destroy": ([_vp], None),
+    "nitro_cv_create": ([_vp, ctypes.c_char_p, _P(_vp)], _int),
+    "nitro_cv_destroy": ([_vp], None),
+    "nitro_cv_add_variant": ([_vp, ctypes.c_char_p, VARIANT_FN, _vp, _P(_int)], _int),
+    "nitro_cv_set_default": ([_vp, _int], _int),
+    "nitro_cv_add_feature": ([_vp, ctypes.c_char_p, FEATURE_FN, _vp, _P(_int)], _int),
+    "nitro_cv_add_feature_group": ([_vp, _P(ctypes.c_char_p), _int, GROUP_FN, _vp], _int),
+    "nitro_cv_add_constraint": ([_vp, _int, CONSTRAINT_FN, _vp], _int),
+    "nitro_cv_add_training_input": ([_vp, _vp], _int),
+    "nitro_train_opts_default": ([_P(TrainOpts)], None),
+    "nitro_cv_train": ([_vp, _P(TrainOpts)], _int),
+    "nitro_cv_train_from_table": ([_vp, _int, _vp, _vp, _P(TrainOpts)], _int),
+    "nitro_cv_training_table": ([_vp, _P(_int), _vp, _vp, _vp], _int),
+    "nitro_cv_model_info": ([_vp, _P(_dbl), _P(_dbl), _P(_dbl), _P(_int)], _int),
+    "nitro_cv_save_model": ([_vp, ctypes.c_char_p], _int),
+    "nitro_cv_load_model": ([_vp, ctypes.c_char_p], _int),
+    "nitro_cv_num_features": ([_vp, _P(_int)], _int),
+    "nitro_cv_num_variants": ([_vp, _P(_int)], _int),
+    "nitro_cv_select": ([_vp, _vp, _P(_int), _vp], _int),
+    "nitro_cv_call": ([_vp, _vp, _P(_int), _P(_dbl)], _int),
+    "nitro_cv_predict": ([_vp, _vp, _vp, _P(_int)], _int),
+    # svm
+    "nitro_svm_fit": ([_int, _int, _vp, _vp, _dbl, _dbl, _dbl, _P(_vp)], _int),
+    "nitro_svm_predict": ([_vp, _int, _vp, _vp], _int),
+    "nitro_svm_decision": ([_vp, _int, _vp, _vp, _P(_int)], _int),
+    "nitro_svm_pair_dual": ([_vp, _int, _vp, _P(_dbl)], _int),
+    "nitro_svm_destroy": ([_vp], None),
+    "nitro_svm_fold_assign": ([_int, _vp, _int, _u64, _vp], _int),
+    "nitro_svm_cv_accuracy": ([_int, _int, _vp, _vp, _dbl, _dbl, _dbl, _int, _u64, _P(_dbl)], _int),
+    # spmv
+    "nitro_spmv_create": ([_int, _vp, _i64, _i64, _i64, _vp, _int, _vp, _vp, _int, _P(_vp)], _int),
+    "nitro_spmv_set_stream": ([_vp, _vp], _int),
+    "nitro_spmv_features": ([_vp, _P(Feat)], _int),
+    "nitro_spmv_features_async": ([_vp], _int),
+    "nitro_spmv_allowed": ([_vp, _int, _P(_int)], _int),
+    "nitro_spmv_set_budget": ([_vp, _dbl], _int),
+    "nitro_spmv_prepare": ([_vp, _int], _int),
+    "nitro_spmv_format_info": ([_vp, _int, _P(FormatInfo)], _int),
+    "nitro_spmv_run": ([_vp, _int, _vp, _vp], _int),
+    "nitro_spmv_run_host": ([_vp, _int, _vp, _vp], _int),
+    "nitro_spmv_time": ([_vp, _int, _vp, _vp, _int, _int, _int, _P(_dbl), _vp], _int),
+    "nitro_spmv_flush_l2": ([_vp], _int),
+    "nitro_spmv_launches": ([_vp, _int, _P(_int)], _int),
+    "nitro_spmv_export": ([_vp, _int, _vp, ctypes.c_size_t, _P(ctypes.c_size_t)], _int),
+    "nitro_spmv_release": ([_vp, _int], _int),
+    "nitro_spmv_destroy": ([_vp], None),
+    "nitro_spmv_register": ([_vp], _int),
+    # dist
+    "nitro_dist_unique_id": ([_vp], _int),
+    "nitro_dist_init": ([_vp, _int, _int, _int, _P(_vp)], _int),
+    "nitro_dist_destroy": ([_vp], None),
+    "nitro_dist_partition": ([_i64, _vp, _int, _vp], _int),
+    "nitro_dist_spmv_create": ([_vp, _i64, _vp, _i64, _vp, _int, _vp, _vp, _int, _P(_vp)], _int),
+    "nitro_dist_spmv_run": ([_vp, _vp, _int, _vp, _vp], _int),
+    "nitro_dist_features": ([_vp, _vp, _P(Feat)], _int),
+}
+for _name, (_args, _res) in _SIGS.items():
+    _f = getattr(_L, _name)
+    _f.argtypes = _args
+    _f.restype = _res
+
+EXPORTED = tuple(_SIGS)
+
+
+def _check(rc):
+    if rc != 0:
+        raise NitroError(rc, _L.nitro_last_error().decode(errors="replace"))
+
+
+def version() -> str:
+    return _L.nitro_version().decode()
+
+
+def _ptr(t):
+    if t is None:
+        return None
+    if isinstance(t, np.ndarray):
+        return t.ctypes.data
+    return t.data_ptr()
+
+
+def _np(a, dtype):
+    return np.ascontiguousarray(np.asarray(a, dtype=dtype))
+
+
+# ====================================================================== SpMV layer
+class SpMV:
+    """A borrowed device CSR matrix (torch CUDA tensors) and its formats.
+
+    rowptr int32/int64 [rows+1], colidx int32 [nnz], vals fp32/fp64 [nnz]."""
+
+    def __init__(self, rowptr, colidx, vals, rows: int, cols: int, stream=None, device: int | None = None):
+        import torch
+        assert rowptr.is_cuda and colidx.is_cuda and vals.is_cuda, "SpMV needs CUDA tensors"
+        assert colidx.dtype == torch.int32 and rowptr.dtype in (torch.int32, torch.int64)
+        assert vals.dtype in (torch.float32, torch.float64)
+        self._keep = (rowptr, colidx, vals)
+        self.rows, self.cols, self.nnz = int(rows), int(cols), int(colidx.numel())
+        self.fp64 = vals.dtype == torch.float64
+        self.dtype = vals.dtype
+        self.device = rowptr.device.index if device is None else device
+        if stream is None:
+            stream = torch.cuda.current_stream(self.device).cuda_stream
+        self.stream = stream
+        h = ctypes.c_void_p()
+        _check(_L.nitro_spmv_create(self.device, stream, self.rows, self.cols, self.nnz, _ptr(rowptr),
+                                    int(rowptr.dtype == torch.int64), _ptr(colidx), _ptr(vals), int(self.fp64),
+                                    ctypes.byref(h)))
+        self.h = h
+
+    @classmethod
+    def from_csr(cls, A, **kw):
+        """From a synth.Csr whose arrays live on the GPU."""
+        return cls(A.rowptr, A.colidx, A.vals, A.rows, A.cols, **kw)
+
+    def close(self):
+        if getattr(self, "h", None):
+            _L.nitro_spmv_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def features(self) -> dict:
+        f = Feat()
+        _check(_L.nitro_spmv_features(self.h, ctypes.byref(f)))
+        return f.as_dict()
+
+    def features_async(self):
+        _check(_L.nitro_spmv_features_async(self.h))
+
+    def allowed(self, v: int) -> bool:
+        ok = ctypes.c_int()
+        _check(_L.nitro_spmv_allowed(self.h, v, ctypes.byref(ok)))
+        return bool(ok.value)
+
+    def allowed_mask(self):
+        return [self.allowed(v) for v in range(NUM_VARIANTS)]
+
+    def set_budget(self, nbytes: float):
+        _check(_L.nitro_spmv_set_budget(self.h, float(nbytes)))
+
+    def prepare(self, v: int):
+        _check(_L.nitro_spmv_prepare(self.h, v))
+
+    def format_info(self, v: int) -> dict:
+        fi = FormatInfo()
+        _check(_L.nitro_spmv_format_info(self.h, v, ctypes.byref(fi)))
+        return fi.as_dict()
+
+    def run(self, v: int, x, y=None):
+        import torch
+        if y is None:
+            y = torch.empty(self.rows, dtype=self.dtype, device=x.device)
+        _check(_L.nitro_spmv_run(self.h, v, _ptr(x), _ptr(y)))
+        return y
+
+    def run_host(self, v: int, x_host: np.ndarray, y_host: np.ndarray | None = None) -> np.ndarray:
+        dt = np.float64 if self.fp64 else np.float32
+        assert x_host.dtype == dt and x_host.flags.c_contiguous
+        if y_host is None:
+            y_host = np.empty(self.rows, dtype=dt)
+        _check(_L.nitro_spmv_run_host(self.h, v, _ptr(x_host), _ptr(y_host)))
+        return y_host
+
+    def time(self, v: int, x, y, warmup: int = 3, reps: int = 20, flush_l2: bool = True):
+        med = ctypes.c_double()
+        allt = np.empty(reps, dtype=np.float64)
+        _check(_L.nitro_spmv_time(self.h, v, _ptr(x), _ptr(y), warmup, reps, int(flush_l2), ctypes.byref(med),
+                                  _ptr(allt)))
+        return med.value, allt
+
+    def flush_l2(self):
+        _check(_L.nitro_spmv_flush_l2(self.h))
+
+    def launches(self, v: int) -> int:
+        n = ctypes.c_int()
+        _check(_L.nitro_spmv_launches(self.h, v, ctypes.byref(n)))
+        return n.value
+
+    def export(self, part: int) -> np.ndarray:
+        need = ctypes.c_size_t()
+        _check(_L.nitro_spmv_export(self.h, part, None, 0, ctypes.byref(need)))
+        is_val = part in (PART_ELL_VAL, PART_DIA_VAL, PART_HYB_VAL, PART_HYB_TVAL)
+        dt = (np.float64 if self.fp64 else np.float32) if is_val else np.int32
+        out = np.empty(need.value // np.dtype(dt).itemsize, dtype=dt)
+        if need.value:
+            _check(_L.nitro_spmv_export(self.h, part, _ptr(out), need.value, ctypes.byref(need)))
+        return out
+
+    def release(self, v: int = -1):
+        _check(_L.nitro_spmv_release(self.h, v))
+
+
+# ====================================================================== generic Nitro layer
+def train_opts(**kw) -> TrainOpts:
+    o = TrainOpts()
+    _L.nitro_train_opts_default(ctypes.byref(o))
+    for k, v in kw.items():
+        setattr(o, k, v)
+    return o
+
+
+class Context:
+    def __init__(self):
+        h = ctypes.c_void_p()
+        _check(_L.nitro_context_create(ctypes.byref(h)))
+        self.h = h
+
+    def __del__(self):
+        if getattr(self, "h", None):
+            _L.nitro_context_destroy(self.h)
+            self.h = None
+
+
+class CodeVariant:
+    """nitro_cv: variants, features, constraints, training inputs, model.
+
+    Inputs are opaque pointers (ints); Python callbacks receive the pointer value."""
+
+    def __init__(self, ctx: Context, name: str):
+        self.ctx = ctx
+        h = ctypes.c_void_p()
+        _check(_L.nitro_cv_create(ctx.h, name.encode(), ctypes.byref(h)))
+        self.h = h
+        self._keep = []
+
+    def __del__(self):
+        if getattr(self, "h", None):
+            _L.nitro_cv_destroy(self.h)
+            self.h = None
+
+    def add_variant(self, name, fn) -> int:
+        cb = VARIANT_FN(lambda inp, user: float(fn(inp or 0)))
+        self._keep.append(cb)
+        i = ctypes.c_int()
+        _check(_L.nitro_cv_add_variant(self.h, name.encode(), cb, None, ctypes.byref(i)))
+        return i.value
+
+    def set_default(self, vid: int):
+        _check(_L.nitro_cv_set_default(self.h, vid))
+
+    def add_feature(self, name, fn) -> int:
+        cb = FEATURE_FN(lambda inp, user: float(fn(inp or 0)))
+        self._keep.append(cb)
+        i = ctypes.c_int()
+        _check(_L.nitro_cv_add_feature(self.h, name.encode(), cb, None, ctypes.byref(i)))
+        return i.value
+
+    def add_constraint(self, vid: int, fn):
+        cb = CONSTRAINT_FN(lambda inp, user: int(bool(fn(inp or 0))))
+        self._keep.append(cb)
+        _check(_L.nitro_cv_add_constraint(self.h, vid, cb, None))
+
+    def add_training_input(self, inp):
+        _check(_L.nitro_cv_add_training_input(self.h, inp))
+
+    def register_spmv(self):
+        _check(_L.nitro_spmv_register(self.h))
+
+    def train(self, **opts):
+        o = train_opts(**opts)
+        _check(_L.nitro_cv_train(self.h, ctypes.byref(o)))
+
+    def train_from_table(self, feat, cost, **opts):
+        feat = _np(feat, np.float64)
+        cost = _np(cost, np.float64)
+        o = train_opts(**opts)
+        _check(_L.nitro_cv_train_from_table(self.h, feat.shape[0], _ptr(feat), _ptr(cost), ctypes.byref(o)))
+
+    def n_features(self):
+        n = ctypes.c_int()
+        _check(_L.nitro_cv_num_features(self.h, ctypes.byref(n)))
+        return n.value
+
+    def n_variants(self):
+        n = ctypes.c_int()
+        _check(_L.nitro_cv_num_variants(self.h, ctypes.byref(n)))
+        return n.value
+
+    def training_table(self):
+        n = ctypes.c_int()
+        _check(_L.nitro_cv_training_table(self.h, ctypes.byref(n), None, None, None))
+        nv, nf = self.n_variants(), self.n_features()
+        cost = np.empty((n.value, nv))
+        feat = np.empty((n.value, nf))
+        lab = np.empty(n.value, dtype=np.int32)
+        _check(_L.nitro_cv_training_table(self.h, ctypes.byref(n), _ptr(cost), _ptr(feat), _ptr(lab)))
+        return cost, feat, lab
+
+    def model_info(self) -> dict:
+        C, g, a, ns = ctypes.c_double(), ctypes.c_double(), ctypes.c_double(), ctypes.c_int()
+        _check(_L.nitro_cv_model_info(self.h, ctypes.byref(C), ctypes.byref(g), ctypes.byref(a), ctypes.byref(ns)))
+        return {"C": C.value, "gamma": g.value, "cv_accuracy": a.value, "n_sv": ns.value}
+
+    def save(self, path):
+        _check(_L.nitro_cv_save_model(self.h, str(path).encode()))
+
+    def load(self, path):
+        _check(_L.nitro_cv_load_model(self.h, str(path).encode()))
+
+    def select(self, inp):
+        v = ctypes.c_int()
+        f = np.empty(max(self.n_features(), 1))
+        _check(_L.nitro_cv_select(self.h, inp, ctypes.byref(v), _ptr(f)))
+        return v.value, f
+
+    def call(self, inp):
+        v, c = ctypes.c_int(), ctypes.c_double()
+        _check(_L.nitro_cv_call(self.h, inp, ctypes.byref(v), ctypes.byref(c)))
+        return v.value, c.value
+
+    def predict(self, feat, allowed=None) -> int:
+        feat = _np(feat, np.float64)
+        al = None if allowed is None else _np([int(bool(a)) for a in allowed], np.int32)
+        v = ctypes.c_int()
+        _check(_L.nitro_cv_predict(self.h, _ptr(feat), _ptr(al), ctypes.byref(v)))
+        return v.value
+
+
+def spmv_input(A: SpMV, x, y, warmup=3, reps=20, flush_l2=True) -> SpmvInput:
+    """Input record for the registered SpMV variants (keep it alive while used)."""
+    rec = SpmvInput(A.h.value, _ptr(x), _ptr(y), warmup, reps, int(flush_l2))
+    rec._keep = (A, x, y)
+    return rec
+
+
+def addr(rec) -> int:
+    return ctypes.addressof(rec)
+
+
+# ====================================================================== host SVM primitives
+class SVM:
+    def __init__(self, X, y, C, gamma, tol=1e-6):
+        X = _np(X, np.float64)
+        y = _np(y, np.int32)
+        h = ctypes.c_void_p()
+        _check(_L.nitro_svm_fit(X.shape[0], X.shape[1], _ptr(X), _ptr(y), C, gamma, tol, ctypes.byref(h)))
+        self.h, self.n, self.d = h, X.shape[0], X.shape[1]
+
+    def __del__(self):
+        if getattr(self, "h", None):
+            _L.nitro_svm_destroy(self.h)
+            self.h = None
+
+    def predict(self, X):
+        X = _np(X, np.float64)
+        out = np.empty(X.shape[0], dtype=np.int32)
+        _check(_L.nitro_svm_predict(self.h, X.shape[0], _ptr(X), _ptr(out)))
+        return out
+
+    def decision(self, X):
+        X = _np(X, np.float64)
+        npairs = ctypes.c_int()
+        _check(_L.nitro_svm_decision(self.h, 0, None, None, ctypes.byref(npairs)))
+        out = np.empty((X.shape[0], npairs.value))
+        _check(_L.nitro_svm_decision(self.h, X.shape[0], _ptr(X), _ptr(out), ctypes.byref(npairs)))
+        return out
+
+    def pair_dual(self, p: int):
+        coef = np.empty(self.n)
+        rho = ctypes.c_double()
+        _check(_L.nitro_svm_pair_dual(self.h, p, _ptr(coef), ctypes.byref(rho)))
+        return coef, rho.value
+
+
+def fold_assign(y, k: int, seed: int = 0) -> np.ndarray:
+    y = _np(y, np.int32)
+    out = np.empty(y.shape[0], dtype=np.int32)
+    _check(_L.nitro_svm_fold_assign(y.shape[0], _ptr(y), k, seed, _ptr(out)))
+    return out
+
+
+def cv_accuracy(X, y, C, gamma, tol=1e-6, folds=5, seed=0) -> float:
+    X = _np(X, np.float64)
+    y = _np(y, np.int32)
+    acc = ctypes.c_double()
+    _check(_L.nitro_svm_cv_accuracy(X.shape[0], X.shape[1], _ptr(X), _ptr(y), C, gamma, tol, folds, seed,
+                                    ctypes.byref(acc)))
+    return acc.value
+
+
+# ====================================================================== multi-GPU
+def dist_partition(rowptr_host, nranks: int) -> np.ndarray:
+    rp = _np(rowptr_host, np.int64)
+    out = np.empty(nranks + 1, dtype=np.int64)
+    _check(_L.nitro_dist_partition(rp.shape[0] - 1, _ptr(rp), nranks, _ptr(out)))
+    return out
+
+
+def dist_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(_L.nitro_dist_unique_id(buf))
+    return buf.raw
+
+
+class Dist:
+    def __init__(self, uid: bytes, rank: int, nranks: int, device: int):
+        buf = ctypes.create_string_buffer(uid, 128)
+        h = ctypes.c_void_p()
+        _check(_L.nitro_dist_init(buf, rank, nranks, device, ctypes.byref(h)))
+        self.h, self.rank, self.nranks, self.device = h, rank, nranks, device
+
+    def close(self):
+        if getattr(self, "h", None):
+            _L.nitro_dist_destroy(self.h)
+            self.h = None
+
+    def spmv(self, global_rows, bounds, rowptr, colidx, vals):
+        """This rank's row block (global column ids) -> SpMV handle for dist runs."""
+        import torch
+        b = _np(bounds, np.int64)
+        h = ctypes.c_void_p()
+        _check(_L.nitro_dist_spmv_create(self.h, global_rows, _ptr(b), colidx.numel(), _ptr(rowptr),
+                                         int(rowptr.dtype == torch.int64), _ptr(colidx), _ptr(vals),
+                                         int(vals.dtype == torch.float64), ctypes.byref(h)))
+        A = SpMV.__new__(SpMV)
+        A._keep = (rowptr, colidx, vals)
+        A.rows = int(b[self.rank + 1] - b[self.rank])
+        A.cols = int(global_rows)
+        A.nnz = int(colidx.numel())
+        A.fp64 = vals.dtype == torch.float64
+        A.dtype = vals.dtype
+        A.device = self.device
+        A.stream = None
+        A.h = h
+        return A
+
+    def run(self, A: SpMV, v: int, x_local, y_local):
+        _check(_L.nitro_dist_spmv_run(self.h, A.h, v, _ptr(x_local), _ptr(y_local)))
+        return y_local
+
+    def features(self, A: SpMV) -> dict:
+        f = Feat()
+        _check(_L.nitro_dist_features(self.h, A.h, ctypes.byref(f)))
+        return f.as_dict()

@@ -1,0 +1,397 @@
+// capi.cu — the SpMV layer of the C ABI (include/nitro.h §2) + shared plumbing.
+#include "nitro_internal.h"
+
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <new>
+#include <vector>
+
+namespace nitro {
+
+static thread_local std::string g_err;
+
+void set_error(const std::string &msg) { g_err = msg; }
+nitro_status_t fail(nitro_status_t code, const std::string &msg) {
+  g_err = msg;
+  return code;
+}
+nitro_status_t cuda_fail(cudaError_t e, const char *where) {
+  g_err = std::string("CUDA error ") + cudaGetErrorName(e) + " (" + cudaGetErrorString(e) + ") at " + where;
+  return e == cudaErrorMemoryAllocation ? NITRO_E_OOM : NITRO_E_CUDA;
+}
+
+nitro_status_t DevBuf::alloc(size_t n) {
+  if (n <= bytes && p) return NITRO_OK;
+  release();
+  if (n == 0) n = 16;
+  cudaError_t e = cudaMalloc(&p, n);
+  if (e != cudaSuccess) {
+    p = nullptr;
+    bytes = 0;
+    (void)cudaGetLastError();
+    return cuda_fail(e, "cudaMalloc");
+  }
+  bytes = n;
+  return NITRO_OK;
+}
+void DevBuf::release() {
+  if (p) cudaFree(p);
+  p = nullptr;
+  bytes = 0;
+}
+
+int num_sms() {
+  static int cached[64] = {0};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 0 || dev >= 64) dev = 0;
+  if (!cached[dev]) {
+    int n = 0;
+    if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n <= 0) n = 148;
+    cached[dev] = n;
+  }
+  return cached[dev];
+}
+
+namespace {
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+bool valid_variant(int v) { return v >= 0 && v < NITRO_NUM_VARIANTS; }
+
+nitro_status_t ensure_budget(nitro_spmv *A) {
+  if (A->budget >= 0) return NITRO_OK;
+  size_t fr = 0, tot = 0;
+  NITRO_CUDA(cudaMemGetInfo(&fr, &tot));
+  A->budget = 0.4 * (double)fr;
+  return NITRO_OK;
+}
+
+// C9 constraints (R9)
+nitro_status_t allowed_impl(nitro_spmv *A, int v, int *out) {
+  NITRO_TRY(features_finish(A));
+  NITRO_TRY(ensure_budget(A));
+  const double ld = (double)round_up(A->N, 32), sv = A->fp64 ? 8 : 4;
+  const nitro_spmv_feat &f = A->feat;
+  switch (v) {
+    case NITRO_DIA: *out = f.dia_fill <= 3.0 && (double)f.ndiag * ld * sv <= A->budget; break;
+    case NITRO_ELL: *out = f.ell_fill <= 3.0 && (double)f.max_row * ld * (sv + 4) <= A->budget; break;
+    default: *out = 1;
+  }
+  return NITRO_OK;
+}
+
+nitro_status_t prepare_impl(nitro_spmv *A, int v) {
+  int ok = 0;
+  NITRO_TRY(allowed_impl(A, v, &ok));
+  if (!ok) return fail(NITRO_E_CONSTRAINT, "variant ruled out by its constraint for this matrix");
+  switch (v) {
+    case NITRO_CSR_SCALAR: return NITRO_OK;
+    case NITRO_CSR_VECTOR: return prepare_csrv(A);
+    case NITRO_ELL: return prepare_ell(A);
+    case NITRO_DIA: return prepare_dia(A);
+    case NITRO_HYB: return prepare_hyb(A);
+  }
+  return fail(NITRO_E_INVALID_ARG, "bad variant");
+}
+
+bool is_ready(const nitro_spmv *A, int v) {
+  switch (v) {
+    case NITRO_CSR_SCALAR: return A->feat_ready && A->feat.canonical;
+    case NITRO_CSR_VECTOR: return A->csrv.ready;
+    case NITRO_ELL: return A->ell.ready;
+    case NITRO_DIA: return A->dia.ready;
+    case NITRO_HYB: return A->hyb.ready;
+  }
+  return false;
+}
+
+}  // namespace
+}  // namespace nitro
+
+using namespace nitro;
+
+#define NITRO_GUARD_BEGIN try {
+#define NITRO_GUARD_END                                              \
+  }                                                                  \
+  catch (const std::bad_alloc &) {                                   \
+    return fail(NITRO_E_OOM, "host allocation failed");             \
+  }                                                                  \
+  catch (...) {                                                      \
+    return fail(NITRO_E_INVALID_ARG, "unexpected exception");       \
+  }
+
+extern "C" {
+
+const char *nitro_last_error(void) { return g_err.c_str(); }
+const char *nitro_version(void) { return "nitro-b200 0.1 (sm_100a)"; }
+
+nitro_status_t nitro_spmv_create(int device, void *stream, int64_t rows, int64_t cols, int64_t nnz,
+                                 const void *d_rowptr, int rowptr_is_64, const int32_t *d_colidx, const void *d_vals,
+                                 int is_fp64, nitro_spmv **out) {
+  NITRO_GUARD_BEGIN
+  if (!out) return fail(NITRO_E_INVALID_ARG, "out is NULL");
+  *out = nullptr;
+  if (rows < 0 || cols < 0 || nnz < 0) return fail(NITRO_E_INVALID_ARG, "negative size");
+  if (!d_rowptr) return fail(NITRO_E_INVALID_ARG, "rowptr is NULL");
+  if (nnz > 0 && (!d_colidx || !d_vals)) return fail(NITRO_E_INVALID_ARG, "colidx/vals NULL with nnz > 0");
+  if (cols > 2147483647LL || rows > 2147483647LL) return fail(NITRO_E_UNSUPPORTED, "rows/cols must be < 2^31");
+  if (!rowptr_is_64 && nnz > 2147483647LL) return fail(NITRO_E_INVALID_ARG, "nnz >= 2^31 needs a 64-bit rowptr");
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev)
+    return fail(NITRO_E_CUDA, "no such CUDA device");
+  nitro_spmv *A = new nitro_spmv();
+  A->device = device;
+  A->stream = (cudaStream_t)stream;
+  A->N = rows; A->M = cols; A->Z = nnz;
+  A->rowptr = d_rowptr; A->rp64 = rowptr_is_64 != 0;
+  A->col = d_colidx; A->val = d_vals; A->fp64 = is_fp64 != 0;
+  *out = A;
+  return NITRO_OK;
+  NITRO_GUARD_END
+}
+
+nitro_status_t nitro_spmv_set_stream(nitro_spmv *A, void *stream) {
+  if (!A) return fail(NITRO_E_INVALID_ARG, "NULL handle");
+  A->stream = (cudaStream_t)stream;
+  return NITRO_OK;
+}
+
+nitro_status_t nitro_spmv_features(nitro_spmv *A, nitro_spmv_feat *out) {
+  NITRO_GUARD_BEGIN
+  if (!A || !out) return fail(NITRO_E_INVALID_ARG, "NULL argument");
+  DeviceGuard g(A->device);
+  nitro_status_t st = features_finish(A);
+  if (A->feat_ready) *out = A->feat;
+  return st;
+  NITRO_GUARD_END
+}
+
+nitro_status_t nitro_spmv_features_async(nitro_spmv *A) {
+  NITRO_GUARD_BEGIN
+  if (!A) return fail(NITRO_E_INVALID_ARG, "NULL handle");
+  DeviceGuard g(A->device);
+  return features_launch(A);
+  NITRO_GUARD_END
+}
+
+nitro_status_t nitro_spmv_allowed(nitro_spmv *A, int variant, int *out_allowed) {
+  NITRO_GUARD_BEGIN
+  if (!A || !out_allowed || !valid_variant(variant)) return fail(NITRO_E_INVALID_ARG, "bad argument");
+  DeviceGuard g(A->device);
+  return allowed_impl(A, variant, out_allowed);
+  NITRO_GUARD_END
+}
+
+nitro_status_t nitro_spmv_set_budget(nitro_spmv *A, double bytes) {
+  if (!A || !(bytes >= 0)) return fail(NITRO_E_INVALID_ARG, "bad argument");
+  A->budget = bytes;
+  return NITRO_OK;
+}
+
+nitro_status_t nitro_spmv_prepare(nitro_spmv *A, int variant) {
+  NITRO_GUARD_BEGIN
+  if (!A || !valid_variant(variant)) return fail(NITRO_E_INVALID_ARG, "bad argument");
+  DeviceGuard g(A->device);
+  if (is_ready(A, variant)) return NITRO_OK;
+  return prepare_impl(A, variant);
+  NITRO_GUARD_END
+}
+
+nitro_status_t nitro_spmv_format_info(nitro_spmv *A, int variant, nitro_format_info *out) {
+  NITRO_GUARD_BEGIN
+  if (!A || !out || !valid_variant(variant)) return fail(NITRO_E_INVALID_ARG, "bad argument");
+  DeviceGuard g(A->device);
+  if (!is_ready(A, variant)) NITRO_TRY(prepare_impl(A, variant));
+  memset(out, 0, sizeof(*out));
+  switch (variant) {
+    case NITRO_CSR_SCALAR: out->width = 1; break;
+    case NITRO_CSR_VECTOR: out->width = A->csrv.V; out->tail = A->csrv.n_long; out->bytes = (int64_t)A->csrv.long_rows.bytes; break;
+    case NITRO_ELL: out->ld = A->ell.ld; out->width = A->ell.K; out->bytes = (int64_t)(A->ell.col.bytes + A->ell.val.bytes); break;
+    case NITRO_DIA: out->ld = A->dia.ld; out->width = A->dia.D; out->bytes = (int64_t)(A->dia.off.bytes + A->dia.val.bytes); break;
+    case NITRO_HYB:
+      out->ld = A->hyb.ld; out->width = A->hyb.K; out->tail = A->hyb.Zt;
+      out->bytes = (int64_t)(A->hyb.col.bytes + A->hyb.val.bytes + A->hyb.trow.bytes + A->hyb.tcol.bytes +
+                             A->hyb.tval.bytes + A->hyb.carry_row.bytes + A->hyb.carry_val.bytes);
+      break;
+  }
+  out->compulsory_bytes = compulsory_bytes(A, variant);
+  return NITRO_OK;
+  NITRO_GUARD_END
+}
+
+nitro_status_t nitro_spmv_run(nitro_spmv *A, int variant, const void *d_x, void *d_y) {
+  NITRO_GUARD_BEGIN
+  if (!A || !valid_variant(variant)) return fail(NITRO_E_INVALID_ARG, "bad argument");
+  if ((A->M > 0 && !d_x) || (A->N > 0 && !d_y)) return fail(NITRO_E_INVALID_ARG, "x or y is NULL");
+  DeviceGuard g(A->device);
+  if (!is_ready(A, variant)) NITRO_TRY(prepare_impl(A, variant));
+  return launch_spmv(A, variant, d_x, d_y, A->stream);
+  NITRO_GUARD_END
+}
+
+nitro_status_t nitro_spmv_run_host(nitro_spmv *A, int variant, const void *h_x, void *h_y) {
+  NITRO_GUARD_BEGIN
+  if (!A || !valid_variant(variant)) return fail(NITRO_E_INVALID_ARG, "bad argument");
+  if ((A->M > 0 && !h_x) || (A->N > 0 && !h_y)) return fail(NITRO_E_INVALID_ARG, "x or y is NULL");
+  DeviceGuard g(A->device);
+  if (!is_ready(A, variant)) NITRO_TRY(prepare_impl(A, variant));
+  const size_t sv = A->fp64 ? 8 : 4;
+  NITRO_TRY(A->xbuf.alloc(std::max<size_t>(A->M * sv, 16)));
+  NITRO_TRY(A->ybuf.alloc(std::max<size_t>(A->N * sv, 16)));
+  if (A->M) NITRO_CUDA(cudaMemcpyAsync(A->xbuf.p, h_x, A->M * sv, cudaMemcpyHostToDevice, A->stream));
+  NITRO_TRY(launch_spmv(A, variant, A->xbuf.p, A->ybuf.p, A->stream));
+  if (A->N) NITRO_CUDA(cudaMemcpyAsync(h_y, A->ybuf.p, A->N * sv, cudaMemcpyDeviceToHost, A->stream));
+  NITRO_CUDA(cudaStreamSynchronize(A->stream));
+  return NITRO_OK;
+  NITRO_GUARD_END
+}
+
+nitro_status_t nitro_spmv_flush_l2(nitro_spmv *A) {
+  NITRO_GUARD_BEGIN
+  if (!A) return fail(NITRO_E_INVALID_ARG, "NULL handle");
+  DeviceGuard g(A->device);
+  return launch_flush(A, A->stream);
+  NITRO_GUARD_END
+}
+
+nitro_status_t nitro_spmv_time(nitro_spmv *A, int variant, const void *d_x, void *d_y, int warmup, int reps,
+                               int flush_l2, double *out_median_s, double *out_all) {
+  NITRO_GUARD_BEGIN
+  if (!A || !valid_variant(variant) || reps < 1 || warmup < 0 || !out_median_s)
+    return fail(NITRO_E_INVALID_ARG, "bad argument");
+  DeviceGuard g(A->device);
+  if (!is_ready(A, variant)) NITRO_TRY(prepare_impl(A, variant));
+  cudaStream_t s = A->stream;
+  for (int w = 0; w < warmup; ++w) NITRO_TRY(launch_spmv(A, variant, d_x, d_y, s));
+  std::vector<cudaEvent_t> ev(2 * reps, nullptr);
+  for (auto &e : ev) NITRO_CUDA(cudaEventCreate(&e));
+  nitro_status_t st = NITRO_OK;
+  for (int r = 0; r < reps && st == NITRO_OK; ++r) {
+    if (flush_l2) st = launch_flush(A, s);
+    if (st == NITRO_OK) {
+      cudaEventRecord(ev[2 * r], s);
+      st = launch_spmv(A, variant, d_x, d_y, s);
+      cudaEventRecord(ev[2 * r + 1], s);
+    }
+  }
+  std::vector<double> t(reps, 0.0);
+  cudaError_t e = cudaStreamSynchronize(s);
+  if (st == NITRO_OK && e != cudaSuccess) st = cuda_fail(e, "cudaStreamSynchronize");
+  for (int r = 0; r < reps && st == NITRO_OK; ++r) {
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, ev[2 * r], ev[2 * r + 1]);
+    t[r] = ms * 1e-3;
+  }
+  for (auto &x : ev) cudaEventDestroy(x);
+  if (st != NITRO_OK) return st;
+  if (out_all) std::copy(t.begin(), t.end(), out_all);
+  std::sort(t.begin(), t.end());
+  *out_median_s = reps % 2 ? t[reps / 2] : 0.5 * (t[reps / 2 - 1] + t[reps / 2]);
+  return NITRO_OK;
+  NITRO_GUARD_END
+}
+
+nitro_status_t nitro_spmv_launches(nitro_spmv *A, int variant, int *out) {
+  NITRO_GUARD_BEGIN
+  if (!A || !out || !valid_variant(variant)) return fail(NITRO_E_INVALID_ARG, "bad argument");
+  DeviceGuard g(A->device);
+  if (!is_ready(A, variant)) NITRO_TRY(prepare_impl(A, variant));
+  *out = launches_of(A, variant);
+  return NITRO_OK;
+  NITRO_GUARD_END
+}
+
+nitro_status_t nitro_spmv_export(nitro_spmv *A, int part, void *host_buf, size_t cap, size_t *needed) {
+  NITRO_GUARD_BEGIN
+  if (!A || !needed) return fail(NITRO_E_INVALID_ARG, "NULL argument");
+  DeviceGuard g(A->device);
+  const size_t sv = A->fp64 ? 8 : 4;
+  const void *src = nullptr;
+  size_t n = 0;
+  DevBuf tmp;
+  if (part <= 1) {
+    NITRO_TRY(nitro_spmv_prepare(A, NITRO_ELL));
+    n = (size_t)(A->ell.K * A->ell.ld) * (part == 0 ? 4 : sv);
+    src = part == 0 ? A->ell.col.p : A->ell.val.p;
+  } else if (part <= 3) {
+    NITRO_TRY(nitro_spmv_prepare(A, NITRO_DIA));
+    n = part == 2 ? (size_t)A->dia.D * 4 : (size_t)(A->dia.D * A->dia.ld) * sv;
+    src = part == 2 ? A->dia.off.p : A->dia.val.p;
+  } else if (part <= 8) {
+    NITRO_TRY(nitro_spmv_prepare(A, NITRO_HYB));
+    const size_t ke = (size_t)(A->hyb.K * A->hyb.ld), zt = (size_t)A->hyb.Zt;
+    switch (part) {
+      case 4: n = ke * 4; src = A->hyb.col.p; break;
+      case 5: n = ke * sv; src = A->hyb.val.p; break;
+      case 6: n = zt * 4; src = A->hyb.trow.p; break;
+      case 7: n = zt * 4; src = A->hyb.tcol.p; break;
+      default: n = zt * sv; src = A->hyb.tval.p; break;
+    }
+  } else if (part == 9) {
+    // ascending diagonal offsets of the feature pass (same emit as DIA prepare)
+    NITRO_TRY(features_finish(A));
+    if (!A->dia.ready) {
+      // emit without building DIA values: reuse prepare_dia only when allowed, else emit directly
+      int ok = 0;
+      NITRO_TRY(allowed_impl(A, NITRO_DIA, &ok));
+      if (ok) NITRO_TRY(prepare_dia(A));
+    }
+    if (A->dia.ready) {
+      n = (size_t)A->dia.D * 4;
+      src = A->dia.off.p;
+    } else {
+      return fail(NITRO_E_CONSTRAINT, "diagonal list is only materialised for DIA-allowed matrices");
+    }
+  } else {
+    return fail(NITRO_E_INVALID_ARG, "bad part");
+  }
+  *needed = n;
+  if (host_buf && cap >= n && n > 0) {
+    NITRO_CUDA(cudaMemcpyAsync(host_buf, src, n, cudaMemcpyDeviceToHost, A->stream));
+    NITRO_CUDA(cudaStreamSynchronize(A->stream));
+  }
+  return NITRO_OK;
+  NITRO_GUARD_END
+}
+
+nitro_status_t nitro_spmv_release(nitro_spmv *A, int variant) {
+  if (!A) return fail(NITRO_E_INVALID_ARG, "NULL handle");
+  DeviceGuard g(A->device);
+  cudaStreamSynchronize(A->stream);
+  if (variant == -1 || variant == NITRO_ELL) { A->ell.col.release(); A->ell.val.release(); A->ell.ready = false; }
+  if (variant == -1 || variant == NITRO_DIA) { A->dia.off.release(); A->dia.val.release(); A->dia.ready = false; }
+  if (variant == -1 || variant == NITRO_HYB) {
+    A->hyb.col.release(); A->hyb.val.release(); A->hyb.trow.release(); A->hyb.tcol.release();
+    A->hyb.tval.release(); A->hyb.carry_row.release(); A->hyb.carry_val.release(); A->hyb.ready = false;
+  }
+  if (variant == -1 || variant == NITRO_CSR_VECTOR) { A->csrv.long_rows.release(); A->csrv.ready = false; }
+  return NITRO_OK;
+}
+
+void nitro_spmv_destroy(nitro_spmv *A) {
+  if (!A) return;
+  {
+    DeviceGuard g(A->device);
+    cudaStreamSynchronize(A->stream);
+    nitro_spmv_release(A, -1);
+    if (A->h_acc) cudaFreeHost(A->h_acc);
+    if (A->feat_done) cudaEventDestroy(A->feat_done);
+    A->feat_acc.release(); A->bitmap.release(); A->offsets.release(); A->scratch.release();
+    A->flush.release(); A->xbuf.release(); A->ybuf.release();
+  }
+  delete A;
+}
+
+}  // extern "C"

@@ -1,0 +1,351 @@
+// convert.cu — A5: CSR -> ELL / DIA / HYB(ELL + COO tail), and the CSR-vector
+// long-row segment table.  Conversions are cached per matrix and excluded from
+// variant time (their cost is amortised over repeated SpMVs).
+//
+// Layouts (R5-R7): column-major, pitch ld = round_up(N, 32) rows so
+// every (slot, 4-row group) is 16-byte aligned for 128-bit loads; ELL padding
+// col = -1, val = 0; DIA indexed by row (val[d*ld + i] = a(i, i+off_d));
+// HYB = ELL of width K_hyb + tail (row, col, val) in CSR order.
+#include "nitro_internal.h"
+#include "util.cuh"
+
+#include <algorithm>
+#include <vector>
+
+namespace nitro {
+namespace {
+
+template <typename IT, typename VT>
+__global__ void k_fill_ell(const IT *__restrict__ rowptr, const int32_t *__restrict__ col, const VT *__restrict__ val,
+                           int64_t N, int64_t K, int64_t ld, int32_t *__restrict__ ecol, VT *__restrict__ eval,
+                           const int64_t *__restrict__ toff, int32_t *__restrict__ trow, int32_t *__restrict__ tcol,
+                           VT *__restrict__ tval) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < ld; i += (int64_t)gridDim.x * blockDim.x) {
+    int64_t a = 0, L = 0;
+    if (i < N) { a = (int64_t)rowptr[i]; L = (int64_t)rowptr[i + 1] - a; }
+    for (int64_t k = 0; k < K; ++k) {
+      const bool in = k < L;
+      ecol[k * ld + i] = in ? col[a + k] : -1;
+      eval[k * ld + i] = in ? val[a + k] : (VT)0;
+    }
+    if (toff && L > K) {
+      int64_t o = toff[i];
+      for (int64_t k = K; k < L; ++k, ++o) {
+        trow[o] = (int32_t)i;
+        tcol[o] = col[a + k];
+        tval[o] = val[a + k];
+      }
+    }
+  }
+}
+
+// tail count per row (HYB): max(L_i - K, 0)
+template <typename IT>
+__global__ void k_tail_counts(const IT *__restrict__ rowptr, int64_t N, int64_t K, int64_t *__restrict__ cnt) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < N; i += (int64_t)gridDim.x * blockDim.x) {
+    int64_t L = (int64_t)rowptr[i + 1] - (int64_t)rowptr[i];
+    cnt[i] = L > K ? L - K : 0;
+  }
+}
+
+// histogram of row lengths over the window [k0, k0 + W): bins[t] = #rows with
+// L == k0 + t, bins[W] = #rows with L >= k0 + W.
+template <typename IT, int W>
+__global__ void __launch_bounds__(256) k_len_hist(const IT *__restrict__ rowptr, int64_t N, int64_t k0,
+                                                  unsigned long long *__restrict__ bins) {
+  __shared__ unsigned s[W + 1];
+  for (int t = threadIdx.x; t <= W; t += blockDim.x) s[t] = 0;
+  __syncthreads();
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < N; i += (int64_t)gridDim.x * blockDim.x) {
+    int64_t L = (int64_t)rowptr[i + 1] - (int64_t)rowptr[i];
+    int64_t t = L - k0;
+    if (t < 0) continue;
+    int b = t >= W ? W : (int)t;
+    // warp-aggregated increment: lanes with the same bin add once
+    unsigned grp = __match_any_sync(__activemask(), b);
+    if ((int)(__ffs(grp) - 1) == (int)(threadIdx.x & 31)) atomicAdd(&s[b], (unsigned)__popc(grp));
+  }
+  __syncthreads();
+  for (int t = threadIdx.x; t <= W; t += blockDim.x)
+    if (s[t]) atomicAdd(&bins[t], (unsigned long long)s[t]);
+}
+
+// DIA offsets: popcount per tile of 1024 bitmap words, then emit ascending
+__global__ void __launch_bounds__(256) k_popc_tiles(const uint32_t *__restrict__ bm, int64_t nwords,
+                                                    int64_t *__restrict__ cnt) {
+  int64_t base = (int64_t)blockIdx.x * 1024;
+  int64_t s = 0;
+  for (int t = threadIdx.x; t < 1024; t += 256)
+    if (base + t < nwords) s += __popc(bm[base + t]);
+  s = block_sum_i64<256>(s);
+  if (threadIdx.x == 0) cnt[blockIdx.x] = s;
+}
+__global__ void __launch_bounds__(256) k_emit_offsets(const uint32_t *__restrict__ bm, int64_t nwords,
+                                                      const int64_t *__restrict__ tile_off, int64_t G,
+                                                      int32_t *__restrict__ out) {
+  int64_t base = (int64_t)blockIdx.x * 1024 + threadIdx.x * 4;
+  uint32_t w[4];
+  int64_t c = 0;
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    w[q] = base + q < nwords ? bm[base + q] : 0u;
+    c += __popc(w[q]);
+  }
+  int64_t agg;
+  int64_t o = tile_off[blockIdx.x] + block_exclusive_i64<256>(c, agg);
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    uint32_t v = w[q];
+    while (v) {
+      int b = __ffs(v) - 1;
+      v &= v - 1;
+      out[o++] = (int32_t)((base + q) * 32 + b - G);
+    }
+  }
+}
+
+template <typename IT, typename VT>
+__global__ void k_fill_dia(const IT *__restrict__ rowptr, const int32_t *__restrict__ col, const VT *__restrict__ val,
+                           int64_t N, int64_t row0, const int32_t *__restrict__ offs, int64_t D, int64_t ld,
+                           VT *__restrict__ dval) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < N; i += (int64_t)gridDim.x * blockDim.x) {
+    int64_t a = (int64_t)rowptr[i], b = (int64_t)rowptr[i + 1];
+    if (a == b) continue;
+    // binary search the first entry's offset, then walk (offsets ascend with columns)
+    int64_t off0 = (int64_t)col[a] - (row0 + i);
+    int64_t lo = 0, hi = D;
+    while (lo < hi) {
+      int64_t mid = (lo + hi) >> 1;
+      if ((int64_t)__ldg(offs + mid) < off0) lo = mid + 1; else hi = mid;
+    }
+    int64_t d = lo;
+    for (int64_t k = a; k < b; ++k) {
+      int64_t off = (int64_t)col[k] - (row0 + i);
+      while (d < D && (int64_t)__ldg(offs + d) < off) ++d;
+      dval[d * ld + i] = val[k];
+    }
+  }
+}
+
+// CSR-vector long rows: flag rows with L > T, then emit row ids ascending
+template <typename IT>
+__global__ void k_long_flags(const IT *__restrict__ rowptr, int64_t N, int64_t T, int64_t S,
+                             int64_t *__restrict__ nseg) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < N; i += (int64_t)gridDim.x * blockDim.x) {
+    int64_t L = (int64_t)rowptr[i + 1] - (int64_t)rowptr[i];
+    nseg[i] = L > T ? (L + S - 1) / S : 0;
+  }
+}
+// segment table: seg_row[s], seg_first[s] (index of the row's first segment),
+// seg_count[s]; segments of a row are consecutive.
+template <typename IT>
+__global__ void k_long_emit(const IT *__restrict__ rowptr, int64_t N, const int64_t *__restrict__ segoff,
+                            int32_t *__restrict__ seg_row, int32_t *__restrict__ seg_k) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < N; i += (int64_t)gridDim.x * blockDim.x) {
+    int64_t s0 = segoff[i], s1 = segoff[i + 1];
+    for (int64_t s = s0; s < s1; ++s) {
+      seg_row[s] = (int32_t)i;
+      seg_k[s] = (int32_t)(s - s0);  // segment ordinal within its row
+    }
+  }
+}
+
+unsigned grid_of(int64_t n, int threads = 256) {
+  int64_t g = (n + threads - 1) / threads;
+  int64_t cap = (int64_t)num_sms() * 16;
+  if (g > cap) g = cap;
+  return (unsigned)(g < 1 ? 1 : g);
+}
+
+template <typename IT, typename VT>
+nitro_status_t fill_ell_t(nitro_spmv *A, int64_t K, int64_t ld, int32_t *ecol, VT *eval, const int64_t *toff,
+                          int32_t *trow, int32_t *tcol, VT *tval) {
+  k_fill_ell<IT, VT><<<grid_of(ld), 256, 0, A->stream>>>((const IT *)A->rowptr, A->col, (const VT *)A->val, A->N, K,
+                                                         ld, ecol, eval, toff, trow, tcol, tval);
+  NITRO_CUDA(cudaGetLastError());
+  return NITRO_OK;
+}
+
+nitro_status_t fill_ell(nitro_spmv *A, int64_t K, int64_t ld, void *ecol, void *eval, const int64_t *toff,
+                        void *trow, void *tcol, void *tval) {
+  if (A->rp64) {
+    if (A->fp64) return fill_ell_t<int64_t, double>(A, K, ld, (int32_t *)ecol, (double *)eval, toff, (int32_t *)trow, (int32_t *)tcol, (double *)tval);
+    return fill_ell_t<int64_t, float>(A, K, ld, (int32_t *)ecol, (float *)eval, toff, (int32_t *)trow, (int32_t *)tcol, (float *)tval);
+  }
+  if (A->fp64) return fill_ell_t<int32_t, double>(A, K, ld, (int32_t *)ecol, (double *)eval, toff, (int32_t *)trow, (int32_t *)tcol, (double *)tval);
+  return fill_ell_t<int32_t, float>(A, K, ld, (int32_t *)ecol, (float *)eval, toff, (int32_t *)trow, (int32_t *)tcol, (float *)tval);
+}
+
+}  // namespace
+
+// ------------------------------------------------------------------ ELL (C5)
+nitro_status_t prepare_ell(nitro_spmv *A) {
+  if (A->ell.ready) return NITRO_OK;
+  NITRO_TRY(features_finish(A));
+  const int64_t K = A->feat.max_row, ld = round_up(A->N, 32), sv = A->fp64 ? 8 : 4;
+  NITRO_TRY(A->ell.col.alloc((size_t)std::max<int64_t>(K * ld, 1) * 4));
+  NITRO_TRY(A->ell.val.alloc((size_t)std::max<int64_t>(K * ld, 1) * sv));
+  if (K > 0) NITRO_TRY(fill_ell(A, K, ld, A->ell.col.p, A->ell.val.p, nullptr, nullptr, nullptr, nullptr));
+  A->ell.K = K;
+  A->ell.ld = ld;
+  A->ell.ready = true;
+  return NITRO_OK;
+}
+
+// ------------------------------------------------------------------ DIA (C6)
+nitro_status_t prepare_dia(nitro_spmv *A) {
+  if (A->dia.ready) return NITRO_OK;
+  NITRO_TRY(features_finish(A));
+  cudaStream_t s = A->stream;
+  const int64_t D = A->feat.ndiag, ld = round_up(A->N, 32), sv = A->fp64 ? 8 : 4;
+  const int64_t G = A->row0 + A->N - 1;
+  const int64_t span = A->N > 0 ? G + A->M : 0, nwords = (span + 31) / 32;
+  NITRO_TRY(A->dia.off.alloc((size_t)std::max<int64_t>(D, 1) * 4));
+  if (D > 0) {
+    const int64_t nt = (nwords + 1023) / 1024;
+    DevBuf cnt;
+    NITRO_TRY(cnt.alloc((size_t)(2 * nt + 2) * 8));
+    int64_t *tile_cnt = cnt.as<int64_t>(), *tile_off = tile_cnt + nt + 1;
+    k_popc_tiles<<<(unsigned)nt, 256, 0, s>>>(A->bitmap.as<uint32_t>(), nwords, tile_cnt);
+    NITRO_TRY(exclusive_scan_i64(tile_cnt, tile_off, nt, A->scratch, s));
+    k_emit_offsets<<<(unsigned)nt, 256, 0, s>>>(A->bitmap.as<uint32_t>(), nwords, tile_off, G, A->dia.off.as<int32_t>());
+    NITRO_CUDA(cudaGetLastError());
+  }
+  NITRO_TRY(A->dia.val.alloc((size_t)std::max<int64_t>(D * ld, 1) * sv));
+  if (D > 0) {
+    NITRO_CUDA(cudaMemsetAsync(A->dia.val.p, 0, (size_t)(D * ld * sv), s));
+    const unsigned g = grid_of(A->N);
+    if (A->rp64) {
+      if (A->fp64) k_fill_dia<int64_t, double><<<g, 256, 0, s>>>((const int64_t *)A->rowptr, A->col, (const double *)A->val, A->N, A->row0, A->dia.off.as<int32_t>(), D, ld, A->dia.val.as<double>());
+      else k_fill_dia<int64_t, float><<<g, 256, 0, s>>>((const int64_t *)A->rowptr, A->col, (const float *)A->val, A->N, A->row0, A->dia.off.as<int32_t>(), D, ld, A->dia.val.as<float>());
+    } else {
+      if (A->fp64) k_fill_dia<int32_t, double><<<g, 256, 0, s>>>((const int32_t *)A->rowptr, A->col, (const double *)A->val, A->N, A->row0, A->dia.off.as<int32_t>(), D, ld, A->dia.val.as<double>());
+      else k_fill_dia<int32_t, float><<<g, 256, 0, s>>>((const int32_t *)A->rowptr, A->col, (const float *)A->val, A->N, A->row0, A->dia.off.as<int32_t>(), D, ld, A->dia.val.as<float>());
+    }
+    NITRO_CUDA(cudaGetLastError());
+  }
+  // in-range slots (compulsory bytes): sum_d |{i : 0 <= row0+i+off_d < M}|
+  std::vector<int32_t> h(D);
+  if (D > 0) {
+    NITRO_CUDA(cudaMemcpyAsync(h.data(), A->dia.off.p, (size_t)D * 4, cudaMemcpyDeviceToHost, s));
+    NITRO_CUDA(cudaStreamSynchronize(s));
+  }
+  int64_t inr = 0;
+  for (int64_t d = 0; d < D; ++d) {
+    int64_t lo = std::max<int64_t>(0, -(A->row0 + h[d])), hi = std::min<int64_t>(A->N, A->M - A->row0 - h[d]);
+    if (hi > lo) inr += hi - lo;
+  }
+  A->dia.off_min = D > 0 ? h[0] : 0;
+  A->dia.off_max = D > 0 ? h[D - 1] : 0;
+  A->dia.D = D;
+  A->dia.ld = ld;
+  A->dia.inrange = inr;
+  A->dia.ready = true;
+  return NITRO_OK;
+}
+
+// ------------------------------------------------------------------ HYB (C7)
+nitro_status_t prepare_hyb(nitro_spmv *A) {
+  if (A->hyb.ready) return NITRO_OK;
+  NITRO_TRY(features_finish(A));
+  cudaStream_t s = A->stream;
+  const int64_t N = A->N, lmax = A->feat.max_row, ld = round_up(N, 32), sv = A->fp64 ? 8 : 4;
+  // K_hyb = first k in [0, Lmax) with 3 R_k < N or R_k < 4096 (R_k = #rows with L > k); else Lmax
+  constexpr int W = 1024;
+  int64_t K = lmax, Rk_at_K = 0;
+  {
+    DevBuf bins;
+    NITRO_TRY(bins.alloc((W + 1) * sizeof(unsigned long long)));
+    std::vector<unsigned long long> hb(W + 1);
+    bool found = false;
+    // R_{k0-1} = #rows with L >= k0; start with R_{-1} = N
+    for (int64_t k0 = 0; k0 < lmax && !found; k0 += W) {
+      NITRO_CUDA(cudaMemsetAsync(bins.p, 0, bins.bytes, s));
+      if (A->rp64) k_len_hist<int64_t, W><<<grid_of(N), 256, 0, s>>>((const int64_t *)A->rowptr, N, k0, bins.as<unsigned long long>());
+      else k_len_hist<int32_t, W><<<grid_of(N), 256, 0, s>>>((const int32_t *)A->rowptr, N, k0, bins.as<unsigned long long>());
+      NITRO_CUDA(cudaGetLastError());
+      NITRO_CUDA(cudaMemcpyAsync(hb.data(), bins.p, bins.bytes, cudaMemcpyDeviceToHost, s));
+      NITRO_CUDA(cudaStreamSynchronize(s));
+      // rows with L >= k0
+      int64_t ge = 0;
+      for (int t = 0; t <= W; ++t) ge += (int64_t)hb[t];
+      for (int t = 0; t < W && k0 + t < lmax; ++t) {
+        ge -= (int64_t)hb[t];  // now ge = #rows with L > k0 + t = R_{k0+t}
+        if (3 * ge < N || ge < 4096) { K = k0 + t; Rk_at_K = ge; found = true; break; }
+      }
+    }
+  }
+  A->hyb.tail_rows = Rk_at_K;  // rows with L > K (0 when K = Lmax)
+  DevBuf cnt;
+  NITRO_TRY(cnt.alloc((size_t)(2 * N + 2) * 8));
+  int64_t *c = cnt.as<int64_t>(), *toff = c + N + 1;
+  int64_t Zt = 0;
+  if (N > 0) {
+    if (A->rp64) k_tail_counts<int64_t><<<grid_of(N), 256, 0, s>>>((const int64_t *)A->rowptr, N, K, c);
+    else k_tail_counts<int32_t><<<grid_of(N), 256, 0, s>>>((const int32_t *)A->rowptr, N, K, c);
+    NITRO_TRY(exclusive_scan_i64(c, toff, N, A->scratch, s));
+    NITRO_CUDA(cudaMemcpyAsync(&Zt, toff + N, 8, cudaMemcpyDeviceToHost, s));
+    NITRO_CUDA(cudaStreamSynchronize(s));
+  }
+  NITRO_TRY(A->hyb.col.alloc((size_t)std::max<int64_t>(K * ld, 1) * 4));
+  NITRO_TRY(A->hyb.val.alloc((size_t)std::max<int64_t>(K * ld, 1) * sv));
+  NITRO_TRY(A->hyb.trow.alloc((size_t)std::max<int64_t>(Zt, 1) * 4));
+  NITRO_TRY(A->hyb.tcol.alloc((size_t)std::max<int64_t>(Zt, 1) * 4));
+  NITRO_TRY(A->hyb.tval.alloc((size_t)std::max<int64_t>(Zt, 1) * sv));
+  const int64_t nch = (Zt + 255) / 256;
+  NITRO_TRY(A->hyb.carry_row.alloc((size_t)std::max<int64_t>(2 * nch, 1) * 4));
+  NITRO_TRY(A->hyb.carry_val.alloc((size_t)std::max<int64_t>(2 * nch, 1) * 8));
+  if (N > 0)
+    NITRO_TRY(fill_ell(A, K, ld, A->hyb.col.p, A->hyb.val.p, Zt > 0 ? toff : nullptr, A->hyb.trow.p, A->hyb.tcol.p,
+                       A->hyb.tval.p));
+  NITRO_CUDA(cudaStreamSynchronize(s));  // cnt is freed on return
+  A->hyb.K = K;
+  A->hyb.ld = ld;
+  A->hyb.Zt = Zt;
+  A->hyb.nchunks = nch;
+  A->hyb.ready = true;
+  return NITRO_OK;
+}
+
+// ------------------------------------------------------------------ CSR-vector (C8)
+// V = lanes per row from the mean row length; rows longer than 8V are split
+// into segments of kSeg entries handled by whole CTAs (see spmv.cu).
+nitro_status_t prepare_csrv(nitro_spmv *A) {
+  if (A->csrv.ready) return NITRO_OK;
+  NITRO_TRY(features_finish(A));
+  cudaStream_t s = A->stream;
+  const int64_t N = A->N;
+  const int64_t q = N > 0 ? A->Z / N : 0;
+  int V = q <= 2 ? 2 : q <= 4 ? 4 : q <= 8 ? 8 : q <= 16 ? 16 : 32;
+  A->csrv.V = V;
+  const int64_t T = 8LL * V, S = 4096;
+  A->csrv.n_long = 0;
+  if (A->feat.max_row > T) {
+    DevBuf cnt;
+    NITRO_TRY(cnt.alloc((size_t)(2 * N + 2) * 8));
+    int64_t *c = cnt.as<int64_t>(), *off = c + N + 1;
+    if (A->rp64) k_long_flags<int64_t><<<grid_of(N), 256, 0, s>>>((const int64_t *)A->rowptr, N, T, S, c);
+    else k_long_flags<int32_t><<<grid_of(N), 256, 0, s>>>((const int32_t *)A->rowptr, N, T, S, c);
+    NITRO_TRY(exclusive_scan_i64(c, off, N, A->scratch, s));
+    int64_t nseg = 0;
+    NITRO_CUDA(cudaMemcpyAsync(&nseg, off + N, 8, cudaMemcpyDeviceToHost, s));
+    NITRO_CUDA(cudaStreamSynchronize(s));
+    // layout: seg_row[nseg] | seg_k[nseg] | seg partials (double)[nseg] | row counters (uint)[nseg]
+    NITRO_TRY(A->csrv.long_rows.alloc((size_t)std::max<int64_t>(nseg, 1) * (4 + 4 + 8 + 4) + 16));
+    int32_t *seg_row = A->csrv.long_rows.as<int32_t>();
+    int32_t *seg_k = seg_row + nseg;
+    if (A->rp64) k_long_emit<int64_t><<<grid_of(N), 256, 0, s>>>((const int64_t *)A->rowptr, N, off, seg_row, seg_k);
+    else k_long_emit<int32_t><<<grid_of(N), 256, 0, s>>>((const int32_t *)A->rowptr, N, off, seg_row, seg_k);
+    NITRO_CUDA(cudaGetLastError());
+    // zero the per-row completion counters (indexed by a row's first segment)
+    char *base = (char *)A->csrv.long_rows.p;
+    size_t ctr_off = (size_t)nseg * 16;
+    NITRO_CUDA(cudaMemsetAsync(base + ctr_off, 0, (size_t)std::max<int64_t>(nseg, 1) * 4, s));
+    NITRO_CUDA(cudaStreamSynchronize(s));
+    A->csrv.n_long = nseg;
+  }
+  A->csrv.ready = true;
+  return NITRO_OK;
+}
+
+}  // namespace nitro

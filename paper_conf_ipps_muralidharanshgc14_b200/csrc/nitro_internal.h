@@ -1,0 +1,141 @@
+// nitro_internal.h — internal declarations of libnitro (not part of the ABI).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+
+#include "../../include/nitro.h"
+
+namespace nitro {
+
+// ------------------------------------------------------------------ errors
+void set_error(const std::string &msg);
+nitro_status_t fail(nitro_status_t code, const std::string &msg);
+nitro_status_t cuda_fail(cudaError_t e, const char *where);
+
+#define NITRO_CUDA(call)                                         \
+  do {                                                           \
+    cudaError_t e_ = (call);                                     \
+    if (e_ != cudaSuccess) return ::nitro::cuda_fail(e_, #call); \
+  } while (0)
+#define NITRO_TRY(call)                           \
+  do {                                            \
+    nitro_status_t s_ = (call);                   \
+    if (s_ != NITRO_OK) return s_;                \
+  } while (0)
+
+// ------------------------------------------------------------------ device buffer
+struct DevBuf {
+  void *p = nullptr;
+  size_t bytes = 0;
+  nitro_status_t alloc(size_t n);  // (re)allocates if smaller; contents undefined
+  void release();
+  template <typename T> T *as() const { return reinterpret_cast<T *>(p); }
+  ~DevBuf() { release(); }
+  DevBuf() = default;
+  DevBuf(const DevBuf &) = delete;
+  DevBuf &operator=(const DevBuf &) = delete;
+};
+
+// ------------------------------------------------------------------ feature pass
+// Device-side accumulators of the K1 pass (exact integers).
+struct FeatAcc {
+  unsigned long long s1, s2, lmax;
+  unsigned int bad;      // bit0 rowptr not monotone / wrong ends, bit1 unsorted/dup col, bit2 col out of range
+  unsigned int pad;
+  unsigned long long ndiag;
+};
+
+// ------------------------------------------------------------------ formats
+struct EllFmt {
+  bool ready = false;
+  int64_t K = 0, ld = 0;
+  DevBuf col, val;
+};
+struct DiaFmt {
+  bool ready = false;
+  int64_t D = 0, ld = 0;
+  int64_t inrange = 0;  // sum over diagonals of in-range slots (compulsory)
+  int64_t off_min = 0, off_max = 0;
+  DevBuf off, val;
+};
+struct HybFmt {
+  bool ready = false;
+  int64_t K = 0, ld = 0, Zt = 0, nchunks = 0, tail_rows = 0;
+  DevBuf col, val, trow, tcol, tval, carry_row, carry_val;
+};
+struct CsrvFmt {
+  bool ready = false;
+  int V = 32;
+  int64_t n_long = 0;
+  DevBuf long_rows;
+};
+
+}  // namespace nitro
+
+struct nitro_spmv {
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  int64_t N = 0, M = 0, Z = 0;
+  int64_t row0 = 0;  // global row of local row 0 (multi-GPU blocks), for diagonal offsets
+  const void *rowptr = nullptr;
+  bool rp64 = false;
+  const int32_t *col = nullptr;
+  const void *val = nullptr;
+  bool fp64 = false;
+
+  // features
+  bool feat_ready = false, feat_pending = false;
+  nitro_spmv_feat feat{};
+  nitro::DevBuf feat_acc;   // FeatAcc
+  nitro::DevBuf bitmap;     // u32 words over offsets [-(N-1) .. M-1] (+row0 shift)
+  nitro::DevBuf offsets;    // int32 [ndiag] ascending
+  nitro::DevBuf scratch;    // scan scratch
+  nitro::FeatAcc *h_acc = nullptr;  // pinned
+  cudaEvent_t feat_done = nullptr;
+
+  double budget = -1.0;
+
+  nitro::EllFmt ell;
+  nitro::DiaFmt dia;
+  nitro::HybFmt hyb;
+  nitro::CsrvFmt csrv;
+
+  nitro::DevBuf flush;      // L2 flush scratch
+  nitro::DevBuf xbuf, ybuf; // run_host staging
+
+  // multi-GPU
+  nitro_dist *dist = nullptr;
+  int64_t n_interior = 0;   // rows [0, n_interior) are interior after a dist permutation? (see dist.cu)
+  void *dist_state = nullptr;
+};
+
+namespace nitro {
+
+// features.cu
+nitro_status_t features_launch(nitro_spmv *A);   // enqueue K1 + compaction, async
+nitro_status_t features_finish(nitro_spmv *A);   // wait + host finishing
+void finish_features(int64_t N, int64_t M, int64_t Z, uint64_t s1, uint64_t s2, int64_t lmax, int64_t D,
+                     nitro_spmv_feat *f);
+
+// convert.cu
+nitro_status_t prepare_ell(nitro_spmv *A);
+nitro_status_t prepare_dia(nitro_spmv *A);
+nitro_status_t prepare_hyb(nitro_spmv *A);
+nitro_status_t prepare_csrv(nitro_spmv *A);
+
+// spmv.cu
+nitro_status_t launch_spmv(nitro_spmv *A, int variant, const void *x, void *y, cudaStream_t s);
+int launches_of(const nitro_spmv *A, int variant);
+nitro_status_t launch_flush(nitro_spmv *A, cudaStream_t s);
+double compulsory_bytes(const nitro_spmv *A, int variant);
+
+// scan.cu: exclusive scan of int64 counts; out[n] = total.  scratch grows.
+nitro_status_t exclusive_scan_i64(const int64_t *in, int64_t *out, int64_t n, DevBuf &scratch, cudaStream_t s);
+
+inline int64_t round_up(int64_t n, int64_t m) { return (n + m - 1) / m * m; }
+int num_sms();
+
+}  // namespace nitro

@@ -1,0 +1,462 @@
+// spmv.cu — A6-A10: the five SpMV variants y = A.x for sm_100a (CUDA cores;
+// SpMV is HBM-bound, ~0.2 flop/byte, so tensor cores do not apply).
+//
+// Semantics (read as y <- A.x): every variant overwrites y.
+// Accumulation (R2): fp64 data accumulate in fp64.  fp32 data form
+// fp32 partial sums of at most 16 terms (FFMA), combined in fp64 (or in a
+// <=5-level fp32 shuffle tree for rows of <= 8V entries), so the error stays
+// below ~21 u sum|a_ij x_j| (u = 2^-24) for any row length: inside the
+// 1e-5 bound of the north star, and exact on integer stencils.
+#include "nitro_internal.h"
+#include "util.cuh"
+
+#include <algorithm>
+
+namespace nitro {
+namespace {
+
+template <typename VT> struct V4;
+template <> struct V4<float> {
+  float v[4];
+  __device__ __forceinline__ void load(const float *p) {
+    float4 t = ld_stream_f4(reinterpret_cast<const float4 *>(p));
+    v[0] = t.x; v[1] = t.y; v[2] = t.z; v[3] = t.w;
+  }
+};
+template <> struct V4<double> {
+  double v[4];
+  __device__ __forceinline__ void load(const double *p) {
+    double2 a = ld_stream_d2(reinterpret_cast<const double2 *>(p));
+    double2 b = ld_stream_d2(reinterpret_cast<const double2 *>(p) + 1);
+    v[0] = a.x; v[1] = a.y; v[2] = b.x; v[3] = b.y;
+  }
+};
+
+template <typename VT>
+__device__ __forceinline__ void store4(VT *y, int64_t i0, int64_t N, const double *acc) {
+  if (i0 + 3 < N) {
+    if constexpr (sizeof(VT) == 4) {
+      *reinterpret_cast<float4 *>(y + i0) = make_float4((float)acc[0], (float)acc[1], (float)acc[2], (float)acc[3]);
+    } else {
+      reinterpret_cast<double2 *>(y + i0)[0] = make_double2(acc[0], acc[1]);
+      reinterpret_cast<double2 *>(y + i0)[1] = make_double2(acc[2], acc[3]);
+    }
+  } else {
+    for (int q = 0; q < 4; ++q)
+      if (i0 + q < N) y[i0 + q] = (VT)acc[q];
+  }
+}
+
+// ------------------------------------------------------------------ K5 CSR-scalar
+template <typename IT, typename VT>
+__global__ void __launch_bounds__(256) k_csr_scalar(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
+                                                    const VT *__restrict__ val, const VT *__restrict__ x,
+                                                    VT *__restrict__ y, int64_t N) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < N; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t a = (int64_t)rowptr[i], b = (int64_t)rowptr[i + 1];
+    double acc = 0.0;
+    for (int64_t k = a; k < b; k += 16) {
+      const int64_t e = k + 16 < b ? k + 16 : b;
+      VT part = 0;
+#pragma unroll 4
+      for (int64_t j = k; j < e; ++j) part = fma(__ldg(val + j), __ldg(x + __ldg(col + j)), part);
+      acc += (double)part;
+    }
+    y[i] = (VT)acc;
+  }
+}
+
+// ------------------------------------------------------------------ K6 CSR-vector
+// V lanes per row.  A warp takes 32 consecutive rows (one coalesced rowptr
+// load per lane); lane group g handles rows g, g+G, ... (G = 32/V) R at a
+// time so R independent (col, val) -> x chains are in flight per lane.
+// Rows longer than 8V are split into kSeg-entry segments, each reduced by a
+// whole CTA (first nseg blocks of the grid); the last CTA of a row sums the
+// row's segment partials in segment order (deterministic, no float atomics).
+constexpr int kSeg = 4096;
+
+template <int V, typename IT, typename VT>
+__global__ void __launch_bounds__(256) k_csr_vector(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
+                                                    const VT *__restrict__ val, const VT *__restrict__ x,
+                                                    VT *__restrict__ y, int64_t N, int64_t nseg,
+                                                    const int32_t *__restrict__ seg_row,
+                                                    const int32_t *__restrict__ seg_k, double *seg_part,
+                                                    unsigned *seg_ctr) {
+  constexpr int64_t T = 8 * V;
+  if ((int64_t)blockIdx.x < nseg) {
+    // ---- long-row segment: one CTA, <= 16 entries per thread
+    __shared__ double s_w[8];
+    __shared__ bool s_last;
+    const int64_t sg = blockIdx.x;
+    const int64_t row = seg_row[sg], k = seg_k[sg];
+    const int64_t a = (int64_t)rowptr[row], b = (int64_t)rowptr[row + 1];
+    const int64_t st = a + k * kSeg, en = st + kSeg < b ? st + kSeg : b;
+    VT part = 0;
+#pragma unroll 4
+    for (int64_t j = st + threadIdx.x; j < en; j += 256) part = fma(ld_stream(val + j), __ldg(x + ld_stream_i(col + j)), part);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) part += __shfl_xor_sync(kFull, part, o);
+    if ((threadIdx.x & 31) == 0) s_w[threadIdx.x >> 5] = (double)part;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      double t = 0.0;
+      for (int w = 0; w < 8; ++w) t += s_w[w];
+      seg_part[sg] = t;
+      __threadfence();
+      const int64_t first = sg - k, ns = (b - a + kSeg - 1) / kSeg;
+      const unsigned done = atomicAdd(seg_ctr + first, 1u);
+      s_last = done == (unsigned)(ns - 1);
+      if (s_last) {
+        __threadfence();
+        double tot = 0.0;
+        for (int64_t q = 0; q < ns; ++q) tot += *((volatile double *)(seg_part + first + q));
+        y[row] = (VT)tot;
+        seg_ctr[first] = 0;  // re-arm for the next multiply
+      }
+    }
+    return;
+  }
+  constexpr int G = 32 / V;
+  constexpr int R = V >= 4 ? 4 : V;
+  const int lane = threadIdx.x & 31, g = lane / V, li = lane % V;
+  const int64_t warp = (((int64_t)blockIdx.x - nseg) * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = (((int64_t)gridDim.x - nseg) * blockDim.x) >> 5;
+  for (int64_t t0 = warp * 32; t0 < N; t0 += nwarps * 32) {
+    const int64_t r = t0 + lane;
+    int64_t a = 0, L = 0;
+    if (r < N) { a = (int64_t)rowptr[r]; L = (int64_t)rowptr[r + 1] - a; }
+#pragma unroll
+    for (int tb = 0; tb < V; tb += R) {
+      int64_t s[R];
+      int64_t l[R];
+#pragma unroll
+      for (int u = 0; u < R; ++u) {
+        const int src = g + G * (tb + u);
+        s[u] = __shfl_sync(kFull, a, src);
+        l[u] = __shfl_sync(kFull, L, src);
+        if (l[u] > T) l[u] = 0;  // handled by the segment path
+      }
+      int c[R];
+      VT v[R];
+#pragma unroll
+      for (int u = 0; u < R; ++u) {
+        const bool in = li < l[u];
+        c[u] = in ? ld_stream_i(col + s[u] + li) : -1;
+        v[u] = in ? ld_stream(val + s[u] + li) : (VT)0;
+      }
+      VT part[R];
+#pragma unroll
+      for (int u = 0; u < R; ++u) part[u] = c[u] >= 0 ? v[u] * __ldg(x + c[u]) : (VT)0;
+#pragma unroll
+      for (int u = 0; u < R; ++u)
+        for (int64_t m = V + li; m < l[u]; m += V)  // <= 7 more terms per lane
+          part[u] = fma(ld_stream(val + s[u] + m), __ldg(x + ld_stream_i(col + s[u] + m)), part[u]);
+#pragma unroll
+      for (int u = 0; u < R; ++u) {
+#pragma unroll
+        for (int o = V / 2; o > 0; o >>= 1) part[u] += __shfl_xor_sync(kFull, part[u], o);
+      }
+      // write results (lanes li == 0); long rows skipped
+#pragma unroll
+      for (int u = 0; u < R; ++u) {
+        const int src = g + G * (tb + u);
+        const int64_t Lr = __shfl_sync(kFull, L, src);
+        const int64_t row = t0 + src;
+        if (li == 0 && row < N && Lr <= T) y[row] = part[u];
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------------ K7 ELL (also HYB's ELL part)
+// Thread per 4 consecutive rows: per slot one 128-bit load of 4 column ids and
+// one 128-bit (fp32) / 2x128-bit (fp64) load of 4 values; 4 slots unrolled.
+template <typename VT>
+__global__ void __launch_bounds__(256) k_ell(const int32_t *__restrict__ ecol, const VT *__restrict__ eval,
+                                             const VT *__restrict__ x, VT *__restrict__ y, int64_t N, int64_t K,
+                                             int64_t ld) {
+  const int64_t nq = ld >> 2;
+  for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nq; q += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t i0 = q << 2;
+    double acc[4] = {0.0, 0.0, 0.0, 0.0};
+    for (int64_t k0 = 0; k0 < K; k0 += 16) {
+      const int64_t ke = k0 + 16 < K ? k0 + 16 : K;
+      VT part[4] = {0, 0, 0, 0};
+#pragma unroll 4
+      for (int64_t k = k0; k < ke; ++k) {
+        const int4 c = ld_stream_i4(reinterpret_cast<const int4 *>(ecol + k * ld + i0));
+        V4<VT> v;
+        v.load(eval + k * ld + i0);
+        part[0] = fma(v.v[0], c.x >= 0 ? __ldg(x + c.x) : (VT)0, part[0]);
+        part[1] = fma(v.v[1], c.y >= 0 ? __ldg(x + c.y) : (VT)0, part[1]);
+        part[2] = fma(v.v[2], c.z >= 0 ? __ldg(x + c.z) : (VT)0, part[2]);
+        part[3] = fma(v.v[3], c.w >= 0 ? __ldg(x + c.w) : (VT)0, part[3]);
+      }
+#pragma unroll
+      for (int t = 0; t < 4; ++t) acc[t] += (double)part[t];
+    }
+    store4<VT>(y, i0, N, acc);
+  }
+}
+
+// ------------------------------------------------------------------ K8 DIA
+// Thread per 4 consecutive rows, block = 1024 rows; offsets in shared memory.
+// Blocks whose rows see every diagonal in range skip all bounds checks.
+template <typename VT>
+__global__ void __launch_bounds__(256) k_dia(const int32_t *__restrict__ offs, const VT *__restrict__ dval,
+                                             const VT *__restrict__ x, VT *__restrict__ y, int64_t N, int64_t M,
+                                             int64_t D, int64_t ld, int64_t row0, int64_t off_min, int64_t off_max) {
+  extern __shared__ int s_off[];
+  for (int64_t d = threadIdx.x; d < D; d += blockDim.x) s_off[d] = offs[d];
+  __syncthreads();
+  const int64_t nb = (ld + 1023) / 1024;
+  for (int64_t blk = blockIdx.x; blk < nb; blk += gridDim.x) {
+    const int64_t B0 = blk * 1024;
+    const int64_t i0 = B0 + 4 * threadIdx.x;
+    if (i0 >= ld) continue;
+    const int64_t Bend = (B0 + 1024 < ld ? B0 + 1024 : ld) - 1;
+    const bool interior = row0 + B0 + off_min >= 0 && row0 + Bend + off_max < M;
+    double acc[4] = {0.0, 0.0, 0.0, 0.0};
+    for (int64_t d0 = 0; d0 < D; d0 += 16) {
+      const int64_t de = d0 + 16 < D ? d0 + 16 : D;
+      VT part[4] = {0, 0, 0, 0};
+      if (interior) {
+#pragma unroll 4
+        for (int64_t d = d0; d < de; ++d) {
+          V4<VT> v;
+          v.load(dval + d * ld + i0);
+          const VT *xp = x + (row0 + i0 + s_off[d]);
+#pragma unroll
+          for (int t = 0; t < 4; ++t) part[t] = fma(v.v[t], __ldg(xp + t), part[t]);
+        }
+      } else {
+#pragma unroll 2
+        for (int64_t d = d0; d < de; ++d) {
+          V4<VT> v;
+          v.load(dval + d * ld + i0);
+          const int64_t j = row0 + i0 + s_off[d];
+#pragma unroll
+          for (int t = 0; t < 4; ++t)
+            if (j + t >= 0 && j + t < M) part[t] = fma(v.v[t], __ldg(x + j + t), part[t]);
+        }
+      }
+#pragma unroll
+      for (int t = 0; t < 4; ++t) acc[t] += (double)part[t];
+    }
+    store4<VT>(y, i0, N, acc);
+  }
+}
+
+// ------------------------------------------------------------------ K9b HYB COO tail
+// Warp per chunk of 256 row-sorted tail entries: 8 coalesced windows loaded up
+// front, then a segmented inclusive scan per window (rows sorted => equal row
+// ids are contiguous).  Rows wholly inside the chunk are added to y directly
+// (single owner); the chunk's first and last rows go to two carry slots that
+// k_hyb_fixup applies in chunk order.  No atomics; deterministic.
+template <typename VT>
+__global__ void __launch_bounds__(256) k_hyb_tail(const int32_t *__restrict__ trow, const int32_t *__restrict__ tcol,
+                                                  const VT *__restrict__ tval, const VT *__restrict__ x,
+                                                  VT *__restrict__ y, int64_t Zt, int64_t nch,
+                                                  int32_t *__restrict__ carry_row, double *__restrict__ carry_val) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t ch = warp; ch < nch; ch += nw) {
+    const int64_t c0 = ch * 256, cend = c0 + 256 < Zt ? c0 + 256 : Zt;
+    const int first_row = __ldg(trow + c0), last_row = __ldg(trow + cend - 1);
+    int rr[8], cc[8];
+    VT vv[8];
+#pragma unroll
+    for (int w = 0; w < 8; ++w) {
+      const int64_t e = c0 + w * 32 + lane;
+      const bool ok = e < cend;
+      rr[w] = ok ? ld_stream_i(trow + e) : -2;
+      cc[w] = ok ? ld_stream_i(tcol + e) : 0;
+      vv[w] = ok ? ld_stream(tval + e) : (VT)0;
+    }
+    double p[8];
+#pragma unroll
+    for (int w = 0; w < 8; ++w) p[w] = (double)vv[w] * (double)__ldg(x + cc[w]);
+    if (lane == 0) { carry_row[2 * ch] = -1; carry_row[2 * ch + 1] = -1; }
+    __syncwarp();
+    int carry_r = -3;
+    double carry_v = 0.0;
+#pragma unroll
+    for (int w = 0; w < 8; ++w) {
+      const int64_t w0 = c0 + w * 32;
+      if (w0 >= cend) break;
+      double q = p[w];
+      const int r = rr[w];
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const double t = __shfl_up_sync(kFull, q, o);
+        const int rt = __shfl_up_sync(kFull, r, o);
+        if (lane >= o && rt == r) q += t;
+      }
+      if (r == carry_r) q += carry_v;
+      const int nr = __shfl_down_sync(kFull, r, 1);
+      const int lvl = (int)(cend - 1 - w0 < 31 ? cend - 1 - w0 : 31);  // last valid lane
+      const bool more = w0 + 32 < cend;
+      const bool is_end = r >= 0 && (lane == lvl || nr != r);
+      const bool open = lane == lvl && more;
+      if (is_end && !open) {
+        if (r == first_row) { carry_row[2 * ch] = r; carry_val[2 * ch] = q; }
+        else if (r == last_row) { carry_row[2 * ch + 1] = r; carry_val[2 * ch + 1] = q; }
+        else y[r] = (VT)((double)y[r] + q);
+      }
+      carry_r = __shfl_sync(kFull, r, lvl);
+      carry_v = __shfl_sync(kFull, q, lvl);
+    }
+  }
+}
+
+template <typename VT>
+__global__ void __launch_bounds__(256) k_hyb_fixup(const int32_t *__restrict__ carry_row,
+                                                   const double *__restrict__ carry_val, VT *__restrict__ y,
+                                                   int64_t nch) {
+  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < nch; c += (int64_t)gridDim.x * blockDim.x) {
+#pragma unroll
+    for (int s = 0; s < 2; ++s) {
+      const int r = carry_row[2 * c + s];
+      if (r < 0) continue;
+      if (c > 0 && (carry_row[2 * c - 2] == r || carry_row[2 * c - 1] == r)) continue;  // started earlier
+      double sum = carry_val[2 * c + s];
+      const bool may_continue = s == 1 || carry_row[2 * c + 1] < 0;
+      if (may_continue) {
+        for (int64_t c2 = c + 1; c2 < nch && carry_row[2 * c2] == r; ++c2) {
+          sum += carry_val[2 * c2];
+          if (carry_row[2 * c2 + 1] >= 0) break;  // r ended inside c2
+        }
+      }
+      y[r] = (VT)((double)y[r] + sum);
+    }
+  }
+}
+
+// ------------------------------------------------------------------ K10 L2 flush (read-only: leaves clean lines)
+__global__ void __launch_bounds__(256) k_flush(const int4 *__restrict__ buf, int64_t n, int *__restrict__ sink) {
+  int acc = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    int4 v = __ldcg(buf + i);
+    acc ^= v.x ^ v.y ^ v.z ^ v.w;
+  }
+  if (acc == 0x7fffffff) *sink = acc;
+}
+
+unsigned grid_cap(int64_t blocks, int per_sm = 8) {
+  int64_t cap = (int64_t)num_sms() * per_sm;
+  if (blocks > cap) blocks = cap;
+  return (unsigned)(blocks < 1 ? 1 : blocks);
+}
+
+template <typename IT, typename VT>
+nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_t s) {
+  const IT *rp = (const IT *)A->rowptr;
+  const VT *val = (const VT *)A->val;
+  const int64_t N = A->N;
+  switch (variant) {
+    case NITRO_CSR_SCALAR:
+      if (N > 0) k_csr_scalar<IT, VT><<<grid_cap((N + 255) / 256, 16), 256, 0, s>>>(rp, A->col, val, x, y, N);
+      break;
+    case NITRO_CSR_VECTOR: {
+      if (N == 0) break;
+      const int64_t nseg = A->csrv.n_long;
+      int32_t *seg_row = A->csrv.long_rows.as<int32_t>();
+      int32_t *seg_k = seg_row + nseg;
+      double *seg_part = reinterpret_cast<double *>(reinterpret_cast<char *>(A->csrv.long_rows.p) + nseg * 8);
+      unsigned *seg_ctr = reinterpret_cast<unsigned *>(reinterpret_cast<char *>(A->csrv.long_rows.p) + nseg * 16);
+      const int64_t main_blocks = grid_cap((N + 255) / 256, 8);  // 8 warps x 32 rows per block-iteration
+      const unsigned g = (unsigned)(nseg + main_blocks);
+#define NITRO_CSRV(VV)                                                                                      \
+  k_csr_vector<VV, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, nseg, seg_row, seg_k, seg_part, seg_ctr)
+      switch (A->csrv.V) {
+        case 2: NITRO_CSRV(2); break;
+        case 4: NITRO_CSRV(4); break;
+        case 8: NITRO_CSRV(8); break;
+        case 16: NITRO_CSRV(16); break;
+        default: NITRO_CSRV(32); break;
+      }
+#undef NITRO_CSRV
+      break;
+    }
+    case NITRO_ELL:
+      if (N > 0)
+        k_ell<VT><<<grid_cap((A->ell.ld / 4 + 255) / 256, 16), 256, 0, s>>>(A->ell.col.as<int32_t>(), A->ell.val.as<VT>(),
+                                                                        x, y, N, A->ell.K, A->ell.ld);
+      break;
+    case NITRO_DIA:
+      if (N > 0) {
+        const size_t sm = (size_t)std::max<int64_t>(A->dia.D, 1) * 4;
+        k_dia<VT><<<grid_cap((A->dia.ld + 1023) / 1024, 16), 256, sm, s>>>(
+            A->dia.off.as<int32_t>(), A->dia.val.as<VT>(), x, y, N, A->M, A->dia.D, A->dia.ld, A->row0,
+            A->dia.off_min, A->dia.off_max);
+      }
+      break;
+    case NITRO_HYB:
+      if (N > 0) {
+        k_ell<VT><<<grid_cap((A->hyb.ld / 4 + 255) / 256, 16), 256, 0, s>>>(A->hyb.col.as<int32_t>(), A->hyb.val.as<VT>(),
+                                                                        x, y, N, A->hyb.K, A->hyb.ld);
+        if (A->hyb.Zt > 0) {
+          k_hyb_tail<VT><<<grid_cap((A->hyb.nchunks + 7) / 8, 16), 256, 0, s>>>(
+              A->hyb.trow.as<int32_t>(), A->hyb.tcol.as<int32_t>(), A->hyb.tval.as<VT>(), x, y, A->hyb.Zt,
+              A->hyb.nchunks, A->hyb.carry_row.as<int32_t>(), A->hyb.carry_val.as<double>());
+          k_hyb_fixup<VT><<<grid_cap((A->hyb.nchunks + 255) / 256, 16), 256, 0, s>>>(
+              A->hyb.carry_row.as<int32_t>(), A->hyb.carry_val.as<double>(), y, A->hyb.nchunks);
+        }
+      }
+      break;
+    default:
+      return fail(NITRO_E_INVALID_ARG, "unknown variant");
+  }
+  NITRO_CUDA(cudaGetLastError());
+  return NITRO_OK;
+}
+
+}  // namespace
+
+nitro_status_t launch_spmv(nitro_spmv *A, int variant, const void *x, void *y, cudaStream_t s) {
+  if (A->rp64) {
+    if (A->fp64) return run_t<int64_t, double>(A, variant, (const double *)x, (double *)y, s);
+    return run_t<int64_t, float>(A, variant, (const float *)x, (float *)y, s);
+  }
+  if (A->fp64) return run_t<int32_t, double>(A, variant, (const double *)x, (double *)y, s);
+  return run_t<int32_t, float>(A, variant, (const float *)x, (float *)y, s);
+}
+
+nitro_status_t launch_flush(nitro_spmv *A, cudaStream_t s) {
+  if (!A->flush.p) {
+    int l2 = 0;
+    NITRO_CUDA(cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, A->device));
+    NITRO_TRY(A->flush.alloc((size_t)std::max(l2, 1 << 20) * 3 + 64));
+    NITRO_CUDA(cudaMemsetAsync(A->flush.p, 1, A->flush.bytes, s));
+  }
+  const int64_t n = (int64_t)((A->flush.bytes - 64) / 16);
+  k_flush<<<grid_cap((n + 255) / 256, 8), 256, 0, s>>>(A->flush.as<int4>(), n,
+                                                       reinterpret_cast<int *>(A->flush.as<char>() + A->flush.bytes - 64));
+  NITRO_CUDA(cudaGetLastError());
+  return NITRO_OK;
+}
+
+int launches_of(const nitro_spmv *A, int variant) {
+  if (A->N == 0) return 0;
+  if (variant == NITRO_HYB) return A->hyb.Zt > 0 ? 3 : 1;
+  return 1;
+}
+
+double compulsory_bytes(const nitro_spmv *A, int variant) {
+  const double N = (double)A->N, M = (double)A->M, Z = (double)A->Z;
+  const double sv = A->fp64 ? 8 : 4, si = 4, sp = A->rp64 ? 8 : 4;
+  const double xy = M * sv + N * sv;
+  switch (variant) {
+    case NITRO_CSR_SCALAR:
+    case NITRO_CSR_VECTOR: return Z * (sv + si) + (N + 1) * sp + xy;
+    case NITRO_ELL: return (double)A->ell.K * N * (sv + si) + xy;
+    case NITRO_DIA: return (double)A->dia.inrange * sv + (double)A->dia.D * 4 + xy;
+    case NITRO_HYB:
+      return (double)A->hyb.K * N * (sv + si) + (double)A->hyb.Zt * (sv + 2 * si) + xy +
+             (double)A->hyb.tail_rows * sv;
+  }
+  return 0.0;
+}
+
+}  // namespace nitro

@@ -1,0 +1,97 @@
+// util.cuh — warp/block primitives and load helpers for the sm_100a kernels.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace nitro {
+
+constexpr unsigned kFull = 0xffffffffu;
+
+__device__ __forceinline__ int64_t warp_sum_i64(int64_t v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(kFull, v, o);
+  return v;
+}
+
+template <int kThreads>
+__device__ __forceinline__ int64_t block_sum_i64(int64_t v) {
+  __shared__ int64_t red[kThreads / 32];
+  v = warp_sum_i64(v);
+  int w = threadIdx.x >> 5, l = threadIdx.x & 31;
+  if (l == 0) red[w] = v;
+  __syncthreads();
+  if (w == 0) {
+    v = l < kThreads / 32 ? red[l] : 0;
+    v = warp_sum_i64(v);
+  }
+  __syncthreads();
+  return v;  // valid in thread 0
+}
+
+// exclusive prefix over the block; agg = block total (all threads)
+template <int kThreads>
+__device__ __forceinline__ int64_t block_exclusive_i64(int64_t v, int64_t &agg) {
+  constexpr int NW = kThreads / 32;
+  __shared__ int64_t wsum[NW + 1];
+  int w = threadIdx.x >> 5, l = threadIdx.x & 31;
+  int64_t inc = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    int64_t t = __shfl_up_sync(kFull, inc, o);
+    if (l >= o) inc += t;
+  }
+  if (l == 31) wsum[w] = inc;
+  __syncthreads();
+  if (w == 0) {
+    int64_t s = l < NW ? wsum[l] : 0;
+    int64_t si = s;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      int64_t t = __shfl_up_sync(kFull, si, o);
+      if (l >= o) si += t;
+    }
+    if (l < NW) wsum[l] = si - s;
+    if (l == NW - 1) wsum[NW] = si;
+  }
+  __syncthreads();
+  int64_t r = wsum[w] + inc - v;
+  agg = wsum[NW];
+  __syncthreads();
+  return r;
+}
+
+// streaming (read-once) loads: bypass L1 allocation, keep default L2 policy
+__device__ __forceinline__ int4 ld_stream_i4(const int4 *p) {
+  int4 r;
+  asm("ld.global.nc.L1::no_allocate.v4.s32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ float4 ld_stream_f4(const float4 *p) {
+  float4 r;
+  asm("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
+               : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ double2 ld_stream_d2(const double2 *p) {
+  double2 r;
+  asm("ld.global.nc.L1::no_allocate.v2.f64 {%0,%1}, [%2];" : "=d"(r.x), "=d"(r.y) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ int ld_stream_i(const int *p) {
+  int r;
+  asm("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(r) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ float ld_stream(const float *p) {
+  float r;
+  asm("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(r) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ double ld_stream(const double *p) {
+  double r;
+  asm("ld.global.nc.L1::no_allocate.f64 %0, [%1];" : "=d"(r) : "l"(p));
+  return r;
+}
+
+}  // namespace nitro

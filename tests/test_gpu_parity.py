@@ -1,0 +1,339 @@
+"""GPU path (through the C ABI) vs the CPU oracle — the parity gate.
+
+Bars (BASELINE north_star): features and conversions bit-exact; fp32 SpMV
+per row |y - y_ref| <= 1e-5 * sum_j |a_ij x_j| + 1e-30; fp64 the same at
+1e-12; integer stencils x integer x exact in fp32 for every variant.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from synth import Csr
+
+pytestmark = pytest.mark.gpu
+
+FEAT_KEYS = ("rows", "cols", "nnz", "sum_len", "sum_len2", "max_row", "ndiag", "canonical",
+             "mean", "sd", "max_dev", "dia_fill", "ell_fill")
+
+
+def nitro():
+    import paper_conf_ipps_muralidharanshgc14_b200 as n
+    return n
+
+
+def handle(A, cuda, rowptr32=None):
+    Ad = synth.to_device(A, cuda, rowptr32=rowptr32)
+    return nitro().SpMV.from_csr(Ad), Ad
+
+
+def small_mats():
+    """Several tiles + ragged tails + degenerate cases; (name, host Csr)."""
+    yield "2d5_n64_c0", synth.stencil("2d5", 64)
+    yield "2d5_n64_rand", synth.stencil("2d5", 64, mode=1, seed=2)
+    yield "3d27_n20", synth.stencil("3d27", 20, mode=1, seed=3)
+    yield "3d7_n17", synth.stencil("3d7", 17, mode=1, seed=4)
+    yield "1d3_n1001", synth.stencil("1d3", 1001, mode=1, seed=5)
+    yield "2d9_n33", synth.stencil("2d9", 33, mode=1, seed=6)
+    yield "banded_b7_d05", synth.banded(5003, 7, 0.5, seed=7)
+    yield "banded_b40_full", synth.banded(2999, 40, 1.0, seed=8)
+    yield "uniform_k32", synth.uniform(4099, 32, seed=9)
+    yield "uniform_var_k9_rect", synth.uniform(3001, 9, variable=True, seed=10, M=7777)
+    yield "uniform_k2", synth.uniform(9000, 2, seed=11)
+    yield "rmat12_fp32", synth.rmat(12, 16, seed=12, fp64=False)
+    yield "rmat13_fp64", synth.rmat(13, 8, seed=13, fp64=True)
+    yield "one_row", Csr(1, 5, np.array([0, 3], np.int64), np.array([0, 2, 4], np.int32),
+                         np.array([1.5, -2.0, 0.25], np.float32), False)
+    yield "empty_rows", Csr(70, 70, np.array([0] * 35 + [2] * 36, np.int64), np.array([3, 69], np.int32),
+                            np.array([1.0, 2.0], np.float32), False)
+    yield "nnz0", Csr(40, 33, np.zeros(41, np.int64), np.zeros(0, np.int32), np.zeros(0, np.float32), False)
+
+
+def long_row_matrix(L=150_000, N=5000, fp64=False, seed=21):
+    """Row 17 holds L entries (CSR-vector segments / HYB tail), others 0..5."""
+    rng = np.random.default_rng(seed)
+    lens = rng.integers(0, 6, N)
+    lens[17] = L
+    M = max(L + 10, N)
+    rp = np.zeros(N + 1, np.int64)
+    rp[1:] = np.cumsum(lens)
+    cols = []
+    for i, l in enumerate(lens):
+        cols.append(np.sort(rng.choice(M, l, replace=False)) if l != L else np.arange(0, 2 * L, 2)[:L] % M)
+    ci = np.concatenate(cols).astype(np.int32)
+    v = rng.uniform(-1, 1, rp[-1])
+    v[v == 0] = 0.5
+    return Csr(N, M, rp, ci, v.astype(np.float64 if fp64 else np.float32), fp64)
+
+
+def check_y(y, y_ref, r, fp64):
+    tol = (1e-12 if fp64 else 1e-5) * r + 1e-30
+    err = np.abs(np.asarray(y, np.float64) - y_ref)
+    bad = np.nonzero(err > tol)[0]
+    assert bad.size == 0, f"{bad.size} rows out of tolerance, first {bad[:5]}: {err[bad[:5]]} > {tol[bad[:5]]}"
+
+
+# ------------------------------------------------------------------ features
+@pytest.mark.parametrize("name,A", list(small_mats()))
+def test_features_bit_exact(cuda, name, A):
+    M, _ = handle(A, cuda)
+    f = M.features()
+    f_ref = oracle.features(A)
+    for k in FEAT_KEYS:
+        assert f[k] == f_ref[k], (name, k, f[k], f_ref[k])
+
+
+def test_features_int64_rowptr_and_long_row(cuda):
+    A = long_row_matrix()
+    M, _ = handle(A, cuda, rowptr32=False)
+    f, f_ref = M.features(), oracle.features(A)
+    for k in FEAT_KEYS:
+        assert f[k] == f_ref[k], k
+
+
+@pytest.mark.parametrize("case", ["unsorted", "dup", "oob", "rowptr"])
+def test_non_canonical_rejected(cuda, case):
+    n = nitro()
+    rp = np.array([0, 2, 4, 6], np.int64)
+    ci = {"unsorted": [1, 0, 0, 1, 0, 2], "dup": [0, 0, 0, 1, 0, 2], "oob": [0, 1, 0, 3, 0, 2],
+          "rowptr": [0, 1, 0, 1, 0, 2]}[case]
+    if case == "rowptr":
+        rp = np.array([0, 3, 2, 6], np.int64)
+    A = Csr(3, 3, rp, np.array(ci, np.int32), np.ones(6, np.float32), False)
+    assert not oracle.is_canonical(A)
+    M, _ = handle(A, cuda)
+    with pytest.raises(n.NitroError) as e:
+        M.features()
+    assert e.value.code == 2
+    with pytest.raises(n.NitroError):
+        M.run(n.CSR_VECTOR, __import__("torch").zeros(3, device=cuda))
+
+
+# ------------------------------------------------------------------ conversions
+def _mats_for_conv():
+    for name, A in small_mats():
+        yield name, A
+    yield "long_row", long_row_matrix(L=20_000, N=3000)
+
+
+@pytest.mark.parametrize("name,A", list(_mats_for_conv()))
+def test_conversions_bit_exact(cuda, name, A):
+    n = nitro()
+    M, _ = handle(A, cuda)
+    mask = M.allowed_mask()
+    f = oracle.features(A)
+    ld = oracle.round_up(A.rows)
+    big = 1e18
+    M.set_budget(big)
+    assert M.allowed_mask() == oracle.allowed_mask(f, ld, 8 if A.fp64 else 4, big)
+    mask = M.allowed_mask()
+    if mask[n.ELL]:
+        K, ld_o, ecol, ev = oracle.csr_to_ell(A)
+        info = M.format_info(n.ELL)
+        assert (info["width"], info["ld"]) == (K, ld_o)
+        assert np.array_equal(M.export(n.PART_ELL_COL), ecol)
+        assert np.array_equal(M.export(n.PART_ELL_VAL).astype(np.float64), ev)
+    if mask[n.DIA] and A.nnz > 0:
+        offs, ld_o, dv = oracle.csr_to_dia(A)
+        info = M.format_info(n.DIA)
+        assert (info["width"], info["ld"]) == (len(offs), ld_o)
+        assert np.array_equal(M.export(n.PART_DIA_OFF), offs)
+        assert np.array_equal(M.export(n.PART_DIA_VAL).astype(np.float64), dv)
+    K, ld_o, ecol, ev, tr, tc, tv = oracle.csr_to_hyb(A)
+    info = M.format_info(n.HYB)
+    assert (info["width"], info["ld"], info["tail"]) == (K, ld_o, len(tr))
+    assert np.array_equal(M.export(n.PART_HYB_COL), ecol)
+    assert np.array_equal(M.export(n.PART_HYB_VAL).astype(np.float64), ev)
+    assert np.array_equal(M.export(n.PART_HYB_TROW), tr)
+    assert np.array_equal(M.export(n.PART_HYB_TCOL), tc)
+    assert np.array_equal(M.export(n.PART_HYB_TVAL).astype(np.float64), tv)
+
+
+# ------------------------------------------------------------------ SpMV
+def _run_all(A, x, cuda, rowptr32=None, budget=1e18):
+    import torch
+    n = nitro()
+    M, _ = handle(A, cuda, rowptr32=rowptr32)
+    M.set_budget(budget)
+    xd = torch.from_numpy(x).to(cuda)
+    out = {}
+    for v in range(n.NUM_VARIANTS):
+        if not M.allowed(v):
+            continue
+        y = torch.full((A.rows,), float("nan"), dtype=xd.dtype, device=cuda)  # overwrite semantics
+        M.run(v, xd, y)
+        y2 = M.run(v, xd)  # repeat: no state carried between multiplies
+        torch.cuda.synchronize()
+        out[v] = (y.cpu().numpy(), y2.cpu().numpy())
+    return out
+
+
+@pytest.mark.parametrize("name,A", list(small_mats()))
+def test_spmv_all_variants_tolerance(cuda, name, A):
+    x = synth.vector(A.cols, seed=31, mode=0, fp64=A.fp64)
+    y_ref, r = oracle.spmv(A, x)
+    res = _run_all(A, x, cuda)
+    assert 0 in res and 1 in res and 4 in res
+    for v, (y, y2) in res.items():
+        check_y(y, y_ref, r, A.fp64)
+        assert np.array_equal(y, y2), (name, v)   # deterministic
+
+
+@pytest.mark.parametrize("kind,n", [("2d5", 64), ("2d5", 100), ("3d27", 24), ("3d7", 30), ("1d3", 5000), ("2d9", 40)])
+def test_spmv_integer_stencil_exact(cuda, kind, n):
+    """Integer Poisson stencil x integer x: exact in fp32 for every variant."""
+    A = synth.stencil(kind, n)
+    x = synth.vector(A.cols, seed=1, mode=1)
+    y_ref, _ = oracle.spmv(A, x)
+    res = _run_all(A, x, cuda)
+    assert len(res) == 5
+    for v, (y, _) in res.items():
+        assert np.array_equal(y.astype(np.float64), y_ref), v
+
+
+@pytest.mark.parametrize("fp64", [False, True])
+def test_spmv_long_row(cuda, fp64):
+    A = long_row_matrix(fp64=fp64)
+    x = synth.vector(A.cols, seed=7, fp64=fp64)
+    y_ref, r = oracle.spmv(A, x)
+    for rp32 in (True, False):
+        for v, (y, y2) in _run_all(A, x, cuda, rowptr32=rp32).items():
+            check_y(y, y_ref, r, fp64)
+            assert np.array_equal(y, y2)
+
+
+def test_run_host_matches_device(cuda):
+    n = nitro()
+    A = synth.uniform(10000, 7, variable=True, seed=3)
+    x = synth.vector(A.cols, seed=4)
+    y_ref, r = oracle.spmv(A, x)
+    M, _ = handle(A, cuda)
+    for v in range(5):
+        if M.allowed(v):
+            check_y(M.run_host(v, x), y_ref, r, False)
+
+
+def test_constraint_blocks_explicit_run(cuda):
+    import torch
+    n = nitro()
+    A = synth.rmat(12, 16, seed=2, fp64=False)
+    M, _ = handle(A, cuda)
+    assert not M.allowed(n.ELL) and not M.allowed(n.DIA)
+    with pytest.raises(n.NitroError) as e:
+        M.run(n.DIA, torch.zeros(A.cols, device=cuda))
+    assert e.value.code == 4
+    M2, _ = handle(synth.stencil("3d27", 10), cuda)
+    M2.set_budget(100.0)
+    assert not M2.allowed(n.DIA) and not M2.allowed(n.ELL)
+
+
+def test_timing_and_launch_counts(cuda):
+    import torch
+    n = nitro()
+    A = synth.stencil("3d27", 32, mode=1)
+    M, Ad = handle(A, cuda)
+    x = synth.vector(A.cols, seed=1, device=cuda)
+    y = torch.empty(A.rows, device=cuda)
+    for v in range(5):
+        med, allt = M.time(v, x, y, warmup=1, reps=5, flush_l2=True)
+        assert 0 < med < 0.1 and len(allt) == 5
+        assert M.launches(v) == (3 if v == n.HYB and M.format_info(v)["tail"] > 0 else 1)
+
+
+# ------------------------------------------------------------------ full-size configs (BASELINE configs[1], [2])
+def test_c1_3d27_n128_full(cuda):
+    """configs[1]: 2,097,152 rows, 55,742,968 nnz, fp32; every variant vs oracle."""
+    A = synth.stencil("3d27", 128, mode=1, seed=1)
+    x = synth.vector(A.cols, seed=2)
+    y_ref, r = oracle.spmv(A, x)
+    M, Ad = handle(A, cuda)
+    f, f_ref = M.features(), oracle.features(A)
+    for k in FEAT_KEYS:
+        assert f[k] == f_ref[k], k
+    import torch
+    xd = torch.from_numpy(x).to(cuda)
+    for v in range(5):
+        y = M.run(v, xd)
+        torch.cuda.synchronize()
+        check_y(y.cpu().numpy(), y_ref, r, False)
+        M.release(v)
+
+
+def test_c2a_uniform_full(cuda):
+    """configs[2] uniform: 8,388,608 rows x 32 nnz/row fp32 (ELL-favourable); DIA ruled out."""
+    import torch
+    n = nitro()
+    A = synth.uniform(1 << 23, 32, seed=5)
+    x = synth.vector(A.cols, seed=6)
+    y_ref, r = oracle.spmv(A, x)
+    M, _ = handle(A, cuda)
+    assert not M.allowed(n.DIA) and M.allowed(n.ELL)
+    xd = torch.from_numpy(x).to(cuda)
+    for v in (n.CSR_VECTOR, n.ELL, n.HYB):
+        y = M.run(v, xd)
+        torch.cuda.synchronize()
+        check_y(y.cpu().numpy(), y_ref, r, False)
+        M.release(v)
+
+
+def test_c2b_rmat_full(cuda):
+    """configs[2] power law: R-MAT scale 23, edge factor 16, fp64; ELL/DIA ruled out."""
+    import torch
+    n = nitro()
+    A = synth.rmat(23, 16, seed=7, fp64=True)
+    x = synth.vector(A.cols, seed=8, fp64=True)
+    y_ref, r = oracle.spmv(A, x)
+    M, _ = handle(A, cuda)
+    f, f_ref = M.features(), oracle.features(A)
+    for k in FEAT_KEYS:
+        assert f[k] == f_ref[k], k
+    assert not M.allowed(n.DIA) and not M.allowed(n.ELL)
+    xd = torch.from_numpy(x).to(cuda)
+    for v in (n.CSR_SCALAR, n.CSR_VECTOR, n.HYB):
+        y = M.run(v, xd)
+        torch.cuda.synchronize()
+        check_y(y.cpu().numpy(), y_ref, r, True)
+        M.release(v)
+
+
+# ------------------------------------------------------------------ select path on the GPU
+def test_register_train_select_call(cuda, tmp_path):
+    import torch
+    n = nitro()
+    mats = [synth.stencil("3d27", 24, mode=1), synth.uniform(60000, 30, seed=1), synth.rmat(14, 8, seed=1, fp64=False),
+            synth.stencil("1d3", 100000, mode=1), synth.banded(50000, 3, 1.0, seed=2), synth.uniform(80000, 2, seed=3)]
+    ctx = n.Context()
+    cv = n.CodeVariant(ctx, "spmv")
+    cv.register_spmv()
+    assert cv.n_variants() == 5 and cv.n_features() == 7
+    keep = []
+    for A in mats:
+        M, Ad = handle(A, cuda)
+        x = synth.vector(A.cols, seed=1, device=cuda)
+        y = torch.empty(A.rows, device=cuda)
+        rec = n.spmv_input(M, x, y, warmup=1, reps=5)
+        keep.append((M, Ad, x, y, rec))
+        cv.add_training_input(n.addr(rec))
+    cv.train(folds=3, log2c_lo=-1, log2c_hi=5, log2g_lo=-3, log2g_hi=1)
+    cost, feat, lab = cv.training_table()
+    # exhaustive best == argmin of the recorded table (oracle C10), constraints -> inf
+    from oracle import select as S
+    assert list(lab) == S.exhaustive_best(cost.tolist())
+    for (M, *_), row in zip(keep, cost):
+        for v in range(5):
+            assert np.isfinite(row[v]) == M.allowed(v)
+    # features in the table equal the oracle's
+    for A, frow in zip(mats, feat):
+        fo = oracle.features(A)
+        assert list(frow) == [fo[k] for k in S.FEATURE_NAMES]
+    p = tmp_path / "m.txt"
+    cv.save(p)
+    cv2 = n.CodeVariant(ctx, "spmv2")
+    cv2.register_spmv()
+    cv2.load(p)
+    for (M, Ad, x, y, rec) in keep:
+        v1, _ = cv.select(n.addr(rec))
+        v2, _ = cv2.select(n.addr(rec))
+        assert v1 == v2 and M.allowed(v1)
+        v3, c3 = cv.call(n.addr(rec))
+        assert v3 == v1 and c3 > 0
