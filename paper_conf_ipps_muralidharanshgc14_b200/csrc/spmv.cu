@@ -125,45 +125,59 @@ __global__ void __launch_bounds__(256) k_csr_vector(const IT *__restrict__ rowpt
     const int64_t r = t0 + lane;
     int64_t a = 0, L = 0;
     if (r < N) { a = (int64_t)rowptr[r]; L = (int64_t)rowptr[r + 1] - a; }
+    // 32-bit row starts relative to the tile's first row (a tile never spans 2^31
+    // entries of short rows; long rows are zeroed below and never dereferenced)
+    const int64_t abase = __shfl_sync(kFull, a, 0);
+    const int rel = (int)(a - abase);
+    const int L32 = L > T ? -1 : (int)L;  // -1 marks a long row (segment path)
+    const int *colt = col + abase;
+    const VT *valt = val + abase;
 #pragma unroll
     for (int tb = 0; tb < V; tb += R) {
-      int64_t s[R];
-      int64_t l[R];
+      int s[R], l[R];
+      unsigned longmask = 0;
 #pragma unroll
       for (int u = 0; u < R; ++u) {
         const int src = g + G * (tb + u);
-        s[u] = __shfl_sync(kFull, a, src);
-        l[u] = __shfl_sync(kFull, L, src);
-        if (l[u] > T) l[u] = 0;  // handled by the segment path
+        s[u] = __shfl_sync(kFull, rel, src);
+        l[u] = __shfl_sync(kFull, L32, src);
+        if (l[u] < 0) { longmask |= 1u << u; l[u] = 0; }
       }
       int c[R];
       VT v[R];
 #pragma unroll
       for (int u = 0; u < R; ++u) {
         const bool in = li < l[u];
-        c[u] = in ? ld_stream_i(col + s[u] + li) : -1;
-        v[u] = in ? ld_stream(val + s[u] + li) : (VT)0;
+        c[u] = in ? ld_stream_i(colt + s[u] + li) : -1;
+        v[u] = in ? ld_stream(valt + s[u] + li) : (VT)0;
       }
       VT part[R];
 #pragma unroll
       for (int u = 0; u < R; ++u) part[u] = c[u] >= 0 ? v[u] * __ldg(x + c[u]) : (VT)0;
 #pragma unroll
       for (int u = 0; u < R; ++u)
-        for (int64_t m = V + li; m < l[u]; m += V)  // <= 7 more terms per lane
-          part[u] = fma(ld_stream(val + s[u] + m), __ldg(x + ld_stream_i(col + s[u] + m)), part[u]);
+        for (int m = V + li; m < l[u]; m += V)  // <= 7 more terms per lane
+          part[u] = fma(ld_stream(valt + s[u] + m), __ldg(x + ld_stream_i(colt + s[u] + m)), part[u]);
+      // transposed reduction: R rows over V lanes in log2(V) + R/2 shuffles;
+      // lane li ends with the total of row ridx (valid where li % (V/R) == 0)
+      int ridx;
+      VT tot;
+      if constexpr (R == 4) {
+        constexpr int o1 = V / 2, o2 = V / 4;
+        const bool h1 = li & o1, h2 = li & o2;
+        const VT a0 = (h1 ? part[2] : part[0]) + __shfl_xor_sync(kFull, h1 ? part[0] : part[2], o1);
+        const VT a1 = (h1 ? part[3] : part[1]) + __shfl_xor_sync(kFull, h1 ? part[1] : part[3], o1);
+        tot = (h2 ? a1 : a0) + __shfl_xor_sync(kFull, h2 ? a0 : a1, o2);
 #pragma unroll
-      for (int u = 0; u < R; ++u) {
-#pragma unroll
-        for (int o = V / 2; o > 0; o >>= 1) part[u] += __shfl_xor_sync(kFull, part[u], o);
+        for (int o = V / 8; o > 0; o >>= 1) tot += __shfl_xor_sync(kFull, tot, o);
+        ridx = (h1 ? 2 : 0) + (h2 ? 1 : 0);
+      } else {  // V == 2, R == 2
+        const bool h = li & 1;
+        tot = (h ? part[1] : part[0]) + __shfl_xor_sync(kFull, h ? part[0] : part[1], 1);
+        ridx = h ? 1 : 0;
       }
-      // write results (lanes li == 0); long rows skipped
-#pragma unroll
-      for (int u = 0; u < R; ++u) {
-        const int src = g + G * (tb + u);
-        const int64_t Lr = __shfl_sync(kFull, L, src);
-        const int64_t row = t0 + src;
-        if (li == 0 && row < N && Lr <= T) y[row] = part[u];
-      }
+      const int64_t row = t0 + g + G * (tb + ridx);
+      if (li % (V / R) == 0 && row < N && !((longmask >> ridx) & 1u)) y[row] = tot;
     }
   }
 }
@@ -287,6 +301,14 @@ __global__ void __launch_bounds__(256) k_hyb_tail(const int32_t *__restrict__ tr
       if (w0 >= cend) break;
       double q = p[w];
       const int r = rr[w];
+      // a segment left open at the previous window's last lane ended exactly
+      // at the window boundary if this window starts a new row: emit it now
+      const int r_first = __shfl_sync(kFull, r, 0);
+      if (carry_r >= 0 && r_first != carry_r && lane == 0) {
+        if (carry_r == first_row) { carry_row[2 * ch] = carry_r; carry_val[2 * ch] = carry_v; }
+        else if (carry_r == last_row) { carry_row[2 * ch + 1] = carry_r; carry_val[2 * ch + 1] = carry_v; }
+        else y[carry_r] = (VT)((double)y[carry_r] + carry_v);
+      }
 #pragma unroll
       for (int o = 1; o < 32; o <<= 1) {
         const double t = __shfl_up_sync(kFull, q, o);
