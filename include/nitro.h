@@ -274,6 +274,19 @@ nitro_status_t nitro_dist_spmv_create(nitro_dist *D, int64_t global_rows, const 
  * a side stream; interior rows overlap the gather, boundary rows follow). */
 nitro_status_t nitro_dist_spmv_run(nitro_dist *D, nitro_spmv *A_local, int variant, const void *d_x_local,
                                    void *d_y_local);
+/* Same multiply from an x that is already gathered in the padded layout
+ * (block q at q*B, B = max block rows, length nranks*B): no communication.
+ * Used when the caller owns the exchange (e.g. a solver that writes y straight
+ * into the next x), and to check every rank's part on one GPU. */
+nitro_status_t nitro_dist_spmv_run_gathered(nitro_dist *D, nitro_spmv *A_local, int variant,
+                                            const void *d_x_gathered, void *d_y_local);
+/* Padded block size B and this rank's [i0, i1) interior row run (rows that
+ * read only local x and overlap the all-gather). */
+nitro_status_t nitro_dist_layout(nitro_spmv *A_local, int64_t *B, int64_t *i0, int64_t *i1);
+/* A communicator-less handle for (rank, nranks): everything but the NCCL
+ * calls works (partition, remap, parts, run_gathered); run/features with
+ * nranks > 1 return NITRO_E_STATE.  For single-GPU checks of multi-rank logic. */
+nitro_status_t nitro_dist_init_local(int rank, int nranks, int device, nitro_dist **out);
 /* Global features from per-rank feature passes (sum / max all-reduce and a
  * union of diagonal offsets): identical to the single-GPU features. */
 nitro_status_t nitro_dist_features(nitro_dist *D, nitro_spmv *A_local, nitro_spmv_feat *out);

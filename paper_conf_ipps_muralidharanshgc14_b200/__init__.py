@@ -144,6 +144,9 @@ _SIGS = {
     "nitro_dist_spmv_create": ([_vp, _i64, _vp, _i64, _vp, _int, _vp, _vp, _int, _P(_vp)], _int),
     "nitro_dist_spmv_run": ([_vp, _vp, _int, _vp, _vp], _int),
     "nitro_dist_features": ([_vp, _vp, _P(Feat)], _int),
+    "nitro_dist_spmv_run_gathered": ([_vp, _vp, _int, _vp, _vp], _int),
+    "nitro_dist_layout": ([_vp, _P(_i64), _P(_i64), _P(_i64)], _int),
+    "nitro_dist_init_local": ([_int, _int, _int, _P(_vp)], _int),
 }
 for _name, (_args, _res) in _SIGS.items():
     _f = getattr(_L, _name)
@@ -489,11 +492,33 @@ def dist_unique_id() -> bytes:
 
 
 class Dist:
-    def __init__(self, uid: bytes, rank: int, nranks: int, device: int):
-        buf = ctypes.create_string_buffer(uid, 128)
+    """One rank of the row-partitioned multi-GPU SpMV (NCCL communicator).
+
+    ``Dist.local(rank, nranks, device)`` builds a communicator-less handle whose
+    ``run_gathered`` computes that rank's rows from an already gathered x."""
+
+    def __init__(self, uid: bytes | None, rank: int, nranks: int, device: int):
         h = ctypes.c_void_p()
-        _check(_L.nitro_dist_init(buf, rank, nranks, device, ctypes.byref(h)))
+        if uid is None:
+            _check(_L.nitro_dist_init_local(rank, nranks, device, ctypes.byref(h)))
+        else:
+            buf = ctypes.create_string_buffer(uid, 128)
+            _check(_L.nitro_dist_init(buf, rank, nranks, device, ctypes.byref(h)))
         self.h, self.rank, self.nranks, self.device = h, rank, nranks, device
+
+    @classmethod
+    def local(cls, rank: int, nranks: int, device: int = 0):
+        return cls(None, rank, nranks, device)
+
+    def run_gathered(self, A: "SpMV", v: int, x_gathered, y_local):
+        _check(_L.nitro_dist_spmv_run_gathered(self.h, A.h, v, _ptr(x_gathered), _ptr(y_local)))
+        return y_local
+
+    @staticmethod
+    def layout(A: "SpMV"):
+        B, i0, i1 = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64()
+        _check(_L.nitro_dist_layout(A.h, ctypes.byref(B), ctypes.byref(i0), ctypes.byref(i1)))
+        return B.value, i0.value, i1.value
 
     def close(self):
         if getattr(self, "h", None):
@@ -516,8 +541,9 @@ class Dist:
         A.fp64 = vals.dtype == torch.float64
         A.dtype = vals.dtype
         A.device = self.device
-        A.stream = None
+        A.stream = torch.cuda.current_stream(self.device).cuda_stream
         A.h = h
+        _check(_L.nitro_spmv_set_stream(h, A.stream))
         return A
 
     def run(self, A: SpMV, v: int, x_local, y_local):

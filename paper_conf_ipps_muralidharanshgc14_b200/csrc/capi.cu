@@ -390,6 +390,7 @@ void nitro_spmv_destroy(nitro_spmv *A) {
     if (A->feat_done) cudaEventDestroy(A->feat_done);
     A->feat_acc.release(); A->bitmap.release(); A->offsets.release(); A->scratch.release();
     A->flush.release(); A->xbuf.release(); A->ybuf.release();
+    if (A->dist_free && A->dist_state) A->dist_free(A->dist_state);
   }
   delete A;
 }

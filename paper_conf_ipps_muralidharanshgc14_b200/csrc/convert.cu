@@ -198,7 +198,7 @@ nitro_status_t prepare_dia(nitro_spmv *A) {
   NITRO_TRY(features_finish(A));
   cudaStream_t s = A->stream;
   const int64_t D = A->feat.ndiag, ld = round_up(A->N, 32), sv = A->fp64 ? 8 : 4;
-  const int64_t G = A->row0 + A->N - 1;
+  const int64_t G = diag_shift(A);
   const int64_t span = A->N > 0 ? G + A->M : 0, nwords = (span + 31) / 32;
   NITRO_TRY(A->dia.off.alloc((size_t)std::max<int64_t>(D, 1) * 4));
   if (D > 0) {

@@ -178,7 +178,7 @@ void finish_features(int64_t N, int64_t M, int64_t Z, uint64_t s1, uint64_t s2, 
 nitro_status_t features_launch(nitro_spmv *A) {
   if (A->feat_ready || A->feat_pending) return NITRO_OK;
   cudaStream_t s = A->stream;
-  const int64_t G = A->row0 + A->N - 1;            // bitmap index = d + G
+  const int64_t G = diag_shift(A);                 // bitmap index = d + G
   const int64_t span = A->N > 0 ? G + A->M : 0;    // offsets in [-G, M-1]
   const int64_t nwords = (span + 31) / 32;
   NITRO_TRY(A->feat_acc.alloc(sizeof(FeatAcc)));

@@ -106,10 +106,11 @@ struct nitro_spmv {
   nitro::DevBuf flush;      // L2 flush scratch
   nitro::DevBuf xbuf, ybuf; // run_host staging
 
-  // multi-GPU
+  // multi-GPU (dist.cu)
+  int64_t feat_G = -1;      // bitmap offset shift override (global-offset bitmaps); -1 = row0 + N - 1
   nitro_dist *dist = nullptr;
-  int64_t n_interior = 0;   // rows [0, n_interior) are interior after a dist permutation? (see dist.cu)
   void *dist_state = nullptr;
+  void (*dist_free)(void *) = nullptr;
 };
 
 namespace nitro {
@@ -136,6 +137,8 @@ double compulsory_bytes(const nitro_spmv *A, int variant);
 nitro_status_t exclusive_scan_i64(const int64_t *in, int64_t *out, int64_t n, DevBuf &scratch, cudaStream_t s);
 
 inline int64_t round_up(int64_t n, int64_t m) { return (n + m - 1) / m * m; }
+// bitmap index of diagonal offset d is d + G; the bitmap spans G + M bits
+inline int64_t diag_shift(const nitro_spmv *A) { return A->feat_G >= 0 ? A->feat_G : A->row0 + A->N - 1; }
 int num_sms();
 
 }  // namespace nitro
