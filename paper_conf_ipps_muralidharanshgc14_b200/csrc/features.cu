@@ -26,7 +26,8 @@ namespace {
 
 constexpr int kThreads = 256;
 constexpr int kWarps = kThreads / 32;
-constexpr int kCache = 512;  // per-block offset cache slots
+constexpr int kCache = 1024;  // per-block offset set slots (8 KB)
+constexpr int kProbe = 4;     // linear-probe length
 
 template <typename IT>
 __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
@@ -99,18 +100,31 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
           }
         }
         // occupied-diagonal bitmap with dedupe
+        // (per-block open-addressing set of offsets already in the bitmap:
+        //  a stencil's few offsets stay resident, so its entries cost only lookups)
         bool want = idx >= 0;
         unsigned h = 0;
         if (want) {
-          h = (unsigned)(((unsigned long long)idx * 0x9E3779B97F4A7C15ull) >> 55) & (kCache - 1);
-          if (s_seen[h] == idx) want = false;
+          h = (unsigned)(((unsigned long long)idx * 0x9E3779B97F4A7C15ull) >> 40);
+#pragma unroll
+          for (int p = 0; p < kProbe; ++p) {
+            const long long cur = s_seen[(h + p) & (kCache - 1)];
+            if (cur == idx) { want = false; break; }
+            if (cur == -1) break;
+          }
         }
         const unsigned need = __ballot_sync(kFull, want);
         if (want) {
           const unsigned grp = __match_any_sync(need, idx);
           if ((int)(__ffs(grp) - 1) == lane) {
             atomicOr(bitmap + (idx >> 5), 1u << (idx & 31));
-            s_seen[h] = idx;
+#pragma unroll
+            for (int p = 0; p < kProbe; ++p) {
+              const unsigned long long prev = atomicCAS(
+                  reinterpret_cast<unsigned long long *>(&s_seen[(h + p) & (kCache - 1)]), ~0ull,
+                  (unsigned long long)idx);
+              if (prev == ~0ull || prev == (unsigned long long)idx) break;
+            }
           }
         }
         const int last_lane = E1 - 1 - w0 < 31 ? (int)(E1 - 1 - w0) : 31;

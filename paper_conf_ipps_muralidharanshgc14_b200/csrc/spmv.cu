@@ -66,6 +66,30 @@ __global__ void __launch_bounds__(256) k_csr_scalar(const IT *__restrict__ rowpt
   }
 }
 
+// Transposed reduction of R per-lane values (one per row) over groups of V
+// lanes: log2(R) exchange steps halve the value count (R-1 shuffles), then
+// log2(V/R) plain butterfly steps.  Lane li returns the total of row ridx;
+// the lanes with li % (V/R) == 0 hold distinct rows.
+template <int V, int R, typename VT>
+__device__ __forceinline__ VT reduce_transpose(VT (&p)[R], int li, int &ridx) {
+  ridx = 0;
+#pragma unroll
+  for (int n = R, o = V / 2; n > 1; n >>= 1, o >>= 1) {
+    const bool h = li & o;
+#pragma unroll
+    for (int j = 0; j < n / 2; ++j) {
+      const VT keep = h ? p[j + n / 2] : p[j];
+      const VT send = h ? p[j] : p[j + n / 2];
+      p[j] = keep + __shfl_xor_sync(kFull, send, o);
+    }
+    ridx = ridx * 2 + (h ? 1 : 0);
+  }
+  VT t = p[0];
+#pragma unroll
+  for (int o = V / (2 * R); o > 0; o >>= 1) t += __shfl_xor_sync(kFull, t, o);
+  return t;
+}
+
 // ------------------------------------------------------------------ K6 CSR-vector
 // V lanes per row.  A warp takes 32 consecutive rows (one coalesced rowptr
 // load per lane); lane group g handles rows g, g+G, ... (G = 32/V) R at a
@@ -116,71 +140,77 @@ __global__ void __launch_bounds__(256) k_csr_vector(const IT *__restrict__ rowpt
     }
     return;
   }
+  // R rows per lane group in flight per batch, TU tiles of 32 rows per warp
+  // iteration, so every lane keeps R*TU = 8 independent (col, val) -> x chains
   constexpr int G = 32 / V;
-  constexpr int R = V >= 4 ? 4 : V;
+  constexpr int R = V >= 8 ? 8 : V;
+  constexpr int TU = 8 / R;
   const int lane = threadIdx.x & 31, g = lane / V, li = lane % V;
   const int64_t warp = (((int64_t)blockIdx.x - nseg) * blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = (((int64_t)gridDim.x - nseg) * blockDim.x) >> 5;
-  for (int64_t t0 = warp * 32; t0 < N; t0 += nwarps * 32) {
-    const int64_t r = t0 + lane;
-    int64_t a = 0, L = 0;
-    if (r < N) { a = (int64_t)rowptr[r]; L = (int64_t)rowptr[r + 1] - a; }
-    // 32-bit row starts relative to the tile's first row (a tile never spans 2^31
-    // entries of short rows; long rows are zeroed below and never dereferenced)
-    const int64_t abase = __shfl_sync(kFull, a, 0);
-    const int rel = (int)(a - abase);
-    const int L32 = L > T ? -1 : (int)L;  // -1 marks a long row (segment path)
+  for (int64_t t0 = warp * (32 * TU); t0 < N; t0 += nwarps * (32 * TU)) {
+    // 32-bit row starts relative to the first row of the TU tiles (short rows
+    // only: long rows are flagged -1 and never dereferenced here)
+    int rel[TU], L32[TU];
+    int64_t abase = 0;
+#pragma unroll
+    for (int tu = 0; tu < TU; ++tu) {
+      const int64_t r = t0 + tu * 32 + lane;
+      int64_t a = 0, L = 0;
+      if (r < N) { a = (int64_t)rowptr[r]; L = (int64_t)rowptr[r + 1] - a; }
+      if (tu == 0) abase = __shfl_sync(kFull, a, 0);
+      rel[tu] = (int)(a - abase);
+      L32[tu] = L > T ? -1 : (int)L;
+    }
     const int *colt = col + abase;
     const VT *valt = val + abase;
 #pragma unroll
     for (int tb = 0; tb < V; tb += R) {
-      int s[R], l[R];
-      unsigned longmask = 0;
+      int s[TU][R], l[TU][R];
+      unsigned longmask[TU];
 #pragma unroll
-      for (int u = 0; u < R; ++u) {
-        const int src = g + G * (tb + u);
-        s[u] = __shfl_sync(kFull, rel, src);
-        l[u] = __shfl_sync(kFull, L32, src);
-        if (l[u] < 0) { longmask |= 1u << u; l[u] = 0; }
+      for (int tu = 0; tu < TU; ++tu) {
+        longmask[tu] = 0;
+#pragma unroll
+        for (int u = 0; u < R; ++u) {
+          const int src = g + G * (tb + u);
+          s[tu][u] = __shfl_sync(kFull, rel[tu], src);
+          l[tu][u] = __shfl_sync(kFull, L32[tu], src);
+          if (l[tu][u] < 0) { longmask[tu] |= 1u << u; l[tu][u] = 0; }
+        }
       }
-      int c[R];
-      VT v[R];
+      int c[TU][R];
+      VT v[TU][R];
 #pragma unroll
-      for (int u = 0; u < R; ++u) {
-        const bool in = li < l[u];
-        c[u] = in ? ld_stream_i(colt + s[u] + li) : -1;
-        v[u] = in ? ld_stream(valt + s[u] + li) : (VT)0;
+      for (int tu = 0; tu < TU; ++tu)
+#pragma unroll
+        for (int u = 0; u < R; ++u) {
+          const bool in = li < l[tu][u];
+          c[tu][u] = in ? ld_stream_i(colt + s[tu][u] + li) : -1;
+          v[tu][u] = in ? ld_stream(valt + s[tu][u] + li) : (VT)0;
+        }
+      VT part[TU][R];
+#pragma unroll
+      for (int tu = 0; tu < TU; ++tu)
+#pragma unroll
+        for (int u = 0; u < R; ++u) part[tu][u] = c[tu][u] >= 0 ? v[tu][u] * __ldg(x + c[tu][u]) : (VT)0;
+#pragma unroll
+      for (int tu = 0; tu < TU; ++tu)
+#pragma unroll
+        for (int u = 0; u < R; ++u)
+          for (int m = V + li; m < l[tu][u]; m += V)  // <= 7 more terms per lane
+            part[tu][u] = fma(ld_stream(valt + s[tu][u] + m), __ldg(x + ld_stream_i(colt + s[tu][u] + m)), part[tu][u]);
+#pragma unroll
+      for (int tu = 0; tu < TU; ++tu) {
+        int ridx;
+        const VT tot = reduce_transpose<V, R>(part[tu], li, ridx);
+        const int64_t row = t0 + tu * 32 + g + G * (tb + ridx);
+        if (li % (V / R) == 0 && row < N && !((longmask[tu] >> ridx) & 1u)) y[row] = tot;
       }
-      VT part[R];
-#pragma unroll
-      for (int u = 0; u < R; ++u) part[u] = c[u] >= 0 ? v[u] * __ldg(x + c[u]) : (VT)0;
-#pragma unroll
-      for (int u = 0; u < R; ++u)
-        for (int m = V + li; m < l[u]; m += V)  // <= 7 more terms per lane
-          part[u] = fma(ld_stream(valt + s[u] + m), __ldg(x + ld_stream_i(colt + s[u] + m)), part[u]);
-      // transposed reduction: R rows over V lanes in log2(V) + R/2 shuffles;
-      // lane li ends with the total of row ridx (valid where li % (V/R) == 0)
-      int ridx;
-      VT tot;
-      if constexpr (R == 4) {
-        constexpr int o1 = V / 2, o2 = V / 4;
-        const bool h1 = li & o1, h2 = li & o2;
-        const VT a0 = (h1 ? part[2] : part[0]) + __shfl_xor_sync(kFull, h1 ? part[0] : part[2], o1);
-        const VT a1 = (h1 ? part[3] : part[1]) + __shfl_xor_sync(kFull, h1 ? part[1] : part[3], o1);
-        tot = (h2 ? a1 : a0) + __shfl_xor_sync(kFull, h2 ? a0 : a1, o2);
-#pragma unroll
-        for (int o = V / 8; o > 0; o >>= 1) tot += __shfl_xor_sync(kFull, tot, o);
-        ridx = (h1 ? 2 : 0) + (h2 ? 1 : 0);
-      } else {  // V == 2, R == 2
-        const bool h = li & 1;
-        tot = (h ? part[1] : part[0]) + __shfl_xor_sync(kFull, h ? part[0] : part[1], 1);
-        ridx = h ? 1 : 0;
-      }
-      const int64_t row = t0 + g + G * (tb + ridx);
-      if (li % (V / R) == 0 && row < N && !((longmask >> ridx) & 1u)) y[row] = tot;
     }
   }
 }
+
 
 // ------------------------------------------------------------------ K7 ELL (also HYB's ELL part)
 // Thread per 4 consecutive rows: per slot one 128-bit load of 4 column ids and

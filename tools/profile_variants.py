@@ -1,6 +1,10 @@
 #!/usr/bin/env python
-"""Run every SpMV variant (and the feature pass) on one BASELINE config, for
-ncu captures.  Usage: python tools/profile_variants.py c1|c2a|c2b [variants...]"""
+"""Run (or time) every SpMV variant and the feature pass on BASELINE configs.
+
+  python tools/profile_variants.py c1 [variants...]        # 2 runs each, for ncu
+  python tools/profile_variants.py --time c1 c2a c2b       # JSON table (median of 20, L2 flushed)
+"""
+import json
 import os
 import sys
 
@@ -10,12 +14,16 @@ sys.path.insert(0, ROOT)
 
 def make(cfg, dev):
     import synth
+    if cfg == "c0":
+        return synth.stencil("2d5", 64, device=dev)
     if cfg == "c1":
         return synth.stencil("3d27", 128, mode=1, seed=1, device=dev)
     if cfg == "c2a":
         return synth.uniform(1 << 23, 32, seed=5, device=dev)
     if cfg == "c2b":
         return synth.rmat(23, 16, seed=7, fp64=True, device=dev)
+    if cfg == "short":   # very short rows (CSR-scalar class): 1D 3-pt, 2^23 rows
+        return synth.stencil("1d3", 1 << 23, mode=1, seed=3, device=dev)
     raise SystemExit(f"unknown config {cfg}")
 
 
@@ -23,26 +31,54 @@ def main():
     import torch
     import paper_conf_ipps_muralidharanshgc14_b200 as nitro
     import synth
-    cfg = sys.argv[1] if len(sys.argv) > 1 else "c1"
-    want = [nitro.VARIANT_NAMES.index(v) for v in sys.argv[2:]] or list(range(5))
+    args = sys.argv[1:]
+    timing = "--time" in args
+    args = [a for a in args if a != "--time"]
+    cfgs = [a for a in args if a in ("c0", "c1", "c2a", "c2b", "short")] or ["c1"]
+    want = [nitro.VARIANT_NAMES.index(v) for v in args if v in nitro.VARIANT_NAMES] or list(range(5))
     dev = torch.device("cuda:0")
-    A = make(cfg, dev)
-    A.rowptr = A.rowptr.to(torch.int32)
-    M = nitro.SpMV.from_csr(A)
-    f = M.features()
-    x = synth.vector(A.cols, seed=2, fp64=A.fp64, device=dev)
-    y = torch.empty(A.rows, dtype=x.dtype, device=dev)
-    for v in want:
-        if not M.allowed(v):
-            continue
-        M.prepare(v)
-        for _ in range(2):
-            M.flush_l2()
-            M.run(v, x, y)
+    table = {}
+    for cfg in cfgs:
+        A = make(cfg, dev)
+        A.rowptr = A.rowptr.to(torch.int32)
+        M = nitro.SpMV.from_csr(A)
+        s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        M2 = nitro.SpMV.from_csr(A)     # fresh handle: time the feature pass alone
+        M2.features()
+        M3 = nitro.SpMV.from_csr(A)
         torch.cuda.synchronize()
-        info = M.format_info(v)
-        print(cfg, nitro.VARIANT_NAMES[v], "bytes", info["compulsory_bytes"], "launches", M.launches(v), flush=True)
-    print(cfg, "features", f)
+        s.record()
+        f = M3.features()
+        e.record()
+        torch.cuda.synchronize()
+        feat_ms = s.elapsed_time(e)
+        M.features()
+        x = synth.vector(A.cols, seed=2, fp64=A.fp64, device=dev)
+        y = torch.empty(A.rows, dtype=x.dtype, device=dev)
+        row = {"rows": A.rows, "nnz": A.nnz, "feature_ms": feat_ms,
+               "feature_GBps": ((A.rows + 1) * 4 + A.nnz * 4) / (feat_ms * 1e-3) / 1e9, "variants": {}}
+        for v in want:
+            if not M.allowed(v):
+                continue
+            M.prepare(v)
+            info = M.format_info(v)
+            if timing:
+                med, allt = M.time(v, x, y, warmup=3, reps=20, flush_l2=True)
+                row["variants"][nitro.VARIANT_NAMES[v]] = {
+                    "ms": med * 1e3, "GBps": info["compulsory_bytes"] / med / 1e9,
+                    "GFLOPs": 2 * A.nnz / med / 1e9, "bytes": info["compulsory_bytes"], "width": info["width"],
+                    "tail": info["tail"], "launches": M.launches(v)}
+            else:
+                for _ in range(2):
+                    M.flush_l2()
+                    M.run(v, x, y)
+                torch.cuda.synchronize()
+                print(cfg, nitro.VARIANT_NAMES[v], "bytes", info["compulsory_bytes"], flush=True)
+            M.release(v)
+        table[cfg] = row
+        del M, M2, M3, A, x, y
+        torch.cuda.empty_cache()
+    print(json.dumps(table, indent=1))
 
 
 if __name__ == "__main__":
