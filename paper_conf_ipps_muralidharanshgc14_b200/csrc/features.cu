@@ -117,7 +117,10 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
         if (want) {
           const unsigned grp = __match_any_sync(need, idx);
           if ((int)(__ffs(grp) - 1) == lane) {
-            atomicOr(bitmap + (idx >> 5), 1u << (idx & 31));
+            // test before set: an L2 read is far cheaper than a contended RED on
+            // the hot words of random matrices (a stale 0 only costs a redundant OR)
+            const unsigned bit = 1u << (idx & 31);
+            if (!(__ldcg(bitmap + (idx >> 5)) & bit)) atomicOr(bitmap + (idx >> 5), bit);
 #pragma unroll
             for (int p = 0; p < kProbe; ++p) {
               const unsigned long long prev = atomicCAS(

@@ -34,7 +34,8 @@ template <> struct V4<double> {
 
 template <typename VT>
 __device__ __forceinline__ void store4(VT *y, int64_t i0, int64_t N, const double *acc) {
-  if (i0 + 3 < N) {
+  // vector store only when y + i0 is 16-byte aligned (y may be a row-offset view)
+  if (i0 + 3 < N && ((reinterpret_cast<uintptr_t>(y + i0) & 15) == 0)) {
     if constexpr (sizeof(VT) == 4) {
       *reinterpret_cast<float4 *>(y + i0) = make_float4((float)acc[0], (float)acc[1], (float)acc[2], (float)acc[3]);
     } else {
@@ -140,77 +141,93 @@ __global__ void __launch_bounds__(256) k_csr_vector(const IT *__restrict__ rowpt
     }
     return;
   }
-  // R rows per lane group in flight per batch, TU tiles of 32 rows per warp
-  // iteration, so every lane keeps R*TU = 8 independent (col, val) -> x chains
+  // Software-pipelined main path.  A "stage" is R rows of one lane group:
+  // row starts/lengths come from the tile's rowptr registers by shuffle, and
+  // the (col, val) loads of the NEXT stage are issued before the current
+  // stage's x gathers and reduction, so loads stay in flight continuously;
+  // the rowptr of the tile after the next is prefetched one tile ahead.
   constexpr int G = 32 / V;
-  constexpr int R = V >= 8 ? 8 : V;
-  constexpr int TU = 8 / R;
+  constexpr int R = V >= 4 ? 4 : 2;
   const int lane = threadIdx.x & 31, g = lane / V, li = lane % V;
   const int64_t warp = (((int64_t)blockIdx.x - nseg) * blockDim.x + threadIdx.x) >> 5;
-  const int64_t nwarps = (((int64_t)gridDim.x - nseg) * blockDim.x) >> 5;
-  for (int64_t t0 = warp * (32 * TU); t0 < N; t0 += nwarps * (32 * TU)) {
-    // 32-bit row starts relative to the first row of the TU tiles (short rows
-    // only: long rows are flagged -1 and never dereferenced here)
-    int rel[TU], L32[TU];
-    int64_t abase = 0;
+  const int64_t stride = ((((int64_t)gridDim.x - nseg) * blockDim.x) >> 5) * 32;
+  int64_t t0 = warp * 32;
+  if (t0 >= N) return;
+  struct Tile { int64_t abase; int rel, len; };
+  struct Stage { int s[R], l[R]; unsigned longmask; int c[R]; VT v[R]; };
+  auto load_rp = [&](int64_t tt, int64_t &a, int64_t &L) {
+    const int64_t r = tt + lane;
+    a = 0; L = 0;
+    if (r < N) { a = (int64_t)rowptr[r]; L = (int64_t)rowptr[r + 1] - a; }
+  };
+  auto make_tile = [&](int64_t a, int64_t L) {
+    Tile t;
+    t.abase = __shfl_sync(kFull, a, 0);
+    t.rel = (int)(a - t.abase);  // 32-bit within a tile of short rows
+    t.len = L > T ? -1 : (int)L; // -1: long row, handled by the segment path
+    return t;
+  };
+  auto issue = [&](const Tile &t, int tb, Stage &st) {
+    st.longmask = 0;
 #pragma unroll
-    for (int tu = 0; tu < TU; ++tu) {
-      const int64_t r = t0 + tu * 32 + lane;
-      int64_t a = 0, L = 0;
-      if (r < N) { a = (int64_t)rowptr[r]; L = (int64_t)rowptr[r + 1] - a; }
-      if (tu == 0) abase = __shfl_sync(kFull, a, 0);
-      rel[tu] = (int)(a - abase);
-      L32[tu] = L > T ? -1 : (int)L;
+    for (int u = 0; u < R; ++u) {
+      const int src = g + G * (tb + u);
+      st.s[u] = __shfl_sync(kFull, t.rel, src);
+      st.l[u] = __shfl_sync(kFull, t.len, src);
+      if (st.l[u] < 0) { st.longmask |= 1u << u; st.l[u] = 0; }
     }
-    const int *colt = col + abase;
-    const VT *valt = val + abase;
 #pragma unroll
-    for (int tb = 0; tb < V; tb += R) {
-      int s[TU][R], l[TU][R];
-      unsigned longmask[TU];
+    for (int u = 0; u < R; ++u) {
+      const bool in = li < st.l[u];
+      st.c[u] = in ? ld_stream_i(col + t.abase + st.s[u] + li) : -1;
+      st.v[u] = in ? ld_stream(val + t.abase + st.s[u] + li) : (VT)0;
+    }
+  };
+  auto finish = [&](const Tile &t, int64_t tt, int tb, Stage &st) {
+    VT part[R];
 #pragma unroll
-      for (int tu = 0; tu < TU; ++tu) {
-        longmask[tu] = 0;
+    for (int u = 0; u < R; ++u) part[u] = st.c[u] >= 0 ? st.v[u] * __ldg(x + st.c[u]) : (VT)0;
 #pragma unroll
-        for (int u = 0; u < R; ++u) {
-          const int src = g + G * (tb + u);
-          s[tu][u] = __shfl_sync(kFull, rel[tu], src);
-          l[tu][u] = __shfl_sync(kFull, L32[tu], src);
-          if (l[tu][u] < 0) { longmask[tu] |= 1u << u; l[tu][u] = 0; }
-        }
-      }
-      int c[TU][R];
-      VT v[TU][R];
-#pragma unroll
-      for (int tu = 0; tu < TU; ++tu)
-#pragma unroll
-        for (int u = 0; u < R; ++u) {
-          const bool in = li < l[tu][u];
-          c[tu][u] = in ? ld_stream_i(colt + s[tu][u] + li) : -1;
-          v[tu][u] = in ? ld_stream(valt + s[tu][u] + li) : (VT)0;
-        }
-      VT part[TU][R];
-#pragma unroll
-      for (int tu = 0; tu < TU; ++tu)
-#pragma unroll
-        for (int u = 0; u < R; ++u) part[tu][u] = c[tu][u] >= 0 ? v[tu][u] * __ldg(x + c[tu][u]) : (VT)0;
-#pragma unroll
-      for (int tu = 0; tu < TU; ++tu)
-#pragma unroll
-        for (int u = 0; u < R; ++u)
-          for (int m = V + li; m < l[tu][u]; m += V)  // <= 7 more terms per lane
-            part[tu][u] = fma(ld_stream(valt + s[tu][u] + m), __ldg(x + ld_stream_i(colt + s[tu][u] + m)), part[tu][u]);
-#pragma unroll
-      for (int tu = 0; tu < TU; ++tu) {
-        int ridx;
-        const VT tot = reduce_transpose<V, R>(part[tu], li, ridx);
-        const int64_t row = t0 + tu * 32 + g + G * (tb + ridx);
-        if (li % (V / R) == 0 && row < N && !((longmask[tu] >> ridx) & 1u)) y[row] = tot;
+    for (int u = 0; u < R; ++u)
+      for (int m = V + li; m < st.l[u]; m += V)  // <= 7 more terms per lane
+        part[u] = fma(ld_stream(val + t.abase + st.s[u] + m), __ldg(x + ld_stream_i(col + t.abase + st.s[u] + m)),
+                      part[u]);
+    int ridx;
+    const VT tot = reduce_transpose<V, R>(part, li, ridx);
+    const int64_t row = tt + g + G * (tb + ridx);
+    if (li % (V / R) == 0 && row < N && !((st.longmask >> ridx) & 1u)) y[row] = tot;
+  };
+  int64_t pa, pL;  // prefetched rowptr data of the next tile
+  int64_t a0, L0;
+  load_rp(t0, a0, L0);
+  load_rp(t0 + stride, pa, pL);
+  Tile cur = make_tile(a0, L0);
+  int tb = 0;
+  Stage st;
+  issue(cur, tb, st);
+  for (;;) {
+    int ntb = tb + R;
+    int64_t nt0 = t0;
+    Tile nxt = cur;
+    if (ntb >= V) {
+      ntb = 0;
+      nt0 = t0 + stride;
+      if (nt0 < N) {
+        nxt = make_tile(pa, pL);
+        load_rp(nt0 + stride, pa, pL);
       }
     }
+    const bool more = nt0 < N;
+    Stage ns;
+    if (more) issue(nxt, ntb, ns);
+    finish(cur, t0, tb, st);
+    if (!more) break;
+    st = ns;
+    cur = nxt;
+    t0 = nt0;
+    tb = ntb;
   }
 }
-
 
 // ------------------------------------------------------------------ K7 ELL (also HYB's ELL part)
 // Thread per 4 consecutive rows: per slot one 128-bit load of 4 column ids and

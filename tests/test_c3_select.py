@@ -1,0 +1,76 @@
+"""configs[3] select-path parity on the committed experiment (CPU only).
+
+tools/train_select.py measured the 100-matrix timing table on a B200 and ran
+the library's training (nitro_cv_train_from_table) and selection.  Here the
+oracle's select path re-derives, from the same table: the exhaustive-best
+labels (C10), the scaled CV grid choice of (C, gamma) and the held-out
+predictions (C11-C12, sklearn/libSVM as the library step), and the Nitro %
+statistics (C13) — and they must match what the library produced.
+The statistic's VALUE is parity-unpinned (no reference GPU timings exist)."""
+import json
+import math
+import os
+
+import numpy as np
+import pytest
+
+from oracle import select as S
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+TABLE = os.path.join(ROOT, "artifacts", "c3_table.json")
+REPORT = os.path.join(ROOT, "artifacts", "c3_report.json")
+MODEL = os.path.join(ROOT, "artifacts", "spmv_model.txt")
+
+pytestmark = pytest.mark.skipif(not os.path.exists(TABLE), reason="configs[3] experiment not run yet")
+
+
+def _load():
+    t = json.load(open(TABLE))
+    rep = json.load(open(REPORT))
+    return t, rep
+
+
+def _costs(rows):
+    return [[math.inf if c is None else c for c in r["cost"]] for r in rows]
+
+
+def test_labels_are_exhaustive_argmin_and_constraints_infinite():
+    t, rep = _load()
+    for r in t["train"] + t["test"]:
+        for a, c in zip(r["allowed"], r["cost"]):
+            assert (not a) == (c is None or math.isinf(c))
+    lab = S.exhaustive_best(_costs(t["train"]))
+    counts = {k: 0 for k in ("csr_scalar", "csr_vector", "ell", "dia", "hyb")}
+    for l in lab:
+        counts[list(counts)[l]] += 1
+    assert counts == rep["train_label_counts"]
+
+
+def test_library_training_matches_oracle():
+    import paper_conf_ipps_muralidharanshgc14_b200 as nitro
+    t, rep = _load()
+    F = np.array([r["features"] for r in t["train"]])
+    lab = S.exhaustive_best(_costs(t["train"]))
+    m = S.train(F, lab)
+    assert (rep["model"]["C"], rep["model"]["gamma"]) == (m.C, m.gamma)
+    assert rep["model"]["cv_accuracy"] == pytest.approx(m.cv_accuracy, abs=1e-12)
+    # the committed model file selects like the oracle model on the held-out set
+    ctx = nitro.Context()
+    cv = nitro.CodeVariant(ctx, "spmv")
+    cv.register_spmv()
+    cv.load(MODEL)
+    sel_lib = [cv.predict(r["features"], r["allowed"]) for r in t["test"]]
+    sel_or = [S.select(m, r["features"], r["allowed"], default=1) for r in t["test"]]
+    agree = sum(a == b for a, b in zip(sel_lib, sel_or))
+    assert agree >= len(sel_lib) - 1, (sel_lib, sel_or)   # at most one near-boundary point may differ
+    names = ("csr_scalar", "csr_vector", "ell", "dia", "hyb")
+    assert [names[v] for v in sel_lib] == rep["selected"]
+
+
+def test_nitro_percent_recomputed():
+    t, rep = _load()
+    names = ("csr_scalar", "csr_vector", "ell", "dia", "hyb")
+    sel = [names.index(s) for s in rep["selected"]]
+    r = S.nitro_percent(_costs(t["test"]), sel)
+    assert r["mean"] == pytest.approx(rep["nitro_pct_mean"], abs=1e-12)
+    assert r["ge70"] == pytest.approx(rep["share_ge_70"]) and r["ge90"] == pytest.approx(rep["share_ge_90"])
