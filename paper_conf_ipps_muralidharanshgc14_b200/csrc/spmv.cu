@@ -231,28 +231,45 @@ __global__ void __launch_bounds__(256) k_csr_vector(const IT *__restrict__ rowpt
 
 // ------------------------------------------------------------------ K7 ELL (also HYB's ELL part)
 // Thread per 4 consecutive rows: per slot one 128-bit load of 4 column ids and
-// one 128-bit (fp32) / 2x128-bit (fp64) load of 4 values; 4 slots unrolled.
+// one 128-bit (fp32) / 2x128-bit (fp64) load of 4 values.  The loads of U
+// slots are all issued before the first FMA (explicit register batches: the
+// compiler otherwise reuses one register quad and serialises the slots), so
+// each thread keeps U x (16 + 16|32) bytes of HBM traffic in flight.
 template <typename VT>
 __global__ void __launch_bounds__(256) k_ell(const int32_t *__restrict__ ecol, const VT *__restrict__ eval,
                                              const VT *__restrict__ x, VT *__restrict__ y, int64_t N, int64_t K,
                                              int64_t ld) {
+  constexpr int U = sizeof(VT) == 4 ? 8 : 4;  // <= 16 terms per fp32 partial
   const int64_t nq = ld >> 2;
   for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nq; q += (int64_t)gridDim.x * blockDim.x) {
     const int64_t i0 = q << 2;
     double acc[4] = {0.0, 0.0, 0.0, 0.0};
-    for (int64_t k0 = 0; k0 < K; k0 += 16) {
-      const int64_t ke = k0 + 16 < K ? k0 + 16 : K;
-      VT part[4] = {0, 0, 0, 0};
-#pragma unroll 4
-      for (int64_t k = k0; k < ke; ++k) {
-        const int4 c = ld_stream_i4(reinterpret_cast<const int4 *>(ecol + k * ld + i0));
-        V4<VT> v;
-        v.load(eval + k * ld + i0);
-        part[0] = fma(v.v[0], c.x >= 0 ? __ldg(x + c.x) : (VT)0, part[0]);
-        part[1] = fma(v.v[1], c.y >= 0 ? __ldg(x + c.y) : (VT)0, part[1]);
-        part[2] = fma(v.v[2], c.z >= 0 ? __ldg(x + c.z) : (VT)0, part[2]);
-        part[3] = fma(v.v[3], c.w >= 0 ? __ldg(x + c.w) : (VT)0, part[3]);
+    for (int64_t k0 = 0; k0 < K; k0 += U) {
+      int4 c[U];
+      V4<VT> v[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (k0 + u < K) {
+          c[u] = ld_stream_i4(reinterpret_cast<const int4 *>(ecol + (k0 + u) * ld + i0));
+          v[u].load(eval + (k0 + u) * ld + i0);
+        } else {
+          c[u] = make_int4(-1, -1, -1, -1);
+          v[u].v[0] = v[u].v[1] = v[u].v[2] = v[u].v[3] = (VT)0;
+        }
       }
+      VT xv[U][4];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        xv[u][0] = c[u].x >= 0 ? __ldg(x + c[u].x) : (VT)0;
+        xv[u][1] = c[u].y >= 0 ? __ldg(x + c[u].y) : (VT)0;
+        xv[u][2] = c[u].z >= 0 ? __ldg(x + c[u].z) : (VT)0;
+        xv[u][3] = c[u].w >= 0 ? __ldg(x + c[u].w) : (VT)0;
+      }
+      VT part[4] = {0, 0, 0, 0};
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+#pragma unroll
+        for (int t = 0; t < 4; ++t) part[t] = fma(v[u].v[t], xv[u][t], part[t]);
 #pragma unroll
       for (int t = 0; t < 4; ++t) acc[t] += (double)part[t];
     }
@@ -277,30 +294,39 @@ __global__ void __launch_bounds__(256) k_dia(const int32_t *__restrict__ offs, c
     if (i0 >= ld) continue;
     const int64_t Bend = (B0 + 1024 < ld ? B0 + 1024 : ld) - 1;
     const bool interior = row0 + B0 + off_min >= 0 && row0 + Bend + off_max < M;
+    // U diagonals per batch: all value and x loads issued before the FMAs
+    constexpr int U = sizeof(VT) == 4 ? 8 : 4;
     double acc[4] = {0.0, 0.0, 0.0, 0.0};
-    for (int64_t d0 = 0; d0 < D; d0 += 16) {
-      const int64_t de = d0 + 16 < D ? d0 + 16 : D;
-      VT part[4] = {0, 0, 0, 0};
-      if (interior) {
-#pragma unroll 4
-        for (int64_t d = d0; d < de; ++d) {
-          V4<VT> v;
-          v.load(dval + d * ld + i0);
-          const VT *xp = x + (row0 + i0 + s_off[d]);
+    for (int64_t d0 = 0; d0 < D; d0 += U) {
+      V4<VT> v[U];
+      VT xv[U][4];
 #pragma unroll
-          for (int t = 0; t < 4; ++t) part[t] = fma(v.v[t], __ldg(xp + t), part[t]);
+      for (int u = 0; u < U; ++u) {
+        if (d0 + u < D) v[u].load(dval + (d0 + u) * ld + i0);
+        else v[u].v[0] = v[u].v[1] = v[u].v[2] = v[u].v[3] = (VT)0;
+      }
+      if (interior) {
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          const bool live = d0 + u < D;  // uniform
+          const VT *xp = x + (row0 + i0 + (live ? s_off[d0 + u] : 0));
+#pragma unroll
+          for (int t = 0; t < 4; ++t) xv[u][t] = live ? __ldg(xp + t) : (VT)0;
         }
       } else {
-#pragma unroll 2
-        for (int64_t d = d0; d < de; ++d) {
-          V4<VT> v;
-          v.load(dval + d * ld + i0);
-          const int64_t j = row0 + i0 + s_off[d];
 #pragma unroll
-          for (int t = 0; t < 4; ++t)
-            if (j + t >= 0 && j + t < M) part[t] = fma(v.v[t], __ldg(x + j + t), part[t]);
+        for (int u = 0; u < U; ++u) {
+          const bool live = d0 + u < D;
+          const int64_t j = row0 + i0 + (live ? s_off[d0 + u] : 0);
+#pragma unroll
+          for (int t = 0; t < 4; ++t) xv[u][t] = (live && j + t >= 0 && j + t < M) ? __ldg(x + j + t) : (VT)0;
         }
       }
+      VT part[4] = {0, 0, 0, 0};
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+#pragma unroll
+        for (int t = 0; t < 4; ++t) part[t] = fma(v[u].v[t], xv[u][t], part[t]);
 #pragma unroll
       for (int t = 0; t < 4; ++t) acc[t] += (double)part[t];
     }
