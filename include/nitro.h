@@ -232,6 +232,10 @@ nitro_status_t nitro_spmv_launches(nitro_spmv *A, int variant, int *out);
  *  9 diagonal offsets from the feature pass (int32 [ndiag], ascending).
  * needed receives the byte size; copies only if cap >= needed.  Syncs. */
 nitro_status_t nitro_spmv_export(nitro_spmv *A, int part, void *host_buf, size_t cap, size_t *needed);
+/* The caller changed the borrowed CSR contents in place: drop the cached
+ * features and every converted format (buffers are kept for reuse).  The
+ * next features/prepare/run recomputes them. */
+nitro_status_t nitro_spmv_invalidate(nitro_spmv *A);
 /* Free one variant's format (variant = -1: all). */
 nitro_status_t nitro_spmv_release(nitro_spmv *A, int variant);
 void nitro_spmv_destroy(nitro_spmv *A);
@@ -275,7 +279,9 @@ nitro_status_t nitro_dist_spmv_create(nitro_dist *D, int64_t global_rows, const 
 nitro_status_t nitro_dist_spmv_run(nitro_dist *D, nitro_spmv *A_local, int variant, const void *d_x_local,
                                    void *d_y_local);
 /* Same multiply from an x that is already gathered in the padded layout
- * (block q at q*B, B = max block rows, length nranks*B): no communication.
+ * (block q at q*B, B = max block rows, length nranks*B; padding entries must
+ * be finite, e.g. 0, because padded formats multiply zero slots by them):
+ * no communication.
  * Used when the caller owns the exchange (e.g. a solver that writes y straight
  * into the next x), and to check every rank's part on one GPU. */
 nitro_status_t nitro_dist_spmv_run_gathered(nitro_dist *D, nitro_spmv *A_local, int variant,

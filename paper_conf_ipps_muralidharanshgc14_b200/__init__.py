@@ -134,6 +134,7 @@ _SIGS = {
     "nitro_spmv_launches": ([_vp, _int, _P(_int)], _int),
     "nitro_spmv_export": ([_vp, _int, _vp, ctypes.c_size_t, _P(ctypes.c_size_t)], _int),
     "nitro_spmv_release": ([_vp, _int], _int),
+    "nitro_spmv_invalidate": ([_vp], _int),
     "nitro_spmv_destroy": ([_vp], None),
     "nitro_spmv_register": ([_vp], _int),
     # dist
@@ -287,6 +288,10 @@ class SpMV:
 
     def release(self, v: int = -1):
         _check(_L.nitro_spmv_release(self.h, v))
+
+    def invalidate(self):
+        """Matrix contents changed in place: recompute features/formats on next use."""
+        _check(_L.nitro_spmv_invalidate(self.h))
 
 
 # ====================================================================== generic Nitro layer

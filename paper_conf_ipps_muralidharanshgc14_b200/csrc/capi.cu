@@ -366,6 +366,15 @@ nitro_status_t nitro_spmv_export(nitro_spmv *A, int part, void *host_buf, size_t
   NITRO_GUARD_END
 }
 
+nitro_status_t nitro_spmv_invalidate(nitro_spmv *A) {
+  if (!A) return fail(NITRO_E_INVALID_ARG, "NULL handle");
+  DeviceGuard g(A->device);
+  NITRO_CUDA(cudaStreamSynchronize(A->stream));
+  A->feat_ready = A->feat_pending = false;
+  A->ell.ready = A->dia.ready = A->hyb.ready = A->csrv.ready = false;
+  return NITRO_OK;
+}
+
 nitro_status_t nitro_spmv_release(nitro_spmv *A, int variant) {
   if (!A) return fail(NITRO_E_INVALID_ARG, "NULL handle");
   DeviceGuard g(A->device);

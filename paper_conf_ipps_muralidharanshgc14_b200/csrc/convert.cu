@@ -309,7 +309,7 @@ nitro_status_t prepare_hyb(nitro_spmv *A) {
 
 // ------------------------------------------------------------------ CSR-vector (C8)
 // V = lanes per row from the mean row length; rows longer than 8V are split
-// into segments of kSeg entries handled by whole CTAs (see spmv.cu).
+// into segments of kCsrvSeg entries, each reduced by one warp (see spmv.cu).
 nitro_status_t prepare_csrv(nitro_spmv *A) {
   if (A->csrv.ready) return NITRO_OK;
   NITRO_TRY(features_finish(A));
@@ -318,7 +318,7 @@ nitro_status_t prepare_csrv(nitro_spmv *A) {
   const int64_t q = N > 0 ? A->Z / N : 0;
   int V = q <= 2 ? 2 : q <= 4 ? 4 : q <= 8 ? 8 : q <= 16 ? 16 : 32;
   A->csrv.V = V;
-  const int64_t T = 8LL * V, S = 4096;
+  const int64_t T = 8LL * V, S = kCsrvSeg;
   A->csrv.n_long = 0;
   if (A->feat.max_row > T) {
     DevBuf cnt;

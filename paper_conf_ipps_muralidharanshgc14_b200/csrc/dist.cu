@@ -254,6 +254,9 @@ nitro_status_t nitro_dist_spmv_create(nitro_dist *D, int64_t global_rows, const 
       st->part[k]->row0 = (int64_t)r * st->B + beg[k];  // rows in the remapped space keep diagonal offsets
     }
     if ((rc = st->xfull.alloc(std::max<int64_t>((int64_t)P * st->B, 1) * sv))) return bail(rc);
+    // padding rows of every block stay 0: padded formats (DIA) multiply their
+    // zero slots by x there, so it must be finite
+    NITRO_CUDA(cudaMemset(st->xfull.p, 0, st->xfull.bytes));
     NITRO_CUDA(cudaDeviceSynchronize());
     // the returned handle: the whole local block over remapped columns
     nitro_spmv *A = nullptr;

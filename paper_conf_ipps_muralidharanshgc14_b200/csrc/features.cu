@@ -103,14 +103,15 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
         // (per-block open-addressing set of offsets already in the bitmap:
         //  a stencil's few offsets stay resident, so its entries cost only lookups)
         bool want = idx >= 0;
-        unsigned h = 0;
+        int free_slot = -1;  // first empty slot of the probe run (insert target)
         if (want) {
-          h = (unsigned)(((unsigned long long)idx * 0x9E3779B97F4A7C15ull) >> 40);
+          const unsigned h = (unsigned)(((unsigned long long)idx * 0x9E3779B97F4A7C15ull) >> 40);
 #pragma unroll
           for (int p = 0; p < kProbe; ++p) {
-            const long long cur = s_seen[(h + p) & (kCache - 1)];
+            const int slot = (int)((h + p) & (kCache - 1));
+            const long long cur = s_seen[slot];
             if (cur == idx) { want = false; break; }
-            if (cur == -1) break;
+            if (cur == -1) { free_slot = slot; break; }
           }
         }
         const unsigned need = __ballot_sync(kFull, want);
@@ -121,13 +122,10 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
             // the hot words of random matrices (a stale 0 only costs a redundant OR)
             const unsigned bit = 1u << (idx & 31);
             if (!(__ldcg(bitmap + (idx >> 5)) & bit)) atomicOr(bitmap + (idx >> 5), bit);
-#pragma unroll
-            for (int p = 0; p < kProbe; ++p) {
-              const unsigned long long prev = atomicCAS(
-                  reinterpret_cast<unsigned long long *>(&s_seen[(h + p) & (kCache - 1)]), ~0ull,
-                  (unsigned long long)idx);
-              if (prev == ~0ull || prev == (unsigned long long)idx) break;
-            }
+            // remember it only if the probe run had room (a full run = a
+            // random-offset matrix: stop caching, keep the lookups cheap)
+            if (free_slot >= 0)
+              atomicCAS(reinterpret_cast<unsigned long long *>(&s_seen[free_slot]), ~0ull, (unsigned long long)idx);
           }
         }
         const int last_lane = E1 - 1 - w0 < 31 ? (int)(E1 - 1 - w0) : 31;

@@ -137,6 +137,7 @@ double compulsory_bytes(const nitro_spmv *A, int variant);
 nitro_status_t exclusive_scan_i64(const int64_t *in, int64_t *out, int64_t n, DevBuf &scratch, cudaStream_t s);
 
 inline int64_t round_up(int64_t n, int64_t m) { return (n + m - 1) / m * m; }
+constexpr int64_t kCsrvSeg = 256;  // CSR-vector long-row segment (one warp, 8 entries per lane)
 // bitmap index of diagonal offset d is d + G; the bitmap spans G + M bits
 inline int64_t diag_shift(const nitro_spmv *A) { return A->feat_G >= 0 ? A->feat_G : A->row0 + A->N - 1; }
 int num_sms();

@@ -95,11 +95,11 @@ __device__ __forceinline__ VT reduce_transpose(VT (&p)[R], int li, int &ridx) {
 // V lanes per row.  A warp takes 32 consecutive rows (one coalesced rowptr
 // load per lane); lane group g handles rows g, g+G, ... (G = 32/V) R at a
 // time so R independent (col, val) -> x chains are in flight per lane.
-// Rows longer than 8V are split into kSeg-entry segments, each reduced by a
-// whole CTA (first nseg blocks of the grid); the last CTA of a row sums the
-// row's segment partials in segment order (deterministic, no float atomics).
-constexpr int kSeg = 4096;
-
+// Rows longer than 8V are split into kCsrvSeg (= 256)-entry segments, each
+// reduced by one whole warp (8 entries per lane, all loads issued first); every
+// warp first works through the segment list (grid-stride), then through row
+// tiles.  A multi-segment row's partials are summed in segment order by the
+// last warp to finish one of its segments (deterministic, no float atomics).
 template <int V, typename IT, typename VT>
 __global__ void __launch_bounds__(256) k_csr_vector(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
                                                     const VT *__restrict__ val, const VT *__restrict__ x,
@@ -108,38 +108,47 @@ __global__ void __launch_bounds__(256) k_csr_vector(const IT *__restrict__ rowpt
                                                     const int32_t *__restrict__ seg_k, double *seg_part,
                                                     unsigned *seg_ctr) {
   constexpr int64_t T = 8 * V;
-  if ((int64_t)blockIdx.x < nseg) {
-    // ---- long-row segment: one CTA, <= 16 entries per thread
-    __shared__ double s_w[8];
-    __shared__ bool s_last;
-    const int64_t sg = blockIdx.x;
-    const int64_t row = seg_row[sg], k = seg_k[sg];
-    const int64_t a = (int64_t)rowptr[row], b = (int64_t)rowptr[row + 1];
-    const int64_t st = a + k * kSeg, en = st + kSeg < b ? st + kSeg : b;
-    VT part = 0;
-#pragma unroll 4
-    for (int64_t j = st + threadIdx.x; j < en; j += 256) part = fma(ld_stream(val + j), __ldg(x + ld_stream_i(col + j)), part);
+  {
+    constexpr int64_t S = kCsrvSeg;
+    const int lane = threadIdx.x & 31;
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t sg = gw; sg < nseg; sg += nw) {
+      const int64_t row = seg_row[sg], k = seg_k[sg];
+      const int64_t a = (int64_t)rowptr[row], b = (int64_t)rowptr[row + 1];
+      const int64_t st = a + k * S, en = st + S < b ? st + S : b;
+      int c[8];
+      VT v[8];
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) part += __shfl_xor_sync(kFull, part, o);
-    if ((threadIdx.x & 31) == 0) s_w[threadIdx.x >> 5] = (double)part;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      double t = 0.0;
-      for (int w = 0; w < 8; ++w) t += s_w[w];
-      seg_part[sg] = t;
-      __threadfence();
-      const int64_t first = sg - k, ns = (b - a + kSeg - 1) / kSeg;
-      const unsigned done = atomicAdd(seg_ctr + first, 1u);
-      s_last = done == (unsigned)(ns - 1);
-      if (s_last) {
-        __threadfence();
-        double tot = 0.0;
-        for (int64_t q = 0; q < ns; ++q) tot += *((volatile double *)(seg_part + first + q));
-        y[row] = (VT)tot;
-        seg_ctr[first] = 0;  // re-arm for the next multiply
+      for (int u = 0; u < 8; ++u) {
+        const int64_t e = st + u * 32 + lane;
+        c[u] = e < en ? ld_stream_i(col + e) : -1;
+        v[u] = e < en ? ld_stream(val + e) : (VT)0;
+      }
+      VT part = 0;
+#pragma unroll
+      for (int u = 0; u < 8; ++u) part = fma(v[u], c[u] >= 0 ? __ldg(x + c[u]) : (VT)0, part);
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) part += __shfl_xor_sync(kFull, part, o);
+      const int64_t ns = (b - a + S - 1) / S;
+      if (lane == 0) {
+        if (ns == 1) {
+          y[row] = part;
+        } else {
+          seg_part[sg] = (double)part;
+          __threadfence();
+          const int64_t first = sg - k;
+          const unsigned done = atomicAdd(seg_ctr + first, 1u);
+          if (done == (unsigned)(ns - 1)) {
+            __threadfence();
+            double tot = 0.0;
+            for (int64_t q = 0; q < ns; ++q) tot += *((volatile double *)(seg_part + first + q));
+            y[row] = (VT)tot;
+            seg_ctr[first] = 0;  // re-arm for the next multiply
+          }
+        }
       }
     }
-    return;
   }
   // Software-pipelined main path.  A "stage" is R rows of one lane group:
   // row starts/lengths come from the tile's rowptr registers by shuffle, and
@@ -149,8 +158,8 @@ __global__ void __launch_bounds__(256) k_csr_vector(const IT *__restrict__ rowpt
   constexpr int G = 32 / V;
   constexpr int R = V >= 4 ? 4 : 2;
   const int lane = threadIdx.x & 31, g = lane / V, li = lane % V;
-  const int64_t warp = (((int64_t)blockIdx.x - nseg) * blockDim.x + threadIdx.x) >> 5;
-  const int64_t stride = ((((int64_t)gridDim.x - nseg) * blockDim.x) >> 5) * 32;
+  const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t stride = (((int64_t)gridDim.x * blockDim.x) >> 5) * 32;
   int64_t t0 = warp * 32;
   if (t0 >= N) return;
   struct Tile { int64_t abase; int rel, len; };
@@ -280,7 +289,10 @@ __global__ void __launch_bounds__(256) k_ell(const int32_t *__restrict__ ecol, c
 // ------------------------------------------------------------------ K8 DIA
 // Thread per 4 consecutive rows, block = 1024 rows; offsets in shared memory.
 // Blocks whose rows see every diagonal in range skip all bounds checks.
-template <typename VT>
+// U diagonals per batch (all value and x loads of a batch issued before the
+// FMAs): larger U = more bytes in flight per thread but more registers, i.e.
+// fewer resident warps; chosen per launch (dia_batch()).
+template <typename VT, int U>
 __global__ void __launch_bounds__(256) k_dia(const int32_t *__restrict__ offs, const VT *__restrict__ dval,
                                              const VT *__restrict__ x, VT *__restrict__ y, int64_t N, int64_t M,
                                              int64_t D, int64_t ld, int64_t row0, int64_t off_min, int64_t off_max) {
@@ -294,8 +306,6 @@ __global__ void __launch_bounds__(256) k_dia(const int32_t *__restrict__ offs, c
     if (i0 >= ld) continue;
     const int64_t Bend = (B0 + 1024 < ld ? B0 + 1024 : ld) - 1;
     const bool interior = row0 + B0 + off_min >= 0 && row0 + Bend + off_max < M;
-    // U diagonals per batch: all value and x loads issued before the FMAs
-    constexpr int U = sizeof(VT) == 4 ? 8 : 4;
     double acc[4] = {0.0, 0.0, 0.0, 0.0};
     for (int64_t d0 = 0; d0 < D; d0 += U) {
       V4<VT> v[U];
@@ -438,6 +448,18 @@ __global__ void __launch_bounds__(256) k_flush(const int4 *__restrict__ buf, int
   if (acc == 0x7fffffff) *sink = acc;
 }
 
+// DIA batch width: NITRO_DIA_U overrides (tuning); default 2 (fp32) / 1 (fp64)
+// keeps registers low enough for full occupancy on bandwidth-bound stencils.
+int dia_batch(int64_t D, size_t sv) {
+  static int env = [] {
+    const char *e = getenv("NITRO_DIA_U");
+    return e ? atoi(e) : 0;
+  }();
+  if (env == 1 || env == 2 || env == 4 || env == 8) return env;
+  (void)D;
+  return sv == 4 ? 2 : 1;
+}
+
 unsigned grid_cap(int64_t blocks, int per_sm = 8) {
   int64_t cap = (int64_t)num_sms() * per_sm;
   if (blocks > cap) blocks = cap;
@@ -460,8 +482,8 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
       int32_t *seg_k = seg_row + nseg;
       double *seg_part = reinterpret_cast<double *>(reinterpret_cast<char *>(A->csrv.long_rows.p) + nseg * 8);
       unsigned *seg_ctr = reinterpret_cast<unsigned *>(reinterpret_cast<char *>(A->csrv.long_rows.p) + nseg * 16);
-      const int64_t main_blocks = grid_cap((N + 255) / 256, 8);  // 8 warps x 32 rows per block-iteration
-      const unsigned g = (unsigned)(nseg + main_blocks);
+      // 8 warps x 32 rows per block-iteration; segments are spread over all warps
+      const unsigned g = grid_cap(std::max<int64_t>((N + 255) / 256, (nseg + 7) / 8), 8);
 #define NITRO_CSRV(VV)                                                                                      \
   k_csr_vector<VV, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, nseg, seg_row, seg_k, seg_part, seg_ctr)
       switch (A->csrv.V) {
@@ -482,9 +504,17 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
     case NITRO_DIA:
       if (N > 0) {
         const size_t sm = (size_t)std::max<int64_t>(A->dia.D, 1) * 4;
-        k_dia<VT><<<grid_cap((A->dia.ld + 1023) / 1024, 16), 256, sm, s>>>(
-            A->dia.off.as<int32_t>(), A->dia.val.as<VT>(), x, y, N, A->M, A->dia.D, A->dia.ld, A->row0,
-            A->dia.off_min, A->dia.off_max);
+        const unsigned g = grid_cap((A->dia.ld + 1023) / 1024, 16);
+#define NITRO_DIA_LAUNCH(UU)                                                                                  \
+  k_dia<VT, UU><<<g, 256, sm, s>>>(A->dia.off.as<int32_t>(), A->dia.val.as<VT>(), x, y, N, A->M, A->dia.D,    \
+                                   A->dia.ld, A->row0, A->dia.off_min, A->dia.off_max)
+        switch (dia_batch(A->dia.D, sizeof(VT))) {
+          case 1: NITRO_DIA_LAUNCH(1); break;
+          case 2: NITRO_DIA_LAUNCH(2); break;
+          case 4: NITRO_DIA_LAUNCH(4); break;
+          default: NITRO_DIA_LAUNCH(8); break;
+        }
+#undef NITRO_DIA_LAUNCH
       }
       break;
     case NITRO_HYB:
