@@ -292,7 +292,8 @@ nitro_status_t prepare_hyb(nitro_spmv *A) {
   NITRO_TRY(A->hyb.trow.alloc((size_t)std::max<int64_t>(Zt, 1) * 4));
   NITRO_TRY(A->hyb.tcol.alloc((size_t)std::max<int64_t>(Zt, 1) * 4));
   NITRO_TRY(A->hyb.tval.alloc((size_t)std::max<int64_t>(Zt, 1) * sv));
-  const int64_t nch = (Zt + 255) / 256;
+  const int64_t chunk = 32 * hyb_windows((size_t)sv);
+  const int64_t nch = (Zt + chunk - 1) / chunk;
   NITRO_TRY(A->hyb.carry_row.alloc((size_t)std::max<int64_t>(2 * nch, 1) * 4));
   NITRO_TRY(A->hyb.carry_val.alloc((size_t)std::max<int64_t>(2 * nch, 1) * 8));
   if (N > 0)

@@ -26,22 +26,34 @@ namespace {
 
 constexpr int kThreads = 256;
 constexpr int kWarps = kThreads / 32;
-constexpr int kCache = 1024;  // per-block offset set slots (8 KB)
-constexpr int kProbe = 4;     // linear-probe length
+constexpr int kCache = 1024;            // per-block open-addressing offset set (u32 keys, 4 KB)
+constexpr int kProbe = 4;               // linear-probe length
+constexpr uint32_t kWin = 1u << 17;     // per-block bitmap of offsets in [-2^16, 2^16) (16 KB)
+constexpr uint32_t kEmpty = 0xffffffffu;
 
+// Offset index idx = col - row + G is < 2^32 (rows, cols < 2^31), so all
+// per-entry arithmetic is 32-bit.  Near-diagonal offsets (stencils, banded)
+// are recorded in a shared-memory bitmap window (LDS + rare shared atomic per
+// entry); the rest go through a small shared-memory set of offsets already in
+// the global bitmap and a test-before-set global OR.  Blocks whose set fills
+// up (random matrices) stop probing it.
 template <typename IT>
 __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
                                                         int64_t N, int64_t M, int64_t Z, int64_t row0, int64_t G,
                                                         FeatAcc *__restrict__ acc, uint32_t *__restrict__ bitmap) {
   __shared__ int8_t s_slot[kWarps][32];
-  __shared__ long long s_seen[kCache];
+  __shared__ uint32_t s_seen[kCache];
+  __shared__ uint32_t s_win[kWin / 32];
   __shared__ unsigned long long s_red[3][kWarps];
-  __shared__ unsigned s_bad;
-  for (int i = threadIdx.x; i < kCache; i += kThreads) s_seen[i] = -1;
-  if (threadIdx.x == 0) s_bad = 0;
+  __shared__ unsigned s_bad, s_full;
+  for (int i = threadIdx.x; i < kCache; i += kThreads) s_seen[i] = kEmpty;
+  for (int i = threadIdx.x; i < (int)(kWin / 32); i += kThreads) s_win[i] = 0u;
+  if (threadIdx.x == 0) { s_bad = 0; s_full = 0; }
   __syncthreads();
 
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const uint32_t G32 = (uint32_t)G, M32 = (uint32_t)M;
+  const uint32_t win_lo = G32 - (kWin >> 1);  // idx of offset -2^16 (may wrap: rel test below is modular)
   unsigned bad = 0;
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     if ((int64_t)rowptr[0] != 0 || (int64_t)rowptr[N] != Z) bad |= 1;
@@ -55,82 +67,81 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
     if (r < N) { a = (int64_t)rowptr[r]; b = (int64_t)rowptr[r + 1]; }
     else { a = b = (int64_t)rowptr[N]; }
     const int64_t L = b - a;
-    if (L < 0) bad |= 1;
     if (L > 0) {
       s1 += (unsigned long long)L;
       s2 += (unsigned long long)L * (unsigned long long)L;
       if ((unsigned long long)L > lmax) lmax = (unsigned long long)L;
     }
-    // a block of rows with a broken rowptr is not walked (already flagged)
-    if (__any_sync(kFull, L < 0 || a < 0 || b > Z)) { bad |= (L < 0 || a < 0 || b > Z) ? 1u : 0u; continue; }
+    // a block of rows with a broken rowptr is not walked (flagged)
+    const bool brk = L < 0 || a < 0 || b > Z;
+    if (__any_sync(kFull, brk)) { bad |= brk ? 1u : 0u; continue; }
     const int64_t E0 = __shfl_sync(kFull, a, 0), E1 = __shfl_sync(kFull, b, 31);
-    int cur_rl = 0;
-    int last_c = 0;
-    const int64_t grow0 = row0 + rb * 32;  // global row of lane 0's row
+    const uint32_t rowbase = (uint32_t)(row0 + rb * 32);  // global row of lane 0's row
+    const bool lane_has = L > 0;
+    int cur_rl = 0, last_c = 0;
     for (int64_t base = E0; base < E1; base += 128) {
       int c[4];
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
-        int64_t e = base + u * 32 + lane;
+        const int64_t e = base + u * 32 + lane;
         c[u] = e < E1 ? ld_stream_i(col + e) : 0;
       }
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
         const int64_t w0 = base + u * 32;
         if (w0 >= E1) break;  // warp-uniform
+        const int nvalid = E1 - w0 < 32 ? (int)(E1 - w0) : 32;
+        // rows whose first entry falls in this window: head bit at their start
         const int64_t pos = a - w0;
-        const bool head = L > 0 && pos >= 0 && pos < 32;
+        const bool head = lane_has && pos >= 0 && pos < 32;
         const unsigned mask = __reduce_or_sync(kFull, head ? (1u << (unsigned)pos) : 0u);
         if (head) s_slot[wib][pos] = (int8_t)lane;
         __syncwarp();
-        const int64_t e = w0 + lane;
-        const bool valid = e < E1;
-        const unsigned upto = lane == 31 ? kFull : ((2u << lane) - 1u);
-        const unsigned hm = mask & upto;
+        const unsigned hm = mask & (kFull >> (31 - lane));
         const int rl = hm ? (int)s_slot[wib][31 - __clz(hm)] : cur_rl;
         int prevc = __shfl_up_sync(kFull, c[u], 1);
         if (lane == 0) prevc = last_c;
-        const bool is_head = (mask >> lane) & 1u;
-        long long idx = -1;
-        if (valid) {
-          if (c[u] < 0 || (int64_t)c[u] >= M) bad |= 4;
+        uint32_t idx = kEmpty;
+        if (lane < nvalid) {
+          if ((uint32_t)c[u] >= M32) bad |= 4;  // also catches c < 0
           else {
-            if (!is_head && c[u] <= prevc) bad |= 2;
-            idx = (long long)c[u] - (long long)(grow0 + rl) + (long long)G;
+            if (!((mask >> lane) & 1u) && c[u] <= prevc) bad |= 2;
+            idx = (uint32_t)c[u] - (rowbase + (uint32_t)rl) + G32;
           }
         }
-        // occupied-diagonal bitmap with dedupe
-        // (per-block open-addressing set of offsets already in the bitmap:
-        //  a stencil's few offsets stay resident, so its entries cost only lookups)
-        bool want = idx >= 0;
-        int free_slot = -1;  // first empty slot of the probe run (insert target)
+        bool want = idx != kEmpty;
         if (want) {
-          const unsigned h = (unsigned)(((unsigned long long)idx * 0x9E3779B97F4A7C15ull) >> 40);
+          const uint32_t rel = idx - win_lo;
+          if (rel < kWin) {
+            const uint32_t bit = 1u << (rel & 31);
+            if (!(s_win[rel >> 5] & bit)) atomicOr(&s_win[rel >> 5], bit);
+            want = false;
+          }
+        }
+        int free_slot = -1;
+        if (want && !s_full) {
+          const uint32_t h = idx * 0x9E3779B1u >> 22;  // 10-bit hash
 #pragma unroll
           for (int p = 0; p < kProbe; ++p) {
             const int slot = (int)((h + p) & (kCache - 1));
-            const long long cur = s_seen[slot];
+            const uint32_t cur = s_seen[slot];
             if (cur == idx) { want = false; break; }
-            if (cur == -1) { free_slot = slot; break; }
+            if (cur == kEmpty) { free_slot = slot; break; }
           }
         }
         const unsigned need = __ballot_sync(kFull, want);
         if (want) {
           const unsigned grp = __match_any_sync(need, idx);
           if ((int)(__ffs(grp) - 1) == lane) {
-            // test before set: an L2 read is far cheaper than a contended RED on
-            // the hot words of random matrices (a stale 0 only costs a redundant OR)
-            const unsigned bit = 1u << (idx & 31);
+            // test before set: an L2 read is far cheaper than a contended RED
+            const uint32_t bit = 1u << (idx & 31);
             if (!(__ldcg(bitmap + (idx >> 5)) & bit)) atomicOr(bitmap + (idx >> 5), bit);
-            // remember it only if the probe run had room (a full run = a
-            // random-offset matrix: stop caching, keep the lookups cheap)
-            if (free_slot >= 0)
-              atomicCAS(reinterpret_cast<unsigned long long *>(&s_seen[free_slot]), ~0ull, (unsigned long long)idx);
+            if (free_slot >= 0) atomicCAS(&s_seen[free_slot], kEmpty, idx);
+            else if (!s_full) s_full = 1;  // probe run full: stop using the set
           }
         }
-        const int last_lane = E1 - 1 - w0 < 31 ? (int)(E1 - 1 - w0) : 31;
-        cur_rl = __shfl_sync(kFull, rl, last_lane);
-        last_c = __shfl_sync(kFull, c[u], last_lane);
+        cur_rl = __shfl_sync(kFull, rl, nvalid - 1);
+        last_c = __shfl_sync(kFull, c[u], nvalid - 1);
         __syncwarp();
       }
     }
@@ -149,6 +160,17 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
     if (bad) atomicOr(&s_bad, bad);
   }
   __syncthreads();
+  // merge the near-diagonal window into the global bitmap (nonzero words only)
+  const int64_t span = G + M;
+  for (int i = threadIdx.x; i < (int)(kWin / 32); i += kThreads) {
+    uint32_t w = s_win[i];
+    while (w) {
+      const int bpos = __ffs(w) - 1;
+      w &= w - 1;
+      const uint32_t gidx = win_lo + (uint32_t)(i * 32 + bpos);
+      if ((int64_t)gidx < span) atomicOr(bitmap + (gidx >> 5), 1u << (gidx & 31));
+    }
+  }
   if (threadIdx.x == 0) {
     unsigned long long a1 = 0, a2 = 0, am = 0;
     for (int w = 0; w < kWarps; ++w) {

@@ -138,6 +138,8 @@ nitro_status_t exclusive_scan_i64(const int64_t *in, int64_t *out, int64_t n, De
 
 inline int64_t round_up(int64_t n, int64_t m) { return (n + m - 1) / m * m; }
 constexpr int64_t kCsrvSeg = 256;  // CSR-vector long-row segment (one warp, 8 entries per lane)
+// HYB tail chunk = 32 * hyb_windows entries per warp (fewer for fp64: registers)
+constexpr int hyb_windows(size_t sv) { return sv == 8 ? 4 : 8; }
 // bitmap index of diagonal offset d is d + G; the bitmap spans G + M bits
 inline int64_t diag_shift(const nitro_spmv *A) { return A->feat_G >= 0 ? A->feat_G : A->row0 + A->N - 1; }
 int num_sms();

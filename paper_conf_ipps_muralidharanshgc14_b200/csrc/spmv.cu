@@ -345,45 +345,67 @@ __global__ void __launch_bounds__(256) k_dia(const int32_t *__restrict__ offs, c
 }
 
 // ------------------------------------------------------------------ K9b HYB COO tail
-// Warp per chunk of 256 row-sorted tail entries: 8 coalesced windows loaded up
+// Warp per chunk of 32*W row-sorted tail entries: W coalesced windows loaded up
 // front, then a segmented inclusive scan per window (rows sorted => equal row
 // ids are contiguous).  Rows wholly inside the chunk are added to y directly
 // (single owner); the chunk's first and last rows go to two carry slots that
 // k_hyb_fixup applies in chunk order.  No atomics; deterministic.
-template <typename VT>
+template <typename VT, int W>
 __global__ void __launch_bounds__(256) k_hyb_tail(const int32_t *__restrict__ trow, const int32_t *__restrict__ tcol,
                                                   const VT *__restrict__ tval, const VT *__restrict__ x,
                                                   VT *__restrict__ y, int64_t Zt, int64_t nch,
                                                   int32_t *__restrict__ carry_row, double *__restrict__ carry_val) {
+  constexpr int64_t CH = 32 * W;  // chunk = W windows of 32 entries
   const int lane = threadIdx.x & 31;
   const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  for (int64_t ch = warp; ch < nch; ch += nw) {
-    const int64_t c0 = ch * 256, cend = c0 + 256 < Zt ? c0 + 256 : Zt;
-    const int first_row = __ldg(trow + c0), last_row = __ldg(trow + cend - 1);
-    int rr[8], cc[8];
-    VT vv[8];
+  // software pipeline over the warp's chunks: the next chunk's (row, col, val)
+  // loads are issued right after the current chunk's x gathers, so they are in
+  // flight while the current chunk's segmented scans run
+  int rr[W], cc[W];
+  VT vv[W];
+  auto load_chunk = [&](int64_t c0, int64_t cend) {
 #pragma unroll
-    for (int w = 0; w < 8; ++w) {
+    for (int w = 0; w < W; ++w) {
       const int64_t e = c0 + w * 32 + lane;
       const bool ok = e < cend;
       rr[w] = ok ? ld_stream_i(trow + e) : -2;
       cc[w] = ok ? ld_stream_i(tcol + e) : 0;
       vv[w] = ok ? ld_stream(tval + e) : (VT)0;
     }
-    double p[8];
+  };
+  if (warp < nch) load_chunk(warp * CH, warp * CH + CH < Zt ? warp * CH + CH : Zt);
+  for (int64_t ch = warp; ch < nch; ch += nw) {
+    const int64_t c0 = ch * CH, cend = c0 + CH < Zt ? c0 + CH : Zt;
+    const int first_row = __shfl_sync(kFull, rr[0], 0);
+    const int wl = (int)((cend - 1 - c0) >> 5), ll = (int)((cend - 1 - c0) & 31);
+    int last_row = 0;
 #pragma unroll
-    for (int w = 0; w < 8; ++w) p[w] = (double)vv[w] * (double)__ldg(x + cc[w]);
+    for (int w = 0; w < W; ++w) {
+      const int t = __shfl_sync(kFull, rr[w], ll);
+      if (w == wl) last_row = t;
+    }
+    double p[W];
+    int rcur[W];
+#pragma unroll
+    for (int w = 0; w < W; ++w) {
+      p[w] = (double)vv[w] * (double)__ldg(x + cc[w]);
+      rcur[w] = rr[w];
+    }
+    {
+      const int64_t n0 = ch + nw;
+      if (n0 < nch) load_chunk(n0 * CH, n0 * CH + CH < Zt ? n0 * CH + CH : Zt);
+    }
     if (lane == 0) { carry_row[2 * ch] = -1; carry_row[2 * ch + 1] = -1; }
     __syncwarp();
     int carry_r = -3;
     double carry_v = 0.0;
 #pragma unroll
-    for (int w = 0; w < 8; ++w) {
+    for (int w = 0; w < W; ++w) {
       const int64_t w0 = c0 + w * 32;
       if (w0 >= cend) break;
       double q = p[w];
-      const int r = rr[w];
+      const int r = rcur[w];
       // a segment left open at the previous window's last lane ended exactly
       // at the window boundary if this window starts a new row: emit it now
       const int r_first = __shfl_sync(kFull, r, 0);
@@ -448,8 +470,9 @@ __global__ void __launch_bounds__(256) k_flush(const int4 *__restrict__ buf, int
   if (acc == 0x7fffffff) *sink = acc;
 }
 
-// DIA batch width: NITRO_DIA_U overrides (tuning); default 2 (fp32) / 1 (fp64)
-// keeps registers low enough for full occupancy on bandwidth-bound stencils.
+// DIA batch width: NITRO_DIA_U overrides (tuning); default 4 (fp32) / 2 (fp64)
+// (B200 sweep on configs[1]: U=1 4925, 2 5112, 4 5139, 8 4544 GB/s — U=8's
+// 124 registers cost more occupancy than its extra bytes in flight buy).
 int dia_batch(int64_t D, size_t sv) {
   static int env = [] {
     const char *e = getenv("NITRO_DIA_U");
@@ -457,7 +480,7 @@ int dia_batch(int64_t D, size_t sv) {
   }();
   if (env == 1 || env == 2 || env == 4 || env == 8) return env;
   (void)D;
-  return sv == 4 ? 2 : 1;
+  return sv == 4 ? 4 : 2;
 }
 
 unsigned grid_cap(int64_t blocks, int per_sm = 8) {
@@ -522,7 +545,7 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
         k_ell<VT><<<grid_cap((A->hyb.ld / 4 + 255) / 256, 16), 256, 0, s>>>(A->hyb.col.as<int32_t>(), A->hyb.val.as<VT>(),
                                                                         x, y, N, A->hyb.K, A->hyb.ld);
         if (A->hyb.Zt > 0) {
-          k_hyb_tail<VT><<<grid_cap((A->hyb.nchunks + 7) / 8, 16), 256, 0, s>>>(
+          k_hyb_tail<VT, hyb_windows(sizeof(VT))><<<grid_cap((A->hyb.nchunks + 7) / 8, 16), 256, 0, s>>>(
               A->hyb.trow.as<int32_t>(), A->hyb.tcol.as<int32_t>(), A->hyb.tval.as<VT>(), x, y, A->hyb.Zt,
               A->hyb.nchunks, A->hyb.carry_row.as<int32_t>(), A->hyb.carry_val.as<double>());
           k_hyb_fixup<VT><<<grid_cap((A->hyb.nchunks + 255) / 256, 16), 256, 0, s>>>(
