@@ -168,11 +168,12 @@ def run_nitro(args):
     x_local = synth.vector(N, seed=2, device=dev, j0=row0)
     y = torch.empty(N, dtype=torch.float32, device=dev)
 
-    if world == 1:
+    use_dist = world > 1 or args.dist   # --dist: the multi-GPU code path even at N = 1
+    if not use_dist:
         M = nitro.SpMV(A.rowptr, A.colidx, A.vals, N, A.cols)
         x = x_local
     else:
-        D = _dist_setup(nitro, dist, rank, world, local)
+        D = _dist_setup(nitro, dist if world > 1 else None, rank, world, local)
         bounds = np.array([r * n * n * n for r in range(world + 1)], dtype=np.int64)
         M = D.spmv(A.cols, bounds, A.rowptr, A.colidx, A.vals)
         x = x_local
@@ -180,10 +181,10 @@ def run_nitro(args):
     # --- one end-to-end pass of the hot path (features -> select -> prepare -> run)
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     t0 = time.perf_counter()
-    feats = M.features() if world == 1 else D.features(M)   # first call: allocates its buffers
+    feats = M.features() if not use_dist else D.features(M)   # first call: allocates its buffers
     feature_first_ms = (time.perf_counter() - t0) * 1e3
     feature_ms = None
-    if world == 1:                                          # warm feature pass (+ host finishing)
+    if not use_dist:                                        # warm feature pass (+ host finishing)
         M.invalidate()
         ev0.record(stream)
         feats = M.features()
@@ -191,7 +192,7 @@ def run_nitro(args):
         torch.cuda.synchronize()
         feature_ms = ev0.elapsed_time(ev1)
     fvec = [feats[k] for k in nitro.FEATURE_NAMES]
-    allowed = M.allowed_mask() if world == 1 else [True] * 5
+    allowed = M.allowed_mask() if not use_dist else [True] * 5   # dist parts check their own constraints
     ctx = nitro.Context()
     cv = nitro.CodeVariant(ctx, "spmv")
     cv.register_spmv()
@@ -206,7 +207,7 @@ def run_nitro(args):
 
     # exhaustive reference: every allowed variant timed the same way (median of R, L2 flushed)
     exhaustive = {}
-    if world == 1:
+    if not use_dist:
         for v in range(5):
             if allowed[v]:
                 med, _ = M.time(v, x, y, warmup=3, reps=20, flush_l2=True)
@@ -221,7 +222,7 @@ def run_nitro(args):
         if sel is None:
             sel = nitro.DIA
     vname = nitro.VARIANT_NAMES[sel]
-    if world == 1:
+    if not use_dist:
         M.prepare(sel)
         nbytes = M.format_info(sel)["compulsory_bytes"]
         launches = M.launches(sel)
@@ -230,7 +231,7 @@ def run_nitro(args):
         launches = 1
 
     def step():
-        if world == 1:
+        if not use_dist:
             M.run(sel, x, y)
         else:
             D.run(M, sel, x, y)
@@ -264,8 +265,31 @@ def run_nitro(args):
 
     # --- e2e through the C ABI with host buffers (pinned), copies inside the timed region
     e2e = None
-    if world == 1:
-        hx = torch.empty(N, dtype=torch.float32).pin_memory()
+    hx = torch.empty(N, dtype=torch.float32).pin_memory()
+    hx.copy_(x.cpu())
+    hy = torch.empty(N, dtype=torch.float32).pin_memory()
+    if use_dist:   # no host-buffer entry in the dist API: pinned copies around nitro_dist_spmv_run
+        xs = torch.empty_like(x)
+        et = []
+        for i in range(args.steps + 3):
+            M.flush_l2()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            xs.copy_(hx, non_blocking=True)
+            D.run(M, sel, xs, y)
+            hy.copy_(y, non_blocking=True)
+            b.record(stream)
+            b.synchronize()
+            if i >= 3:
+                et.append(a.elapsed_time(b))
+        e2e_ms = sum(et) / len(et)
+        if world > 1:
+            t = torch.tensor([e2e_ms], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            e2e_ms = float(t.item())
+        e2e = {"value": nbytes * world / (e2e_ms * 1e-3) / 1e9, "unit": "GB/s", "ms_per_step": e2e_ms,
+               "h2d_bytes_per_step": N * 4 * world, "d2h_bytes_per_step": N * 4 * world}
+    else:
         hx.copy_(x.cpu())
         hy = torch.empty(N, dtype=torch.float32).pin_memory()
         hxn, hyn = hx.numpy(), hy.numpy()
@@ -306,7 +330,7 @@ def run_nitro(args):
         "data": "synthetic",
         "config": {"workload": WORKLOAD if world == 1 else f"3d27pt_stencil_128x128x{128 * world}_fp32 (128^3 rows/rank)",
                    "rows_per_gpu": N, "nnz_per_gpu": Z, "l2": "flushed between steps (read of 3x L2)",
-                   "parallelism": "single GPU" if world == 1 else f"row-partitioned x{world}, NCCL x all-gather",
+                   "parallelism": "single GPU" if not use_dist else f"row-partitioned x{world}, NCCL x all-gather",
                    "selection": selection, "selected_variant": vname},
         "selected_variant": vname,
         "gflops": 2.0 * Z * world / (ms * 1e-3) / 1e9,
@@ -338,9 +362,11 @@ def D_bytes(M, nitro, v):
 def _dist_setup(nitro, dist, rank, world, local):
     import torch
     uid = nitro.dist_unique_id() if rank == 0 else bytes(128)
-    t = torch.tensor(list(uid), dtype=torch.uint8, device="cuda")
-    dist.broadcast(t, 0)
-    return nitro.Dist(bytes(t.cpu().tolist()), rank, world, local)
+    if dist is not None:
+        t = torch.tensor(list(uid), dtype=torch.uint8, device="cuda")
+        dist.broadcast(t, 0)
+        uid = bytes(t.cpu().tolist())
+    return nitro.Dist(uid, rank, world, local)
 
 
 def main():
@@ -350,6 +376,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="nitro", choices=["nitro", "reference"])
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--dist", action="store_true", help="use the multi-GPU (NCCL) code path even at N=1")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     if args.impl == "reference":

@@ -33,6 +33,8 @@ if want prof; then
     ncu -i /tmp/prof_$cfg.ncu-rep --page details --csv > gpurun_out/prof_${cfg}_details.csv 2>/dev/null
     ncu -i /tmp/prof_$cfg.ncu-rep --page source --csv -k regex:k_dia > gpurun_out/prof_${cfg}_src_dia.csv 2>/dev/null
     ncu -i /tmp/prof_$cfg.ncu-rep --page source --csv -k regex:k_csr_vector > gpurun_out/prof_${cfg}_src_csrv.csv 2>/dev/null
+    ncu -i /tmp/prof_$cfg.ncu-rep --page source --csv -k regex:k_features > gpurun_out/prof_${cfg}_src_feat.csv 2>/dev/null
+    ncu -i /tmp/prof_$cfg.ncu-rep --page source --csv -k regex:k_hyb_tail > gpurun_out/prof_${cfg}_src_tail.csv 2>/dev/null
     ls -la /tmp/prof_$cfg.ncu-rep gpurun_out/prof_${cfg}_*
   done
   du -sh gpurun_out
