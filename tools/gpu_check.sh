@@ -1,11 +1,11 @@
 # GPU-box check: parity tests, smoke, bench, variant table, ncu launch list +
 # full captures (exported to CSV on the box; the .ncu-rep files are too big
-# to bring back).  usage: bash tools/gpu_check.sh [tests|bench|prof]...  (default: all)
+# to bring back).  usage: bash tools/gpu_check.sh [tests|bench|table|prof]...  (default: all)
 set -x
 mkdir -p gpurun_out
-want() { [ $# -eq 0 ] && return 0; for a in $ALL; do [ "$a" = "$1" ] && return 0; done; return 1; }
 ALL="$*"
 [ -z "$ALL" ] && ALL="tests bench table prof"
+want() { for a in $ALL; do [ "$a" = "$1" ] && return 0; done; return 1; }
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,memory.total --format=csv
 if want tests; then
   timeout 1500 python -m pytest tests -m gpu -q -rf --durations=10 > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?"
@@ -30,12 +30,14 @@ if want prof; then
         -o /tmp/prof_$cfg -f python tools/profile_variants.py $cfg > gpurun_out/prof_$cfg.log 2>&1
     echo "ncu full $cfg rc=$?"
     ncu -i /tmp/prof_$cfg.ncu-rep --page raw --csv > gpurun_out/prof_${cfg}_raw.csv 2>/dev/null
-    ncu -i /tmp/prof_$cfg.ncu-rep --page details --csv > gpurun_out/prof_${cfg}_details.csv 2>/dev/null
-    ncu -i /tmp/prof_$cfg.ncu-rep --page source --csv -k regex:k_dia > gpurun_out/prof_${cfg}_src_dia.csv 2>/dev/null
-    ncu -i /tmp/prof_$cfg.ncu-rep --page source --csv -k regex:k_csr_vector > gpurun_out/prof_${cfg}_src_csrv.csv 2>/dev/null
-    ncu -i /tmp/prof_$cfg.ncu-rep --page source --csv -k regex:k_features > gpurun_out/prof_${cfg}_src_feat.csv 2>/dev/null
-    ncu -i /tmp/prof_$cfg.ncu-rep --page source --csv -k regex:k_hyb_tail > gpurun_out/prof_${cfg}_src_tail.csv 2>/dev/null
-    ls -la /tmp/prof_$cfg.ncu-rep gpurun_out/prof_${cfg}_*
+    case $cfg in
+      c1)  srcs="dia csr_vector features ell" ;;
+      c2b) srcs="hyb_tail csr_vector" ;;
+      *)   srcs="" ;;
+    esac
+    for k in $srcs; do
+      ncu -i /tmp/prof_$cfg.ncu-rep --page source --csv -k regex:k_$k -c 1 > gpurun_out/prof_${cfg}_src_$k.csv 2>/dev/null
+    done
   done
   du -sh gpurun_out
 fi
