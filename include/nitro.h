@@ -115,6 +115,30 @@ nitro_status_t nitro_cv_train(nitro_cv *cv, const nitro_train_opts *opts);
  * feat[n_in * n_feat], cost[n_in * n_var] (row-major). */
 nitro_status_t nitro_cv_train_from_table(nitro_cv *cv, int n_in, const double *feat, const double *cost,
                                          const nitro_train_opts *opts);
+/* Incremental tuning: features of every training input are
+ * computed first (they are cheap); then only a subset is labelled by
+ * exhaustive search: `init` inputs in a seeded order (extended until two
+ * labels are present), then one input per iteration chosen by the
+ * Best-vs-Second-Best rule (smallest gap between the two largest class
+ * probabilities of the current model, P:L188 [20]), refitting after each.
+ * Stops after `iters` picks ("iter") or once the accuracy on the
+ * labelled test set reaches `acc` ("acc"), or when the pool is empty. */
+typedef struct {
+  int init;                 /* initial labelled inputs (default: number of variants) */
+  int iters;                /* max BvSB picks; <= 0 = until the pool is exhausted */
+  double acc;               /* target test accuracy in (0,1]; 0 = off */
+  uint64_t seed;            /* order of the initial picks */
+  int prob_folds;           /* Platt CV folds (default 5) */
+  int n_test;               /* optional labelled test set (0 = none) */
+  const double *test_feat;  /* [n_test * n_feat] raw features */
+  const double *test_cost;  /* [n_test * n_var] costs (+INF = ruled out); label = argmin */
+} nitro_itune_opts;
+void nitro_itune_opts_default(nitro_itune_opts *o);
+nitro_status_t nitro_cv_itune(nitro_cv *cv, const nitro_train_opts *train, const nitro_itune_opts *it);
+/* One entry per refit: labelled count, input picked after it (-1 = none),
+ * test accuracy and test performance (mean t_best / t_selected), NaN without a test set. */
+nitro_status_t nitro_cv_itune_history(const nitro_cv *cv, int *n_steps, int *n_labelled, int *picked,
+                                      double *test_acc, double *test_perf);
 /* Copies out the training table; any pointer may be NULL.  Sizes: cost
  * [n_in*n_var], feat [n_in*n_feat], label [n_in]. */
 nitro_status_t nitro_cv_training_table(const nitro_cv *cv, int *n_in, double *cost, double *feat, int *label);
@@ -146,6 +170,14 @@ nitro_status_t nitro_svm_decision(const nitro_svm *m, int n, const double *X, do
 /* dual coefficients y_i*alpha_i of pair p for training sample ids (dense [n_train]) and rho */
 nitro_status_t nitro_svm_pair_dual(const nitro_svm *m, int p, double *coef_dense, double *rho);
 void nitro_svm_destroy(nitro_svm *m);
+/* Probability model (libSVM's method, used by BvSB active learning):
+ * per pair a Platt sigmoid fitted on decision values of an internal `folds`-fold
+ * CV (deterministic stratified folds from `seed`), then pairwise coupling. */
+nitro_status_t nitro_svm_fit_prob(int n, int d, const double *X, const int *y, double C, double gamma, double tol,
+                                  int folds, uint64_t seed, nitro_svm **out);
+/* class probabilities [n * n_classes] in ascending-label order */
+nitro_status_t nitro_svm_probability(const nitro_svm *m, int n, const double *X, double *out, int *n_classes);
+nitro_status_t nitro_svm_pair_sigmoid(const nitro_svm *m, int p, double *A, double *B);
 /* deterministic stratified folds (R12) */
 nitro_status_t nitro_svm_fold_assign(int n, const int *y, int k, uint64_t seed, int *out_fold);
 nitro_status_t nitro_svm_cv_accuracy(int n, int d, const double *X, const int *y, double C, double gamma,

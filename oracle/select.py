@@ -167,3 +167,151 @@ def select(model: Model, feat_vec, allowed, default: int = 1) -> int:
     """Predict; a disallowed prediction reverts to the default."""
     lab = int(model.predict(np.asarray([feat_vec], dtype=np.float64))[0])
     return lab if allowed[lab] else default
+
+
+# ---------------------------------------------------------------- probabilities + BvSB (NEXT f1, P:L181-190)
+def sigmoid_predict(f, A, B):
+    fApB = f * A + B
+    return math.exp(-fApB) / (1.0 + math.exp(-fApB)) if fApB >= 0 else 1.0 / (1.0 + math.exp(fApB))
+
+
+def sigmoid_train(dec, y):
+    """Platt's sigmoid P(+1|f) = 1/(1+exp(A f + B)), Newton with backtracking as
+    written in Lin, Lin & Weng (2007), Algorithm 1 (the method libSVM uses)."""
+    dec = [float(v) for v in dec]
+    prior1 = sum(1 for v in y if v > 0)
+    prior0 = len(y) - prior1
+    hi, lo = (prior1 + 1.0) / (prior1 + 2.0), 1.0 / (prior0 + 2.0)
+    t = [hi if v > 0 else lo for v in y]
+    A, B = 0.0, math.log((prior0 + 1.0) / (prior1 + 1.0))
+
+    def F(a, b):
+        s = 0.0
+        for f, ti in zip(dec, t):
+            z = f * a + b
+            s += ti * z + math.log1p(math.exp(-z)) if z >= 0 else (ti - 1) * z + math.log1p(math.exp(z))
+        return s
+
+    fval = F(A, B)
+    for _ in range(100):
+        h11 = h22 = 1e-12
+        h21 = g1 = g2 = 0.0
+        for f, ti in zip(dec, t):
+            z = f * A + B
+            if z >= 0:
+                p, q = math.exp(-z) / (1 + math.exp(-z)), 1 / (1 + math.exp(-z))
+            else:
+                p, q = 1 / (1 + math.exp(z)), math.exp(z) / (1 + math.exp(z))
+            d2 = p * q
+            h11 += f * f * d2
+            h22 += d2
+            h21 += f * d2
+            d1 = ti - p
+            g1 += f * d1
+            g2 += d1
+        if abs(g1) < 1e-5 and abs(g2) < 1e-5:
+            break
+        det = h11 * h22 - h21 * h21
+        dA, dB = -(h22 * g1 - h21 * g2) / det, -(-h21 * g1 + h11 * g2) / det
+        gd = g1 * dA + g2 * dB
+        step = 1.0
+        while step >= 1e-10:
+            nA, nB = A + step * dA, B + step * dB
+            nf = F(nA, nB)
+            if nf < fval + 0.0001 * step * gd:
+                A, B, fval = nA, nB, nf
+                break
+            step /= 2.0
+        if step < 1e-10:
+            break
+    return A, B
+
+
+def pair_cv_decisions(Xp, ypm, C, gamma, folds, seed, tol=1e-6):
+    """Decision values of a binary (+1/-1) problem by internal CV (libSVM
+    svm_binary_svc_probability; folds stratified as fold_assign)."""
+    from sklearn.svm import SVC
+    Xp = np.asarray(Xp, dtype=np.float64)
+    ypm = np.asarray(ypm)
+    fa = fold_assign([0 if v > 0 else 1 for v in ypm], folds, seed)
+    dec = np.zeros(len(ypm))
+    for f in range(folds):
+        te, tr = fa == f, fa != f
+        if not te.any():
+            continue
+        pc, nc = int((ypm[tr] > 0).sum()), int((ypm[tr] < 0).sum())
+        if pc == 0 or nc == 0:
+            dec[te] = 1.0 if pc > 0 else (-1.0 if nc > 0 else 0.0)
+            continue
+        svc = SVC(kernel="rbf", C=C, gamma=gamma, tol=tol).fit(Xp[tr], ypm[tr])
+        dec[te] = svc.decision_function(Xp[te])      # > 0 <=> +1 (sorted classes [-1, +1])
+    return dec
+
+
+def couple(r):
+    """Wu, Lin & Weng (2004) method 2: p = argmin p'Qp, sum p = 1, solved as the
+    KKT linear system (numpy)."""
+    k = r.shape[0]
+    Q = np.zeros((k, k))
+    for t in range(k):
+        for j in range(k):
+            if j != t:
+                Q[t, t] += r[j, t] ** 2
+                Q[t, j] = -r[j, t] * r[t, j]
+    Mx = np.zeros((k + 1, k + 1))
+    Mx[:k, :k] = Q
+    Mx[:k, k] = 1.0
+    Mx[k, :k] = 1.0
+    rhs = np.zeros(k + 1)
+    rhs[k] = 1.0
+    return np.linalg.solve(Mx, rhs)[:k]
+
+
+class ProbModel:
+    """OvO SVC + per-pair Platt sigmoids + coupling (libSVM's probability model)."""
+
+    def __init__(self, Xs, y, C, gamma, folds=5, seed=0, tol=1e-6):
+        Xs = np.asarray(Xs, dtype=np.float64)
+        y = np.asarray(y)
+        self.classes = sorted(set(y.tolist()))
+        self.svc, _ = svc_fit(Xs, y, C, gamma, tol)
+        self.sig = {}
+        for a in range(len(self.classes)):
+            for b in range(a + 1, len(self.classes)):
+                m = (y == self.classes[a]) | (y == self.classes[b])
+                ypm = np.where(y[m] == self.classes[a], 1, -1)
+                dec = pair_cv_decisions(Xs[m], ypm, C, gamma, folds, seed, tol)
+                self.sig[(a, b)] = sigmoid_train(dec, ypm)
+
+    def proba(self, Xs):
+        Xs = np.asarray(Xs, dtype=np.float64)
+        k = len(self.classes)
+        if k == 1:
+            return np.ones((Xs.shape[0], 1))
+        D = self.svc.decision_function(Xs)           # ovo columns: pairs (a<b), > 0 votes a
+        if D.ndim == 1:                               # 2 classes: sklearn flips the sign
+            D = -D[:, None]
+        out = np.zeros((Xs.shape[0], k))
+        for i in range(Xs.shape[0]):
+            r = np.zeros((k, k))
+            q = 0
+            for a in range(k):
+                for b in range(a + 1, k):
+                    A, B = self.sig[(a, b)]
+                    v = min(max(sigmoid_predict(D[i, q], A, B), 1e-7), 1 - 1e-7)
+                    r[a, b], r[b, a] = v, 1 - v
+                    q += 1
+            out[i] = couple(r)
+        return out
+
+
+def bvsb_pick(P, candidates):
+    """Best-vs-Second-Best: the candidate with the smallest gap between its two
+    largest class probabilities (ties -> first candidate)."""
+    best, pick = math.inf, None
+    for row, c in zip(P, candidates):
+        s = sorted(row, reverse=True)
+        gap = s[0] - (s[1] if len(s) > 1 else 0.0)
+        if gap < best:
+            best, pick = gap, c
+    return pick

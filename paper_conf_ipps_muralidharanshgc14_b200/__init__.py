@@ -71,6 +71,12 @@ class TrainOpts(ctypes.Structure):
                 ("verbose", ctypes.c_int)]
 
 
+class ItuneOpts(ctypes.Structure):
+    _fields_ = [("init", ctypes.c_int), ("iters", ctypes.c_int), ("acc", ctypes.c_double),
+                ("seed", ctypes.c_uint64), ("prob_folds", ctypes.c_int), ("n_test", ctypes.c_int),
+                ("test_feat", ctypes.c_void_p), ("test_cost", ctypes.c_void_p)]
+
+
 class SpmvInput(ctypes.Structure):
     _fields_ = [("A", ctypes.c_void_p), ("d_x", ctypes.c_void_p), ("d_y", ctypes.c_void_p),
                 ("warmup", ctypes.c_int), ("reps", ctypes.c_int), ("flush_l2", ctypes.c_int)]
@@ -118,6 +124,12 @@ _SIGS = {
     "nitro_svm_destroy": ([_vp], None),
     "nitro_svm_fold_assign": ([_int, _vp, _int, _u64, _vp], _int),
     "nitro_svm_cv_accuracy": ([_int, _int, _vp, _vp, _dbl, _dbl, _dbl, _int, _u64, _P(_dbl)], _int),
+    "nitro_svm_fit_prob": ([_int, _int, _vp, _vp, _dbl, _dbl, _dbl, _int, _u64, _P(_vp)], _int),
+    "nitro_svm_probability": ([_vp, _int, _vp, _vp, _P(_int)], _int),
+    "nitro_svm_pair_sigmoid": ([_vp, _int, _P(_dbl), _P(_dbl)], _int),
+    "nitro_itune_opts_default": ([_P(ItuneOpts)], None),
+    "nitro_cv_itune": ([_vp, _P(TrainOpts), _P(ItuneOpts)], _int),
+    "nitro_cv_itune_history": ([_vp, _P(_int), _vp, _vp, _vp, _vp], _int),
     # spmv
     "nitro_spmv_create": ([_int, _vp, _i64, _i64, _i64, _vp, _int, _vp, _vp, _int, _P(_vp)], _int),
     "nitro_spmv_set_stream": ([_vp, _vp], _int),
@@ -412,6 +424,28 @@ class CodeVariant:
         _check(_L.nitro_cv_call(self.h, inp, ctypes.byref(v), ctypes.byref(c)))
         return v.value, c.value
 
+    def itune(self, init=0, iters=0, acc=0.0, seed=0, prob_folds=5, test_feat=None, test_cost=None, **train):
+        """Incremental tuning: label a BvSB-chosen subset only.
+        Returns the history dict (one entry per refit)."""
+        io = ItuneOpts()
+        _L.nitro_itune_opts_default(ctypes.byref(io))
+        io.init, io.iters, io.acc, io.seed, io.prob_folds = init, iters, acc, seed, prob_folds
+        keep = []
+        if test_feat is not None:
+            tf, tc = _np(test_feat, np.float64), _np(test_cost, np.float64)
+            keep = [tf, tc]
+            io.n_test, io.test_feat, io.test_cost = tf.shape[0], _ptr(tf), _ptr(tc)
+        o = train_opts(**train)
+        _check(_L.nitro_cv_itune(self.h, ctypes.byref(o), ctypes.byref(io)))
+        del keep
+        ns = ctypes.c_int()
+        _check(_L.nitro_cv_itune_history(self.h, ctypes.byref(ns), None, None, None, None))
+        k = ns.value
+        nl, pk = np.empty(k, np.int32), np.empty(k, np.int32)
+        ac, pf = np.empty(k), np.empty(k)
+        _check(_L.nitro_cv_itune_history(self.h, ctypes.byref(ns), _ptr(nl), _ptr(pk), _ptr(ac), _ptr(pf)))
+        return {"n_labelled": nl.tolist(), "picked": pk.tolist(), "test_acc": ac.tolist(), "test_perf": pf.tolist()}
+
     def predict(self, feat, allowed=None) -> int:
         feat = _np(feat, np.float64)
         al = None if allowed is None else _np([int(bool(a)) for a in allowed], np.int32)
@@ -433,12 +467,29 @@ def addr(rec) -> int:
 
 # ====================================================================== host SVM primitives
 class SVM:
-    def __init__(self, X, y, C, gamma, tol=1e-6):
+    def __init__(self, X, y, C, gamma, tol=1e-6, probability=False, prob_folds=5, seed=0):
         X = _np(X, np.float64)
         y = _np(y, np.int32)
         h = ctypes.c_void_p()
-        _check(_L.nitro_svm_fit(X.shape[0], X.shape[1], _ptr(X), _ptr(y), C, gamma, tol, ctypes.byref(h)))
+        if probability:
+            _check(_L.nitro_svm_fit_prob(X.shape[0], X.shape[1], _ptr(X), _ptr(y), C, gamma, tol, prob_folds, seed,
+                                         ctypes.byref(h)))
+        else:
+            _check(_L.nitro_svm_fit(X.shape[0], X.shape[1], _ptr(X), _ptr(y), C, gamma, tol, ctypes.byref(h)))
         self.h, self.n, self.d = h, X.shape[0], X.shape[1]
+
+    def probability(self, X):
+        X = _np(X, np.float64)
+        k = ctypes.c_int()
+        _check(_L.nitro_svm_probability(self.h, 0, None, None, ctypes.byref(k)))
+        out = np.empty((X.shape[0], k.value))
+        _check(_L.nitro_svm_probability(self.h, X.shape[0], _ptr(X), _ptr(out), ctypes.byref(k)))
+        return out
+
+    def pair_sigmoid(self, p: int):
+        A, B = ctypes.c_double(), ctypes.c_double()
+        _check(_L.nitro_svm_pair_sigmoid(self.h, p, ctypes.byref(A), ctypes.byref(B)))
+        return A.value, B.value
 
     def __del__(self):
         if getattr(self, "h", None):

@@ -3,6 +3,7 @@
 // (exhaustive search + scaling + CV grid + RBF C-SVC), model I/O,
 // selection and call; plus nitro_spmv_register, which
 // plugs the five GPU SpMV variants into it.
+#include <algorithm>
 #include <cmath>
 #include <cstdio>
 #include <cstring>
@@ -52,6 +53,9 @@ struct nitro_cv {
   std::vector<double> lo, hi;
   double C = 1.0, gamma = 1.0, cv_acc = 0.0;
   nitro::SvmModel svm;
+  // incremental tuning history (one entry per refit)
+  std::vector<int> h_nlab, h_pick;
+  std::vector<double> h_acc, h_perf;
 };
 
 using namespace nitro;
@@ -93,15 +97,27 @@ int predict_raw(const nitro_cv *cv, const double *f) {
   return svm_predict_one(cv->svm, xs.data());
 }
 
-nitro_status_t fit(nitro_cv *cv, const nitro_train_opts &o) {
-  const int n = cv->n_in, d = cv->n_feat;
+void scale_from(nitro_cv *cv, const double *F, int n) {
+  const int d = cv->n_feat;
   cv->lo.assign(d, kInf);
   cv->hi.assign(d, -kInf);
   for (int i = 0; i < n; ++i)
     for (int j = 0; j < d; ++j) {
-      cv->lo[j] = std::min(cv->lo[j], cv->t_feat[(size_t)i * d + j]);
-      cv->hi[j] = std::max(cv->hi[j], cv->t_feat[(size_t)i * d + j]);
+      cv->lo[j] = std::min(cv->lo[j], F[(size_t)i * d + j]);
+      cv->hi[j] = std::max(cv->hi[j], F[(size_t)i * d + j]);
     }
+}
+
+// grid + refit on the training table with the scaler already set
+nitro_status_t fit_scaled(nitro_cv *cv, const nitro_train_opts &o);
+
+nitro_status_t fit(nitro_cv *cv, const nitro_train_opts &o) {
+  scale_from(cv, cv->t_feat.data(), cv->n_in);
+  return fit_scaled(cv, o);
+}
+
+nitro_status_t fit_scaled(nitro_cv *cv, const nitro_train_opts &o) {
+  const int n = cv->n_in, d = cv->n_feat;
   std::vector<double> Xs((size_t)n * d);
   for (int i = 0; i < n; ++i) scale_row(cv, &cv->t_feat[(size_t)i * d], &Xs[(size_t)i * d]);
   // inputs every variant failed on (label -1) carry no information: dropped
@@ -297,6 +313,176 @@ nitro_status_t nitro_cv_train_from_table(nitro_cv *cv, int n_in, const double *f
   }
   return fit(cv, o);
   GUARD_END
+}
+
+void nitro_itune_opts_default(nitro_itune_opts *o) {
+  if (!o) return;
+  o->init = 0;
+  o->iters = 0;
+  o->acc = 0.0;
+  o->seed = 0;
+  o->prob_folds = 5;
+  o->n_test = 0;
+  o->test_feat = nullptr;
+  o->test_cost = nullptr;
+}
+
+nitro_status_t nitro_cv_itune(nitro_cv *cv, const nitro_train_opts *topts, const nitro_itune_opts *iopts) {
+  GUARD_BEGIN
+  if (!cv) return fail(NITRO_E_INVALID_ARG, "NULL cv");
+  if (cv->variants.empty() || cv->n_feat == 0 || cv->inputs.empty())
+    return fail(NITRO_E_STATE, "need variants, features and training inputs");
+  nitro_train_opts o;
+  if (topts) o = *topts; else nitro_train_opts_default(&o);
+  nitro_itune_opts it;
+  if (iopts) it = *iopts; else nitro_itune_opts_default(&it);
+  if (it.n_test > 0 && (!it.test_feat || !it.test_cost)) return fail(NITRO_E_INVALID_ARG, "test set arrays missing");
+  const int n = (int)cv->inputs.size(), d = cv->n_feat, V = (int)cv->variants.size();
+  // 1. features of every input first: they are cheap next to running variants
+  std::vector<double> F((size_t)n * d);
+  for (int i = 0; i < n; ++i) NITRO_TRY(eval_features(cv, cv->inputs[i], &F[(size_t)i * d]));
+  scale_from(cv, F.data(), n);  // the whole pool's features are known: scale with them
+  // seeded order of the initial picks (same key as the CV folds, R15)
+  std::vector<int> order(n);
+  for (int i = 0; i < n; ++i) order[i] = i;
+  const uint64_t s0 = [](uint64_t z) {
+    z += 0x9E3779B97F4A7C15ULL; z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL; return z ^ (z >> 31);
+  }(it.seed);
+  auto key = [&](int i) {
+    uint64_t z = s0 ^ (uint64_t)i;
+    z += 0x9E3779B97F4A7C15ULL; z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL; return z ^ (z >> 31);
+  };
+  std::stable_sort(order.begin(), order.end(), [&](int a, int b) {
+    const uint64_t ka = key(a), kb = key(b);
+    return ka != kb ? ka < kb : a < b;
+  });
+  std::vector<char> done(n, 0);
+  std::vector<int> labelled, label_of(n, -1);
+  std::vector<double> cost((size_t)n * V, kInf);
+  auto label_input = [&](int i) {  // exhaustive search on one input
+    void *in = cv->inputs[i];
+    double best = kInf;
+    for (int v = 0; v < V; ++v) {
+      double c = allowed(cv, v, in) ? cv->variants[v].fn(in, cv->variants[v].user) : kInf;
+      if (std::isnan(c)) c = kInf;
+      cost[(size_t)i * V + v] = c;
+      if (c < best) { best = c; label_of[i] = v; }
+    }
+    done[i] = 1;
+    labelled.push_back(i);
+  };
+  auto distinct = [&]() {
+    std::vector<char> seen(V, 0);
+    int k = 0;
+    for (int i : labelled)
+      if (label_of[i] >= 0 && !seen[label_of[i]]) { seen[label_of[i]] = 1; ++k; }
+    return k;
+  };
+  const int init = it.init > 0 ? it.init : V;
+  size_t pos = 0;
+  while (pos < order.size() && ((int)labelled.size() < init || distinct() < 2)) label_input(order[pos++]);
+  // test-set labels (argmin of the given costs, ties -> lowest id)
+  std::vector<int> tlab(std::max(it.n_test, 0), -1);
+  for (int t = 0; t < it.n_test; ++t) {
+    double b = kInf;
+    for (int v = 0; v < V; ++v)
+      if (it.test_cost[(size_t)t * V + v] < b) { b = it.test_cost[(size_t)t * V + v]; tlab[t] = v; }
+  }
+  cv->h_nlab.clear(); cv->h_pick.clear(); cv->h_acc.clear(); cv->h_perf.clear();
+  int picks = 0;
+  for (;;) {
+    // refit on the labelled inputs (labelling order)
+    const int m = (int)labelled.size();
+    cv->n_in = m;
+    cv->t_feat.resize((size_t)m * d);
+    cv->t_cost.resize((size_t)m * V);
+    cv->t_label.resize(m);
+    for (int r = 0; r < m; ++r) {
+      const int i = labelled[r];
+      std::copy(&F[(size_t)i * d], &F[(size_t)(i + 1) * d], &cv->t_feat[(size_t)r * d]);
+      std::copy(&cost[(size_t)i * V], &cost[(size_t)(i + 1) * V], &cv->t_cost[(size_t)r * V]);
+      cv->t_label[r] = label_of[i];
+    }
+    NITRO_TRY(fit_scaled(cv, o));
+    double acc = std::numeric_limits<double>::quiet_NaN(), perf = acc;
+    if (it.n_test > 0) {
+      int ok = 0, cnt = 0;
+      double ps = 0.0;
+      for (int t = 0; t < it.n_test; ++t) {
+        if (tlab[t] < 0) continue;
+        int v = predict_raw(cv, &it.test_feat[(size_t)t * d]);
+        if (v < 0 || v >= V || !std::isfinite(it.test_cost[(size_t)t * V + v])) v = cv->default_id;
+        ++cnt;
+        ok += v == tlab[t];
+        const double cs = it.test_cost[(size_t)t * V + v], cb = it.test_cost[(size_t)t * V + tlab[t]];
+        ps += std::isfinite(cs) ? cb / cs : 0.0;
+      }
+      if (cnt) { acc = (double)ok / cnt; perf = ps / cnt; }
+    }
+    cv->h_nlab.push_back(m);
+    cv->h_pick.push_back(-1);
+    cv->h_acc.push_back(acc);
+    cv->h_perf.push_back(perf);
+    if (it.acc > 0 && acc >= it.acc) break;
+    if (it.iters > 0 && picks >= it.iters) break;
+    std::vector<int> pool;
+    for (int i = 0; i < n; ++i)
+      if (!done[i]) pool.push_back(i);
+    if (pool.empty()) break;
+    int pick = -1;
+    if (cv->svm.const_label >= 0 || cv->svm.classes.size() < 2) {
+      for (int i : order)
+        if (!done[i]) { pick = i; break; }
+    } else {
+      // Best-vs-Second-Best: smallest gap between the two largest probabilities
+      std::vector<double> X;
+      std::vector<int> y;
+      for (int i : labelled)
+        if (label_of[i] >= 0) {
+          std::vector<double> xs(d);
+          scale_row(cv, &F[(size_t)i * d], xs.data());
+          X.insert(X.end(), xs.begin(), xs.end());
+          y.push_back(label_of[i]);
+        }
+      SvmModel pm;
+      svm_fit_prob_impl((int)y.size(), d, X.data(), y.data(), cv->C, cv->gamma, o.tol,
+                        std::max(2, it.prob_folds), it.seed, pm);
+      const int k = (int)pm.classes.size();
+      std::vector<double> xs(d), p(std::max(k, 1));
+      double best_gap = kInf;
+      for (int i : pool) {
+        scale_row(cv, &F[(size_t)i * d], xs.data());
+        svm_probability_impl(pm, xs.data(), p.data());
+        double p1 = -kInf, p2 = -kInf;
+        for (int c = 0; c < k; ++c) {
+          if (p[c] > p1) { p2 = p1; p1 = p[c]; }
+          else if (p[c] > p2) p2 = p[c];
+        }
+        const double gap = p1 - p2;
+        if (gap < best_gap) { best_gap = gap; pick = i; }  // ties -> lowest input index
+      }
+    }
+    cv->h_pick.back() = pick;
+    label_input(pick);
+    ++picks;
+  }
+  cv->trained = true;
+  cv->frozen = true;
+  return NITRO_OK;
+  GUARD_END
+}
+
+nitro_status_t nitro_cv_itune_history(const nitro_cv *cv, int *n_steps, int *n_labelled, int *picked,
+                                      double *test_acc, double *test_perf) {
+  if (!cv || !n_steps) return fail(NITRO_E_INVALID_ARG, "NULL argument");
+  *n_steps = (int)cv->h_nlab.size();
+  if (n_labelled) std::copy(cv->h_nlab.begin(), cv->h_nlab.end(), n_labelled);
+  if (picked) std::copy(cv->h_pick.begin(), cv->h_pick.end(), picked);
+  if (test_acc) std::copy(cv->h_acc.begin(), cv->h_acc.end(), test_acc);
+  if (test_perf) std::copy(cv->h_perf.begin(), cv->h_perf.end(), test_perf);
+  return NITRO_OK;
 }
 
 nitro_status_t nitro_cv_training_table(const nitro_cv *cv, int *n_in, double *cost, double *feat, int *label) {

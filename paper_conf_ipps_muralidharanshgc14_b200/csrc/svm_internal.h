@@ -11,6 +11,7 @@ struct SvmPair {
   double rho = 0.0;
   std::vector<int> sv;         // training-sample ids
   std::vector<double> coef;    // y_i * alpha_i
+  double probA = 0.0, probB = 0.0;  // Platt sigmoid P(ca | f) = 1 / (1 + exp(A f + B))
 };
 
 struct SvmModel {
@@ -20,7 +21,18 @@ struct SvmModel {
   std::vector<int> classes;    // ascending labels
   std::vector<double> X;       // training points [n_train * d] (SVs index into it)
   std::vector<SvmPair> pairs;
+  bool prob = false;           // pairs carry Platt sigmoids
 };
+
+// Probability outputs (for BvSB active learning, P:L188 [20]): libSVM's method —
+// per pair a Platt sigmoid fitted (Lin, Lin & Weng 2007 Newton) on decision
+// values from an internal k-fold CV, then pairwise coupling (Wu, Lin & Weng
+// 2004, method 2), solved exactly.
+double sigmoid_predict(double f, double A, double B);
+void sigmoid_train(int l, const double *dec, const int8_t *y, double &A, double &B);
+void svm_fit_prob_impl(int n, int d, const double *X, const int *y, double C, double gamma, double tol, int folds,
+                       uint64_t seed, SvmModel &m);
+void svm_probability_impl(const SvmModel &m, const double *x, double *p /* [classes] */);
 
 double rbf(const double *a, const double *b, int d, double gamma);
 void svm_fit_impl(int n, int d, const double *X, const int *y, double C, double gamma, double tol, SvmModel &m);
