@@ -28,8 +28,10 @@ constexpr int kThreads = 256;
 constexpr int kWarps = kThreads / 32;
 constexpr int kCache = 1024;            // per-block open-addressing offset set (u32 keys, 4 KB)
 constexpr int kProbe = 4;               // linear-probe length
-constexpr uint32_t kWin = 1u << 17;     // per-block bitmap of offsets in [-2^16, 2^16) (16 KB)
+constexpr uint32_t kWin = 1u << 16;     // per-block bitmap of offsets in [-2^15, 2^15) (8 KB)
 constexpr uint32_t kEmpty = 0xffffffffu;
+constexpr int kStage = 1024;            // per-warp staging buffer (entries) of the short-row path
+constexpr int kRowCap = 64;             // rows longer than this use the windowed path
 
 // Offset index idx = col - row + G is < 2^32 (rows, cols < 2^31), so all
 // per-entry arithmetic is 32-bit.  Near-diagonal offsets (stencils, banded)
@@ -42,6 +44,7 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
                                                         int64_t N, int64_t M, int64_t Z, int64_t row0, int64_t G,
                                                         FeatAcc *__restrict__ acc, uint32_t *__restrict__ bitmap) {
   __shared__ int8_t s_slot[kWarps][32];
+  __shared__ int s_stage[kWarps][kStage];
   __shared__ uint32_t s_seen[kCache];
   __shared__ uint32_t s_win[kWin / 32];
   __shared__ unsigned long long s_red[3][kWarps];
@@ -53,7 +56,7 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
 
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   const uint32_t G32 = (uint32_t)G, M32 = (uint32_t)M;
-  const uint32_t win_lo = G32 - (kWin >> 1);  // idx of offset -2^16 (may wrap: rel test below is modular)
+  const uint32_t win_lo = G32 - (kWin >> 1);  // idx of offset -kWin/2 (may wrap: rel test below is modular)
   unsigned bad = 0;
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     if ((int64_t)rowptr[0] != 0 || (int64_t)rowptr[N] != Z) bad |= 1;
@@ -78,6 +81,64 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
     const int64_t E0 = __shfl_sync(kFull, a, 0), E1 = __shfl_sync(kFull, b, 31);
     const uint32_t rowbase = (uint32_t)(row0 + rb * 32);  // global row of lane 0's row
     const bool lane_has = L > 0;
+    // ---- fast path (short rows, e.g. stencils / banded): stage the block's
+    // colidx span in shared memory with coalesced loads, then every lane walks
+    // its own row (row id known, ~10 instructions per entry, no shuffles)
+    const int Lmax_blk = (int)__reduce_max_sync(kFull, (unsigned)(L > kRowCap ? kRowCap + 1 : L));
+    if (E1 - E0 <= kStage && Lmax_blk <= kRowCap) {
+      int *buf = s_stage[wib];
+      const int span = (int)(E1 - E0);
+      for (int e0 = 0; e0 < span; e0 += 128) {
+        int v[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int e = e0 + u * 32 + lane;
+          v[u] = e < span ? ld_stream_i(col + E0 + e) : 0;
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int e = e0 + u * 32 + lane;
+          if (e < span) buf[e] = v[u];
+        }
+      }
+      __syncwarp();
+      const int rel0 = (int)(a - E0);
+      const uint32_t myrow = rowbase + (uint32_t)lane;
+      int prev = -1;
+      for (int k = 0; k < (int)L; ++k) {
+        const int c = buf[rel0 + k];
+        if ((uint32_t)c >= M32) { bad |= 4; continue; }
+        if (c <= prev) bad |= 2;
+        prev = c;
+        const uint32_t idx = (uint32_t)c - myrow + G32;
+        const uint32_t rel = idx - win_lo;
+        if (rel < kWin) {
+          const uint32_t bit = 1u << (rel & 31);
+          if (!(s_win[rel >> 5] & bit)) atomicOr(&s_win[rel >> 5], bit);
+        } else {
+          // far from the diagonal: shared offset set, then test-before-set global OR
+          bool hit = false;
+          int free_slot = -1;
+          if (!s_full) {
+            const uint32_t h = idx * 0x9E3779B1u >> 22;
+            for (int p = 0; p < kProbe; ++p) {
+              const int slot = (int)((h + p) & (kCache - 1));
+              const uint32_t cur = s_seen[slot];
+              if (cur == idx) { hit = true; break; }
+              if (cur == kEmpty) { free_slot = slot; break; }
+            }
+          }
+          if (!hit) {
+            const uint32_t gbit = 1u << (idx & 31);
+            if (!(__ldcg(bitmap + (idx >> 5)) & gbit)) atomicOr(bitmap + (idx >> 5), gbit);
+            if (free_slot >= 0) atomicCAS(&s_seen[free_slot], kEmpty, idx);
+            else if (!s_full) s_full = 1;
+          }
+        }
+      }
+      __syncwarp();  // the staging buffer is reused by the next block of rows
+      continue;
+    }
     int cur_rl = 0, last_c = 0;
     for (int64_t base = E0; base < E1; base += 128) {
       int c[4];

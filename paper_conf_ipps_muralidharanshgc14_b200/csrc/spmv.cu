@@ -483,6 +483,19 @@ int dia_batch(int64_t D, size_t sv) {
   return sv == 4 ? 4 : 2;
 }
 
+}  // namespace
+
+// DIA implementation: NITRO_DIA_TMA=1 selects the TMA-streamed kernel
+bool dia_use_tma() {
+  static int v = [] {
+    const char *e = getenv("NITRO_DIA_TMA");
+    return e ? atoi(e) : 0;
+  }();
+  return v != 0;
+}
+
+namespace {
+
 unsigned grid_cap(int64_t blocks, int per_sm = 8) {
   int64_t cap = (int64_t)num_sms() * per_sm;
   if (blocks > cap) blocks = cap;
@@ -525,6 +538,7 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
                                                                         x, y, N, A->ell.K, A->ell.ld);
       break;
     case NITRO_DIA:
+      if (N > 0 && A->dia.D > 0 && dia_use_tma()) return launch_dia_tma(A, x, y, s);
       if (N > 0) {
         const size_t sm = (size_t)std::max<int64_t>(A->dia.D, 1) * 4;
         const unsigned g = grid_cap((A->dia.ld + 1023) / 1024, 16);
