@@ -318,6 +318,12 @@ nitro_status_t prepare_csrv(nitro_spmv *A) {
   const int64_t N = A->N;
   const int64_t q = N > 0 ? A->Z / N : 0;
   int V = q <= 2 ? 2 : q <= 4 ? 4 : q <= 8 ? 8 : q <= 16 ? 16 : 32;
+  // tuning hook: NITRO_CSRV_SHIFT=k divides V by 2^k (more entries per lane)
+  static int shift = [] {
+    const char *e = getenv("NITRO_CSRV_SHIFT");
+    return e ? atoi(e) : 0;
+  }();
+  for (int k = 0; k < shift && V > 2; ++k) V >>= 1;
   A->csrv.V = V;
   const int64_t T = 8LL * V, S = kCsrvSeg;
   A->csrv.n_long = 0;

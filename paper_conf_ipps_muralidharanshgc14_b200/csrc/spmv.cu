@@ -244,11 +244,10 @@ __global__ void __launch_bounds__(256) k_csr_vector(const IT *__restrict__ rowpt
 // slots are all issued before the first FMA (explicit register batches: the
 // compiler otherwise reuses one register quad and serialises the slots), so
 // each thread keeps U x (16 + 16|32) bytes of HBM traffic in flight.
-template <typename VT>
+template <typename VT, int U>  // U <= 16: terms per fp32 partial
 __global__ void __launch_bounds__(256) k_ell(const int32_t *__restrict__ ecol, const VT *__restrict__ eval,
                                              const VT *__restrict__ x, VT *__restrict__ y, int64_t N, int64_t K,
                                              int64_t ld) {
-  constexpr int U = sizeof(VT) == 4 ? 8 : 4;  // <= 16 terms per fp32 partial
   const int64_t nq = ld >> 2;
   for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nq; q += (int64_t)gridDim.x * blockDim.x) {
     const int64_t i0 = q << 2;
@@ -483,6 +482,29 @@ int dia_batch(int64_t D, size_t sv) {
   return sv == 4 ? 4 : 2;
 }
 
+// ELL slot batch width: NITRO_ELL_U overrides (2/4/8); default 8 (fp32) / 4 (fp64)
+int ell_batch(size_t sv) {
+  static int env = [] {
+    const char *e = getenv("NITRO_ELL_U");
+    return e ? atoi(e) : 0;
+  }();
+  if (env == 2 || env == 4 || env == 8) return env;
+  return sv == 4 ? 8 : 4;
+}
+
+unsigned grid_cap(int64_t blocks, int per_sm);
+
+template <typename VT>
+void launch_ell(const int32_t *col, const VT *val, const VT *x, VT *y, int64_t N, int64_t K, int64_t ld,
+                cudaStream_t s) {
+  const unsigned g = grid_cap((ld / 4 + 255) / 256, 16);
+  switch (ell_batch(sizeof(VT))) {
+    case 2: k_ell<VT, 2><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld); break;
+    case 4: k_ell<VT, 4><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld); break;
+    default: k_ell<VT, 8><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld); break;
+  }
+}
+
 }  // namespace
 
 // DIA implementation: NITRO_DIA_TMA=1 selects the TMA-streamed kernel
@@ -533,9 +555,7 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
       break;
     }
     case NITRO_ELL:
-      if (N > 0)
-        k_ell<VT><<<grid_cap((A->ell.ld / 4 + 255) / 256, 16), 256, 0, s>>>(A->ell.col.as<int32_t>(), A->ell.val.as<VT>(),
-                                                                        x, y, N, A->ell.K, A->ell.ld);
+      if (N > 0) launch_ell<VT>(A->ell.col.as<int32_t>(), A->ell.val.as<VT>(), x, y, N, A->ell.K, A->ell.ld, s);
       break;
     case NITRO_DIA:
       if (N > 0 && A->dia.D > 0 && dia_use_tma()) return launch_dia_tma(A, x, y, s);
@@ -556,8 +576,7 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
       break;
     case NITRO_HYB:
       if (N > 0) {
-        k_ell<VT><<<grid_cap((A->hyb.ld / 4 + 255) / 256, 16), 256, 0, s>>>(A->hyb.col.as<int32_t>(), A->hyb.val.as<VT>(),
-                                                                        x, y, N, A->hyb.K, A->hyb.ld);
+        launch_ell<VT>(A->hyb.col.as<int32_t>(), A->hyb.val.as<VT>(), x, y, N, A->hyb.K, A->hyb.ld, s);
         if (A->hyb.Zt > 0) {
           k_hyb_tail<VT, hyb_windows(sizeof(VT))><<<grid_cap((A->hyb.nchunks + 7) / 8, 16), 256, 0, s>>>(
               A->hyb.trow.as<int32_t>(), A->hyb.tcol.as<int32_t>(), A->hyb.tval.as<VT>(), x, y, A->hyb.Zt,

@@ -54,6 +54,25 @@ __global__ void __launch_bounds__(kThr) k_dia_tma(const int32_t *__restrict__ of
   };
   if (tid == 0)
     for (int64_t q = 0; q < Q && q < kStages; ++q) issue(q);
+  // x values of stage qq for this thread's 4 rows (L1/L2 gathers)
+  auto gather = [&](int64_t qq, VT (&xo)[GD][4]) {
+    const int64_t tl = blockIdx.x + (qq / ng) * gridDim.x;
+    const int gg = (int)(qq % ng);
+    const int64_t b0 = tl * kRows, ii = b0 + 4 * tid;
+    const int64_t be = (b0 + kRows < ld ? b0 + kRows : ld) - 1;
+    const bool inter = row0 + b0 + off_min >= 0 && row0 + be + off_max < M;
+    const int ndd = (int)(D - (int64_t)gg * GD < GD ? D - (int64_t)gg * GD : GD);
+#pragma unroll
+    for (int j = 0; j < GD; ++j) {
+      const bool live = j < ndd && ii < ld;
+      const int64_t jx = row0 + ii + (live ? __ldg(offs + (int64_t)gg * GD + j) : 0);
+#pragma unroll
+      for (int t = 0; t < 4; ++t)
+        xo[j][t] = (live && (inter || (jx + t >= 0 && jx + t < M))) ? __ldg(x + jx + t) : (VT)0;
+    }
+  };
+  VT xcur[GD][4];
+  if (Q > 0) gather(0, xcur);
   double acc[4] = {0.0, 0.0, 0.0, 0.0};
   for (int64_t q = 0; q < Q; ++q) {
     const int s = (int)(q % kStages);
@@ -64,9 +83,13 @@ __global__ void __launch_bounds__(kThr) k_dia_tma(const int32_t *__restrict__ of
     const int64_t Bend = (B0 + kRows < ld ? B0 + kRows : ld) - 1;
     const bool interior = row0 + B0 + off_min >= 0 && row0 + Bend + off_max < M;
     const int nd = (int)(D - (int64_t)g * GD < GD ? D - (int64_t)g * GD : GD);
+    (void)interior;
+    // the x gathers do not depend on the TMA data: issue the next stage's now
+    VT xnext[GD][4];
+    if (q + 1 < Q) gather(q + 1, xnext);
     mbar_wait(&full[s], (uint32_t)((q / kStages) & 1));
     if (i0 < ld) {
-      VT v[GD][4], xv[GD][4];
+      VT v[GD][4];
 #pragma unroll
       for (int j = 0; j < GD; ++j) {
         if (j < nd) {
@@ -79,20 +102,16 @@ __global__ void __launch_bounds__(kThr) k_dia_tma(const int32_t *__restrict__ of
             const double2 t1 = reinterpret_cast<const double2 *>(sp)[1];
             v[j][0] = t0.x; v[j][1] = t0.y; v[j][2] = t1.x; v[j][3] = t1.y;
           }
-          const int64_t jx = row0 + i0 + __ldg(offs + (int64_t)g * GD + j);
-#pragma unroll
-          for (int t = 0; t < 4; ++t)
-            xv[j][t] = (interior || (jx + t >= 0 && jx + t < M)) ? __ldg(x + jx + t) : (VT)0;
         } else {
 #pragma unroll
-          for (int t = 0; t < 4; ++t) { v[j][t] = (VT)0; xv[j][t] = (VT)0; }
+          for (int t = 0; t < 4; ++t) v[j][t] = (VT)0;
         }
       }
       VT part[4] = {0, 0, 0, 0};
 #pragma unroll
       for (int j = 0; j < GD; ++j)
 #pragma unroll
-        for (int t = 0; t < 4; ++t) part[t] = fma(v[j][t], xv[j][t], part[t]);
+        for (int t = 0; t < 4; ++t) part[t] = fma(v[j][t], xcur[j][t], part[t]);
 #pragma unroll
       for (int t = 0; t < 4; ++t) acc[t] += (double)part[t];
       if (g == ng - 1) {  // tile complete
@@ -114,6 +133,10 @@ __global__ void __launch_bounds__(kThr) k_dia_tma(const int32_t *__restrict__ of
     }
     __syncthreads();  // stage s fully consumed
     if (tid == 0 && q + kStages < Q) issue(q + kStages);
+#pragma unroll
+    for (int j = 0; j < GD; ++j)
+#pragma unroll
+      for (int t = 0; t < 4; ++t) xcur[j][t] = xnext[j][t];
   }
 }
 
