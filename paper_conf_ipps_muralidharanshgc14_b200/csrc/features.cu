@@ -129,8 +129,9 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
             }
           }
           if (!hit) {
-            const uint32_t gbit = 1u << (idx & 31);
-            if (!(__ldcg(bitmap + (idx >> 5)) & gbit)) atomicOr(bitmap + (idx >> 5), gbit);
+            // fire-and-forget OR (no returned value, so no per-entry dependent
+            // L2 round trip in this per-lane sequential loop)
+            atomicOr(bitmap + (idx >> 5), 1u << (idx & 31));
             if (free_slot >= 0) atomicCAS(&s_seen[free_slot], kEmpty, idx);
             else if (!s_full) s_full = 1;
           }

@@ -53,15 +53,30 @@ template <typename IT, typename VT>
 __global__ void __launch_bounds__(256) k_csr_scalar(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
                                                     const VT *__restrict__ val, const VT *__restrict__ x,
                                                     VT *__restrict__ y, int64_t N) {
+  // thread per row; the first kHead entries of the row are loaded as one
+  // predicated batch (short rows — this variant's class — then cost a single
+  // load round trip), longer rows continue sequentially in 16-term chunks
+  constexpr int kHead = 4;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < N; i += (int64_t)gridDim.x * blockDim.x) {
     const int64_t a = (int64_t)rowptr[i], b = (int64_t)rowptr[i + 1];
-    double acc = 0.0;
-    for (int64_t k = a; k < b; k += 16) {
+    int c[kHead];
+    VT v[kHead];
+#pragma unroll
+    for (int k = 0; k < kHead; ++k) {
+      const bool in = a + k < b;
+      c[k] = in ? __ldg(col + a + k) : -1;
+      v[k] = in ? __ldg(val + a + k) : (VT)0;
+    }
+    VT part = 0;
+#pragma unroll
+    for (int k = 0; k < kHead; ++k) part = fma(v[k], c[k] >= 0 ? __ldg(x + c[k]) : (VT)0, part);
+    double acc = (double)part;
+    for (int64_t k = a + kHead; k < b; k += 16) {
       const int64_t e = k + 16 < b ? k + 16 : b;
-      VT part = 0;
+      VT p2 = 0;
 #pragma unroll 4
-      for (int64_t j = k; j < e; ++j) part = fma(__ldg(val + j), __ldg(x + __ldg(col + j)), part);
-      acc += (double)part;
+      for (int64_t j = k; j < e; ++j) p2 = fma(__ldg(val + j), __ldg(x + __ldg(col + j)), p2);
+      acc += (double)p2;
     }
     y[i] = (VT)acc;
   }
@@ -294,7 +309,8 @@ __global__ void __launch_bounds__(256) k_ell(const int32_t *__restrict__ ecol, c
 template <typename VT, int U>
 __global__ void __launch_bounds__(256) k_dia(const int32_t *__restrict__ offs, const VT *__restrict__ dval,
                                              const VT *__restrict__ x, VT *__restrict__ y, int64_t N, int64_t M,
-                                             int64_t D, int64_t ld, int64_t row0, int64_t off_min, int64_t off_max) {
+                                             int64_t D, int64_t ld, int64_t row0, int64_t off_min, int64_t off_max,
+                                             bool x_aligned) {
   extern __shared__ int s_off[];
   for (int64_t d = threadIdx.x; d < D; d += blockDim.x) s_off[d] = offs[d];
   __syncthreads();
@@ -305,6 +321,8 @@ __global__ void __launch_bounds__(256) k_dia(const int32_t *__restrict__ offs, c
     if (i0 >= ld) continue;
     const int64_t Bend = (B0 + 1024 < ld ? B0 + 1024 : ld) - 1;
     const bool interior = row0 + B0 + off_min >= 0 && row0 + Bend + off_max < M;
+    // vector x path: aligned windows may reach 3 floats left / 4 right of the needed ones
+    const bool xvec = x_aligned && row0 + B0 + off_min - 3 >= 0 && row0 + Bend + off_max + 4 < M;
     double acc[4] = {0.0, 0.0, 0.0, 0.0};
     for (int64_t d0 = 0; d0 < D; d0 += U) {
       V4<VT> v[U];
@@ -314,7 +332,33 @@ __global__ void __launch_bounds__(256) k_dia(const int32_t *__restrict__ offs, c
         if (d0 + u < D) v[u].load(dval + (d0 + u) * ld + i0);
         else v[u].v[0] = v[u].v[1] = v[u].v[2] = v[u].v[3] = (VT)0;
       }
-      if (interior) {
+      if (sizeof(VT) == 4 && xvec) {
+        // fp32, x 16-byte aligned at row0: the 4 values x[j..j+3] (j = row0 + i0 +
+        // off) come from the aligned 8-float window at j - (off & 3): two 128-bit
+        // loads instead of four 32-bit ones (half the L1 wavefronts); off & 3 is
+        // uniform across the warp (i0 is a multiple of 4)
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          const bool live = d0 + u < D;
+          const int off = live ? s_off[d0 + u] : 0;
+          const int r = off & 3;
+          const float *xb = reinterpret_cast<const float *>(x) + (row0 + i0 + off - r);
+          float4 lo = make_float4(0.f, 0.f, 0.f, 0.f), hi = lo;
+          if (live) {
+            lo = __ldg(reinterpret_cast<const float4 *>(xb));
+            if (r) hi = __ldg(reinterpret_cast<const float4 *>(xb) + 1);
+          }
+          float w[4];
+          switch (r) {
+            case 0: w[0] = lo.x; w[1] = lo.y; w[2] = lo.z; w[3] = lo.w; break;
+            case 1: w[0] = lo.y; w[1] = lo.z; w[2] = lo.w; w[3] = hi.x; break;
+            case 2: w[0] = lo.z; w[1] = lo.w; w[2] = hi.x; w[3] = hi.y; break;
+            default: w[0] = lo.w; w[1] = hi.x; w[2] = hi.y; w[3] = hi.z; break;
+          }
+#pragma unroll
+          for (int t = 0; t < 4; ++t) xv[u][t] = (VT)w[t];
+        }
+      } else if (interior) {
 #pragma unroll
         for (int u = 0; u < U; ++u) {
           const bool live = d0 + u < D;  // uniform
@@ -482,14 +526,17 @@ int dia_batch(int64_t D, size_t sv) {
   return sv == 4 ? 4 : 2;
 }
 
-// ELL slot batch width: NITRO_ELL_U overrides (2/4/8); default 8 (fp32) / 4 (fp64)
+// ELL slot batch width: NITRO_ELL_U overrides (1/2/4/8); default 2.  B200 sweep
+// on configs[1] (fp32): U=2 6372, U=4 5461, U=8 4681 GB/s — fewer registers and
+// more resident warps beat deeper per-thread batches for this gather pattern.
 int ell_batch(size_t sv) {
   static int env = [] {
     const char *e = getenv("NITRO_ELL_U");
     return e ? atoi(e) : 0;
   }();
-  if (env == 2 || env == 4 || env == 8) return env;
-  return sv == 4 ? 8 : 4;
+  (void)sv;
+  if (env == 1 || env == 2 || env == 4 || env == 8) return env;
+  return 2;
 }
 
 unsigned grid_cap(int64_t blocks, int per_sm);
@@ -499,6 +546,7 @@ void launch_ell(const int32_t *col, const VT *val, const VT *x, VT *y, int64_t N
                 cudaStream_t s) {
   const unsigned g = grid_cap((ld / 4 + 255) / 256, 16);
   switch (ell_batch(sizeof(VT))) {
+    case 1: k_ell<VT, 1><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld); break;
     case 2: k_ell<VT, 2><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld); break;
     case 4: k_ell<VT, 4><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld); break;
     default: k_ell<VT, 8><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld); break;
@@ -562,9 +610,10 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
       if (N > 0) {
         const size_t sm = (size_t)std::max<int64_t>(A->dia.D, 1) * 4;
         const unsigned g = grid_cap((A->dia.ld + 1023) / 1024, 16);
+        const bool x_al = ((reinterpret_cast<uintptr_t>(x) & 15) == 0) && (A->row0 % 4 == 0);
 #define NITRO_DIA_LAUNCH(UU)                                                                                  \
   k_dia<VT, UU><<<g, 256, sm, s>>>(A->dia.off.as<int32_t>(), A->dia.val.as<VT>(), x, y, N, A->M, A->dia.D,    \
-                                   A->dia.ld, A->row0, A->dia.off_min, A->dia.off_max)
+                                   A->dia.ld, A->row0, A->dia.off_min, A->dia.off_max, x_al)
         switch (dia_batch(A->dia.D, sizeof(VT))) {
           case 1: NITRO_DIA_LAUNCH(1); break;
           case 2: NITRO_DIA_LAUNCH(2); break;
