@@ -244,6 +244,15 @@ nitro_status_t prepare_dia(nitro_spmv *A) {
   return NITRO_OK;
 }
 
+int hyb_windows(size_t sv) {
+  static int env = [] {
+    const char *e = getenv("NITRO_HYB_W");
+    return e ? atoi(e) : 0;
+  }();
+  if (env == 2 || env == 4 || env == 8) return env;
+  return sv == 8 ? 4 : 8;
+}
+
 // ------------------------------------------------------------------ HYB (C7)
 nitro_status_t prepare_hyb(nitro_spmv *A) {
   if (A->hyb.ready) return NITRO_OK;
@@ -292,7 +301,8 @@ nitro_status_t prepare_hyb(nitro_spmv *A) {
   NITRO_TRY(A->hyb.trow.alloc((size_t)std::max<int64_t>(Zt, 1) * 4));
   NITRO_TRY(A->hyb.tcol.alloc((size_t)std::max<int64_t>(Zt, 1) * 4));
   NITRO_TRY(A->hyb.tval.alloc((size_t)std::max<int64_t>(Zt, 1) * sv));
-  const int64_t chunk = 32 * hyb_windows((size_t)sv);
+  A->hyb.W = hyb_windows((size_t)sv);
+  const int64_t chunk = 32 * A->hyb.W;
   const int64_t nch = (Zt + chunk - 1) / chunk;
   NITRO_TRY(A->hyb.carry_row.alloc((size_t)std::max<int64_t>(2 * nch, 1) * 4));
   NITRO_TRY(A->hyb.carry_val.alloc((size_t)std::max<int64_t>(2 * nch, 1) * 8));

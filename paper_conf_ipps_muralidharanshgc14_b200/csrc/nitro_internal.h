@@ -64,6 +64,7 @@ struct DiaFmt {
 struct HybFmt {
   bool ready = false;
   int64_t K = 0, ld = 0, Zt = 0, nchunks = 0, tail_rows = 0;
+  int W = 8;  // tail windows per chunk
   DevBuf col, val, trow, tcol, tval, carry_row, carry_val;
 };
 struct CsrvFmt {
@@ -141,8 +142,9 @@ nitro_status_t exclusive_scan_i64(const int64_t *in, int64_t *out, int64_t n, De
 
 inline int64_t round_up(int64_t n, int64_t m) { return (n + m - 1) / m * m; }
 constexpr int64_t kCsrvSeg = 256;  // CSR-vector long-row segment (one warp, 8 entries per lane)
-// HYB tail chunk = 32 * hyb_windows entries per warp (fewer for fp64: registers)
-constexpr int hyb_windows(size_t sv) { return sv == 8 ? 4 : 8; }
+// HYB tail chunk = 32 * W entries per warp; W = 8 (fp32) / 4 (fp64: registers),
+// NITRO_HYB_W overrides (2/4/8).  Fixed per matrix at prepare time.
+int hyb_windows(size_t sv);
 // bitmap index of diagonal offset d is d + G; the bitmap spans G + M bits
 inline int64_t diag_shift(const nitro_spmv *A) { return A->feat_G >= 0 ? A->feat_G : A->row0 + A->N - 1; }
 int num_sms();

@@ -306,25 +306,31 @@ __global__ void __launch_bounds__(256) k_ell(const int32_t *__restrict__ ecol, c
 // U diagonals per batch (all value and x loads of a batch issued before the
 // FMAs): larger U = more bytes in flight per thread but more registers, i.e.
 // fewer resident warps; chosen per launch (dia_batch()).
-template <typename VT, int U>
+// DS ("diagonal split") adjacent lanes share one 4-row quad, lane q taking the
+// diagonals d = q, q + DS, ...: each thread's serial chain of dependent
+// (value, x) loads is DS times shorter; the DS partial sums are combined by a
+// fixed xor butterfly (deterministic).
+template <typename VT, int U, int DS>
 __global__ void __launch_bounds__(256) k_dia(const int32_t *__restrict__ offs, const VT *__restrict__ dval,
                                              const VT *__restrict__ x, VT *__restrict__ y, int64_t N, int64_t M,
                                              int64_t D, int64_t ld, int64_t row0, int64_t off_min, int64_t off_max,
                                              bool x_aligned) {
+  constexpr int64_t RB = 1024 / DS;  // rows per block iteration
   extern __shared__ int s_off[];
   for (int64_t d = threadIdx.x; d < D; d += blockDim.x) s_off[d] = offs[d];
   __syncthreads();
-  const int64_t nb = (ld + 1023) / 1024;
+  const int q = (int)(threadIdx.x % DS);
+  const int64_t nb = (ld + RB - 1) / RB;
   for (int64_t blk = blockIdx.x; blk < nb; blk += gridDim.x) {
-    const int64_t B0 = blk * 1024;
-    const int64_t i0 = B0 + 4 * threadIdx.x;
-    if (i0 >= ld) continue;
-    const int64_t Bend = (B0 + 1024 < ld ? B0 + 1024 : ld) - 1;
+    const int64_t B0 = blk * RB;
+    const int64_t i0 = B0 + 4 * (threadIdx.x / DS);
+    const bool active = i0 < ld;  // whole DS groups share i0: uniform within a group
+    const int64_t Bend = (B0 + RB < ld ? B0 + RB : ld) - 1;
     const bool interior = row0 + B0 + off_min >= 0 && row0 + Bend + off_max < M;
     // vector x path: aligned windows may reach 3 floats left / 4 right of the needed ones
     const bool xvec = x_aligned && row0 + B0 + off_min - 3 >= 0 && row0 + Bend + off_max + 4 < M;
     double acc[4] = {0.0, 0.0, 0.0, 0.0};
-    for (int64_t d0 = 0; d0 < D; d0 += U) {
+    for (int64_t d0 = (int64_t)q * U; active && d0 < D; d0 += (int64_t)DS * U) {
       V4<VT> v[U];
       VT xv[U][4];
 #pragma unroll
@@ -383,7 +389,11 @@ __global__ void __launch_bounds__(256) k_dia(const int32_t *__restrict__ offs, c
 #pragma unroll
       for (int t = 0; t < 4; ++t) acc[t] += (double)part[t];
     }
-    store4<VT>(y, i0, N, acc);
+#pragma unroll
+    for (int o = 1; o < DS; o <<= 1)
+#pragma unroll
+      for (int t = 0; t < 4; ++t) acc[t] += __shfl_xor_sync(kFull, acc[t], o);
+    if (active && q == 0) store4<VT>(y, i0, N, acc);
   }
 }
 
@@ -513,17 +523,29 @@ __global__ void __launch_bounds__(256) k_flush(const int4 *__restrict__ buf, int
   if (acc == 0x7fffffff) *sink = acc;
 }
 
-// DIA batch width: NITRO_DIA_U overrides (tuning); default 4 (fp32) / 2 (fp64)
-// (B200 sweep on configs[1]: U=1 4925, 2 5112, 4 5139, 8 4544 GB/s — U=8's
-// 124 registers cost more occupancy than its extra bytes in flight buy).
+// DIA batch width: NITRO_DIA_U overrides (1/2/4); default 1.  B200 sweep on
+// configs[1] with vectorised x loads: U=1 5373, 2 4916, 4 4561, 8 3033 GB/s —
+// registers (resident warps) matter more than per-thread bytes in flight.
 int dia_batch(int64_t D, size_t sv) {
   static int env = [] {
     const char *e = getenv("NITRO_DIA_U");
     return e ? atoi(e) : 0;
   }();
-  if (env == 1 || env == 2 || env == 4 || env == 8) return env;
+  if (env == 1 || env == 2 || env == 4) return env;
   (void)D;
-  return sv == 4 ? 4 : 2;
+  (void)sv;
+  return 1;
+}
+
+// DIA diagonal split: NITRO_DIA_DS overrides (1/2/4); default 2 when there are
+// enough diagonals to share
+int dia_split(int64_t D) {
+  static int env = [] {
+    const char *e = getenv("NITRO_DIA_DS");
+    return e ? atoi(e) : 0;
+  }();
+  if (env == 1 || env == 2 || env == 4) return env;
+  return D >= 8 ? 2 : 1;
 }
 
 // ELL slot batch width: NITRO_ELL_U overrides (1/2/4/8); default 2.  B200 sweep
@@ -609,17 +631,24 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
       if (N > 0 && A->dia.D > 0 && dia_use_tma()) return launch_dia_tma(A, x, y, s);
       if (N > 0) {
         const size_t sm = (size_t)std::max<int64_t>(A->dia.D, 1) * 4;
-        const unsigned g = grid_cap((A->dia.ld + 1023) / 1024, 16);
         const bool x_al = ((reinterpret_cast<uintptr_t>(x) & 15) == 0) && (A->row0 % 4 == 0);
-#define NITRO_DIA_LAUNCH(UU)                                                                                  \
-  k_dia<VT, UU><<<g, 256, sm, s>>>(A->dia.off.as<int32_t>(), A->dia.val.as<VT>(), x, y, N, A->M, A->dia.D,    \
-                                   A->dia.ld, A->row0, A->dia.off_min, A->dia.off_max, x_al)
-        switch (dia_batch(A->dia.D, sizeof(VT))) {
-          case 1: NITRO_DIA_LAUNCH(1); break;
-          case 2: NITRO_DIA_LAUNCH(2); break;
-          case 4: NITRO_DIA_LAUNCH(4); break;
-          default: NITRO_DIA_LAUNCH(8); break;
+        const int U = dia_batch(A->dia.D, sizeof(VT)), DS = dia_split(A->dia.D);
+        const unsigned g = grid_cap((A->dia.ld + 1024 / DS - 1) / (1024 / DS), 16);
+#define NITRO_DIA_LAUNCH(UU, SS)                                                                                   \
+  k_dia<VT, UU, SS><<<g, 256, sm, s>>>(A->dia.off.as<int32_t>(), A->dia.val.as<VT>(), x, y, N, A->M, A->dia.D,     \
+                                       A->dia.ld, A->row0, A->dia.off_min, A->dia.off_max, x_al)
+#define NITRO_DIA_U(SS)                      \
+  switch (U) {                               \
+    case 2: NITRO_DIA_LAUNCH(2, SS); break;  \
+    case 4: NITRO_DIA_LAUNCH(4, SS); break;  \
+    default: NITRO_DIA_LAUNCH(1, SS); break; \
+  }
+        switch (DS) {
+          case 2: NITRO_DIA_U(2); break;
+          case 4: NITRO_DIA_U(4); break;
+          default: NITRO_DIA_U(1); break;
         }
+#undef NITRO_DIA_U
 #undef NITRO_DIA_LAUNCH
       }
       break;
@@ -627,9 +656,17 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
       if (N > 0) {
         launch_ell<VT>(A->hyb.col.as<int32_t>(), A->hyb.val.as<VT>(), x, y, N, A->hyb.K, A->hyb.ld, s);
         if (A->hyb.Zt > 0) {
-          k_hyb_tail<VT, hyb_windows(sizeof(VT))><<<grid_cap((A->hyb.nchunks + 7) / 8, 16), 256, 0, s>>>(
-              A->hyb.trow.as<int32_t>(), A->hyb.tcol.as<int32_t>(), A->hyb.tval.as<VT>(), x, y, A->hyb.Zt,
-              A->hyb.nchunks, A->hyb.carry_row.as<int32_t>(), A->hyb.carry_val.as<double>());
+          const unsigned gt = grid_cap((A->hyb.nchunks + 7) / 8, 16);
+#define NITRO_TAIL(WW)                                                                                        \
+  k_hyb_tail<VT, WW><<<gt, 256, 0, s>>>(A->hyb.trow.as<int32_t>(), A->hyb.tcol.as<int32_t>(), A->hyb.tval.as<VT>(), \
+                                        x, y, A->hyb.Zt, A->hyb.nchunks, A->hyb.carry_row.as<int32_t>(),          \
+                                        A->hyb.carry_val.as<double>())
+          switch (A->hyb.W) {
+            case 2: NITRO_TAIL(2); break;
+            case 4: NITRO_TAIL(4); break;
+            default: NITRO_TAIL(8); break;
+          }
+#undef NITRO_TAIL
           k_hyb_fixup<VT><<<grid_cap((A->hyb.nchunks + 255) / 256, 16), 256, 0, s>>>(
               A->hyb.carry_row.as<int32_t>(), A->hyb.carry_val.as<double>(), y, A->hyb.nchunks);
         }

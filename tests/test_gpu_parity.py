@@ -337,3 +337,19 @@ def test_register_train_select_call(cuda, tmp_path):
         assert v1 == v2 and M.allowed(v1)
         v3, c3 = cv.call(n.addr(rec))
         assert v3 == v1 and c3 > 0
+
+
+def test_features_async_then_select(cuda):
+    """fix_inputs analogue: the feature pass is enqueued early,
+    other GPU work overlaps it, the later features()/select waits for it."""
+    import torch
+    n = nitro()
+    A = synth.stencil("3d27", 40, mode=1, seed=4)
+    M, _ = handle(A, cuda)
+    M.features_async()
+    z = torch.randn(1 << 22, device=cuda).sum()       # unrelated work while K1 runs
+    f = M.features()
+    f_ref = oracle.features(A)
+    for k in FEAT_KEYS:
+        assert f[k] == f_ref[k], k
+    assert torch.isfinite(z)
