@@ -311,7 +311,8 @@ __global__ void __launch_bounds__(256) k_ell(const int32_t *__restrict__ ecol, c
 // (value, x) loads is DS times shorter; the DS partial sums are combined by a
 // fixed xor butterfly (deterministic).
 template <typename VT, int U, int DS>
-__global__ void __launch_bounds__(256) k_dia(const int32_t *__restrict__ offs, const VT *__restrict__ dval,
+__global__ void __launch_bounds__(256, (U == 1 && sizeof(VT) == 4) ? 8 : 1)  // U=1 fp32: <= 32 regs, full occupancy
+    k_dia(const int32_t *__restrict__ offs, const VT *__restrict__ dval,
                                              const VT *__restrict__ x, VT *__restrict__ y, int64_t N, int64_t M,
                                              int64_t D, int64_t ld, int64_t row0, int64_t off_min, int64_t off_max,
                                              bool x_aligned) {
@@ -325,12 +326,15 @@ __global__ void __launch_bounds__(256) k_dia(const int32_t *__restrict__ offs, c
     const int64_t B0 = blk * RB;
     const int64_t i0 = B0 + 4 * (threadIdx.x / DS);
     const bool active = i0 < ld;  // whole DS groups share i0: uniform within a group
+    if constexpr (DS == 1) {
+      if (!active) continue;      // no cross-lane combine needed
+    }
     const int64_t Bend = (B0 + RB < ld ? B0 + RB : ld) - 1;
     const bool interior = row0 + B0 + off_min >= 0 && row0 + Bend + off_max < M;
     // vector x path: aligned windows may reach 3 floats left / 4 right of the needed ones
     const bool xvec = x_aligned && row0 + B0 + off_min - 3 >= 0 && row0 + Bend + off_max + 4 < M;
     double acc[4] = {0.0, 0.0, 0.0, 0.0};
-    for (int64_t d0 = (int64_t)q * U; active && d0 < D; d0 += (int64_t)DS * U) {
+    for (int64_t d0 = (int64_t)q * U; (DS == 1 || active) && d0 < D; d0 += (int64_t)DS * U) {
       V4<VT> v[U];
       VT xv[U][4];
 #pragma unroll
@@ -537,15 +541,17 @@ int dia_batch(int64_t D, size_t sv) {
   return 1;
 }
 
-// DIA diagonal split: NITRO_DIA_DS overrides (1/2/4); default 2 when there are
-// enough diagonals to share
+// DIA diagonal split: NITRO_DIA_DS overrides (1/2/4); default 1 (B200 sweep on
+// configs[1]: DS=2 4076, DS=4 3115 GB/s — the extra registers and butterfly
+// cost more than the shorter per-thread chains gain)
 int dia_split(int64_t D) {
   static int env = [] {
     const char *e = getenv("NITRO_DIA_DS");
     return e ? atoi(e) : 0;
   }();
+  (void)D;
   if (env == 1 || env == 2 || env == 4) return env;
-  return D >= 8 ? 2 : 1;
+  return 1;
 }
 
 // ELL slot batch width: NITRO_ELL_U overrides (1/2/4/8); default 2.  B200 sweep
