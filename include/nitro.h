@@ -297,8 +297,9 @@ void nitro_dist_destroy(nitro_dist *D);
 /* nnz-balanced contiguous partition: rank r owns rows [bounds[r], bounds[r+1]),
  * bounds[r] = first row i with rowptr[i] >= ceil(r*nnz/P) (host rowptr). */
 nitro_status_t nitro_dist_partition(int64_t rows, const int64_t *h_rowptr, int nranks, int64_t *bounds);
-/* Per-rank matrix: this rank's row block of the global matrix, with GLOBAL
- * column ids, borrowed like nitro_spmv_create.  bounds[nranks+1] is the global
+/* Per-rank matrix: this rank's row block of a SQUARE global matrix (x is
+ * partitioned like y), with GLOBAL column ids < global_rows (checked by the
+ * feature pass: NITRO_E_BAD_MATRIX), borrowed like nitro_spmv_create.  bounds[nranks+1] is the global
  * row partition (x is distributed the same way).  Splits interior rows (all
  * columns owned locally) from boundary rows and remaps columns into the
  * gathered-x layout (block r at r*B, B = max block rows). */

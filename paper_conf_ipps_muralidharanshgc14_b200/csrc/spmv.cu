@@ -494,6 +494,119 @@ __global__ void __launch_bounds__(256) k_hyb_tail(const int32_t *__restrict__ tr
   }
 }
 
+// K9b' (default): lane-sequential variant.  Lane l of a chunk owns the EP
+// consecutive entries [c0 + l*EP, c0 + (l+1)*EP) (128-bit vector loads of
+// row/col ids), sums them sequentially per row, writes rows that start and end
+// inside the lane directly, and one segmented scan ACROSS LANES (5 steps)
+// joins the runs that cross lane boundaries — 1 scan per 32*EP entries
+// instead of one per 32.  Same chunk-level ownership/carry rule as k_hyb_tail.
+template <typename VT, int EP>
+__global__ void __launch_bounds__(256) k_hyb_tail_ls(const int32_t *__restrict__ trow, const int32_t *__restrict__ tcol,
+                                                     const VT *__restrict__ tval, const VT *__restrict__ x,
+                                                     VT *__restrict__ y, int64_t Zt, int64_t nch,
+                                                     int32_t *__restrict__ carry_row, double *__restrict__ carry_val) {
+  static_assert(EP == 4 || EP == 8, "EP");
+  constexpr int64_t CH = 32 * EP;
+  const int lane = threadIdx.x & 31;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t ch = warp; ch < nch; ch += nw) {
+    const int64_t c0 = ch * CH, cend = c0 + CH < Zt ? c0 + CH : Zt;
+    const int64_t e0 = c0 + (int64_t)lane * EP;
+    const int nv = e0 >= cend ? 0 : (cend - e0 < EP ? (int)(cend - e0) : EP);  // valid entries of this lane
+    int r[EP], c[EP];
+    VT v[EP];
+    if (nv == EP) {  // full lane: vector loads (e0 is a multiple of EP, arrays 16-byte aligned)
+#pragma unroll
+      for (int k = 0; k < EP; k += 4) {
+        const int4 rr = ld_stream_i4(reinterpret_cast<const int4 *>(trow + e0 + k));
+        const int4 cc = ld_stream_i4(reinterpret_cast<const int4 *>(tcol + e0 + k));
+        r[k] = rr.x; r[k + 1] = rr.y; r[k + 2] = rr.z; r[k + 3] = rr.w;
+        c[k] = cc.x; c[k + 1] = cc.y; c[k + 2] = cc.z; c[k + 3] = cc.w;
+        V4<VT> vv;
+        vv.load(tval + e0 + k);
+        v[k] = vv.v[0]; v[k + 1] = vv.v[1]; v[k + 2] = vv.v[2]; v[k + 3] = vv.v[3];
+      }
+    } else {
+#pragma unroll
+      for (int k = 0; k < EP; ++k) {
+        const bool ok = k < nv;
+        r[k] = ok ? ld_stream_i(trow + e0 + k) : -2;
+        c[k] = ok ? ld_stream_i(tcol + e0 + k) : 0;
+        v[k] = ok ? ld_stream(tval + e0 + k) : (VT)0;
+      }
+    }
+    double p[EP];
+#pragma unroll
+    for (int k = 0; k < EP; ++k) p[k] = k < nv ? (double)v[k] * (double)__ldg(x + c[k]) : 0.0;
+    // chunk's first / last row (lane 0's first entry; last valid entry)
+    const int first_row = __shfl_sync(kFull, r[0], 0);
+    const int lastl = (int)((cend - 1 - c0) / EP), lastk = (int)((cend - 1 - c0) % EP);
+    int my_last_k = 0;
+#pragma unroll
+    for (int k = 0; k < EP; ++k) my_last_k = k == lastk ? r[k] : my_last_k;
+    const int last_row = __shfl_sync(kFull, my_last_k, lastl);
+    if (lane == 0) { carry_row[2 * ch] = -1; carry_row[2 * ch + 1] = -1; }
+    __syncwarp();
+    auto emit = [&](int row, double val) {  // a completed row segment (chunk ownership rule)
+      if (row == first_row) { carry_row[2 * ch] = row; carry_val[2 * ch] = val; }
+      else if (row == last_row) { carry_row[2 * ch + 1] = row; carry_val[2 * ch + 1] = val; }
+      else y[row] = (VT)((double)y[row] + val);
+    };
+    // lane-sequential runs
+    const int fr = nv > 0 ? r[0] : -2;
+    int cur = fr;
+    double acc = 0.0, pf = 0.0;
+    bool boundary = false;
+#pragma unroll
+    for (int k = 0; k < EP; ++k) {
+      if (k < nv) {
+        if (r[k] != cur) {
+          if (!boundary) { pf = acc; boundary = true; }
+          else emit(cur, acc);  // a row wholly inside this lane
+          cur = r[k];
+          acc = 0.0;
+        }
+        acc += p[k];
+      }
+    }
+    const int lr = cur;                  // this lane's last run row
+    double s = acc;                      // value of the last run
+    // segmented inclusive scan across lanes of the last-run values; a lane heads
+    // a new segment if its last run starts inside it or its row differs from the
+    // previous lane's last row
+    const int prev_lr = __shfl_up_sync(kFull, lr, 1);
+    bool f = boundary || lane == 0 || fr != prev_lr;  // segment head flag
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {  // (s, f) segmented inclusive scan
+      const double t = __shfl_up_sync(kFull, s, o);
+      const bool tf = __shfl_up_sync(kFull, f, o);
+      if (lane >= o) {
+        if (!f) s += t;
+        f = f || tf;
+      }
+    }
+    // s = total of the run ending at this lane's end.  Previous lane's run total:
+    const double prev_s = __shfl_up_sync(kFull, s, 1);
+    if (nv > 0) {
+      if (boundary) {
+        // first run of this lane completes here; it continues a run from the
+        // previous lane iff that lane's last row equals it
+        const double tot = pf + ((lane > 0 && prev_lr == fr) ? prev_s : 0.0);
+        emit(fr, tot);
+      }
+      // the run ending at this lane: complete unless it continues into the next lane
+      const int next_fr = __shfl_down_sync(kFull, fr, 1);
+      const bool next_valid = __shfl_down_sync(kFull, nv, 1) > 0 && lane < 31;
+      const bool continues = next_valid && next_fr == lr;
+      if (!continues) emit(lr, s);
+    } else {
+      (void)__shfl_down_sync(kFull, fr, 1);
+      (void)__shfl_down_sync(kFull, nv, 1);
+    }
+  }
+}
+
 template <typename VT>
 __global__ void __launch_bounds__(256) k_hyb_fixup(const int32_t *__restrict__ carry_row,
                                                    const double *__restrict__ carry_val, VT *__restrict__ y,
@@ -667,11 +780,20 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
   k_hyb_tail<VT, WW><<<gt, 256, 0, s>>>(A->hyb.trow.as<int32_t>(), A->hyb.tcol.as<int32_t>(), A->hyb.tval.as<VT>(), \
                                         x, y, A->hyb.Zt, A->hyb.nchunks, A->hyb.carry_row.as<int32_t>(),          \
                                         A->hyb.carry_val.as<double>())
+#define NITRO_TAIL_LS(WW)                                                                                      \
+  k_hyb_tail_ls<VT, WW><<<gt, 256, 0, s>>>(A->hyb.trow.as<int32_t>(), A->hyb.tcol.as<int32_t>(),                \
+                                           A->hyb.tval.as<VT>(), x, y, A->hyb.Zt, A->hyb.nchunks,               \
+                                           A->hyb.carry_row.as<int32_t>(), A->hyb.carry_val.as<double>())
+          static const bool ls = [] {
+            const char *e = getenv("NITRO_HYB_LS");
+            return e ? atoi(e) != 0 : true;
+          }();
           switch (A->hyb.W) {
             case 2: NITRO_TAIL(2); break;
-            case 4: NITRO_TAIL(4); break;
-            default: NITRO_TAIL(8); break;
+            case 4: if (ls) NITRO_TAIL_LS(4); else NITRO_TAIL(4); break;
+            default: if (ls) NITRO_TAIL_LS(8); else NITRO_TAIL(8); break;
           }
+#undef NITRO_TAIL_LS
 #undef NITRO_TAIL
           k_hyb_fixup<VT><<<grid_cap((A->hyb.nchunks + 255) / 256, 16), 256, 0, s>>>(
               A->hyb.carry_row.as<int32_t>(), A->hyb.carry_val.as<double>(), y, A->hyb.nchunks);

@@ -1,4 +1,4 @@
-# quick check of the default kernels on the four configs + sanitizers
-t() { timeout 300 python tools/profile_variants.py --time $1 $2 2>/dev/null | python -c "import json,sys; t=json.load(sys.stdin); print({c: {k: round(v['GBps']) for k,v in r['variants'].items()} for c,r in t.items()}, {c: round(r['feature_ms'],3) for c,r in t.items()})"; }
-echo "defaults"; t "c1 c2a c2b short" ""
-echo "DIA U=2"; NITRO_DIA_U=2 t "c1 short" dia
+t() { timeout 300 python tools/profile_variants.py --time $1 $2 2>/dev/null | python -c "import json,sys; t=json.load(sys.stdin); print({c: {k: round(v['GBps']) for k,v in r['variants'].items()} for c,r in t.items()})"; }
+echo "HYB ls default"; t "c2b c0" hyb
+echo "HYB ls W=8"; NITRO_HYB_W=8 t "c2b" hyb
+echo "HYB old"; NITRO_HYB_LS=0 t "c2b" hyb
