@@ -307,14 +307,33 @@ nitro_status_t nitro_dist_spmv_create(nitro_dist *D, int64_t global_rows, const 
                                       int64_t local_nnz, const void *d_rowptr, int rowptr_is_64,
                                       const int32_t *d_colidx, const void *d_vals, int is_fp64,
                                       nitro_spmv **out_local);
-/* y_local = A_local * x (x all-gathered from every rank's x_local with NCCL on
- * a side stream; interior rows overlap the gather, boundary rows follow). */
+/* Same, choosing the x exchange: -1 auto (halo when the largest per-rank halo
+ * is < 1/4 of the all-gather volume), 0 all-gather (layout: P*B padded
+ * blocks), 1 halo (layout: [x_local (n) | halo (nh)], grouped send/recv of
+ * only the referenced remote entries).  Collective when the
+ * handle has a communicator (every rank must call it). */
+nitro_status_t nitro_dist_spmv_create_ex(nitro_dist *D, int64_t global_rows, const int64_t *bounds,
+                                         int64_t local_nnz, const void *d_rowptr, int rowptr_is_64,
+                                         const int32_t *d_colidx, const void *d_vals, int is_fp64, int exchange,
+                                         nitro_spmv **out_local);
+/* Exchange facts: mode (0 all-gather, 1 halo), x layout length, halo entries
+ * this rank receives, entries it sends. */
+nitro_status_t nitro_dist_exchange_info(nitro_spmv *A_local, int *mode, int64_t *layout_len, int64_t *halo_len,
+                                        int64_t *send_len);
+/* The sorted global column ids of the halo (host array of halo_len entries). */
+nitro_status_t nitro_dist_halo_cols(nitro_spmv *A_local, int32_t *h_out);
+/* Device address where this rank's x block lives inside the exchange layout:
+ * passing it as d_x_local to nitro_dist_spmv_run (e.g. a solver writing its
+ * next x there directly) skips the per-multiply copy. */
+nitro_status_t nitro_dist_x_local(nitro_spmv *A_local, void **ptr);
+/* y_local = A_local * x (x exchanged with NCCL on a side stream — all-gather or
+ * halo send/recv; interior rows overlap the exchange, boundary rows follow). */
 nitro_status_t nitro_dist_spmv_run(nitro_dist *D, nitro_spmv *A_local, int variant, const void *d_x_local,
                                    void *d_y_local);
-/* Same multiply from an x that is already gathered in the padded layout
- * (block q at q*B, B = max block rows, length nranks*B; padding entries must
- * be finite, e.g. 0, because padded formats multiply zero slots by them):
- * no communication.
+/* Same multiply from an x that is already exchanged into this handle's layout
+ * (all-gather: block q at q*B, B = max block rows, length nranks*B; halo:
+ * [x_local | x[halo_cols]]; padding entries must be finite, e.g. 0, because
+ * padded formats multiply zero slots by them): no communication.
  * Used when the caller owns the exchange (e.g. a solver that writes y straight
  * into the next x), and to check every rank's part on one GPU. */
 nitro_status_t nitro_dist_spmv_run_gathered(nitro_dist *D, nitro_spmv *A_local, int variant,

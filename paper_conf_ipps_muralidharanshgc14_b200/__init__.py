@@ -160,6 +160,10 @@ _SIGS = {
     "nitro_dist_spmv_run_gathered": ([_vp, _vp, _int, _vp, _vp], _int),
     "nitro_dist_layout": ([_vp, _P(_i64), _P(_i64), _P(_i64)], _int),
     "nitro_dist_init_local": ([_int, _int, _int, _P(_vp)], _int),
+    "nitro_dist_spmv_create_ex": ([_vp, _i64, _vp, _i64, _vp, _int, _vp, _vp, _int, _int, _P(_vp)], _int),
+    "nitro_dist_exchange_info": ([_vp, _P(_int), _P(_i64), _P(_i64), _P(_i64)], _int),
+    "nitro_dist_halo_cols": ([_vp, _vp], _int),
+    "nitro_dist_x_local": ([_vp, _P(_vp)], _int),
 }
 for _name, (_args, _res) in _SIGS.items():
     _f = getattr(_L, _name)
@@ -534,6 +538,18 @@ def cv_accuracy(X, y, C, gamma, tol=1e-6, folds=5, seed=0) -> float:
 
 
 # ====================================================================== multi-GPU
+def _wrap_device(ptr: int, n: int, dtype, device: int):
+    """A torch tensor over library-owned device memory (no copy, not owning)."""
+    import torch
+    itemsize = torch.empty((), dtype=dtype).element_size()
+
+    class _CAI:
+        __cuda_array_interface__ = {"shape": (n,), "typestr": "<f8" if itemsize == 8 else "<f4",
+                                    "data": (ptr, False), "version": 3, "strides": None}
+    with torch.cuda.device(device):
+        return torch.as_tensor(_CAI(), device=f"cuda:{device}")
+
+
 def dist_partition(rowptr_host, nranks: int) -> np.ndarray:
     rp = _np(rowptr_host, np.int64)
     out = np.empty(nranks + 1, dtype=np.int64)
@@ -571,6 +587,29 @@ class Dist:
         return y_local
 
     @staticmethod
+    def exchange_info(A: "SpMV") -> dict:
+        m, L, nh, ns = ctypes.c_int(), ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64()
+        _check(_L.nitro_dist_exchange_info(A.h, ctypes.byref(m), ctypes.byref(L), ctypes.byref(nh), ctypes.byref(ns)))
+        return {"mode": ("allgather", "halo")[m.value], "layout_len": L.value, "halo_len": nh.value,
+                "send_len": ns.value}
+
+    @staticmethod
+    def halo_cols(A: "SpMV") -> np.ndarray:
+        info = Dist.exchange_info(A)
+        out = np.empty(info["halo_len"], dtype=np.int32)
+        _check(_L.nitro_dist_halo_cols(A.h, _ptr(out) if out.size else None))
+        return out
+
+    @staticmethod
+    def x_local(A: "SpMV"):
+        """torch view of this rank's x block inside the exchange buffer (write x
+        there and pass it to run() to skip the per-multiply copy)."""
+        import torch
+        p = ctypes.c_void_p()
+        _check(_L.nitro_dist_x_local(A.h, ctypes.byref(p)))
+        return _wrap_device(p.value, A.rows, A.dtype, A.device)
+
+    @staticmethod
     def layout(A: "SpMV"):
         B, i0, i1 = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64()
         _check(_L.nitro_dist_layout(A.h, ctypes.byref(B), ctypes.byref(i0), ctypes.byref(i1)))
@@ -581,14 +620,15 @@ class Dist:
             _L.nitro_dist_destroy(self.h)
             self.h = None
 
-    def spmv(self, global_rows, bounds, rowptr, colidx, vals):
-        """This rank's row block (global column ids) -> SpMV handle for dist runs."""
+    def spmv(self, global_rows, bounds, rowptr, colidx, vals, exchange: int = -1):
+        """This rank's row block (global column ids) -> SpMV handle for dist runs.
+        exchange: -1 auto, 0 all-gather, 1 halo."""
         import torch
         b = _np(bounds, np.int64)
         h = ctypes.c_void_p()
-        _check(_L.nitro_dist_spmv_create(self.h, global_rows, _ptr(b), colidx.numel(), _ptr(rowptr),
-                                         int(rowptr.dtype == torch.int64), _ptr(colidx), _ptr(vals),
-                                         int(vals.dtype == torch.float64), ctypes.byref(h)))
+        _check(_L.nitro_dist_spmv_create_ex(self.h, global_rows, _ptr(b), colidx.numel(), _ptr(rowptr),
+                                            int(rowptr.dtype == torch.int64), _ptr(colidx), _ptr(vals),
+                                            int(vals.dtype == torch.float64), exchange, ctypes.byref(h)))
         A = SpMV.__new__(SpMV)
         A._keep = (rowptr, colidx, vals)
         A.rows = int(b[self.rank + 1] - b[self.rank])

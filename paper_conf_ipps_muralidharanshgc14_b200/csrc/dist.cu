@@ -1,22 +1,30 @@
 // dist.cu — A13: multi-GPU row-partitioned SpMV (include/nitro.h §3).
 //
 // One process per GPU.  Rank r owns the contiguous, nnz-balanced row block
-// [bounds[r], bounds[r+1]) (R14) and the matching block of x.
-// Every multiply all-gathers x with NCCL (in place, into a padded layout where
-// block r starts at r*B, B = max block rows); columns are remapped once to that
-// layout.  Local rows are split into head [0,i0) / interior [i0,i1) / tail
-// [i1,n): interior rows only touch locally owned columns, so they run on the
-// compute stream while the all-gather is in flight on the comm stream; head
-// and tail rows run after it.  Each part is an ordinary nitro_spmv over a
-// rebased CSR slice, so every variant (and its constraint) works unchanged.
-// Global features: per-rank K1 over a global-offset bitmap, integer moments
-// all-reduced (sum / max), occupied diagonals unioned (max over u8 flags).
+// [bounds[r], bounds[r+1]) (R14) and the matching block of x.  Two
+// x-exchange modes, fixed when the handle is created:
+//  * all-gather: every multiply all-gathers x in place with NCCL into a padded
+//    layout where block q starts at q*B (B = max block rows);
+//  * halo: only the x entries this rank's rows reference on
+//    other ranks are exchanged (grouped ncclSend/ncclRecv of packed lists),
+//    into a layout [x_local (n) | halo (nh)] — for stencil/banded partitions a
+//    few planes instead of the whole vector.  Chosen automatically when the
+//    largest halo is under a quarter of the all-gather volume.
+// Columns are remapped once to the chosen layout.  Local rows are split into
+// head [0,i0) / interior [i0,i1) / tail [i1,n): interior rows only touch
+// locally owned columns, so they run on the compute stream while the exchange
+// is in flight on the comm stream; head and tail rows run after it.  Each part
+// is an ordinary nitro_spmv over a rebased CSR slice, so every variant (and
+// its constraint) works unchanged.  Global features: per-rank K1 over a
+// global-offset bitmap, integer moments all-reduced (sum / max), occupied
+// diagonals unioned (max over u8 flags).
 #include <nccl.h>
 
 #include <algorithm>
 #include <vector>
 
 #include "nitro_internal.h"
+#include "util.cuh"
 
 struct nitro_dist {
   ncclComm_t comm = nullptr;
@@ -28,20 +36,29 @@ struct nitro_dist {
 namespace nitro {
 namespace {
 
-#define NITRO_NCCL(call)                                                                    \
-  do {                                                                                      \
-    ncclResult_t r_ = (call);                                                               \
+#define NITRO_NCCL(call)                                                                                         \
+  do {                                                                                                           \
+    ncclResult_t r_ = (call);                                                                                    \
     if (r_ != ncclSuccess) return fail(NITRO_E_NCCL, std::string("NCCL: ") + ncclGetErrorString(r_) + " at " #call); \
   } while (0)
+
+enum { kAllGather = 0, kHalo = 1 };
 
 struct DistState {
   nitro_dist *D = nullptr;
   int64_t global_rows = 0, B = 0, n = 0, row_begin = 0, i0 = 0, i1 = 0;
+  int mode = kAllGather;
   std::vector<int64_t> bounds;
-  DevBuf colmap, rp_part[3], xfull, flags;
+  DevBuf colmap, rp_part[3], xbuf, flags;
+  // halo mode
+  int64_t nh = 0, ns = 0;
+  std::vector<int64_t> recv_off, send_off;  // [P+1] offsets into the halo / send lists
+  DevBuf halo_cols, send_idx, sendbuf;
   nitro_spmv *part[3] = {nullptr, nullptr, nullptr};
   nitro_spmv *feat = nullptr;  // original global columns, for global features
   int64_t part_begin[3] = {0, 0, 0};
+  int64_t layout_len() const { return mode == kHalo ? n + nh : (int64_t)D->nranks * B; }
+  int64_t x_offset() const { return mode == kHalo ? 0 : (int64_t)D->rank * B; }
 };
 
 void free_state(void *p) {
@@ -52,8 +69,14 @@ void free_state(void *p) {
   delete st;
 }
 
-__global__ void k_remap(const int32_t *__restrict__ col, int64_t Z, const int64_t *__restrict__ bounds, int P,
-                        int64_t B, int32_t *__restrict__ out) {
+unsigned grid_n(int64_t n) {
+  int64_t g = (n + 255) / 256, cap = (int64_t)num_sms() * 16;
+  return (unsigned)std::max<int64_t>(1, std::min(g, cap));
+}
+
+// all-gather layout: owner(c) * B + (c - bounds[owner])
+__global__ void k_remap_ag(const int32_t *__restrict__ col, int64_t Z, const int64_t *__restrict__ bounds, int P,
+                           int64_t B, int32_t *__restrict__ out) {
   for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < Z; k += (int64_t)gridDim.x * blockDim.x) {
     const int64_t c = col[k];
     int lo = 0, hi = P - 1;  // owner = last r with bounds[r] <= c
@@ -62,6 +85,64 @@ __global__ void k_remap(const int32_t *__restrict__ col, int64_t Z, const int64_
       if (bounds[mid] <= c) lo = mid; else hi = mid - 1;
     }
     out[k] = (int32_t)((int64_t)lo * B + (c - bounds[lo]));
+  }
+}
+
+// halo layout: local c -> c - lo; remote c -> n + position of c in the sorted halo list
+__global__ void k_remap_halo(const int32_t *__restrict__ col, int64_t Z, int64_t lo, int64_t hi, int64_t n,
+                             const int32_t *__restrict__ H, int64_t nh, int32_t *__restrict__ out) {
+  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < Z; k += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t c = col[k];
+    if (c >= lo && c < hi) { out[k] = (int32_t)(c - lo); continue; }
+    int64_t a = 0, b = nh;
+    while (a < b) {
+      const int64_t m = (a + b) >> 1;
+      if ((int64_t)H[m] < c) a = m + 1; else b = m;
+    }
+    out[k] = (int32_t)(n + a);
+  }
+}
+
+// mark remote columns in a bitmap over the global columns
+__global__ void k_mark_remote(const int32_t *__restrict__ col, int64_t Z, int64_t lo, int64_t hi,
+                              uint32_t *__restrict__ bm) {
+  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < Z; k += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t c = col[k];
+    if (c < lo || c >= hi) {
+      const uint32_t bit = 1u << (c & 31);
+      if (!(__ldcg(bm + (c >> 5)) & bit)) atomicOr(bm + (c >> 5), bit);
+    }
+  }
+}
+__global__ void __launch_bounds__(256) k_bm_tile_counts(const uint32_t *__restrict__ bm, int64_t nwords,
+                                                        int64_t *__restrict__ cnt) {
+  const int64_t base = (int64_t)blockIdx.x * 1024;
+  int64_t s = 0;
+  for (int t = threadIdx.x; t < 1024; t += 256)
+    if (base + t < nwords) s += __popc(bm[base + t]);
+  s = block_sum_i64<256>(s);
+  if (threadIdx.x == 0) cnt[blockIdx.x] = s;
+}
+__global__ void __launch_bounds__(256) k_bm_emit(const uint32_t *__restrict__ bm, int64_t nwords,
+                                                 const int64_t *__restrict__ tile_off, int32_t *__restrict__ out) {
+  const int64_t base = (int64_t)blockIdx.x * 1024 + threadIdx.x * 4;
+  uint32_t w[4];
+  int64_t c = 0;
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    w[q] = base + q < nwords ? bm[base + q] : 0u;
+    c += __popc(w[q]);
+  }
+  int64_t agg;
+  int64_t o = tile_off[blockIdx.x] + block_exclusive_i64<256>(c, agg);
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    uint32_t v = w[q];
+    while (v) {
+      const int b = __ffs(v) - 1;
+      v &= v - 1;
+      out[o++] = (int32_t)((base + q) * 32 + b);
+    }
   }
 }
 
@@ -83,6 +164,17 @@ __global__ void k_rebase(const IT *__restrict__ rowptr, int64_t s, int64_t cnt, 
     out[i] = (int32_t)((int64_t)rowptr[s + i] - base);
 }
 
+__global__ void k_to_local(int32_t *__restrict__ ids, int64_t n, int64_t lo) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    ids[i] = (int32_t)((int64_t)ids[i] - lo);
+}
+
+template <typename VT>
+__global__ void k_pack(const VT *__restrict__ xl, const int32_t *__restrict__ idx, int64_t n, VT *__restrict__ out) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    out[i] = xl[idx[i]];
+}
+
 __global__ void k_bits_to_flags(const uint32_t *__restrict__ bm, int64_t nbits, uint8_t *__restrict__ f) {
   for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < nbits; t += (int64_t)gridDim.x * blockDim.x)
     f[t] = (bm[t >> 5] >> (t & 31)) & 1u;
@@ -99,9 +191,79 @@ __global__ void k_pack_acc(const FeatAcc *a, unsigned long long *sum2, unsigned 
   sum2[0] = a->s1; sum2[1] = a->s2; max2[0] = a->lmax; max2[1] = a->bad;
 }
 
-unsigned grid_n(int64_t n) {
-  int64_t g = (n + 255) / 256, cap = (int64_t)num_sms() * 16;
-  return (unsigned)std::max<int64_t>(1, std::min(g, cap));
+// sorted list of the remote global columns referenced by this rank's rows
+nitro_status_t halo_list(DistState *st, const int32_t *col, int64_t Z, DevBuf &out, int64_t &nh) {
+  const int64_t M = st->global_rows, nwords = (M + 31) / 32, nt = (nwords + 1023) / 1024;
+  DevBuf bm, cnt, scratch;
+  NITRO_TRY(bm.alloc((size_t)std::max<int64_t>(nwords, 1) * 4));
+  NITRO_CUDA(cudaMemset(bm.p, 0, (size_t)std::max<int64_t>(nwords, 1) * 4));
+  if (Z > 0) k_mark_remote<<<grid_n(Z), 256>>>(col, Z, st->bounds[st->D->rank], st->bounds[st->D->rank + 1],
+                                               bm.as<uint32_t>());
+  NITRO_TRY(cnt.alloc((size_t)(2 * nt + 2) * 8));
+  int64_t *tc = cnt.as<int64_t>(), *to = tc + nt + 1;
+  nh = 0;
+  if (nt > 0) {
+    k_bm_tile_counts<<<(unsigned)nt, 256>>>(bm.as<uint32_t>(), nwords, tc);
+    NITRO_TRY(exclusive_scan_i64(tc, to, nt, scratch, nullptr));
+    NITRO_CUDA(cudaMemcpy(&nh, to + nt, 8, cudaMemcpyDeviceToHost));
+  }
+  NITRO_TRY(out.alloc((size_t)std::max<int64_t>(nh, 1) * 4));
+  if (nh > 0) k_bm_emit<<<(unsigned)nt, 256>>>(bm.as<uint32_t>(), nwords, to, out.as<int32_t>());
+  NITRO_CUDA(cudaGetLastError());
+  NITRO_CUDA(cudaDeviceSynchronize());
+  return NITRO_OK;
+}
+
+// halo plan: what to receive from each owner, and (via NCCL) what to send to each requester
+nitro_status_t halo_plan(DistState *st) {
+  nitro_dist *D = st->D;
+  const int P = D->nranks, me = D->rank;
+  std::vector<int32_t> H(st->nh);
+  if (st->nh) NITRO_CUDA(cudaMemcpy(H.data(), st->halo_cols.p, st->nh * 4, cudaMemcpyDeviceToHost));
+  st->recv_off.assign(P + 1, 0);
+  for (int q = 0, k = 0; q < P; ++q) {
+    while (k < (int)st->nh && H[k] < st->bounds[q + 1]) ++k;
+    st->recv_off[q + 1] = k;
+  }
+  st->send_off.assign(P + 1, 0);
+  st->ns = 0;
+  if (!D->comm || P == 1) return NITRO_OK;  // communicator-less: the caller supplies the layout
+  // need matrix: row r = counts rank r receives from each owner
+  DevBuf need;
+  NITRO_TRY(need.alloc((size_t)P * P * 8));
+  std::vector<int64_t> mine(P), all((size_t)P * P);
+  for (int q = 0; q < P; ++q) mine[q] = st->recv_off[q + 1] - st->recv_off[q];
+  NITRO_CUDA(cudaMemcpy(need.as<int64_t>() + (size_t)me * P, mine.data(), P * 8, cudaMemcpyHostToDevice));
+  NITRO_NCCL(ncclAllGather(need.as<int64_t>() + (size_t)me * P, need.p, P, ncclInt64, D->comm, D->comm_stream));
+  NITRO_CUDA(cudaStreamSynchronize(D->comm_stream));
+  NITRO_CUDA(cudaMemcpy(all.data(), need.p, (size_t)P * P * 8, cudaMemcpyDeviceToHost));
+  for (int r = 0; r < P; ++r) st->send_off[r + 1] = st->send_off[r] + all[(size_t)r * P + me];
+  st->ns = st->send_off[P];
+  NITRO_TRY(st->send_idx.alloc((size_t)std::max<int64_t>(st->ns, 1) * 4));
+  // requesters send me the global ids they need from me
+  NITRO_NCCL(ncclGroupStart());
+  for (int q = 0; q < P; ++q) {
+    if (q == me) continue;
+    const int64_t rc = st->recv_off[q + 1] - st->recv_off[q];
+    const int64_t sc = st->send_off[q + 1] - st->send_off[q];
+    if (rc > 0) NITRO_NCCL(ncclSend(st->halo_cols.as<int32_t>() + st->recv_off[q], rc, ncclInt32, q, D->comm, D->comm_stream));
+    if (sc > 0) NITRO_NCCL(ncclRecv(st->send_idx.as<int32_t>() + st->send_off[q], sc, ncclInt32, q, D->comm, D->comm_stream));
+  }
+  NITRO_NCCL(ncclGroupEnd());
+  NITRO_CUDA(cudaStreamSynchronize(D->comm_stream));
+  if (st->ns > 0) k_to_local<<<grid_n(st->ns), 256>>>(st->send_idx.as<int32_t>(), st->ns, st->bounds[me]);
+  NITRO_CUDA(cudaDeviceSynchronize());
+  return NITRO_OK;
+}
+
+nitro_status_t run_part(DistState *st, int k, int variant, cudaStream_t s, const void *xg, void *y, size_t sv) {
+  nitro_spmv *P = st->part[k];
+  if (!P) return NITRO_OK;
+  P->stream = s;
+  int ok = 0, v = variant;
+  NITRO_TRY(nitro_spmv_allowed(P, v, &ok));
+  if (!ok) v = NITRO_CSR_VECTOR;  // part-level constraint fallback (P:L134)
+  return nitro_spmv_run(P, v, xg, (char *)y + (size_t)st->part_begin[k] * sv);
 }
 
 }  // namespace
@@ -139,6 +301,18 @@ nitro_status_t nitro_dist_init(const void *id128, int rank, int nranks, int devi
   return NITRO_OK;
 }
 
+nitro_status_t nitro_dist_init_local(int rank, int nranks, int device, nitro_dist **out) {
+  if (!out || nranks < 1 || rank < 0 || rank >= nranks) return fail(NITRO_E_INVALID_ARG, "bad argument");
+  NITRO_CUDA(cudaSetDevice(device));
+  nitro_dist *D = new nitro_dist();
+  D->rank = rank; D->nranks = nranks; D->device = device;
+  NITRO_CUDA(cudaStreamCreateWithFlags(&D->comm_stream, cudaStreamNonBlocking));
+  NITRO_CUDA(cudaEventCreateWithFlags(&D->ev_x, cudaEventDisableTiming));
+  NITRO_CUDA(cudaEventCreateWithFlags(&D->ev_g, cudaEventDisableTiming));
+  *out = D;
+  return NITRO_OK;
+}
+
 void nitro_dist_destroy(nitro_dist *D) {
   if (!D) return;
   cudaSetDevice(D->device);
@@ -167,11 +341,12 @@ nitro_status_t nitro_dist_partition(int64_t rows, const int64_t *h_rowptr, int n
   return NITRO_OK;
 }
 
-nitro_status_t nitro_dist_spmv_create(nitro_dist *D, int64_t global_rows, const int64_t *bounds, int64_t local_nnz,
-                                      const void *d_rowptr, int rowptr_is_64, const int32_t *d_colidx,
-                                      const void *d_vals, int is_fp64, nitro_spmv **out_local) {
+nitro_status_t nitro_dist_spmv_create_ex(nitro_dist *D, int64_t global_rows, const int64_t *bounds, int64_t local_nnz,
+                                         const void *d_rowptr, int rowptr_is_64, const int32_t *d_colidx,
+                                         const void *d_vals, int is_fp64, int exchange, nitro_spmv **out_local) {
   try {
-    if (!D || !bounds || !d_rowptr || !out_local || local_nnz < 0) return fail(NITRO_E_INVALID_ARG, "bad argument");
+    if (!D || !bounds || !d_rowptr || !out_local || local_nnz < 0 || exchange < -1 || exchange > 1)
+      return fail(NITRO_E_INVALID_ARG, "bad argument");
     *out_local = nullptr;
     const int P = D->nranks, r = D->rank;
     for (int q = 0; q < P; ++q)
@@ -185,9 +360,7 @@ nitro_status_t nitro_dist_spmv_create(nitro_dist *D, int64_t global_rows, const 
     st->row_begin = bounds[r];
     st->n = bounds[r + 1] - bounds[r];
     for (int q = 0; q < P; ++q) st->B = std::max(st->B, bounds[q + 1] - bounds[q]);
-    if ((int64_t)P * st->B > 2147483647LL) { free_state(st); return fail(NITRO_E_UNSUPPORTED, "P*B must be < 2^31"); }
     const size_t sv = is_fp64 ? 8 : 4;
-    cudaStream_t s = nullptr;
     auto bail = [&](nitro_status_t code) { free_state(st); return code; };
     // features handle over the original columns (global rows start at row_begin)
     nitro_status_t rc = nitro_spmv_create(D->device, nullptr, st->n, global_rows, local_nnz, d_rowptr, rowptr_is_64,
@@ -195,24 +368,50 @@ nitro_status_t nitro_dist_spmv_create(nitro_dist *D, int64_t global_rows, const 
     if (rc) return bail(rc);
     st->feat->row0 = st->row_begin;
     st->feat->feat_G = global_rows - 1;
+    // ---- exchange mode: halo when the largest halo is < 1/4 of the all-gather volume
+    if ((rc = halo_list(st, d_colidx, local_nnz, st->halo_cols, st->nh))) return bail(rc);
+    int64_t max_nh = st->nh;
+    if (D->comm && P > 1) {
+      DevBuf t;
+      if ((rc = t.alloc(8))) return bail(rc);
+      NITRO_CUDA(cudaMemcpy(t.p, &max_nh, 8, cudaMemcpyHostToDevice));
+      NITRO_NCCL(ncclAllReduce(t.p, t.p, 1, ncclInt64, ncclMax, D->comm, D->comm_stream));
+      NITRO_CUDA(cudaStreamSynchronize(D->comm_stream));
+      NITRO_CUDA(cudaMemcpy(&max_nh, t.p, 8, cudaMemcpyDeviceToHost));
+    }
+    st->mode = exchange == -1 ? (4 * max_nh < (int64_t)(P - 1) * st->B || P == 1 ? kHalo : kAllGather) : exchange;
+    if (st->mode == kAllGather && (int64_t)P * st->B > 2147483647LL)
+      return bail(fail(NITRO_E_UNSUPPORTED, "all-gather layout needs P*B < 2^31"));
+    if (st->mode == kHalo) {
+      if (st->n + st->nh > 2147483647LL) return bail(fail(NITRO_E_UNSUPPORTED, "n + halo must be < 2^31"));
+      if ((rc = halo_plan(st))) return bail(rc);
+      if ((rc = st->sendbuf.alloc((size_t)std::max<int64_t>(st->ns, 1) * sv))) return bail(rc);
+    }
     // remapped columns
     if ((rc = st->colmap.alloc(std::max<int64_t>(local_nnz, 1) * 4))) return bail(rc);
-    DevBuf dbounds;
-    if ((rc = dbounds.alloc((P + 1) * 8))) return bail(rc);
-    NITRO_CUDA(cudaMemcpy(dbounds.p, bounds, (P + 1) * 8, cudaMemcpyHostToDevice));
-    if (local_nnz > 0)
-      k_remap<<<grid_n(local_nnz), 256, 0, s>>>(d_colidx, local_nnz, dbounds.as<int64_t>(), P, st->B,
-                                                 st->colmap.as<int32_t>());
+    if (local_nnz > 0) {
+      if (st->mode == kHalo) {
+        k_remap_halo<<<grid_n(local_nnz), 256>>>(d_colidx, local_nnz, bounds[r], bounds[r + 1], st->n,
+                                                 st->halo_cols.as<int32_t>(), st->nh, st->colmap.as<int32_t>());
+      } else {
+        DevBuf dbounds;
+        if ((rc = dbounds.alloc((P + 1) * 8))) return bail(rc);
+        NITRO_CUDA(cudaMemcpy(dbounds.p, bounds, (P + 1) * 8, cudaMemcpyHostToDevice));
+        k_remap_ag<<<grid_n(local_nnz), 256>>>(d_colidx, local_nnz, dbounds.as<int64_t>(), P, st->B,
+                                               st->colmap.as<int32_t>());
+        NITRO_CUDA(cudaDeviceSynchronize());
+      }
+    }
     // interior rows (all columns inside this rank's block) -> contiguous run [i0, i1)
     std::vector<uint8_t> hf(st->n);
     if (st->n > 0) {
       if ((rc = st->flags.alloc(st->n))) return bail(rc);
       if (rowptr_is_64)
-        k_interior<int64_t><<<grid_n(st->n), 256, 0, s>>>((const int64_t *)d_rowptr, d_colidx, st->n, bounds[r],
-                                                          bounds[r + 1], st->flags.as<uint8_t>());
+        k_interior<int64_t><<<grid_n(st->n), 256>>>((const int64_t *)d_rowptr, d_colidx, st->n, bounds[r],
+                                                    bounds[r + 1], st->flags.as<uint8_t>());
       else
-        k_interior<int32_t><<<grid_n(st->n), 256, 0, s>>>((const int32_t *)d_rowptr, d_colidx, st->n, bounds[r],
-                                                          bounds[r + 1], st->flags.as<uint8_t>());
+        k_interior<int32_t><<<grid_n(st->n), 256>>>((const int32_t *)d_rowptr, d_colidx, st->n, bounds[r],
+                                                    bounds[r + 1], st->flags.as<uint8_t>());
       NITRO_CUDA(cudaGetLastError());
       NITRO_CUDA(cudaMemcpy(hf.data(), st->flags.p, st->n, cudaMemcpyDeviceToHost));
     }
@@ -222,9 +421,9 @@ nitro_status_t nitro_dist_spmv_create(nitro_dist *D, int64_t global_rows, const 
     while (i1 < st->n && hf[i1]) ++i1;
     st->i0 = i0;
     st->i1 = i1;
+    const int64_t Mx = st->layout_len(), xoff = st->x_offset();
     // three part handles over rebased CSR slices with remapped columns
     const int64_t beg[3] = {0, i0, i1}, end[3] = {i0, i1, st->n};
-    std::vector<int64_t> hrp(4, 0);
     for (int k = 0; k < 3; ++k) {
       const int64_t cnt = end[k] - beg[k];
       st->part_begin[k] = beg[k];
@@ -243,27 +442,26 @@ nitro_status_t nitro_dist_spmv_create(nitro_dist *D, int64_t global_rows, const 
       if (pz > 2147483647LL) return bail(fail(NITRO_E_UNSUPPORTED, "a rank part needs < 2^31 nonzeros"));
       if ((rc = st->rp_part[k].alloc((cnt + 1) * 4))) return bail(rc);
       if (rowptr_is_64)
-        k_rebase<int64_t><<<grid_n(cnt + 1), 256, 0, s>>>((const int64_t *)d_rowptr, beg[k], cnt, st->rp_part[k].as<int32_t>());
+        k_rebase<int64_t><<<grid_n(cnt + 1), 256>>>((const int64_t *)d_rowptr, beg[k], cnt, st->rp_part[k].as<int32_t>());
       else
-        k_rebase<int32_t><<<grid_n(cnt + 1), 256, 0, s>>>((const int32_t *)d_rowptr, beg[k], cnt, st->rp_part[k].as<int32_t>());
+        k_rebase<int32_t><<<grid_n(cnt + 1), 256>>>((const int32_t *)d_rowptr, beg[k], cnt, st->rp_part[k].as<int32_t>());
       NITRO_CUDA(cudaGetLastError());
-      rc = nitro_spmv_create(D->device, nullptr, cnt, (int64_t)P * st->B, pz, st->rp_part[k].p, 0,
-                             st->colmap.as<int32_t>() + ab[0], (const char *)d_vals + ab[0] * sv, is_fp64,
-                             &st->part[k]);
+      rc = nitro_spmv_create(D->device, nullptr, cnt, Mx, pz, st->rp_part[k].p, 0, st->colmap.as<int32_t>() + ab[0],
+                             (const char *)d_vals + ab[0] * sv, is_fp64, &st->part[k]);
       if (rc) return bail(rc);
-      st->part[k]->row0 = (int64_t)r * st->B + beg[k];  // rows in the remapped space keep diagonal offsets
+      st->part[k]->row0 = xoff + beg[k];  // local row i sits at layout index xoff + i: diagonal offsets kept
     }
-    if ((rc = st->xfull.alloc(std::max<int64_t>((int64_t)P * st->B, 1) * sv))) return bail(rc);
-    // padding rows of every block stay 0: padded formats (DIA) multiply their
-    // zero slots by x there, so it must be finite
-    NITRO_CUDA(cudaMemset(st->xfull.p, 0, st->xfull.bytes));
+    if ((rc = st->xbuf.alloc(std::max<int64_t>(Mx, 1) * sv))) return bail(rc);
+    // padding / not-yet-exchanged entries stay 0: padded formats (DIA) multiply
+    // their zero slots by x there, so it must be finite
+    NITRO_CUDA(cudaMemset(st->xbuf.p, 0, st->xbuf.bytes));
     NITRO_CUDA(cudaDeviceSynchronize());
     // the returned handle: the whole local block over remapped columns
     nitro_spmv *A = nullptr;
-    rc = nitro_spmv_create(D->device, nullptr, st->n, (int64_t)P * st->B, local_nnz, d_rowptr, rowptr_is_64,
-                           st->colmap.as<int32_t>(), d_vals, is_fp64, &A);
+    rc = nitro_spmv_create(D->device, nullptr, st->n, Mx, local_nnz, d_rowptr, rowptr_is_64, st->colmap.as<int32_t>(),
+                           d_vals, is_fp64, &A);
     if (rc) return bail(rc);
-    A->row0 = (int64_t)r * st->B;
+    A->row0 = xoff;
     A->dist = D;
     A->dist_state = st;
     A->dist_free = free_state;
@@ -274,15 +472,11 @@ nitro_status_t nitro_dist_spmv_create(nitro_dist *D, int64_t global_rows, const 
   }
 }
 
-static nitro_status_t run_part(DistState *st, int k, int variant, cudaStream_t s, const void *xg, void *y,
-                               size_t sv) {
-  nitro_spmv *P = st->part[k];
-  if (!P) return NITRO_OK;
-  P->stream = s;
-  int ok = 0, v = variant;
-  NITRO_TRY(nitro_spmv_allowed(P, v, &ok));
-  if (!ok) v = NITRO_CSR_VECTOR;  // part-level constraint fallback (P:L134)
-  return nitro_spmv_run(P, v, xg, (char *)y + (size_t)st->part_begin[k] * sv);
+nitro_status_t nitro_dist_spmv_create(nitro_dist *D, int64_t global_rows, const int64_t *bounds, int64_t local_nnz,
+                                      const void *d_rowptr, int rowptr_is_64, const int32_t *d_colidx,
+                                      const void *d_vals, int is_fp64, nitro_spmv **out_local) {
+  return nitro_dist_spmv_create_ex(D, global_rows, bounds, local_nnz, d_rowptr, rowptr_is_64, d_colidx, d_vals,
+                                   is_fp64, -1, out_local);
 }
 
 nitro_status_t nitro_dist_spmv_run(nitro_dist *D, nitro_spmv *A, int variant, const void *d_x_local, void *d_y_local) {
@@ -293,19 +487,37 @@ nitro_status_t nitro_dist_spmv_run(nitro_dist *D, nitro_spmv *A, int variant, co
   NITRO_CUDA(cudaSetDevice(D->device));
   const size_t sv = A->fp64 ? 8 : 4;
   cudaStream_t s = A->stream;
-  char *xfull = st->xfull.as<char>();
-  char *mine = xfull + (size_t)D->rank * st->B * sv;
-  if (st->n > 0) NITRO_CUDA(cudaMemcpyAsync(mine, d_x_local, st->n * sv, cudaMemcpyDeviceToDevice, s));
+  char *xb = st->xbuf.as<char>();
+  char *mine = xb + (size_t)st->x_offset() * sv;
+  if (st->n > 0 && d_x_local != mine)  // callers that write x in place (nitro_dist_x_local) skip this copy
+    NITRO_CUDA(cudaMemcpyAsync(mine, d_x_local, st->n * sv, cudaMemcpyDeviceToDevice, s));
+  const ncclDataType_t dt = A->fp64 ? ncclFloat64 : ncclFloat32;
+  if (st->mode == kHalo && st->ns > 0) {
+    if (A->fp64) k_pack<double><<<grid_n(st->ns), 256, 0, s>>>((const double *)mine, st->send_idx.as<int32_t>(), st->ns, st->sendbuf.as<double>());
+    else k_pack<float><<<grid_n(st->ns), 256, 0, s>>>((const float *)mine, st->send_idx.as<int32_t>(), st->ns, st->sendbuf.as<float>());
+    NITRO_CUDA(cudaGetLastError());
+  }
   NITRO_CUDA(cudaEventRecord(D->ev_x, s));
   NITRO_CUDA(cudaStreamWaitEvent(D->comm_stream, D->ev_x, 0));
-  if (D->nranks > 1)
-    NITRO_NCCL(ncclAllGather(mine, xfull, (size_t)st->B, A->fp64 ? ncclFloat64 : ncclFloat32, D->comm,
-                             D->comm_stream));
+  if (D->nranks > 1) {
+    if (st->mode == kAllGather) {
+      NITRO_NCCL(ncclAllGather(mine, xb, (size_t)st->B, dt, D->comm, D->comm_stream));
+    } else {
+      NITRO_NCCL(ncclGroupStart());
+      for (int q = 0; q < D->nranks; ++q) {
+        if (q == D->rank) continue;
+        const int64_t sc = st->send_off[q + 1] - st->send_off[q], rc = st->recv_off[q + 1] - st->recv_off[q];
+        if (sc > 0) NITRO_NCCL(ncclSend(st->sendbuf.as<char>() + (size_t)st->send_off[q] * sv, sc, dt, q, D->comm, D->comm_stream));
+        if (rc > 0) NITRO_NCCL(ncclRecv(xb + (size_t)(st->n + st->recv_off[q]) * sv, rc, dt, q, D->comm, D->comm_stream));
+      }
+      NITRO_NCCL(ncclGroupEnd());
+    }
+  }
   NITRO_CUDA(cudaEventRecord(D->ev_g, D->comm_stream));
-  NITRO_TRY(run_part(st, 1, variant, s, xfull, d_y_local, sv));  // interior: overlaps the all-gather
+  NITRO_TRY(run_part(st, 1, variant, s, xb, d_y_local, sv));  // interior: overlaps the exchange
   NITRO_CUDA(cudaStreamWaitEvent(s, D->ev_g, 0));
-  NITRO_TRY(run_part(st, 0, variant, s, xfull, d_y_local, sv));
-  NITRO_TRY(run_part(st, 2, variant, s, xfull, d_y_local, sv));
+  NITRO_TRY(run_part(st, 0, variant, s, xb, d_y_local, sv));
+  NITRO_TRY(run_part(st, 2, variant, s, xb, d_y_local, sv));
   return NITRO_OK;
 }
 
@@ -329,15 +541,28 @@ nitro_status_t nitro_dist_layout(nitro_spmv *A, int64_t *B, int64_t *i0, int64_t
   return NITRO_OK;
 }
 
-nitro_status_t nitro_dist_init_local(int rank, int nranks, int device, nitro_dist **out) {
-  if (!out || nranks < 1 || rank < 0 || rank >= nranks) return fail(NITRO_E_INVALID_ARG, "bad argument");
-  NITRO_CUDA(cudaSetDevice(device));
-  nitro_dist *D = new nitro_dist();
-  D->rank = rank; D->nranks = nranks; D->device = device;
-  NITRO_CUDA(cudaStreamCreateWithFlags(&D->comm_stream, cudaStreamNonBlocking));
-  NITRO_CUDA(cudaEventCreateWithFlags(&D->ev_x, cudaEventDisableTiming));
-  NITRO_CUDA(cudaEventCreateWithFlags(&D->ev_g, cudaEventDisableTiming));
-  *out = D;
+nitro_status_t nitro_dist_exchange_info(nitro_spmv *A, int *mode, int64_t *layout_len, int64_t *halo_len,
+                                        int64_t *send_len) {
+  if (!A || !A->dist_state) return fail(NITRO_E_INVALID_ARG, "not a dist handle");
+  DistState *st = (DistState *)A->dist_state;
+  if (mode) *mode = st->mode;
+  if (layout_len) *layout_len = st->layout_len();
+  if (halo_len) *halo_len = st->nh;
+  if (send_len) *send_len = st->ns;
+  return NITRO_OK;
+}
+
+nitro_status_t nitro_dist_halo_cols(nitro_spmv *A, int32_t *h_out) {
+  if (!A || !A->dist_state) return fail(NITRO_E_INVALID_ARG, "not a dist handle");
+  DistState *st = (DistState *)A->dist_state;
+  if (h_out && st->nh) NITRO_CUDA(cudaMemcpy(h_out, st->halo_cols.p, st->nh * 4, cudaMemcpyDeviceToHost));
+  return NITRO_OK;
+}
+
+nitro_status_t nitro_dist_x_local(nitro_spmv *A, void **ptr) {
+  if (!A || !A->dist_state || !ptr) return fail(NITRO_E_INVALID_ARG, "not a dist handle");
+  DistState *st = (DistState *)A->dist_state;
+  *ptr = st->xbuf.as<char>() + (size_t)st->x_offset() * (A->fp64 ? 8 : 4);
   return NITRO_OK;
 }
 

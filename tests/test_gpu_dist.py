@@ -55,7 +55,7 @@ def test_emulated_ranks_match_single_gpu(cuda, name, A, P):
     for q in range(P):
         D = n.Dist.local(q, P, 0)
         blk = synth.to_device(block(A, bounds[q], bounds[q + 1]), cuda)
-        Mq = D.spmv(A.rows, bounds, blk.rowptr, blk.colidx, blk.vals)
+        Mq = D.spmv(A.rows, bounds, blk.rowptr, blk.colidx, blk.vals, exchange=0)
         assert n.Dist.layout(Mq)[0] == B
         ranks.append((D, Mq, blk))
     tol = 1e-12 if A.fp64 else 1e-5
@@ -90,7 +90,7 @@ def test_interior_run_of_stencil_slabs(cuda):
     for q in range(4):
         D = n.Dist.local(q, 4, 0)
         blk = synth.to_device(block(A, bounds[q], bounds[q + 1]), cuda)
-        Mq = D.spmv(A.rows, bounds, blk.rowptr, blk.colidx, blk.vals)
+        Mq = D.spmv(A.rows, bounds, blk.rowptr, blk.colidx, blk.vals, exchange=0)
         B, i0, i1 = n.Dist.layout(Mq)
         assert B == nx ** 3
         assert i0 == (0 if q == 0 else nx * nx)
@@ -114,6 +114,81 @@ def test_nccl_single_rank(cuda):
         y1 = M1.run(v, xd)
         yd = torch.empty_like(y1)
         D.run(Md, v, xd, yd)
+        torch.cuda.synchronize()
+        assert torch.equal(y1, yd), v
+    D.close()
+
+
+@pytest.mark.parametrize("P", [2, 4, 8])
+@pytest.mark.parametrize("name,A", list(mats()))
+def test_emulated_ranks_halo_layout(cuda, name, A, P):
+    """Halo exchange: each rank's layout is [x_local | x[halo]],
+    halo = the sorted remote columns its rows reference."""
+    import torch
+    n = nitro()
+    x = synth.vector(A.cols, seed=12, fp64=A.fp64)
+    y_ref, r = oracle.spmv(A, x)
+    xd = torch.from_numpy(x).to(cuda)
+    rp = np.asarray(A.rowptr, np.int64)
+    bounds = n.dist_partition(rp, P)
+    tol = 1e-12 if A.fp64 else 1e-5
+    ranks = []
+    for q in range(P):
+        lo, hi = int(bounds[q]), int(bounds[q + 1])
+        D = n.Dist.local(q, P, 0)
+        blk = synth.to_device(block(A, lo, hi), cuda)
+        Mq = D.spmv(A.rows, bounds, blk.rowptr, blk.colidx, blk.vals, exchange=1)
+        info = n.Dist.exchange_info(Mq)
+        H = n.Dist.halo_cols(Mq)
+        a, b = rp[lo], rp[hi]
+        cols = np.asarray(A.colidx[a:b], np.int64)
+        want = np.unique(cols[(cols < lo) | (cols >= hi)])
+        assert info["mode"] == "halo" and np.array_equal(H, want)
+        assert info["layout_len"] == (hi - lo) + len(H)
+        xe = torch.cat([xd[lo:hi], xd[torch.from_numpy(H.astype(np.int64)).to(cuda)]]) if len(H) else xd[lo:hi].clone()
+        ranks.append((D, Mq, blk, xe))
+    for v in range(n.NUM_VARIANTS):
+        ys = []
+        for D, Mq, blk, xe in ranks:
+            yq = torch.full((Mq.rows,), float("nan"), dtype=xd.dtype, device=cuda)
+            D.run_gathered(Mq, v, xe, yq)
+            ys.append(yq)
+        yd = torch.cat(ys)
+        torch.cuda.synchronize()
+        err = np.abs(yd.cpu().numpy().astype(np.float64) - y_ref)
+        assert np.all(err <= tol * r + 1e-30), (name, P, v)
+
+
+def test_halo_is_small_for_stencil_slabs(cuda):
+    """3D 27-point z-slabs: the halo is the neighbouring plane(s), so auto mode picks it."""
+    n = nitro()
+    nx = 16
+    A = synth.stencil("3d27", (nx, nx, 4 * nx), mode=1, seed=1)
+    bounds = np.array([q * nx ** 3 for q in range(5)], np.int64)
+    for q in range(4):
+        D = n.Dist.local(q, 4, 0)
+        blk = synth.to_device(block(A, bounds[q], bounds[q + 1]), cuda)
+        Mq = D.spmv(A.rows, bounds, blk.rowptr, blk.colidx, blk.vals)   # auto
+        info = n.Dist.exchange_info(Mq)
+        assert info["mode"] == "halo"
+        assert info["halo_len"] == nx * nx * (1 if q in (0, 3) else 2)
+
+
+def test_nccl_single_rank_halo_in_place_x(cuda):
+    import torch
+    n = nitro()
+    A = synth.stencil("3d27", 24, mode=1, seed=5)
+    x = synth.vector(A.cols, seed=6)
+    Ad = synth.to_device(A, cuda)
+    M1 = n.SpMV.from_csr(Ad)
+    D = n.Dist(n.dist_unique_id(), 0, 1, 0)
+    Md = D.spmv(A.rows, np.array([0, A.rows], np.int64), Ad.rowptr, Ad.colidx, Ad.vals, exchange=1)
+    xl = n.Dist.x_local(Md)             # write x straight into the exchange buffer: no copy per multiply
+    xl.copy_(torch.from_numpy(x).to(cuda))
+    for v in range(5):
+        y1 = M1.run(v, xl)
+        yd = torch.empty_like(y1)
+        D.run(Md, v, xl, yd)
         torch.cuda.synchronize()
         assert torch.equal(y1, yd), v
     D.close()
