@@ -175,8 +175,10 @@ def run_nitro(args):
     else:
         D = _dist_setup(nitro, dist if world > 1 else None, rank, world, local)
         bounds = np.array([r * n * n * n for r in range(world + 1)], dtype=np.int64)
-        M = D.spmv(A.cols, bounds, A.rowptr, A.colidx, A.vals)
-        x = x_local
+        M = D.spmv(A.cols, bounds, A.rowptr, A.colidx, A.vals, exchange=args.exchange)
+        exch = nitro.Dist.exchange_info(M)
+        x = nitro.Dist.x_local(M)      # x lives inside the exchange buffer: no per-multiply copy
+        x.copy_(x_local)
 
     # --- one end-to-end pass of the hot path (features -> select -> prepare -> run)
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -330,7 +332,8 @@ def run_nitro(args):
         "data": "synthetic",
         "config": {"workload": WORKLOAD if world == 1 else f"3d27pt_stencil_128x128x{128 * world}_fp32 (128^3 rows/rank)",
                    "rows_per_gpu": N, "nnz_per_gpu": Z, "l2": "flushed between steps (read of 3x L2)",
-                   "parallelism": "single GPU" if not use_dist else f"row-partitioned x{world}, NCCL x all-gather",
+                   "parallelism": "single GPU" if not use_dist else
+                   f"row-partitioned x{world}, NCCL x {exch['mode']} ({exch['halo_len']} halo entries/rank)",
                    "selection": selection, "selected_variant": vname},
         "selected_variant": vname,
         "gflops": 2.0 * Z * world / (ms * 1e-3) / 1e9,
@@ -377,6 +380,7 @@ def main():
     ap.add_argument("--impl", default="nitro", choices=["nitro", "reference"])
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--dist", action="store_true", help="use the multi-GPU (NCCL) code path even at N=1")
+    ap.add_argument("--exchange", type=int, default=-1, help="multi-GPU x exchange: -1 auto, 0 all-gather, 1 halo")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     if args.impl == "reference":

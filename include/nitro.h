@@ -309,7 +309,7 @@ nitro_status_t nitro_dist_spmv_create(nitro_dist *D, int64_t global_rows, const 
                                       nitro_spmv **out_local);
 /* Same, choosing the x exchange: -1 auto (halo when the largest per-rank halo
  * is < 1/4 of the all-gather volume), 0 all-gather (layout: P*B padded
- * blocks), 1 halo (layout: [x_local (n) | halo (nh)], grouped send/recv of
+ * blocks), 1 halo (layout: [x[halo < lo] | x_local | x[halo >= hi]], monotone in the global column; grouped send/recv of
  * only the referenced remote entries).  Collective when the
  * handle has a communicator (every rank must call it). */
 nitro_status_t nitro_dist_spmv_create_ex(nitro_dist *D, int64_t global_rows, const int64_t *bounds,
@@ -332,7 +332,7 @@ nitro_status_t nitro_dist_spmv_run(nitro_dist *D, nitro_spmv *A_local, int varia
                                    void *d_y_local);
 /* Same multiply from an x that is already exchanged into this handle's layout
  * (all-gather: block q at q*B, B = max block rows, length nranks*B; halo:
- * [x_local | x[halo_cols]]; padding entries must be finite, e.g. 0, because
+ * [x[halo below] | x_local | x[halo above]]; padding entries must be finite, e.g. 0, because
  * padded formats multiply zero slots by them): no communication.
  * Used when the caller owns the exchange (e.g. a solver that writes y straight
  * into the next x), and to check every rank's part on one GPU. */

@@ -51,14 +51,16 @@ struct DistState {
   std::vector<int64_t> bounds;
   DevBuf colmap, rp_part[3], xbuf, flags;
   // halo mode
-  int64_t nh = 0, ns = 0;
+  int64_t nh = 0, ns = 0, nb = 0;           // halo entries, send entries, halo entries below lo
   std::vector<int64_t> recv_off, send_off;  // [P+1] offsets into the halo / send lists
   DevBuf halo_cols, send_idx, sendbuf;
   nitro_spmv *part[3] = {nullptr, nullptr, nullptr};
   nitro_spmv *feat = nullptr;  // original global columns, for global features
   int64_t part_begin[3] = {0, 0, 0};
   int64_t layout_len() const { return mode == kHalo ? n + nh : (int64_t)D->nranks * B; }
-  int64_t x_offset() const { return mode == kHalo ? 0 : (int64_t)D->rank * B; }
+  int64_t x_offset() const { return mode == kHalo ? nb : (int64_t)D->rank * B; }
+  // layout index of halo position k (halo mode)
+  int64_t halo_dest(int64_t k) const { return k < nb ? k : n + k; }
 };
 
 void free_state(void *p) {
@@ -88,18 +90,20 @@ __global__ void k_remap_ag(const int32_t *__restrict__ col, int64_t Z, const int
   }
 }
 
-// halo layout: local c -> c - lo; remote c -> n + position of c in the sorted halo list
+// halo layout [x[H_below] | x_local | x[H_above]] (monotone in the global
+// column, so remapped rows stay sorted): c < lo -> its position k in the sorted
+// halo list H; local c -> nb + (c - lo); c >= hi -> n + k  (nb = |H_below|)
 __global__ void k_remap_halo(const int32_t *__restrict__ col, int64_t Z, int64_t lo, int64_t hi, int64_t n,
-                             const int32_t *__restrict__ H, int64_t nh, int32_t *__restrict__ out) {
+                             int64_t nb, const int32_t *__restrict__ H, int64_t nh, int32_t *__restrict__ out) {
   for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < Z; k += (int64_t)gridDim.x * blockDim.x) {
     const int64_t c = col[k];
-    if (c >= lo && c < hi) { out[k] = (int32_t)(c - lo); continue; }
+    if (c >= lo && c < hi) { out[k] = (int32_t)(nb + c - lo); continue; }
     int64_t a = 0, b = nh;
     while (a < b) {
       const int64_t m = (a + b) >> 1;
       if ((int64_t)H[m] < c) a = m + 1; else b = m;
     }
-    out[k] = (int32_t)(n + a);
+    out[k] = (int32_t)(c < lo ? a : n + a);
   }
 }
 
@@ -225,6 +229,7 @@ nitro_status_t halo_plan(DistState *st) {
     while (k < (int)st->nh && H[k] < st->bounds[q + 1]) ++k;
     st->recv_off[q + 1] = k;
   }
+  st->nb = st->recv_off[me];  // halo entries owned by lower ranks (columns < lo)
   st->send_off.assign(P + 1, 0);
   st->ns = 0;
   if (!D->comm || P == 1) return NITRO_OK;  // communicator-less: the caller supplies the layout
@@ -391,7 +396,7 @@ nitro_status_t nitro_dist_spmv_create_ex(nitro_dist *D, int64_t global_rows, con
     if ((rc = st->colmap.alloc(std::max<int64_t>(local_nnz, 1) * 4))) return bail(rc);
     if (local_nnz > 0) {
       if (st->mode == kHalo) {
-        k_remap_halo<<<grid_n(local_nnz), 256>>>(d_colidx, local_nnz, bounds[r], bounds[r + 1], st->n,
+        k_remap_halo<<<grid_n(local_nnz), 256>>>(d_colidx, local_nnz, bounds[r], bounds[r + 1], st->n, st->nb,
                                                  st->halo_cols.as<int32_t>(), st->nh, st->colmap.as<int32_t>());
       } else {
         DevBuf dbounds;
@@ -508,7 +513,8 @@ nitro_status_t nitro_dist_spmv_run(nitro_dist *D, nitro_spmv *A, int variant, co
         if (q == D->rank) continue;
         const int64_t sc = st->send_off[q + 1] - st->send_off[q], rc = st->recv_off[q + 1] - st->recv_off[q];
         if (sc > 0) NITRO_NCCL(ncclSend(st->sendbuf.as<char>() + (size_t)st->send_off[q] * sv, sc, dt, q, D->comm, D->comm_stream));
-        if (rc > 0) NITRO_NCCL(ncclRecv(xb + (size_t)(st->n + st->recv_off[q]) * sv, rc, dt, q, D->comm, D->comm_stream));
+        if (rc > 0)
+          NITRO_NCCL(ncclRecv(xb + (size_t)st->halo_dest(st->recv_off[q]) * sv, rc, dt, q, D->comm, D->comm_stream));
       }
       NITRO_NCCL(ncclGroupEnd());
     }

@@ -145,7 +145,9 @@ def test_emulated_ranks_halo_layout(cuda, name, A, P):
         want = np.unique(cols[(cols < lo) | (cols >= hi)])
         assert info["mode"] == "halo" and np.array_equal(H, want)
         assert info["layout_len"] == (hi - lo) + len(H)
-        xe = torch.cat([xd[lo:hi], xd[torch.from_numpy(H.astype(np.int64)).to(cuda)]]) if len(H) else xd[lo:hi].clone()
+        Hd = torch.from_numpy(H.astype(np.int64)).to(cuda)
+        below = int((H < lo).sum())
+        xe = torch.cat([xd[Hd[:below]], xd[lo:hi], xd[Hd[below:]]])   # [x[H_below] | x_local | x[H_above]]
         ranks.append((D, Mq, blk, xe))
     for v in range(n.NUM_VARIANTS):
         ys = []
