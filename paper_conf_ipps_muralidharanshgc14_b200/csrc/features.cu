@@ -191,15 +191,21 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
             if (cur == kEmpty) { free_slot = slot; break; }
           }
         }
-        const unsigned need = __ballot_sync(kFull, want);
-        if (want) {
-          const unsigned grp = __match_any_sync(need, idx);
-          if ((int)(__ffs(grp) - 1) == lane) {
-            // test before set: an L2 read is far cheaper than a contended RED
-            const uint32_t bit = 1u << (idx & 31);
-            if (!(__ldcg(bitmap + (idx >> 5)) & bit)) atomicOr(bitmap + (idx >> 5), bit);
-            if (free_slot >= 0) atomicCAS(&s_seen[free_slot], kEmpty, idx);
-            else if (!s_full) s_full = 1;  // probe run full: stop using the set
+        const bool saturated = s_full != 0;  // random offsets: dedupe would not pay
+        if (saturated) {
+          // fire-and-forget OR per entry: no match_any, no dependent L2 read
+          if (want) atomicOr(bitmap + (idx >> 5), 1u << (idx & 31));
+        } else {
+          const unsigned need = __ballot_sync(kFull, want);
+          if (want) {
+            const unsigned grp = __match_any_sync(need, idx);
+            if ((int)(__ffs(grp) - 1) == lane) {
+              // test before set: an L2 read is far cheaper than a contended RED
+              const uint32_t bit = 1u << (idx & 31);
+              if (!(__ldcg(bitmap + (idx >> 5)) & bit)) atomicOr(bitmap + (idx >> 5), bit);
+              if (free_slot >= 0) atomicCAS(&s_seen[free_slot], kEmpty, idx);
+              else if (!s_full) s_full = 1;  // probe run full: stop using the set
+            }
           }
         }
         cur_rl = __shfl_sync(kFull, rl, nvalid - 1);
