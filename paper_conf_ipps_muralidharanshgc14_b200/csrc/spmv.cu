@@ -22,12 +22,21 @@ template <> struct V4<float> {
     float4 t = ld_stream_f4(reinterpret_cast<const float4 *>(p));
     v[0] = t.x; v[1] = t.y; v[2] = t.z; v[3] = t.w;
   }
+  __device__ __forceinline__ void load(const float *p, uint64_t pol) {
+    float4 t = ld_stream_f4(reinterpret_cast<const float4 *>(p), pol);
+    v[0] = t.x; v[1] = t.y; v[2] = t.z; v[3] = t.w;
+  }
 };
 template <> struct V4<double> {
   double v[4];
   __device__ __forceinline__ void load(const double *p) {
     double2 a = ld_stream_d2(reinterpret_cast<const double2 *>(p));
     double2 b = ld_stream_d2(reinterpret_cast<const double2 *>(p) + 1);
+    v[0] = a.x; v[1] = a.y; v[2] = b.x; v[3] = b.y;
+  }
+  __device__ __forceinline__ void load(const double *p, uint64_t pol) {
+    double2 a = ld_stream_d2(reinterpret_cast<const double2 *>(p), pol);
+    double2 b = ld_stream_d2(reinterpret_cast<const double2 *>(p) + 1, pol);
     v[0] = a.x; v[1] = a.y; v[2] = b.x; v[3] = b.y;
   }
 };
@@ -262,7 +271,8 @@ __global__ void __launch_bounds__(256) k_csr_vector(const IT *__restrict__ rowpt
 template <typename VT, int U>  // U <= 16: terms per fp32 partial
 __global__ void __launch_bounds__(256) k_ell(const int32_t *__restrict__ ecol, const VT *__restrict__ eval,
                                              const VT *__restrict__ x, VT *__restrict__ y, int64_t N, int64_t K,
-                                             int64_t ld) {
+                                             int64_t ld, bool l2ef) {
+  const uint64_t pol = l2_policy(l2ef);
   const int64_t nq = ld >> 2;
   for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nq; q += (int64_t)gridDim.x * blockDim.x) {
     const int64_t i0 = q << 2;
@@ -273,8 +283,8 @@ __global__ void __launch_bounds__(256) k_ell(const int32_t *__restrict__ ecol, c
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         if (k0 + u < K) {
-          c[u] = ld_stream_i4(reinterpret_cast<const int4 *>(ecol + (k0 + u) * ld + i0));
-          v[u].load(eval + (k0 + u) * ld + i0);
+          c[u] = ld_stream_i4(reinterpret_cast<const int4 *>(ecol + (k0 + u) * ld + i0), pol);
+          v[u].load(eval + (k0 + u) * ld + i0, pol);
         } else {
           c[u] = make_int4(-1, -1, -1, -1);
           v[u].v[0] = v[u].v[1] = v[u].v[2] = v[u].v[3] = (VT)0;
@@ -504,9 +514,11 @@ template <typename VT, int EP>
 __global__ void __launch_bounds__(256) k_hyb_tail_ls(const int32_t *__restrict__ trow, const int32_t *__restrict__ tcol,
                                                      const VT *__restrict__ tval, const VT *__restrict__ x,
                                                      VT *__restrict__ y, int64_t Zt, int64_t nch,
-                                                     int32_t *__restrict__ carry_row, double *__restrict__ carry_val) {
+                                                     int32_t *__restrict__ carry_row, double *__restrict__ carry_val,
+                                                     bool l2ef) {
   static_assert(EP == 4 || EP == 8, "EP");
   constexpr int64_t CH = 32 * EP;
+  const uint64_t pol = l2_policy(l2ef);
   const int lane = threadIdx.x & 31;
   const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -519,21 +531,21 @@ __global__ void __launch_bounds__(256) k_hyb_tail_ls(const int32_t *__restrict__
     if (nv == EP) {  // full lane: vector loads (e0 is a multiple of EP, arrays 16-byte aligned)
 #pragma unroll
       for (int k = 0; k < EP; k += 4) {
-        const int4 rr = ld_stream_i4(reinterpret_cast<const int4 *>(trow + e0 + k));
-        const int4 cc = ld_stream_i4(reinterpret_cast<const int4 *>(tcol + e0 + k));
+        const int4 rr = ld_stream_i4(reinterpret_cast<const int4 *>(trow + e0 + k), pol);
+        const int4 cc = ld_stream_i4(reinterpret_cast<const int4 *>(tcol + e0 + k), pol);
         r[k] = rr.x; r[k + 1] = rr.y; r[k + 2] = rr.z; r[k + 3] = rr.w;
         c[k] = cc.x; c[k + 1] = cc.y; c[k + 2] = cc.z; c[k + 3] = cc.w;
         V4<VT> vv;
-        vv.load(tval + e0 + k);
+        vv.load(tval + e0 + k, pol);
         v[k] = vv.v[0]; v[k + 1] = vv.v[1]; v[k + 2] = vv.v[2]; v[k + 3] = vv.v[3];
       }
     } else {
 #pragma unroll
       for (int k = 0; k < EP; ++k) {
         const bool ok = k < nv;
-        r[k] = ok ? ld_stream_i(trow + e0 + k) : -2;
-        c[k] = ok ? ld_stream_i(tcol + e0 + k) : 0;
-        v[k] = ok ? ld_stream(tval + e0 + k) : (VT)0;
+        r[k] = ok ? ld_stream_i(trow + e0 + k, pol) : -2;
+        c[k] = ok ? ld_stream_i(tcol + e0 + k, pol) : 0;
+        v[k] = ok ? ld_stream(tval + e0 + k, pol) : (VT)0;
       }
     }
     double p[EP];
@@ -667,6 +679,15 @@ int dia_split(int64_t D) {
   return 1;
 }
 
+// streamed matrix arrays use an L2 evict-first policy (NITRO_L2EF=0 disables)
+bool l2_evict_first() {
+  static bool v = [] {
+    const char *e = getenv("NITRO_L2EF");
+    return e ? atoi(e) != 0 : true;
+  }();
+  return v;
+}
+
 // ELL slot batch width: NITRO_ELL_U overrides (1/2/4/8); default 2.  B200 sweep
 // on configs[1] (fp32): U=2 6372, U=4 5461, U=8 4681 GB/s — fewer registers and
 // more resident warps beat deeper per-thread batches for this gather pattern.
@@ -687,10 +708,10 @@ void launch_ell(const int32_t *col, const VT *val, const VT *x, VT *y, int64_t N
                 cudaStream_t s) {
   const unsigned g = grid_cap((ld / 4 + 255) / 256, 16);
   switch (ell_batch(sizeof(VT))) {
-    case 1: k_ell<VT, 1><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld); break;
-    case 2: k_ell<VT, 2><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld); break;
-    case 4: k_ell<VT, 4><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld); break;
-    default: k_ell<VT, 8><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld); break;
+    case 1: k_ell<VT, 1><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, l2_evict_first()); break;
+    case 2: k_ell<VT, 2><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, l2_evict_first()); break;
+    case 4: k_ell<VT, 4><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, l2_evict_first()); break;
+    default: k_ell<VT, 8><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, l2_evict_first()); break;
   }
 }
 
@@ -783,7 +804,8 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
 #define NITRO_TAIL_LS(WW)                                                                                      \
   k_hyb_tail_ls<VT, WW><<<gt, 256, 0, s>>>(A->hyb.trow.as<int32_t>(), A->hyb.tcol.as<int32_t>(),                \
                                            A->hyb.tval.as<VT>(), x, y, A->hyb.Zt, A->hyb.nchunks,               \
-                                           A->hyb.carry_row.as<int32_t>(), A->hyb.carry_val.as<double>())
+                                           A->hyb.carry_row.as<int32_t>(), A->hyb.carry_val.as<double>(),     \
+                                           l2_evict_first())
           static const bool ls = [] {
             const char *e = getenv("NITRO_HYB_LS");
             return e ? atoi(e) != 0 : true;
