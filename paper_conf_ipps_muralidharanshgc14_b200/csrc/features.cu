@@ -88,19 +88,13 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
     if (E1 - E0 <= kStage && Lmax_blk <= kRowCap) {
       int *buf = s_stage[wib];
       const int span = (int)(E1 - E0);
-      for (int e0 = 0; e0 < span; e0 += 128) {
-        int v[4];
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          const int e = e0 + u * 32 + lane;
-          v[u] = e < span ? ld_stream_i(col + E0 + e) : 0;
-        }
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          const int e = e0 + u * 32 + lane;
-          if (e < span) buf[e] = v[u];
-        }
-      }
+      // cp.async (LDGSTS): the whole span is in flight at once, no registers,
+      // one memory round trip per block of rows
+      for (int e = lane; e < span; e += 32)
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"((uint32_t)__cvta_generic_to_shared(buf + e)),
+                     "l"(col + E0 + e)
+                     : "memory");
+      asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
       __syncwarp();
       const int rel0 = (int)(a - E0);
       const uint32_t myrow = rowbase + (uint32_t)lane;

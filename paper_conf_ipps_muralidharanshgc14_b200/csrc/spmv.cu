@@ -130,8 +130,9 @@ __global__ void __launch_bounds__(256) k_csr_vector(const IT *__restrict__ rowpt
                                                     VT *__restrict__ y, int64_t N, int64_t nseg,
                                                     const int32_t *__restrict__ seg_row,
                                                     const int32_t *__restrict__ seg_k, double *seg_part,
-                                                    unsigned *seg_ctr) {
+                                                    unsigned *seg_ctr, bool l2ef) {
   constexpr int64_t T = 8 * V;
+  const uint64_t pol = l2_policy(l2ef);
   {
     constexpr int64_t S = kCsrvSeg;
     const int lane = threadIdx.x & 31;
@@ -146,8 +147,8 @@ __global__ void __launch_bounds__(256) k_csr_vector(const IT *__restrict__ rowpt
 #pragma unroll
       for (int u = 0; u < 8; ++u) {
         const int64_t e = st + u * 32 + lane;
-        c[u] = e < en ? ld_stream_i(col + e) : -1;
-        v[u] = e < en ? ld_stream(val + e) : (VT)0;
+        c[u] = e < en ? ld_stream_i(col + e, pol) : -1;
+        v[u] = e < en ? ld_stream(val + e, pol) : (VT)0;
       }
       VT part = 0;
 #pragma unroll
@@ -212,8 +213,8 @@ __global__ void __launch_bounds__(256) k_csr_vector(const IT *__restrict__ rowpt
 #pragma unroll
     for (int u = 0; u < R; ++u) {
       const bool in = li < st.l[u];
-      st.c[u] = in ? ld_stream_i(col + t.abase + st.s[u] + li) : -1;
-      st.v[u] = in ? ld_stream(val + t.abase + st.s[u] + li) : (VT)0;
+      st.c[u] = in ? ld_stream_i(col + t.abase + st.s[u] + li, pol) : -1;
+      st.v[u] = in ? ld_stream(val + t.abase + st.s[u] + li, pol) : (VT)0;
     }
   };
   auto finish = [&](const Tile &t, int64_t tt, int tb, Stage &st) {
@@ -223,7 +224,7 @@ __global__ void __launch_bounds__(256) k_csr_vector(const IT *__restrict__ rowpt
 #pragma unroll
     for (int u = 0; u < R; ++u)
       for (int m = V + li; m < st.l[u]; m += V)  // <= 7 more terms per lane
-        part[u] = fma(ld_stream(val + t.abase + st.s[u] + m), __ldg(x + ld_stream_i(col + t.abase + st.s[u] + m)),
+        part[u] = fma(ld_stream(val + t.abase + st.s[u] + m, pol), __ldg(x + ld_stream_i(col + t.abase + st.s[u] + m, pol)),
                       part[u]);
     int ridx;
     const VT tot = reduce_transpose<V, R>(part, li, ridx);
@@ -325,8 +326,9 @@ __global__ void __launch_bounds__(256, (U == 1 && sizeof(VT) == 4) ? 8 : 1)  // 
     k_dia(const int32_t *__restrict__ offs, const VT *__restrict__ dval,
                                              const VT *__restrict__ x, VT *__restrict__ y, int64_t N, int64_t M,
                                              int64_t D, int64_t ld, int64_t row0, int64_t off_min, int64_t off_max,
-                                             bool x_aligned) {
+                                             bool x_aligned, bool l2ef) {
   constexpr int64_t RB = 1024 / DS;  // rows per block iteration
+  const uint64_t pol = l2_policy(l2ef);
   extern __shared__ int s_off[];
   for (int64_t d = threadIdx.x; d < D; d += blockDim.x) s_off[d] = offs[d];
   __syncthreads();
@@ -349,7 +351,7 @@ __global__ void __launch_bounds__(256, (U == 1 && sizeof(VT) == 4) ? 8 : 1)  // 
       VT xv[U][4];
 #pragma unroll
       for (int u = 0; u < U; ++u) {
-        if (d0 + u < D) v[u].load(dval + (d0 + u) * ld + i0);
+        if (d0 + u < D) v[u].load(dval + (d0 + u) * ld + i0, pol);
         else v[u].v[0] = v[u].v[1] = v[u].v[2] = v[u].v[3] = (VT)0;
       }
       if (sizeof(VT) == 4 && xvec) {
@@ -753,7 +755,7 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
       // 8 warps x 32 rows per block-iteration; segments are spread over all warps
       const unsigned g = grid_cap(std::max<int64_t>((N + 255) / 256, (nseg + 7) / 8), 8);
 #define NITRO_CSRV(VV)                                                                                      \
-  k_csr_vector<VV, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, nseg, seg_row, seg_k, seg_part, seg_ctr)
+  k_csr_vector<VV, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, nseg, seg_row, seg_k, seg_part, seg_ctr, l2_evict_first())
       switch (A->csrv.V) {
         case 2: NITRO_CSRV(2); break;
         case 4: NITRO_CSRV(4); break;
@@ -776,7 +778,7 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
         const unsigned g = grid_cap((A->dia.ld + 1024 / DS - 1) / (1024 / DS), 16);
 #define NITRO_DIA_LAUNCH(UU, SS)                                                                                   \
   k_dia<VT, UU, SS><<<g, 256, sm, s>>>(A->dia.off.as<int32_t>(), A->dia.val.as<VT>(), x, y, N, A->M, A->dia.D,     \
-                                       A->dia.ld, A->row0, A->dia.off_min, A->dia.off_max, x_al)
+                                       A->dia.ld, A->row0, A->dia.off_min, A->dia.off_max, x_al, l2_evict_first())
 #define NITRO_DIA_U(SS)                      \
   switch (U) {                               \
     case 2: NITRO_DIA_LAUNCH(2, SS); break;  \
