@@ -265,6 +265,27 @@ def run_nitro(args):
         ms = float(t.item())
     gbps = nbytes * world / (ms * 1e-3) / 1e9
 
+    # --- size-matched ceiling: a device copy moving the same byte count (half read,
+    # half write), timed the same way (L2 flushed, median of 20): at 242 MB the
+    # DRAM ramp/drain is a visible share of a ~45 us kernel
+    copy_gbps = None
+    if world == 1:
+        half = max(nbytes // 8, 1)
+        ca = torch.ones(half, dtype=torch.float32, device=dev)
+        cb = torch.empty_like(ca)
+        cts = []
+        for i in range(23):
+            M.flush_l2()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            cb.copy_(ca)
+            b.record(stream)
+            b.synchronize()
+            if i >= 3:
+                cts.append(a.elapsed_time(b))
+        copy_gbps = 8 * half / (statistics.median(cts) * 1e-3) / 1e9
+        del ca, cb
+
     # --- e2e through the C ABI with host buffers (pinned), copies inside the timed region
     e2e = None
     hx = torch.empty(N, dtype=torch.float32).pin_memory()
@@ -345,6 +366,8 @@ def run_nitro(args):
         "roofline": {"bound": "hbm", "achieved": per_gpu, "peak": peak, "unit": "GB/s", "frac": per_gpu / peak,
                      "traffic": traffic, "peak_kind": f"{pk_kind} hbm_gbs (copy)",
                      "kernel": f"{vname} ({launches} launch/step)",
+                     "size_matched_copy_gbs": copy_gbps,
+                     "frac_of_size_matched_copy": (per_gpu / copy_gbps) if copy_gbps else None,
                      "bytes_per_launch": nbytes},
         "gpu_launches": args.steps * (launches + 1),
         "gpu_launches_note": f"{args.steps} x ({launches} SpMV + 1 L2-flush) kernels of libnitro",

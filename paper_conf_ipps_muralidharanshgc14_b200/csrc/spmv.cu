@@ -125,7 +125,7 @@ __device__ __forceinline__ VT reduce_transpose(VT (&p)[R], int li, int &ridx) {
 // tiles.  A multi-segment row's partials are summed in segment order by the
 // last warp to finish one of its segments (deterministic, no float atomics).
 template <int V, typename IT, typename VT>
-__global__ void __launch_bounds__(256) k_csr_vector(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
+__global__ void __launch_bounds__(256, sizeof(VT) == 4 ? 4 : 3) k_csr_vector(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
                                                     const VT *__restrict__ val, const VT *__restrict__ x,
                                                     VT *__restrict__ y, int64_t N, int64_t nseg,
                                                     const int32_t *__restrict__ seg_row,
@@ -322,7 +322,7 @@ __global__ void __launch_bounds__(256) k_ell(const int32_t *__restrict__ ecol, c
 // (value, x) loads is DS times shorter; the DS partial sums are combined by a
 // fixed xor butterfly (deterministic).
 template <typename VT, int U, int DS>
-__global__ void __launch_bounds__(256, (U == 1 && sizeof(VT) == 4) ? 8 : 1)  // U=1 fp32: <= 32 regs, full occupancy
+__global__ void __launch_bounds__(256, (U == 1 && DS == 1 && sizeof(VT) == 4) ? 8 : 1)  // U=1 fp32: <= 32 regs, full occupancy
     k_dia(const int32_t *__restrict__ offs, const VT *__restrict__ dval,
                                              const VT *__restrict__ x, VT *__restrict__ y, int64_t N, int64_t M,
                                              int64_t D, int64_t ld, int64_t row0, int64_t off_min, int64_t off_max,
@@ -681,6 +681,16 @@ int dia_split(int64_t D) {
   return 1;
 }
 
+// DIA grid cap in blocks per SM: NITRO_DIA_GRID overrides; default 16
+// (one wave-free launch of every 1024-row block at configs[1])
+int dia_blocks_per_sm() {
+  static int env = [] {
+    const char *e = getenv("NITRO_DIA_GRID");
+    return e ? atoi(e) : 0;
+  }();
+  return env > 0 ? env : 16;
+}
+
 // streamed matrix arrays use an L2 evict-first policy (NITRO_L2EF=0 disables)
 bool l2_evict_first() {
   static bool v = [] {
@@ -755,7 +765,7 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
       // 8 warps x 32 rows per block-iteration; segments are spread over all warps
       const unsigned g = grid_cap(std::max<int64_t>((N + 255) / 256, (nseg + 7) / 8), 8);
 #define NITRO_CSRV(VV)                                                                                      \
-  k_csr_vector<VV, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, nseg, seg_row, seg_k, seg_part, seg_ctr, l2_evict_first())
+  k_csr_vector<VV, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, nseg, seg_row, seg_k, seg_part, seg_ctr, l2_evict_first() && VV >= 16)
       switch (A->csrv.V) {
         case 2: NITRO_CSRV(2); break;
         case 4: NITRO_CSRV(4); break;
@@ -775,7 +785,7 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
         const size_t sm = (size_t)std::max<int64_t>(A->dia.D, 1) * 4;
         const bool x_al = ((reinterpret_cast<uintptr_t>(x) & 15) == 0) && (A->row0 % 4 == 0);
         const int U = dia_batch(A->dia.D, sizeof(VT)), DS = dia_split(A->dia.D);
-        const unsigned g = grid_cap((A->dia.ld + 1024 / DS - 1) / (1024 / DS), 16);
+        const unsigned g = grid_cap((A->dia.ld + 1024 / DS - 1) / (1024 / DS), dia_blocks_per_sm());
 #define NITRO_DIA_LAUNCH(UU, SS)                                                                                   \
   k_dia<VT, UU, SS><<<g, 256, sm, s>>>(A->dia.off.as<int32_t>(), A->dia.val.as<VT>(), x, y, N, A->M, A->dia.D,     \
                                        A->dia.ld, A->row0, A->dia.off_min, A->dia.off_max, x_al, l2_evict_first())

@@ -18,6 +18,8 @@ def make(cfg, dev):
         return synth.stencil("2d5", 64, device=dev)
     if cfg == "c1":
         return synth.stencil("3d27", 128, mode=1, seed=1, device=dev)
+    if cfg == "c1big":   # 3D 27-pt 256^3: the asymptotic (ramp-free) DIA/ELL rate
+        return synth.stencil("3d27", 256, mode=1, seed=1, device=dev)
     if cfg == "c2a":
         return synth.uniform(1 << 23, 32, seed=5, device=dev)
     if cfg == "c2b":
@@ -34,7 +36,7 @@ def main():
     args = sys.argv[1:]
     timing = "--time" in args
     args = [a for a in args if a != "--time"]
-    cfgs = [a for a in args if a in ("c0", "c1", "c2a", "c2b", "short")] or ["c1"]
+    cfgs = [a for a in args if a in ("c0", "c1", "c1big", "c2a", "c2b", "short")] or ["c1"]
     want = [nitro.VARIANT_NAMES.index(v) for v in args if v in nitro.VARIANT_NAMES] or list(range(5))
     dev = torch.device("cuda:0")
     table = {}
