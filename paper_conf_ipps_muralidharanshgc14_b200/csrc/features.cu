@@ -8,17 +8,23 @@
 // bit for bit.
 //
 // Layout of the pass: a warp owns 32 consecutive rows (lane j <-> row j, row
-// lengths from two coalesced rowptr loads), then streams the rows' colidx
-// range [rowptr[r0], rowptr[r0+32]) with coalesced 32-entry windows.  The row
-// of each entry is recovered in O(1) per window from a head mask
-// (__reduce_or_sync of 1<<(row start - window base)) and a per-warp row slot
-// table, so short and long rows cost the same per entry.  Occupied diagonals
-// go to a bitmap over the offset range; a per-block direct-mapped cache of
-// recently set offsets plus __match_any_sync dedupe keep the atomics off the
-// hot words (a 3D stencil hits only 27 offsets with 3.6e9 entries).
+// lengths from two coalesced rowptr loads).  Rows of up to kRowCap entries are
+// walked by their own lane (row id known, no shuffles), from a shared-memory
+// copy of the rows' colidx span when it fits (cp.async, bank-skewed), else
+// straight from global memory in 8-entry batches.  Longer rows are walked by
+// the whole warp, 32 coalesced entries at a time; rows longer than kLong are
+// deferred to k_features_long, which splits them into kChunk-entry chunks
+// spread over every warp of the grid (an R-MAT hub row of 1.5e5 entries would
+// otherwise serialise on one warp).  Occupied diagonals go to a bitmap over the
+// offset range: near-diagonal offsets through a per-block shared-memory window,
+// the rest through a per-block set of offsets already set (until it fills up:
+// random matrices) and fire-and-forget global ORs, merged per 32-bit word
+// across a warp's window by a segmented OR scan (a dense row then costs one
+// OR per word, not per entry).
 #include "nitro_internal.h"
 #include "util.cuh"
 
+#include <algorithm>
 #include <cmath>
 
 namespace nitro {
@@ -30,21 +36,149 @@ constexpr int kCache = 1024;            // per-block open-addressing offset set 
 constexpr int kProbe = 4;               // linear-probe length
 constexpr uint32_t kWin = 1u << 16;     // per-block bitmap of offsets in [-2^15, 2^15) (8 KB)
 constexpr uint32_t kEmpty = 0xffffffffu;
-constexpr int kStage = 1024;            // per-warp staging buffer (entries) of the short-row path
-constexpr int kRowCap = 64;             // rows longer than this use the windowed path
+constexpr int kStage = 1024;            // per-warp staging buffer (entries)
+constexpr int kRowCap = 64;             // lane-per-row walk only for rows up to this length
+constexpr int64_t kLong = 4096;         // rows longer than this go to k_features_long
+constexpr int64_t kChunk = 4096;        // entries per task of k_features_long
+
+// staging slot of span entry e: one pad word per 32 entries, so lanes walking
+// rows of 32 (or 16, 8 ...) entries hit distinct banks
+__device__ __forceinline__ int skew(int e) { return e + (e >> 5); }
+
+// The offset bits of one 32-entry window held one per lane (key = bitmap word
+// or kEmpty, bits = its bit): a segmented inclusive OR scan merges runs of
+// equal adjacent keys, and the last lane of each run issues one global OR (a
+// dense row costs one OR per word, not per entry).
+__device__ __forceinline__ void or_window(uint32_t key, uint32_t bits, int lane, uint32_t *__restrict__ bitmap) {
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t tb = __shfl_up_sync(kFull, bits, o);
+    const uint32_t tk = __shfl_up_sync(kFull, key, o);
+    if (lane >= o && tk == key) bits |= tb;
+  }
+  const uint32_t nk = __shfl_down_sync(kFull, key, 1);
+  if (key != kEmpty && (lane == 31 || nk != key)) atomicOr(bitmap + key, bits);
+}
+
+// Offset index idx of an entry -> near-diagonal window bit (shared) or a
+// (key, bits) pair for or_window.
+__device__ __forceinline__ void classify(uint32_t idx, uint32_t win_lo, uint32_t *s_win, uint32_t &key,
+                                         uint32_t &bits) {
+  const uint32_t rel = idx - win_lo;
+  if (s_win && rel < kWin) {
+    const uint32_t bit = 1u << (rel & 31);
+    if (!(s_win[rel >> 5] & bit)) atomicOr(&s_win[rel >> 5], bit);
+  } else {
+    key = idx >> 5;
+    bits = 1u << (idx & 31);
+  }
+}
+
+// Whole-warp walk of one row's entries [st, en) (row start a, global row grow):
+// canonical checks against the previous entry, offsets to the window / bitmap.
+__device__ __forceinline__ void walk_row_warp(const int32_t *__restrict__ col, int64_t st, int64_t en, int64_t a,
+                                              uint32_t grow, uint32_t G32, uint32_t M32, uint32_t win_lo,
+                                              uint32_t *s_win, uint32_t *__restrict__ bitmap, int lane,
+                                              unsigned &bad) {
+  int last_c = st > a ? __ldg(col + st - 1) : -1;
+  for (int64_t base = st; base < en; base += 128) {
+    int c[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int64_t e = base + u * 32 + lane;
+      c[u] = e < en ? ld_stream_i(col + e) : 0;
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int64_t w0 = base + u * 32;
+      if (w0 >= en) break;  // warp-uniform
+      int prevc = __shfl_up_sync(kFull, c[u], 1);
+      if (lane == 0) prevc = last_c;
+      uint32_t key = kEmpty, bits = 0;
+      if (w0 + lane < en) {
+        if ((uint32_t)c[u] >= M32) bad |= 4;  // also catches c < 0
+        else {
+          if (c[u] <= prevc) bad |= 2;
+          classify((uint32_t)c[u] - grow + G32, win_lo, s_win, key, bits);
+        }
+      }
+      or_window(key, bits, lane, bitmap);
+      last_c = __shfl_sync(kFull, c[u], 31);
+    }
+  }
+}
+
+// Whole-warp walk of the contiguous entry range [st, en) of the rows
+// (lanes) flagged in_run of a 32-row block, entries from the staging buffer
+// (SMEM, slots relative to E0) or global memory.  The row of each entry comes
+// from the head mask of the window (bit p set <=> a row starts at window entry
+// p, __reduce_or_sync) and a per-warp table head position -> lane.
+template <bool SMEM>
+__device__ __forceinline__ void walk_span_warp(const int32_t *__restrict__ src, int64_t st, int64_t en, int64_t E0,
+                                               int64_t a, bool in_run, uint32_t rowbase, uint32_t G32,
+                                               uint32_t M32, uint32_t win_lo, uint32_t *s_win, int8_t *slot,
+                                               uint32_t *__restrict__ bitmap, int lane, unsigned &bad) {
+  int cur_rl = 0, last_c = 0;
+  for (int64_t base = st; base < en; base += 128) {
+    int c[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int64_t e = base + u * 32 + lane;
+      c[u] = e < en ? (SMEM ? src[skew((int)(e - E0))] : ld_stream_i(src + e)) : 0;
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int64_t w0 = base + u * 32;
+      if (w0 >= en) break;  // warp-uniform
+      const int nvalid = en - w0 < 32 ? (int)(en - w0) : 32;
+      const int64_t pos = a - w0;
+      const bool head = in_run && pos >= 0 && pos < nvalid;
+      const unsigned mask = __reduce_or_sync(kFull, head ? (1u << (unsigned)pos) : 0u);
+      if (head) slot[pos] = (int8_t)lane;  // in_run excludes empty rows: one head per position
+      __syncwarp();
+      const unsigned hm = mask & (kFull >> (31 - lane));
+      const int rl = hm ? (int)slot[31 - __clz(hm)] : cur_rl;
+      int prevc = __shfl_up_sync(kFull, c[u], 1);
+      if (lane == 0) prevc = last_c;
+      uint32_t key = kEmpty, bits = 0;
+      if (lane < nvalid) {
+        if ((uint32_t)c[u] >= M32) bad |= 4;
+        else {
+          if (!((mask >> lane) & 1u) && c[u] <= prevc) bad |= 2;
+          classify((uint32_t)c[u] - (rowbase + (uint32_t)rl) + G32, win_lo, s_win, key, bits);
+        }
+      }
+      or_window(key, bits, lane, bitmap);
+      cur_rl = __shfl_sync(kFull, rl, nvalid - 1);
+      last_c = __shfl_sync(kFull, c[u], nvalid - 1);
+      __syncwarp();
+    }
+  }
+}
+
+// merge a block's near-diagonal window into the global bitmap (nonzero words only)
+__device__ __forceinline__ void merge_window(const uint32_t *s_win, uint32_t win_lo, int64_t span,
+                                             uint32_t *__restrict__ bitmap) {
+  for (int i = threadIdx.x; i < (int)(kWin / 32); i += blockDim.x) {
+    uint32_t w = s_win[i];
+    while (w) {
+      const int bpos = __ffs(w) - 1;
+      w &= w - 1;
+      const uint32_t gidx = win_lo + (uint32_t)(i * 32 + bpos);
+      if ((int64_t)gidx < span) atomicOr(bitmap + (gidx >> 5), 1u << (gidx & 31));
+    }
+  }
+}
 
 // Offset index idx = col - row + G is < 2^32 (rows, cols < 2^31), so all
-// per-entry arithmetic is 32-bit.  Near-diagonal offsets (stencils, banded)
-// are recorded in a shared-memory bitmap window (LDS + rare shared atomic per
-// entry); the rest go through a small shared-memory set of offsets already in
-// the global bitmap and a test-before-set global OR.  Blocks whose set fills
-// up (random matrices) stop probing it.
+// per-entry arithmetic is 32-bit.
 template <typename IT>
 __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
                                                         int64_t N, int64_t M, int64_t Z, int64_t row0, int64_t G,
-                                                        FeatAcc *__restrict__ acc, uint32_t *__restrict__ bitmap) {
+                                                        FeatAcc *__restrict__ acc, uint32_t *__restrict__ bitmap,
+                                                        int2 *__restrict__ tasks) {
+  __shared__ int s_stage[kWarps][kStage + kStage / 32];
   __shared__ int8_t s_slot[kWarps][32];
-  __shared__ int s_stage[kWarps][kStage];
   __shared__ uint32_t s_seen[kCache];
   __shared__ uint32_t s_win[kWin / 32];
   __shared__ unsigned long long s_red[3][kWarps];
@@ -61,6 +195,27 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     if ((int64_t)rowptr[0] != 0 || (int64_t)rowptr[N] != Z) bad |= 1;
   }
+  // a far (off-window) offset of a lane-walked row: shared offset set (until it
+  // fills: full), then a fire-and-forget global OR (no returned value, so no
+  // dependent L2 round trip)
+  auto lane_far = [&](uint32_t idx, bool full) {
+    if (full) { atomicOr(bitmap + (idx >> 5), 1u << (idx & 31)); return; }
+    bool hit = false;
+    int free_slot = -1;
+    const uint32_t h = idx * 0x9E3779B1u >> 22;
+    for (int p = 0; p < kProbe; ++p) {
+      const int slot = (int)((h + p) & (kCache - 1));
+      const uint32_t cur = s_seen[slot];
+      if (cur == idx) { hit = true; break; }
+      if (cur == kEmpty) { free_slot = slot; break; }
+    }
+    if (!hit) {
+      atomicOr(bitmap + (idx >> 5), 1u << (idx & 31));
+      if (free_slot >= 0) atomicCAS(&s_seen[free_slot], kEmpty, idx);
+      else s_full = 1;
+    }
+  };
+
   unsigned long long s1 = 0, s2 = 0, lmax = 0;
   const int64_t nblk = (N + 31) / 32;
   const int64_t gw = (int64_t)blockIdx.x * kWarps + wib, nw = (int64_t)gridDim.x * kWarps;
@@ -79,134 +234,78 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
     const bool brk = L < 0 || a < 0 || b > Z;
     if (__any_sync(kFull, brk)) { bad |= brk ? 1u : 0u; continue; }
     const int64_t E0 = __shfl_sync(kFull, a, 0), E1 = __shfl_sync(kFull, b, 31);
-    const uint32_t rowbase = (uint32_t)(row0 + rb * 32);  // global row of lane 0's row
-    const bool lane_has = L > 0;
-    // ---- fast path (short rows, e.g. stencils / banded): stage the block's
-    // colidx span in shared memory with coalesced loads, then every lane walks
-    // its own row (row id known, ~10 instructions per entry, no shuffles)
-    const int Lmax_blk = (int)__reduce_max_sync(kFull, (unsigned)(L > kRowCap ? kRowCap + 1 : L));
-    if (E1 - E0 <= kStage && Lmax_blk <= kRowCap) {
-      int *buf = s_stage[wib];
-      const int span = (int)(E1 - E0);
+    const uint32_t rowbase = (uint32_t)(row0 + rb * 32), myrow = rowbase + (uint32_t)lane;
+    // long rows: their kChunk-entry chunks become tasks of k_features_long
+    const bool is_long = L > kLong;
+    if (is_long) {
+      const int nc = (int)((L + kChunk - 1) / kChunk);
+      const unsigned t0 = atomicAdd(&acc->nlong, (unsigned)nc);
+      for (int j = 0; j < nc; ++j) tasks[t0 + j] = make_int2((int)r, j);
+    }
+    const unsigned long_mask = __ballot_sync(kFull, is_long);
+    const bool staged = E1 - E0 <= kStage;  // implies no long row
+    int *buf = s_stage[wib];
+    if (staged) {
       // cp.async (LDGSTS): the whole span is in flight at once, no registers,
       // one memory round trip per block of rows
+      const int span = (int)(E1 - E0);
       for (int e = lane; e < span; e += 32)
-        asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"((uint32_t)__cvta_generic_to_shared(buf + e)),
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"((uint32_t)__cvta_generic_to_shared(buf + skew(e))),
                      "l"(col + E0 + e)
                      : "memory");
       asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
       __syncwarp();
-      const int rel0 = (int)(a - E0);
-      const uint32_t myrow = rowbase + (uint32_t)lane;
-      int prev = -1;
-      for (int k = 0; k < (int)L; ++k) {
-        const int c = buf[rel0 + k];
-        if ((uint32_t)c >= M32) { bad |= 4; continue; }
-        if (c <= prev) bad |= 2;
-        prev = c;
-        const uint32_t idx = (uint32_t)c - myrow + G32;
-        const uint32_t rel = idx - win_lo;
-        if (rel < kWin) {
-          const uint32_t bit = 1u << (rel & 31);
-          if (!(s_win[rel >> 5] & bit)) atomicOr(&s_win[rel >> 5], bit);
-        } else {
-          // far from the diagonal: shared offset set, then test-before-set global OR
-          bool hit = false;
-          int free_slot = -1;
-          if (!s_full) {
-            const uint32_t h = idx * 0x9E3779B1u >> 22;
-            for (int p = 0; p < kProbe; ++p) {
-              const int slot = (int)((h + p) & (kCache - 1));
-              const uint32_t cur = s_seen[slot];
-              if (cur == idx) { hit = true; break; }
-              if (cur == kEmpty) { free_slot = slot; break; }
-            }
-          }
-          if (!hit) {
-            // fire-and-forget OR (no returned value, so no per-entry dependent
-            // L2 round trip in this per-lane sequential loop)
-            atomicOr(bitmap + (idx >> 5), 1u << (idx & 31));
-            if (free_slot >= 0) atomicCAS(&s_seen[free_slot], kEmpty, idx);
-            else if (!s_full) s_full = 1;
-          }
-        }
-      }
-      __syncwarp();  // the staging buffer is reused by the next block of rows
-      continue;
     }
-    int cur_rl = 0, last_c = 0;
-    for (int64_t base = E0; base < E1; base += 128) {
-      int c[4];
-#pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        const int64_t e = base + u * 32 + lane;
-        c[u] = e < E1 ? ld_stream_i(col + e) : 0;
-      }
-#pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        const int64_t w0 = base + u * 32;
-        if (w0 >= E1) break;  // warp-uniform
-        const int nvalid = E1 - w0 < 32 ? (int)(E1 - w0) : 32;
-        // rows whose first entry falls in this window: head bit at their start
-        const int64_t pos = a - w0;
-        const bool head = lane_has && pos >= 0 && pos < 32;
-        const unsigned mask = __reduce_or_sync(kFull, head ? (1u << (unsigned)pos) : 0u);
-        if (head) s_slot[wib][pos] = (int8_t)lane;
-        __syncwarp();
-        const unsigned hm = mask & (kFull >> (31 - lane));
-        const int rl = hm ? (int)s_slot[wib][31 - __clz(hm)] : cur_rl;
-        int prevc = __shfl_up_sync(kFull, c[u], 1);
-        if (lane == 0) prevc = last_c;
-        uint32_t idx = kEmpty;
-        if (lane < nvalid) {
-          if ((uint32_t)c[u] >= M32) bad |= 4;  // also catches c < 0
-          else {
-            if (!((mask >> lane) & 1u) && c[u] <= prevc) bad |= 2;
-            idx = (uint32_t)c[u] - (rowbase + (uint32_t)rl) + G32;
-          }
-        }
-        bool want = idx != kEmpty;
-        if (want) {
+    // lane per row when the rows are short and of similar length (stencils,
+    // uniform rows: no divergence), else the whole warp over the entry span
+    const int64_t Ln = is_long ? 0 : L;
+    const unsigned maxL = __reduce_max_sync(kFull, (unsigned)(Ln > kRowCap ? kRowCap + 1 : Ln));
+    const unsigned sumL = __reduce_add_sync(kFull, (unsigned)(Ln > kRowCap ? kRowCap + 1 : Ln));
+    if (maxL <= (unsigned)kRowCap && maxL * 32u <= 2u * sumL) {
+      if (Ln > 0) {
+        const bool full = *(volatile unsigned *)&s_full != 0;
+        int prev = -1;
+        // per-entry body; the staged / global source is hoisted out of the loop
+        auto entry = [&](int c) {
+          if ((uint32_t)c >= M32) { bad |= 4; return; }
+          if (c <= prev) bad |= 2;
+          prev = c;
+          const uint32_t idx = (uint32_t)c - myrow + G32;
           const uint32_t rel = idx - win_lo;
           if (rel < kWin) {
             const uint32_t bit = 1u << (rel & 31);
             if (!(s_win[rel >> 5] & bit)) atomicOr(&s_win[rel >> 5], bit);
-            want = false;
+          } else {
+            lane_far(idx, full);
           }
-        }
-        int free_slot = -1;
-        if (want && !s_full) {
-          const uint32_t h = idx * 0x9E3779B1u >> 22;  // 10-bit hash
-#pragma unroll
-          for (int p = 0; p < kProbe; ++p) {
-            const int slot = (int)((h + p) & (kCache - 1));
-            const uint32_t cur = s_seen[slot];
-            if (cur == idx) { want = false; break; }
-            if (cur == kEmpty) { free_slot = slot; break; }
-          }
-        }
-        const bool saturated = s_full != 0;  // random offsets: dedupe would not pay
-        if (saturated) {
-          // fire-and-forget OR per entry: no match_any, no dependent L2 read
-          if (want) atomicOr(bitmap + (idx >> 5), 1u << (idx & 31));
+        };
+        if (staged) {
+          const int rel0 = (int)(a - E0);
+          for (int k = 0; k < (int)Ln; ++k) entry(buf[skew(rel0 + k)]);
         } else {
-          const unsigned need = __ballot_sync(kFull, want);
-          if (want) {
-            const unsigned grp = __match_any_sync(need, idx);
-            if ((int)(__ffs(grp) - 1) == lane) {
-              // test before set: an L2 read is far cheaper than a contended RED
-              const uint32_t bit = 1u << (idx & 31);
-              if (!(__ldcg(bitmap + (idx >> 5)) & bit)) atomicOr(bitmap + (idx >> 5), bit);
-              if (free_slot >= 0) atomicCAS(&s_seen[free_slot], kEmpty, idx);
-              else if (!s_full) s_full = 1;  // probe run full: stop using the set
-            }
-          }
+          for (int k = 0; k < (int)Ln; ++k) entry(__ldg(col + a + k));
         }
-        cur_rl = __shfl_sync(kFull, rl, nvalid - 1);
-        last_c = __shfl_sync(kFull, c[u], nvalid - 1);
-        __syncwarp();
+      }
+    } else if (staged) {
+      walk_span_warp<true>(buf, E0, E1, E0, a, L > 0, rowbase, G32, M32, win_lo, s_win, s_slot[wib], bitmap, lane,
+                           bad);
+    } else {
+      // runs of consecutive non-long rows between the long ones
+      int s = 0;
+      while (s < 32) {
+        const unsigned rest = long_mask >> s;
+        const int l = rest ? s + __ffs(rest) - 1 : 32;  // first long lane at or after s
+        if (l > s) {
+          const int64_t st = __shfl_sync(kFull, a, s);
+          const int64_t en = __shfl_sync(kFull, a, l & 31);
+          const int64_t en2 = l < 32 ? en : E1;
+          walk_span_warp<false>(col, st, en2, 0, a, lane >= s && lane < l && L > 0, rowbase, G32, M32, win_lo, s_win,
+                                s_slot[wib], bitmap, lane, bad);
+        }
+        s = l + 1;
       }
     }
+    __syncwarp();  // the staging buffer is reused by the next block of rows
   }
   // reduce s1, s2 (sum) and lmax (max) over the block
 #pragma unroll
@@ -222,17 +321,7 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
     if (bad) atomicOr(&s_bad, bad);
   }
   __syncthreads();
-  // merge the near-diagonal window into the global bitmap (nonzero words only)
-  const int64_t span = G + M;
-  for (int i = threadIdx.x; i < (int)(kWin / 32); i += kThreads) {
-    uint32_t w = s_win[i];
-    while (w) {
-      const int bpos = __ffs(w) - 1;
-      w &= w - 1;
-      const uint32_t gidx = win_lo + (uint32_t)(i * 32 + bpos);
-      if ((int64_t)gidx < span) atomicOr(bitmap + (gidx >> 5), 1u << (gidx & 31));
-    }
-  }
+  merge_window(s_win, win_lo, G + M, bitmap);
   if (threadIdx.x == 0) {
     unsigned long long a1 = 0, a2 = 0, am = 0;
     for (int w = 0; w < kWarps; ++w) {
@@ -244,6 +333,30 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
     if (am) atomicMax(&acc->lmax, am);
     if (s_bad) atomicOr(&acc->bad, s_bad);
   }
+}
+
+// The long rows' chunks (row, j) listed by k_features, one warp per task,
+// grid-stride over the task list.
+template <typename IT>
+__global__ void __launch_bounds__(kThreads) k_features_long(const IT *__restrict__ rowptr,
+                                                             const int32_t *__restrict__ col, int64_t M, int64_t row0,
+                                                             int64_t G, FeatAcc *__restrict__ acc,
+                                                             uint32_t *__restrict__ bitmap,
+                                                             const int2 *__restrict__ tasks) {
+  const unsigned n = *(volatile unsigned *)&acc->nlong;
+  const int lane = threadIdx.x & 31;
+  const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const uint32_t G32 = (uint32_t)G, M32 = (uint32_t)M;
+  unsigned bad = 0;
+  for (int64_t t = gw; t < (int64_t)n; t += nw) {
+    const int2 tk = tasks[t];
+    const int64_t a = (int64_t)rowptr[tk.x], b = (int64_t)rowptr[tk.x + 1];
+    const int64_t st = a + (int64_t)tk.y * kChunk, en = st + kChunk < b ? st + kChunk : b;
+    walk_row_warp(col, st, en, a, (uint32_t)(row0 + tk.x), G32, M32, 0u, nullptr, bitmap, lane, bad);
+  }
+  bad = __reduce_or_sync(kFull, bad);
+  if (lane == 0 && bad) atomicOr(&acc->bad, bad);
 }
 
 __global__ void __launch_bounds__(256) k_popc(const uint32_t *__restrict__ bm, int64_t nwords, FeatAcc *acc) {
@@ -287,17 +400,31 @@ nitro_status_t features_launch(nitro_spmv *A) {
   FeatAcc *acc = A->feat_acc.as<FeatAcc>();
   NITRO_CUDA(cudaMemsetAsync(acc, 0, sizeof(FeatAcc), s));
   if (nwords) NITRO_CUDA(cudaMemsetAsync(A->bitmap.p, 0, (size_t)nwords * 4, s));
+
   const int64_t nblk = (A->N + 31) / 32;
   int64_t grid = (nblk + kWarps - 1) / kWarps;
   const int64_t cap = (int64_t)num_sms() * 8;
   if (grid > cap) grid = cap;
   if (grid < 1) grid = 1;
-  if (A->rp64)
+  // long-row chunk tasks: at most Z / kChunk + (number of long rows <= Z / kLong) entries
+  const int64_t cap_tasks = A->Z / kChunk + A->Z / kLong + 1;
+  NITRO_TRY(A->feat_long.alloc((size_t)cap_tasks * sizeof(int2)));
+  int2 *tasks = A->feat_long.as<int2>();
+  const unsigned glong = (unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)num_sms() * 4,
+                                                                           (A->Z / kChunk + kWarps - 1) / kWarps));
+  if (A->rp64) {
     k_features<int64_t><<<(unsigned)grid, kThreads, 0, s>>>((const int64_t *)A->rowptr, A->col, A->N, A->M, A->Z,
-                                                            A->row0, G, acc, A->bitmap.as<uint32_t>());
-  else
+                                                            A->row0, G, acc, A->bitmap.as<uint32_t>(), tasks);
+    if (A->Z > kLong)
+      k_features_long<int64_t><<<glong, kThreads, 0, s>>>((const int64_t *)A->rowptr, A->col, A->M, A->row0, G, acc,
+                                                          A->bitmap.as<uint32_t>(), tasks);
+  } else {
     k_features<int32_t><<<(unsigned)grid, kThreads, 0, s>>>((const int32_t *)A->rowptr, A->col, A->N, A->M, A->Z,
-                                                            A->row0, G, acc, A->bitmap.as<uint32_t>());
+                                                            A->row0, G, acc, A->bitmap.as<uint32_t>(), tasks);
+    if (A->Z > kLong)
+      k_features_long<int32_t><<<glong, kThreads, 0, s>>>((const int32_t *)A->rowptr, A->col, A->M, A->row0, G, acc,
+                                                          A->bitmap.as<uint32_t>(), tasks);
+  }
   if (nwords) {
     int64_t g2 = (nwords + 255) / 256;
     if (g2 > (int64_t)num_sms() * 8) g2 = (int64_t)num_sms() * 8;

@@ -44,7 +44,7 @@ struct DevBuf {
 struct FeatAcc {
   unsigned long long s1, s2, lmax;
   unsigned int bad;      // bit0 rowptr not monotone / wrong ends, bit1 unsorted/dup col, bit2 col out of range
-  unsigned int pad;
+  unsigned int nlong;    // rows deferred to the long-row pass (k_features_long)
   unsigned long long ndiag;
 };
 
@@ -92,6 +92,7 @@ struct nitro_spmv {
   nitro_spmv_feat feat{};
   nitro::DevBuf feat_acc;   // FeatAcc
   nitro::DevBuf bitmap;     // u32 words over offsets [-(N-1) .. M-1] (+row0 shift)
+  nitro::DevBuf feat_long;  // int32 row ids of the rows longer than the feature pass's kLong
   nitro::DevBuf offsets;    // int32 [ndiag] ascending
   nitro::DevBuf scratch;    // scan scratch
   nitro::FeatAcc *h_acc = nullptr;  // pinned

@@ -91,6 +91,77 @@ def test_features_int64_rowptr_and_long_row(cuda):
         assert f[k] == f_ref[k], k
 
 
+def mixed_matrix(seed=31, N=3000, M=20000, fp64=False):
+    """Every walk of the feature pass in one matrix: rows of similar short length
+    (lane per row), groups of very different lengths (whole-warp span walk),
+    medium rows, long rows of several kChunk (= 4096) chunks including exact
+    multiples, a dense row (runs of equal bitmap words), near-diagonal rows,
+    empty rows."""
+    rng = np.random.default_rng(seed)
+    lens = rng.integers(0, 10, N)
+    lens[:320] = 7                                   # 10 groups of equal short rows
+    med = rng.choice(np.arange(320, N), 60, replace=False)
+    lens[med] = rng.integers(65, 2000, 60)
+    longs = {700: 9000, 1201: 4097, 1202: 8192, 2500: 12289, 2999: 4096}
+    for r, l in longs.items():
+        lens[r] = l
+    dense = 5
+    lens[dense] = 6000
+    lens[400:460] = 0                                # empty run
+    cols = []
+    for i, l in enumerate(lens):
+        if i == dense:
+            cols.append(np.arange(100, 100 + l))
+        elif 2000 <= i < 2100 and l:
+            lo = max(0, i - 4)
+            cols.append(np.arange(lo, min(M, lo + l)))
+            lens[i] = len(cols[-1])
+        else:
+            cols.append(np.sort(rng.choice(M, l, replace=False)))
+    rp = np.zeros(N + 1, np.int64)
+    rp[1:] = np.cumsum(lens)
+    ci = np.concatenate(cols).astype(np.int32)
+    v = rng.uniform(-1, 1, rp[-1])
+    v[v == 0] = 0.5
+    return Csr(N, M, rp, ci, v.astype(np.float64 if fp64 else np.float32), fp64)
+
+
+@pytest.mark.parametrize("rp32", [True, False])
+def test_features_mixed_walks(cuda, rp32):
+    A = mixed_matrix()
+    assert oracle.is_canonical(A)
+    M, _ = handle(A, cuda, rowptr32=rp32)
+    f, f_ref = M.features(), oracle.features(A)
+    for k in FEAT_KEYS:
+        assert f[k] == f_ref[k], k
+
+
+@pytest.mark.parametrize("where", ["long_chunk_boundary", "long_dup", "medium", "short_var", "short_equal"])
+def test_non_canonical_in_every_walk(cuda, where):
+    """A broken row is caught whichever walk of the feature pass visits it."""
+    n = nitro()
+    A = mixed_matrix()
+    ci = A.colidx.copy()
+    rp = A.rowptr
+    row = {"long_chunk_boundary": 700, "long_dup": 2500, "medium": None, "short_var": None, "short_equal": 100}[where]
+    if where == "medium":
+        row = int(np.nonzero(np.diff(rp) > 64)[0][3])
+    if where == "short_var":
+        row = int(np.nonzero((np.diff(rp) >= 3) & (np.arange(A.rows) > 500) & (np.diff(rp) < 10))[0][0])
+    a = int(rp[row])
+    k = {"long_chunk_boundary": 4095, "long_dup": 8192, "short_equal": 1}.get(where, 1)
+    if where == "long_dup":
+        ci[a + k] = ci[a + k - 1]
+    else:
+        ci[a + k - 1], ci[a + k] = ci[a + k], ci[a + k - 1]
+    B = Csr(A.rows, A.cols, rp, ci, A.vals, A.fp64)
+    assert not oracle.is_canonical(B)
+    M, _ = handle(B, cuda)
+    with pytest.raises(n.NitroError) as e:
+        M.features()
+    assert e.value.code == 2
+
+
 @pytest.mark.parametrize("case", ["unsorted", "dup", "oob", "rowptr"])
 def test_non_canonical_rejected(cuda, case):
     n = nitro()

@@ -37,7 +37,7 @@ def main():
     timing = "--time" in args
     args = [a for a in args if a != "--time"]
     cfgs = [a for a in args if a in ("c0", "c1", "c1big", "c2a", "c2b", "short")] or ["c1"]
-    want = [nitro.VARIANT_NAMES.index(v) for v in args if v in nitro.VARIANT_NAMES] or list(range(5))
+    want = [] if "none" in args else ([nitro.VARIANT_NAMES.index(v) for v in args if v in nitro.VARIANT_NAMES] or list(range(5)))
     dev = torch.device("cuda:0")
     table = {}
     for cfg in cfgs:
@@ -46,13 +46,17 @@ def main():
         M = nitro.SpMV.from_csr(A)
         s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         M.features()                    # allocates the feature buffers
-        M.invalidate()                  # then time a warm feature pass
-        torch.cuda.synchronize()
-        s.record()
-        f = M.features()
-        e.record()
-        torch.cuda.synchronize()
-        feat_ms = s.elapsed_time(e)
+        fts = []
+        for _ in range(7 if timing else 1):   # then time warm feature passes (median)
+            M.invalidate()
+            M.flush_l2()
+            torch.cuda.synchronize()
+            s.record()
+            f = M.features()
+            e.record()
+            torch.cuda.synchronize()
+            fts.append(s.elapsed_time(e))
+        feat_ms = sorted(fts)[len(fts) // 2]
         x = synth.vector(A.cols, seed=2, fp64=A.fp64, device=dev)
         y = torch.empty(A.rows, dtype=x.dtype, device=dev)
         row = {"rows": A.rows, "nnz": A.nnz, "feature_ms": feat_ms,
