@@ -270,7 +270,7 @@ def run_nitro(args):
     # DRAM ramp/drain is a visible share of a ~45 us kernel
     copy_gbps = None
     if world == 1:
-        half = max(nbytes // 8, 1)
+        half = max(int(nbytes) // 8, 1)
         ca = torch.ones(half, dtype=torch.float32, device=dev)
         cb = torch.empty_like(ca)
         cts = []

@@ -241,6 +241,91 @@ nitro_status_t nitro_spmv_run(nitro_spmv *A, int variant, const void *d_x, void 
   NITRO_GUARD_END
 }
 
+}  // extern "C"
+
+namespace {
+// Row chunks of the pipelined host-buffer call: the row-separable variants
+// (CSR-scalar, ELL, DIA) of matrices of >= 2^18 rows; NITRO_RUN_HOST_CHUNKS
+// overrides the count (1 = no pipeline).
+int run_host_chunks(const nitro_spmv *A, int variant) {
+  static int env = [] {
+    const char *e = getenv("NITRO_RUN_HOST_CHUNKS");
+    return e ? atoi(e) : 0;
+  }();
+  if (variant != NITRO_CSR_SCALAR && variant != NITRO_ELL && variant != NITRO_DIA) return 1;
+  if (variant == NITRO_DIA && nitro::dia_use_tma()) return 1;
+  const int want = env > 0 ? env : 8;
+  if (want <= 1 || A->N < (int64_t)want * 32768) return 1;
+  return want;
+}
+
+// x arrives in column pieces on s_in, chunk c's multiply (rows [r_c, r_c+1))
+// starts on the handle's stream as soon as the columns its rows reference are
+// in, and its y rows leave on s_out while later chunks compute: the two copy
+// directions overlap each other and the kernels.
+nitro_status_t run_host_pipelined(nitro_spmv *A, int variant, const void *h_x, void *h_y, int nch) {
+  const size_t sv = A->fp64 ? 8 : 4;
+  if (!A->s_in) NITRO_CUDA(cudaStreamCreateWithFlags(&A->s_in, cudaStreamNonBlocking));
+  if (!A->s_out) NITRO_CUDA(cudaStreamCreateWithFlags(&A->s_out, cudaStreamNonBlocking));
+  const size_t nev = (size_t)(2 * nch + 2);
+  while (A->ev_pipe.size() < nev) {
+    cudaEvent_t e;
+    NITRO_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    A->ev_pipe.push_back(e);
+  }
+  // chunk ends: multiples of 1024 rows
+  std::vector<int64_t> ends(nch);
+  const int64_t step = round_up((A->N + nch - 1) / nch, 1024);
+  for (int c = 0; c < nch; ++c) ends[c] = std::min<int64_t>(A->N, (int64_t)(c + 1) * step);
+  ends[nch - 1] = A->N;
+  // columns each chunk needs: DIA from its offsets (+8: the aligned x windows
+  // may touch a few entries past the last one used), else from the rows
+  std::vector<int64_t> xhi(nch);
+  if (variant == NITRO_DIA) {
+    for (int c = 0; c < nch; ++c)
+      xhi[c] = std::min<int64_t>(A->M, std::max<int64_t>(0, A->row0 + ends[c] + A->dia.off_max + 8));
+  } else {
+    if (!A->xhi_ready || A->csr_xhi.size() != (size_t)nch) {
+      NITRO_TRY(csr_chunk_xhi(A, ends, A->csr_xhi));
+      A->xhi_ready = true;
+    }
+    xhi = A->csr_xhi;
+  }
+  xhi[nch - 1] = A->M;  // everything in by the last chunk
+  cudaEvent_t *ev_in = A->ev_pipe.data(), *ev_k = ev_in + nch, ev_start = ev_in[2 * nch], ev_done = ev_in[2 * nch + 1];
+  // order after earlier work on the handle's stream
+  NITRO_CUDA(cudaEventRecord(ev_start, A->stream));
+  NITRO_CUDA(cudaStreamWaitEvent(A->s_in, ev_start, 0));
+  NITRO_CUDA(cudaStreamWaitEvent(A->s_out, ev_start, 0));
+  int64_t lo = 0;
+  for (int c = 0; c < nch; ++c) {
+    const int64_t hi = std::max(lo, xhi[c]);
+    if (hi > lo)
+      NITRO_CUDA(cudaMemcpyAsync(A->xbuf.as<char>() + lo * sv, (const char *)h_x + lo * sv, (size_t)(hi - lo) * sv,
+                                 cudaMemcpyHostToDevice, A->s_in));
+    NITRO_CUDA(cudaEventRecord(ev_in[c], A->s_in));
+    lo = hi;
+  }
+  int64_t r0 = 0;
+  for (int c = 0; c < nch; ++c) {
+    NITRO_CUDA(cudaStreamWaitEvent(A->stream, ev_in[c], 0));
+    NITRO_TRY(launch_spmv_rows(A, variant, A->xbuf.p, A->ybuf.p, A->stream, r0, ends[c]));
+    NITRO_CUDA(cudaEventRecord(ev_k[c], A->stream));
+    NITRO_CUDA(cudaStreamWaitEvent(A->s_out, ev_k[c], 0));
+    if (ends[c] > r0)
+      NITRO_CUDA(cudaMemcpyAsync((char *)h_y + r0 * sv, A->ybuf.as<char>() + r0 * sv, (size_t)(ends[c] - r0) * sv,
+                                 cudaMemcpyDeviceToHost, A->s_out));
+    r0 = ends[c];
+  }
+  NITRO_CUDA(cudaEventRecord(ev_done, A->s_out));
+  NITRO_CUDA(cudaStreamWaitEvent(A->stream, ev_done, 0));
+  NITRO_CUDA(cudaStreamSynchronize(A->stream));
+  return NITRO_OK;
+}
+}  // namespace
+
+extern "C" {
+
 nitro_status_t nitro_spmv_run_host(nitro_spmv *A, int variant, const void *h_x, void *h_y) {
   NITRO_GUARD_BEGIN
   if (!A || !valid_variant(variant)) return fail(NITRO_E_INVALID_ARG, "bad argument");
@@ -250,6 +335,8 @@ nitro_status_t nitro_spmv_run_host(nitro_spmv *A, int variant, const void *h_x, 
   const size_t sv = A->fp64 ? 8 : 4;
   NITRO_TRY(A->xbuf.alloc(std::max<size_t>(A->M * sv, 16)));
   NITRO_TRY(A->ybuf.alloc(std::max<size_t>(A->N * sv, 16)));
+  const int nch = run_host_chunks(A, variant);
+  if (nch > 1) return run_host_pipelined(A, variant, h_x, h_y, nch);
   if (A->M) NITRO_CUDA(cudaMemcpyAsync(A->xbuf.p, h_x, A->M * sv, cudaMemcpyHostToDevice, A->stream));
   NITRO_TRY(launch_spmv(A, variant, A->xbuf.p, A->ybuf.p, A->stream));
   if (A->N) NITRO_CUDA(cudaMemcpyAsync(h_y, A->ybuf.p, A->N * sv, cudaMemcpyDeviceToHost, A->stream));
@@ -372,6 +459,7 @@ nitro_status_t nitro_spmv_invalidate(nitro_spmv *A) {
   NITRO_CUDA(cudaStreamSynchronize(A->stream));
   A->feat_ready = A->feat_pending = false;
   A->ell.ready = A->dia.ready = A->hyb.ready = A->csrv.ready = false;
+  A->xhi_ready = false;
   return NITRO_OK;
 }
 
@@ -397,6 +485,9 @@ void nitro_spmv_destroy(nitro_spmv *A) {
     nitro_spmv_release(A, -1);
     if (A->h_acc) cudaFreeHost(A->h_acc);
     if (A->feat_done) cudaEventDestroy(A->feat_done);
+    for (auto e : A->ev_pipe) cudaEventDestroy(e);
+    if (A->s_in) cudaStreamDestroy(A->s_in);
+    if (A->s_out) cudaStreamDestroy(A->s_out);
     A->feat_acc.release(); A->bitmap.release(); A->offsets.release(); A->scratch.release();
     A->flush.release(); A->xbuf.release(); A->ybuf.release();
     if (A->dist_free && A->dist_state) A->dist_free(A->dist_state);

@@ -2,6 +2,7 @@
 #pragma once
 
 #include <cuda_runtime.h>
+#include <vector>
 #include <stdint.h>
 
 #include <string>
@@ -107,6 +108,11 @@ struct nitro_spmv {
 
   nitro::DevBuf flush;      // L2 flush scratch
   nitro::DevBuf xbuf, ybuf; // run_host staging
+  // run_host row-chunk pipeline (H2D of x / multiply / D2H of y on three streams)
+  cudaStream_t s_in = nullptr, s_out = nullptr;
+  std::vector<cudaEvent_t> ev_pipe;
+  bool xhi_ready = false;            // csr_xhi valid (cleared by invalidate)
+  std::vector<int64_t> csr_xhi;      // per run_host chunk: 1 + max column of the rows before its end
 
   // multi-GPU (dist.cu)
   int64_t feat_G = -1;      // bitmap offset shift override (global-offset bitmaps); -1 = row0 + N - 1
@@ -131,6 +137,11 @@ nitro_status_t prepare_csrv(nitro_spmv *A);
 
 // spmv.cu
 nitro_status_t launch_spmv(nitro_spmv *A, int variant, const void *x, void *y, cudaStream_t s);
+// rows [r0, r1) only (CSR-scalar, ELL, DIA: row-separable launches; r0 a multiple of 32)
+nitro_status_t launch_spmv_rows(nitro_spmv *A, int variant, const void *x, void *y, cudaStream_t s, int64_t r0,
+                                int64_t r1);
+// per-chunk maximum column + 1 of the rows below each chunk end (run_host pipeline)
+nitro_status_t csr_chunk_xhi(nitro_spmv *A, const std::vector<int64_t> &ends, std::vector<int64_t> &xhi);
 int launches_of(const nitro_spmv *A, int variant);
 nitro_status_t launch_flush(nitro_spmv *A, cudaStream_t s);
 // spmv_dia_tma.cu: DIA with TMA-streamed diagonal slabs

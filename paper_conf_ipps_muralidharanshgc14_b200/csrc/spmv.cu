@@ -272,9 +272,10 @@ __global__ void __launch_bounds__(256, sizeof(VT) == 4 ? 4 : 3) k_csr_vector(con
 template <typename VT, int U>  // U <= 16: terms per fp32 partial
 __global__ void __launch_bounds__(256) k_ell(const int32_t *__restrict__ ecol, const VT *__restrict__ eval,
                                              const VT *__restrict__ x, VT *__restrict__ y, int64_t N, int64_t K,
-                                             int64_t ld, bool l2ef) {
+                                             int64_t ld, int64_t nr, bool l2ef) {
+  // rows [0, nr) (nr <= ld: ld for a whole multiply incl. padding, less for a row chunk)
   const uint64_t pol = l2_policy(l2ef);
-  const int64_t nq = ld >> 2;
+  const int64_t nq = (nr + 3) >> 2;
   for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nq; q += (int64_t)gridDim.x * blockDim.x) {
     const int64_t i0 = q << 2;
     double acc[4] = {0.0, 0.0, 0.0, 0.0};
@@ -325,23 +326,23 @@ template <typename VT, int U, int DS>
 __global__ void __launch_bounds__(256, (U == 1 && DS == 1 && sizeof(VT) == 4) ? 8 : 1)  // U=1 fp32: <= 32 regs, full occupancy
     k_dia(const int32_t *__restrict__ offs, const VT *__restrict__ dval,
                                              const VT *__restrict__ x, VT *__restrict__ y, int64_t N, int64_t M,
-                                             int64_t D, int64_t ld, int64_t row0, int64_t off_min, int64_t off_max,
-                                             bool x_aligned, bool l2ef) {
+                                             int64_t D, int64_t ld, int64_t nr, int64_t row0, int64_t off_min,
+                                             int64_t off_max, bool x_aligned, bool l2ef) {
   constexpr int64_t RB = 1024 / DS;  // rows per block iteration
   const uint64_t pol = l2_policy(l2ef);
   extern __shared__ int s_off[];
   for (int64_t d = threadIdx.x; d < D; d += blockDim.x) s_off[d] = offs[d];
   __syncthreads();
   const int q = (int)(threadIdx.x % DS);
-  const int64_t nb = (ld + RB - 1) / RB;
+  const int64_t nb = (nr + RB - 1) / RB;  // rows [0, nr), nr <= ld (a row chunk: less)
   for (int64_t blk = blockIdx.x; blk < nb; blk += gridDim.x) {
     const int64_t B0 = blk * RB;
     const int64_t i0 = B0 + 4 * (threadIdx.x / DS);
-    const bool active = i0 < ld;  // whole DS groups share i0: uniform within a group
+    const bool active = i0 < nr;  // whole DS groups share i0: uniform within a group
     if constexpr (DS == 1) {
       if (!active) continue;      // no cross-lane combine needed
     }
-    const int64_t Bend = (B0 + RB < ld ? B0 + RB : ld) - 1;
+    const int64_t Bend = (B0 + RB < nr ? B0 + RB : nr) - 1;
     const bool interior = row0 + B0 + off_min >= 0 && row0 + Bend + off_max < M;
     // vector x path: aligned windows may reach 3 floats left / 4 right of the needed ones
     const bool xvec = x_aligned && row0 + B0 + off_min - 3 >= 0 && row0 + Bend + off_max + 4 < M;
@@ -717,13 +718,14 @@ unsigned grid_cap(int64_t blocks, int per_sm);
 
 template <typename VT>
 void launch_ell(const int32_t *col, const VT *val, const VT *x, VT *y, int64_t N, int64_t K, int64_t ld,
-                cudaStream_t s) {
-  const unsigned g = grid_cap((ld / 4 + 255) / 256, 16);
+                cudaStream_t s, int64_t nr = -1) {
+  if (nr < 0) nr = ld;
+  const unsigned g = grid_cap(((nr + 3) / 4 + 255) / 256, 16);
   switch (ell_batch(sizeof(VT))) {
-    case 1: k_ell<VT, 1><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, l2_evict_first()); break;
-    case 2: k_ell<VT, 2><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, l2_evict_first()); break;
-    case 4: k_ell<VT, 4><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, l2_evict_first()); break;
-    default: k_ell<VT, 8><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, l2_evict_first()); break;
+    case 1: k_ell<VT, 1><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first()); break;
+    case 2: k_ell<VT, 2><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first()); break;
+    case 4: k_ell<VT, 4><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first()); break;
+    default: k_ell<VT, 8><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first()); break;
   }
 }
 
@@ -747,15 +749,22 @@ unsigned grid_cap(int64_t blocks, int per_sm = 8) {
 }
 
 template <typename IT, typename VT>
-nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_t s) {
-  const IT *rp = (const IT *)A->rowptr;
+nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_t s, int64_t r0 = 0,
+                     int64_t r1 = -1) {
+  // rows [r0, r1) (default: all).  Partial ranges only for the row-separable
+  // CSR-scalar / ELL / DIA launches (launch_spmv_rows); r0 % 32 == 0.
+  const bool part = r1 >= 0;
+  if (!part) r1 = A->N;
+  const IT *rp = (const IT *)A->rowptr + r0;
   const VT *val = (const VT *)A->val;
-  const int64_t N = A->N;
+  const int64_t N = r1 - r0;
+  y += r0;
   switch (variant) {
     case NITRO_CSR_SCALAR:
       if (N > 0) k_csr_scalar<IT, VT><<<grid_cap((N + 255) / 256, 16), 256, 0, s>>>(rp, A->col, val, x, y, N);
       break;
     case NITRO_CSR_VECTOR: {
+      if (part) return fail(NITRO_E_INVALID_ARG, "CSR-vector has no row-range launch");
       if (N == 0) break;
       const int64_t nseg = A->csrv.n_long;
       int32_t *seg_row = A->csrv.long_rows.as<int32_t>();
@@ -777,18 +786,22 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
       break;
     }
     case NITRO_ELL:
-      if (N > 0) launch_ell<VT>(A->ell.col.as<int32_t>(), A->ell.val.as<VT>(), x, y, N, A->ell.K, A->ell.ld, s);
+      if (N > 0)
+        launch_ell<VT>(A->ell.col.as<int32_t>() + r0, A->ell.val.as<VT>() + r0, x, y, N, A->ell.K, A->ell.ld, s,
+                       part ? round_up(N, 32) : A->ell.ld);
       break;
     case NITRO_DIA:
-      if (N > 0 && A->dia.D > 0 && dia_use_tma()) return launch_dia_tma(A, x, y, s);
+      if (N > 0 && A->dia.D > 0 && dia_use_tma() && !part) return launch_dia_tma(A, x, y, s);
       if (N > 0) {
         const size_t sm = (size_t)std::max<int64_t>(A->dia.D, 1) * 4;
-        const bool x_al = ((reinterpret_cast<uintptr_t>(x) & 15) == 0) && (A->row0 % 4 == 0);
+        const int64_t row0 = A->row0 + r0, nr = part ? round_up(N, 32) : A->dia.ld;
+        const bool x_al = ((reinterpret_cast<uintptr_t>(x) & 15) == 0) && (row0 % 4 == 0);
         const int U = dia_batch(A->dia.D, sizeof(VT)), DS = dia_split(A->dia.D);
-        const unsigned g = grid_cap((A->dia.ld + 1024 / DS - 1) / (1024 / DS), dia_blocks_per_sm());
+        const unsigned g = grid_cap((nr + 1024 / DS - 1) / (1024 / DS), dia_blocks_per_sm());
 #define NITRO_DIA_LAUNCH(UU, SS)                                                                                   \
-  k_dia<VT, UU, SS><<<g, 256, sm, s>>>(A->dia.off.as<int32_t>(), A->dia.val.as<VT>(), x, y, N, A->M, A->dia.D,     \
-                                       A->dia.ld, A->row0, A->dia.off_min, A->dia.off_max, x_al, l2_evict_first())
+  k_dia<VT, UU, SS><<<g, 256, sm, s>>>(A->dia.off.as<int32_t>(), A->dia.val.as<VT>() + r0, x, y, N, A->M,         \
+                                       A->dia.D, A->dia.ld, nr, row0, A->dia.off_min, A->dia.off_max, x_al,      \
+                                       l2_evict_first())
 #define NITRO_DIA_U(SS)                      \
   switch (U) {                               \
     case 2: NITRO_DIA_LAUNCH(2, SS); break;  \
@@ -805,6 +818,7 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
       }
       break;
     case NITRO_HYB:
+      if (part) return fail(NITRO_E_INVALID_ARG, "HYB has no row-range launch");
       if (N > 0) {
         launch_ell<VT>(A->hyb.col.as<int32_t>(), A->hyb.val.as<VT>(), x, y, N, A->hyb.K, A->hyb.ld, s);
         if (A->hyb.Zt > 0) {
@@ -850,6 +864,59 @@ nitro_status_t launch_spmv(nitro_spmv *A, int variant, const void *x, void *y, c
   }
   if (A->fp64) return run_t<int32_t, double>(A, variant, (const double *)x, (double *)y, s);
   return run_t<int32_t, float>(A, variant, (const float *)x, (float *)y, s);
+}
+
+nitro_status_t launch_spmv_rows(nitro_spmv *A, int variant, const void *x, void *y, cudaStream_t s, int64_t r0,
+                                int64_t r1) {
+  if (r0 < 0 || r1 > A->N || r0 > r1 || r0 % 32) return fail(NITRO_E_INVALID_ARG, "bad row range");
+  if (A->rp64) {
+    if (A->fp64) return run_t<int64_t, double>(A, variant, (const double *)x, (double *)y, s, r0, r1);
+    return run_t<int64_t, float>(A, variant, (const float *)x, (float *)y, s, r0, r1);
+  }
+  if (A->fp64) return run_t<int32_t, double>(A, variant, (const double *)x, (double *)y, s, r0, r1);
+  return run_t<int32_t, float>(A, variant, (const float *)x, (float *)y, s, r0, r1);
+}
+
+namespace {
+// per chunk c: max over rows i < ends[c] of (last column of row i) + 1 (columns
+// ascend within a canonical row); written as a per-chunk max, prefix-maxed on the host
+template <typename IT>
+__global__ void k_chunk_colmax(const IT *__restrict__ rowptr, const int32_t *__restrict__ col, int64_t N,
+                               const int64_t *__restrict__ ends, int nch, unsigned long long *__restrict__ out) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < N; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t b = (int64_t)rowptr[i + 1];
+    if (b == (int64_t)rowptr[i]) continue;
+    int c = 0;
+    while (c < nch - 1 && i >= ends[c]) ++c;
+    atomicMax(out + c, (unsigned long long)col[b - 1] + 1ull);
+  }
+}
+}  // namespace
+
+nitro_status_t csr_chunk_xhi(nitro_spmv *A, const std::vector<int64_t> &ends, std::vector<int64_t> &xhi) {
+  const int nch = (int)ends.size();
+  DevBuf tmp;
+  NITRO_TRY(tmp.alloc((size_t)nch * 16));
+  int64_t *d_ends = tmp.as<int64_t>();
+  unsigned long long *d_out = reinterpret_cast<unsigned long long *>(d_ends + nch);
+  NITRO_CUDA(cudaMemcpyAsync(d_ends, ends.data(), (size_t)nch * 8, cudaMemcpyHostToDevice, A->stream));
+  NITRO_CUDA(cudaMemsetAsync(d_out, 0, (size_t)nch * 8, A->stream));
+  const unsigned g = grid_cap((A->N + 255) / 256, 8);
+  if (A->N > 0) {
+    if (A->rp64) k_chunk_colmax<int64_t><<<g, 256, 0, A->stream>>>((const int64_t *)A->rowptr, A->col, A->N, d_ends, nch, d_out);
+    else k_chunk_colmax<int32_t><<<g, 256, 0, A->stream>>>((const int32_t *)A->rowptr, A->col, A->N, d_ends, nch, d_out);
+    NITRO_CUDA(cudaGetLastError());
+  }
+  std::vector<unsigned long long> h(nch);
+  NITRO_CUDA(cudaMemcpyAsync(h.data(), d_out, (size_t)nch * 8, cudaMemcpyDeviceToHost, A->stream));
+  NITRO_CUDA(cudaStreamSynchronize(A->stream));
+  xhi.assign(nch, 0);
+  int64_t run = 0;
+  for (int c = 0; c < nch; ++c) {
+    run = std::max<int64_t>(run, (int64_t)h[c]);
+    xhi[c] = run;
+  }
+  return NITRO_OK;
 }
 
 nitro_status_t launch_flush(nitro_spmv *A, cudaStream_t s) {

@@ -1,4 +1,8 @@
-# feature-pass timing (median of 7, L2 flushed) + full GPU suite
-f() { timeout 300 python tools/profile_variants.py --time $1 none 2>/dev/null | python -c "import json,sys; t=json.load(sys.stdin); print({c: round(r['feature_ms'],3) for c,r in t.items()})"; }
-f "c0 c1 short c2a c2b"
-timeout 1500 python -m pytest tests -q -x -m gpu 2>&1 | tail -3
+# pipelined run_host: e2e by chunk count
+mkdir -p gpurun_out
+for c in 1 4 8 16; do
+  echo "RUN_HOST_CHUNKS=$c"
+  NITRO_RUN_HOST_CHUNKS=$c timeout 600 python bench.py --steps 20 --warmup 5 --no-cpu > gpurun_out/b_$c.json 2> gpurun_out/b_$c.err
+  tail -3 gpurun_out/b_$c.err
+  python -c "import json,sys; d=json.loads(open('gpurun_out/b_$c.json').read().strip().splitlines()[-1]); print(round(d['value']), d['e2e'], d['roofline'].get('size_matched_copy_gbs'), d['roofline'].get('frac_of_size_matched_copy'))"
+done
