@@ -229,6 +229,14 @@ nitro_status_t nitro_spmv_set_stream(nitro_spmv *A, void *stream);
  * strictly increasing in a row, or out of [0, cols)) returns
  * NITRO_E_BAD_MATRIX with out->canonical = 0.  Cached. */
 nitro_status_t nitro_spmv_features(nitro_spmv *A, nitro_spmv_feat *out);
+/* Cheaper feature level (the Fig. 8 overhead study): one pass over
+ * rowptr only -> rows, cols, nnz, sum_len, sum_len2, max_row, mean, sd,
+ * max_dev, ell_fill exactly as nitro_spmv_features (bit-identical); the
+ * column-dependent fields are not evaluated: ndiag = -1, dia_fill = -1.0,
+ * canonical = -1 (rowptr monotonicity is still checked: a broken rowptr
+ * returns NITRO_E_BAD_MATRIX).  Not cached; does not satisfy constraints.
+ * Syncs the handle's stream. */
+nitro_status_t nitro_spmv_row_features(nitro_spmv *A, nitro_spmv_feat *out);
 /* fix_inputs analogue: enqueue the feature pass now, on the
  * handle's stream, without waiting; the next features/allowed/select waits. */
 nitro_status_t nitro_spmv_features_async(nitro_spmv *A);

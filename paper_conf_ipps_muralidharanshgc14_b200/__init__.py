@@ -134,6 +134,7 @@ _SIGS = {
     "nitro_spmv_create": ([_int, _vp, _i64, _i64, _i64, _vp, _int, _vp, _vp, _int, _P(_vp)], _int),
     "nitro_spmv_set_stream": ([_vp, _vp], _int),
     "nitro_spmv_features": ([_vp, _P(Feat)], _int),
+    "nitro_spmv_row_features": ([_vp, _P(Feat)], _int),
     "nitro_spmv_features_async": ([_vp], _int),
     "nitro_spmv_allowed": ([_vp, _int, _P(_int)], _int),
     "nitro_spmv_set_budget": ([_vp, _dbl], _int),
@@ -238,6 +239,12 @@ class SpMV:
     def features(self) -> dict:
         f = Feat()
         _check(_L.nitro_spmv_features(self.h, ctypes.byref(f)))
+        return f.as_dict()
+
+    def row_features(self) -> dict:
+        """Cheap level: rowptr-only pass (ndiag / dia_fill / canonical = -1, not evaluated)."""
+        f = Feat()
+        _check(_L.nitro_spmv_row_features(self.h, ctypes.byref(f)))
         return f.as_dict()
 
     def features_async(self):

@@ -178,6 +178,14 @@ nitro_status_t nitro_spmv_features(nitro_spmv *A, nitro_spmv_feat *out) {
   NITRO_GUARD_END
 }
 
+nitro_status_t nitro_spmv_row_features(nitro_spmv *A, nitro_spmv_feat *out) {
+  NITRO_GUARD_BEGIN
+  if (!A || !out) return fail(NITRO_E_INVALID_ARG, "NULL argument");
+  DeviceGuard g(A->device);
+  return row_features(A, out);
+  NITRO_GUARD_END
+}
+
 nitro_status_t nitro_spmv_features_async(nitro_spmv *A) {
   NITRO_GUARD_BEGIN
   if (!A) return fail(NITRO_E_INVALID_ARG, "NULL handle");
@@ -471,7 +479,8 @@ nitro_status_t nitro_spmv_release(nitro_spmv *A, int variant) {
   if (variant == -1 || variant == NITRO_DIA) { A->dia.off.release(); A->dia.val.release(); A->dia.ready = false; }
   if (variant == -1 || variant == NITRO_HYB) {
     A->hyb.col.release(); A->hyb.val.release(); A->hyb.trow.release(); A->hyb.tcol.release();
-    A->hyb.tval.release(); A->hyb.carry_row.release(); A->hyb.carry_val.release(); A->hyb.ready = false;
+    A->hyb.tval.release(); A->hyb.carry_row.release(); A->hyb.carry_val.release();
+    A->hyb.fix_seg.release(); A->hyb.fix_long.release(); A->hyb.ready = false;
   }
   if (variant == -1 || variant == NITRO_CSR_VECTOR) { A->csrv.long_rows.release(); A->csrv.ready = false; }
   return NITRO_OK;

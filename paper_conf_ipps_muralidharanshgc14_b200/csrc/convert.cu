@@ -15,6 +15,8 @@
 namespace nitro {
 namespace {
 
+constexpr int64_t kTailThread = 64, kTailPiece = 4096;
+
 template <typename IT, typename VT>
 __global__ void k_fill_ell(const IT *__restrict__ rowptr, const int32_t *__restrict__ col, const VT *__restrict__ val,
                            int64_t N, int64_t K, int64_t ld, int32_t *__restrict__ ecol, VT *__restrict__ eval,
@@ -28,7 +30,7 @@ __global__ void k_fill_ell(const IT *__restrict__ rowptr, const int32_t *__restr
       ecol[k * ld + i] = in ? col[a + k] : -1;
       eval[k * ld + i] = in ? val[a + k] : (VT)0;
     }
-    if (toff && L > K) {
+    if (toff && L > K && L - K <= kTailThread) {  // longer tails: k_fill_tail_tasks
       int64_t o = toff[i];
       for (int64_t k = K; k < L; ++k, ++o) {
         trow[o] = (int32_t)i;
@@ -37,6 +39,70 @@ __global__ void k_fill_ell(const IT *__restrict__ rowptr, const int32_t *__restr
       }
     }
   }
+}
+
+// HYB tails longer than kTailThread entries are copied by whole warps, in
+// (row, piece of kTailPiece entries) tasks spread over the grid (an R-MAT hub
+// row's 1.5e5-entry tail would serialise one thread for milliseconds)
+template <typename IT>
+__global__ void k_tail_tasks_count(const IT *__restrict__ rowptr, int64_t N, int64_t K, int64_t *__restrict__ cnt) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < N; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t t = (int64_t)rowptr[i + 1] - (int64_t)rowptr[i] - K;
+    cnt[i] = t > kTailThread ? (t + kTailPiece - 1) / kTailPiece : 0;
+  }
+}
+__global__ void k_tail_tasks_emit(const int64_t *__restrict__ off, int64_t N, int2 *__restrict__ tasks) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < N; i += (int64_t)gridDim.x * blockDim.x)
+    for (int64_t t = off[i]; t < off[i + 1]; ++t) tasks[t] = make_int2((int)i, (int)(t - off[i]));
+}
+template <typename IT, typename VT>
+__global__ void k_fill_tail_tasks(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
+                                  const VT *__restrict__ val, int64_t K, const int64_t *__restrict__ toff,
+                                  const int2 *__restrict__ tasks, int64_t ntask, int32_t *__restrict__ trow,
+                                  int32_t *__restrict__ tcol, VT *__restrict__ tval) {
+  const int lane = threadIdx.x & 31;
+  const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t t = gw; t < ntask; t += nw) {
+    const int2 tk = tasks[t];
+    const int64_t a = (int64_t)rowptr[tk.x], b = (int64_t)rowptr[tk.x + 1];
+    const int64_t st = a + K + (int64_t)tk.y * kTailPiece, en = st + kTailPiece < b ? st + kTailPiece : b;
+    const int64_t o = toff[tk.x] + (int64_t)tk.y * kTailPiece - st;
+#pragma unroll 4
+    for (int64_t e = st + lane; e < en; e += 32) {
+      trow[o + e] = tk.x;
+      tcol[o + e] = col[e];
+      tval[o + e] = val[e];
+    }
+  }
+}
+
+// HYB fixup plan: the carry slots a tail multiply fills are fixed by the
+// structure — slot 2c = row of chunk c's first entry, slot 2c+1 = row of its
+// last (left empty by the tail kernel when it equals the first).  With
+// eff[2c+1] = that last row either way, slots of one row are a contiguous run.
+__global__ void k_fix_eff(const int32_t *__restrict__ trow, int64_t Zt, int64_t CH, int64_t nch,
+                          int32_t *__restrict__ eff) {
+  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < nch; c += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t s0 = c * CH, e1 = (s0 + CH < Zt ? s0 + CH : Zt) - 1;
+    eff[2 * c] = trow[s0];
+    eff[2 * c + 1] = trow[e1];
+  }
+}
+__global__ void k_fix_heads(const int32_t *__restrict__ eff, int64_t n, int64_t *__restrict__ h) {
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x)
+    h[j] = (j == 0 || eff[j] != eff[j - 1]) ? 1 : 0;
+}
+__global__ void k_fix_emit(const int32_t *__restrict__ eff, const int64_t *__restrict__ pos, int64_t n,
+                           int32_t *__restrict__ seg) {
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x)
+    if (j == 0 || eff[j] != eff[j - 1]) seg[pos[j]] = (int32_t)j;
+  if (blockIdx.x == 0 && threadIdx.x == 0) seg[pos[n]] = (int32_t)n;
+}
+__global__ void k_fix_long(const int32_t *__restrict__ seg, int64_t S, int32_t *__restrict__ lst,
+                           unsigned long long *__restrict__ cnt) {
+  for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < S; s += (int64_t)gridDim.x * blockDim.x)
+    if (seg[s + 1] - seg[s] > 32) lst[atomicAdd(cnt, 1ull)] = (int32_t)s;
 }
 
 // tail count per row (HYB): max(L_i - K, 0)
@@ -309,6 +375,60 @@ nitro_status_t prepare_hyb(nitro_spmv *A) {
   if (N > 0)
     NITRO_TRY(fill_ell(A, K, ld, A->hyb.col.p, A->hyb.val.p, Zt > 0 ? toff : nullptr, A->hyb.trow.p, A->hyb.tcol.p,
                        A->hyb.tval.p));
+  if (Zt > 0 && lmax - K > kTailThread) {
+    // long tails: (row, piece) tasks, one warp each
+    DevBuf tc;
+    NITRO_TRY(tc.alloc((size_t)(2 * N + 2) * 8));
+    int64_t *tcnt = tc.as<int64_t>(), *tof = tcnt + N + 1;
+    if (A->rp64) k_tail_tasks_count<int64_t><<<grid_of(N), 256, 0, s>>>((const int64_t *)A->rowptr, N, K, tcnt);
+    else k_tail_tasks_count<int32_t><<<grid_of(N), 256, 0, s>>>((const int32_t *)A->rowptr, N, K, tcnt);
+    NITRO_TRY(exclusive_scan_i64(tcnt, tof, N, A->scratch, s));
+    int64_t ntask = 0;
+    NITRO_CUDA(cudaMemcpyAsync(&ntask, tof + N, 8, cudaMemcpyDeviceToHost, s));
+    NITRO_CUDA(cudaStreamSynchronize(s));
+    DevBuf tk;
+    NITRO_TRY(tk.alloc((size_t)std::max<int64_t>(ntask, 1) * sizeof(int2)));
+    k_tail_tasks_emit<<<grid_of(N), 256, 0, s>>>(tof, N, tk.as<int2>());
+    const unsigned gt = (unsigned)std::max<int64_t>(1, std::min<int64_t>((ntask + 7) / 8, (int64_t)num_sms() * 8));
+#define NITRO_TT(IT, VT)                                                                                        \
+  k_fill_tail_tasks<IT, VT><<<gt, 256, 0, s>>>((const IT *)A->rowptr, A->col, (const VT *)A->val, K, toff,    \
+                                              tk.as<int2>(), ntask, A->hyb.trow.as<int32_t>(),                \
+                                              A->hyb.tcol.as<int32_t>(), A->hyb.tval.as<VT>())
+    if (A->rp64) { if (A->fp64) NITRO_TT(int64_t, double); else NITRO_TT(int64_t, float); }
+    else { if (A->fp64) NITRO_TT(int32_t, double); else NITRO_TT(int32_t, float); }
+#undef NITRO_TT
+    NITRO_CUDA(cudaGetLastError());
+    NITRO_CUDA(cudaStreamSynchronize(s));  // tc / tk are freed on return
+  }
+  // fixup plan (see k_fix_eff)
+  A->hyb.fix_S = A->hyb.fix_nlong = 0;
+  if (Zt > 0) {
+    const int64_t nslot = 2 * nch;
+    DevBuf fx;
+    NITRO_TRY(fx.alloc((size_t)nslot * 4 + (size_t)(2 * nslot + 2) * 8 + 8));
+    int32_t *eff = fx.as<int32_t>();
+    int64_t *hd = reinterpret_cast<int64_t *>(fx.as<char>() + round_up(nslot * 4, 8)), *pos = hd + nslot + 1;
+    k_fix_eff<<<grid_of(nch), 256, 0, s>>>(A->hyb.trow.as<int32_t>(), Zt, chunk, nch, eff);
+    k_fix_heads<<<grid_of(nslot), 256, 0, s>>>(eff, nslot, hd);
+    NITRO_TRY(exclusive_scan_i64(hd, pos, nslot, A->scratch, s));
+    int64_t S = 0;
+    NITRO_CUDA(cudaMemcpyAsync(&S, pos + nslot, 8, cudaMemcpyDeviceToHost, s));
+    NITRO_CUDA(cudaStreamSynchronize(s));
+    NITRO_TRY(A->hyb.fix_seg.alloc((size_t)(S + 1) * 4));
+    NITRO_TRY(A->hyb.fix_long.alloc((size_t)std::max<int64_t>(S, 1) * 4));
+    k_fix_emit<<<grid_of(nslot), 256, 0, s>>>(eff, pos, nslot, A->hyb.fix_seg.as<int32_t>());
+    DevBuf lc;
+    NITRO_TRY(lc.alloc(8));
+    NITRO_CUDA(cudaMemsetAsync(lc.p, 0, 8, s));
+    k_fix_long<<<grid_of(S), 256, 0, s>>>(A->hyb.fix_seg.as<int32_t>(), S, A->hyb.fix_long.as<int32_t>(),
+                                          lc.as<unsigned long long>());
+    NITRO_CUDA(cudaGetLastError());
+    unsigned long long nl = 0;
+    NITRO_CUDA(cudaMemcpyAsync(&nl, lc.p, 8, cudaMemcpyDeviceToHost, s));
+    NITRO_CUDA(cudaStreamSynchronize(s));
+    A->hyb.fix_S = S;
+    A->hyb.fix_nlong = (int64_t)nl;
+  }
   NITRO_CUDA(cudaStreamSynchronize(s));  // cnt is freed on return
   A->hyb.K = K;
   A->hyb.ld = ld;

@@ -359,6 +359,47 @@ __global__ void __launch_bounds__(kThreads) k_features_long(const IT *__restrict
   if (lane == 0 && bad) atomicOr(&acc->bad, bad);
 }
 
+// Row-length moments only (the cheap feature level): rowptr read once.
+template <typename IT>
+__global__ void __launch_bounds__(256) k_rowstats(const IT *__restrict__ rowptr, int64_t N, int64_t Z,
+                                                  FeatAcc *__restrict__ acc) {
+  __shared__ unsigned long long s_red[3][8];
+  unsigned long long s1 = 0, s2 = 0, lmax = 0;
+  unsigned bad = 0;
+  if (blockIdx.x == 0 && threadIdx.x == 0 && ((int64_t)rowptr[0] != 0 || (int64_t)rowptr[N] != Z)) bad |= 1;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < N; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t L = (int64_t)rowptr[i + 1] - (int64_t)rowptr[i];
+    if (L < 0) { bad |= 1; continue; }
+    s1 += (unsigned long long)L;
+    s2 += (unsigned long long)L * (unsigned long long)L;
+    lmax = (unsigned long long)L > lmax ? (unsigned long long)L : lmax;
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    s1 += __shfl_xor_sync(kFull, s1, o);
+    s2 += __shfl_xor_sync(kFull, s2, o);
+    const unsigned long long t = __shfl_xor_sync(kFull, lmax, o);
+    lmax = t > lmax ? t : lmax;
+  }
+  bad = __reduce_or_sync(kFull, bad);
+  const int w = threadIdx.x >> 5;
+  if ((threadIdx.x & 31) == 0) {
+    s_red[0][w] = s1; s_red[1][w] = s2; s_red[2][w] = lmax;
+    if (bad) atomicOr(&acc->bad, bad);
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long a1 = 0, a2 = 0, am = 0;
+    for (int k = 0; k < 8; ++k) {
+      a1 += s_red[0][k]; a2 += s_red[1][k];
+      am = s_red[2][k] > am ? s_red[2][k] : am;
+    }
+    if (a1) atomicAdd(&acc->s1, a1);
+    if (a2) atomicAdd(&acc->s2, a2);
+    if (am) atomicMax(&acc->lmax, am);
+  }
+}
+
 __global__ void __launch_bounds__(256) k_popc(const uint32_t *__restrict__ bm, int64_t nwords, FeatAcc *acc) {
   unsigned long long s = 0;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nwords; i += (int64_t)gridDim.x * blockDim.x)
@@ -434,6 +475,29 @@ nitro_status_t features_launch(nitro_spmv *A) {
   NITRO_CUDA(cudaMemcpyAsync(A->h_acc, acc, sizeof(FeatAcc), cudaMemcpyDeviceToHost, s));
   NITRO_CUDA(cudaEventRecord(A->feat_done, s));
   A->feat_pending = true;
+  return NITRO_OK;
+}
+
+nitro_status_t row_features(nitro_spmv *A, nitro_spmv_feat *out) {
+  cudaStream_t s = A->stream;
+  DevBuf acc_buf;
+  NITRO_TRY(acc_buf.alloc(sizeof(FeatAcc)));
+  FeatAcc *acc = acc_buf.as<FeatAcc>();
+  NITRO_CUDA(cudaMemsetAsync(acc, 0, sizeof(FeatAcc), s));
+  if (A->N > 0) {
+    const unsigned g = (unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)num_sms() * 8, (A->N + 255) / 256));
+    if (A->rp64) k_rowstats<int64_t><<<g, 256, 0, s>>>((const int64_t *)A->rowptr, A->N, A->Z, acc);
+    else k_rowstats<int32_t><<<g, 256, 0, s>>>((const int32_t *)A->rowptr, A->N, A->Z, acc);
+    NITRO_CUDA(cudaGetLastError());
+  }
+  FeatAcc h{};
+  NITRO_CUDA(cudaMemcpyAsync(&h, acc, sizeof(FeatAcc), cudaMemcpyDeviceToHost, s));
+  NITRO_CUDA(cudaStreamSynchronize(s));
+  finish_features(A->N, A->M, A->Z, h.s1, h.s2, (int64_t)h.lmax, 0, out);
+  out->ndiag = -1;
+  out->dia_fill = -1.0;
+  out->canonical = -1;
+  if (h.bad) return fail(NITRO_E_BAD_MATRIX, "non-canonical CSR: rowptr not monotone from 0 to nnz");
   return NITRO_OK;
 }
 

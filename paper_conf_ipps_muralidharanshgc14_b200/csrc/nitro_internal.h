@@ -67,6 +67,10 @@ struct HybFmt {
   int64_t K = 0, ld = 0, Zt = 0, nchunks = 0, tail_rows = 0;
   int W = 8;  // tail windows per chunk
   DevBuf col, val, trow, tcol, tval, carry_row, carry_val;
+  // fixup plan (static per matrix): carry slots grouped by row into segments
+  // [fix_seg[s], fix_seg[s+1]); segments longer than 32 slots listed in fix_long
+  DevBuf fix_seg, fix_long;
+  int64_t fix_S = 0, fix_nlong = 0;
 };
 struct CsrvFmt {
   bool ready = false;
@@ -126,6 +130,7 @@ namespace nitro {
 // features.cu
 nitro_status_t features_launch(nitro_spmv *A);   // enqueue K1 + compaction, async
 nitro_status_t features_finish(nitro_spmv *A);   // wait + host finishing
+nitro_status_t row_features(nitro_spmv *A, nitro_spmv_feat *out);  // rowptr-only level, syncs
 void finish_features(int64_t N, int64_t M, int64_t Z, uint64_t s1, uint64_t s2, int64_t lmax, int64_t D,
                      nitro_spmv_feat *f);
 

@@ -419,7 +419,7 @@ __global__ void __launch_bounds__(256, (U == 1 && DS == 1 && sizeof(VT) == 4) ? 
 // front, then a segmented inclusive scan per window (rows sorted => equal row
 // ids are contiguous).  Rows wholly inside the chunk are added to y directly
 // (single owner); the chunk's first and last rows go to two carry slots that
-// k_hyb_fixup applies in chunk order.  No atomics; deterministic.
+// k_hyb_fixup_seg applies per row in slot order.  No atomics; deterministic.
 template <typename VT, int W>
 __global__ void __launch_bounds__(256) k_hyb_tail(const int32_t *__restrict__ trow, const int32_t *__restrict__ tcol,
                                                   const VT *__restrict__ tval, const VT *__restrict__ x,
@@ -622,25 +622,43 @@ __global__ void __launch_bounds__(256) k_hyb_tail_ls(const int32_t *__restrict__
   }
 }
 
+// Carry fixup by the static plan of prepare_hyb: segment s = the carry slots
+// [seg[s], seg[s+1]) of one row, summed in slot order (slots left empty by the
+// tail kernel, row -1, skipped) and added to y once.  Segments of <= 32 slots:
+// a thread each (blocks [0, nshort)); longer ones (rows spanning many chunks,
+// e.g. R-MAT hubs): a warp each, lane-strided partial sums + a fixed xor tree.
 template <typename VT>
-__global__ void __launch_bounds__(256) k_hyb_fixup(const int32_t *__restrict__ carry_row,
-                                                   const double *__restrict__ carry_val, VT *__restrict__ y,
-                                                   int64_t nch) {
-  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < nch; c += (int64_t)gridDim.x * blockDim.x) {
+__global__ void __launch_bounds__(256) k_hyb_fixup_seg(const int32_t *__restrict__ carry_row,
+                                                       const double *__restrict__ carry_val,
+                                                       const int32_t *__restrict__ seg, int64_t S,
+                                                       const int32_t *__restrict__ lst, int64_t nlong,
+                                                       unsigned nshort, VT *__restrict__ y) {
+  if (blockIdx.x < nshort) {
+    for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < S; s += (int64_t)nshort * blockDim.x) {
+      const int j0 = seg[s], j1 = seg[s + 1];
+      if (j1 - j0 > 32) continue;
+      double tot = 0.0;
+      for (int j = j0; j < j1; ++j)
+        if (carry_row[j] >= 0) tot += carry_val[j];
+      const int r = carry_row[j0];
+      y[r] = (VT)((double)y[r] + tot);
+    }
+    return;
+  }
+  const int lane = threadIdx.x & 31;
+  const int64_t w = ((blockIdx.x - nshort) * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)(gridDim.x - nshort) * blockDim.x) >> 5;
+  for (int64_t q = w; q < nlong; q += nw) {
+    const int s = lst[q];
+    const int j0 = seg[s], j1 = seg[s + 1];
+    double t = 0.0;
+    for (int j = j0 + lane; j < j1; j += 32)
+      if (carry_row[j] >= 0) t += carry_val[j];
 #pragma unroll
-    for (int s = 0; s < 2; ++s) {
-      const int r = carry_row[2 * c + s];
-      if (r < 0) continue;
-      if (c > 0 && (carry_row[2 * c - 2] == r || carry_row[2 * c - 1] == r)) continue;  // started earlier
-      double sum = carry_val[2 * c + s];
-      const bool may_continue = s == 1 || carry_row[2 * c + 1] < 0;
-      if (may_continue) {
-        for (int64_t c2 = c + 1; c2 < nch && carry_row[2 * c2] == r; ++c2) {
-          sum += carry_val[2 * c2];
-          if (carry_row[2 * c2 + 1] >= 0) break;  // r ended inside c2
-        }
-      }
-      y[r] = (VT)((double)y[r] + sum);
+    for (int o = 16; o > 0; o >>= 1) t += __shfl_xor_sync(kFull, t, o);
+    if (lane == 0) {
+      const int r = carry_row[j0];
+      y[r] = (VT)((double)y[r] + t);
     }
   }
 }
@@ -843,8 +861,12 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
           }
 #undef NITRO_TAIL_LS
 #undef NITRO_TAIL
-          k_hyb_fixup<VT><<<grid_cap((A->hyb.nchunks + 255) / 256, 16), 256, 0, s>>>(
-              A->hyb.carry_row.as<int32_t>(), A->hyb.carry_val.as<double>(), y, A->hyb.nchunks);
+          const unsigned nshort = grid_cap((A->hyb.fix_S + 255) / 256, 8);
+          const unsigned nlong_blk =
+              A->hyb.fix_nlong > 0 ? (unsigned)std::min<int64_t>((A->hyb.fix_nlong + 7) / 8, (int64_t)num_sms() * 4) : 0;
+          k_hyb_fixup_seg<VT><<<nshort + nlong_blk, 256, 0, s>>>(
+              A->hyb.carry_row.as<int32_t>(), A->hyb.carry_val.as<double>(), A->hyb.fix_seg.as<int32_t>(),
+              A->hyb.fix_S, A->hyb.fix_long.as<int32_t>(), A->hyb.fix_nlong, nshort, y);
         }
       }
       break;

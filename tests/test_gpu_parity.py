@@ -126,6 +126,30 @@ def mixed_matrix(seed=31, N=3000, M=20000, fp64=False):
     return Csr(N, M, rp, ci, v.astype(np.float64 if fp64 else np.float32), fp64)
 
 
+ROW_KEYS = ("rows", "cols", "nnz", "sum_len", "sum_len2", "max_row", "mean", "sd", "max_dev", "ell_fill")
+
+
+@pytest.mark.parametrize("name,A", list(small_mats()) + [("mixed", mixed_matrix())])
+def test_row_features_level_bit_exact(cuda, name, A):
+    """The rowptr-only feature level equals the full pass on every row-length
+    feature and reports the column-dependent ones as not evaluated."""
+    M, _ = handle(A, cuda, rowptr32=(name != "mixed"))
+    f, f_ref = M.row_features(), oracle.features(A)
+    for k in ROW_KEYS:
+        assert f[k] == f_ref[k], (name, k, f[k], f_ref[k])
+    assert f["ndiag"] == -1 and f["dia_fill"] == -1.0 and f["canonical"] == -1
+
+
+def test_row_features_rejects_broken_rowptr(cuda):
+    n = nitro()
+    A = Csr(3, 3, np.array([0, 3, 2, 6], np.int64), np.array([0, 1, 2, 0, 1, 2], np.int32),
+            np.ones(6, np.float32), False)
+    M, _ = handle(A, cuda)
+    with pytest.raises(n.NitroError) as e:
+        M.row_features()
+    assert e.value.code == 2
+
+
 @pytest.mark.parametrize("rp32", [True, False])
 def test_features_mixed_walks(cuda, rp32):
     A = mixed_matrix()
