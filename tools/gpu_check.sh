@@ -26,7 +26,7 @@ if want prof; then
   echo "ncu launches rc=$?"
   for cfg in c1 c2a c2b; do
     timeout 900 ncu --set full --clock-control none --import-source on \
-        -k 'regex:k_(features|csr_scalar|csr_vector|ell|dia|hyb_tail)' -c 16 \
+        -k 'regex:k_(features|csr_scalar|csr_vector|ell|dia|hyb_tail|hyb_fixup)' -c 24 \
         -o /tmp/prof_$cfg -f python tools/profile_variants.py $cfg > gpurun_out/prof_$cfg.log 2>&1
     echo "ncu full $cfg rc=$?"
     ncu -i /tmp/prof_$cfg.ncu-rep --page raw --csv > gpurun_out/prof_${cfg}_raw.csv 2>/dev/null

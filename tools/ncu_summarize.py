@@ -51,7 +51,8 @@ def load(path):
 
 
 def short(name):
-    for k in ("k_features", "k_csr_scalar", "k_csr_vector", "k_hyb_tail", "k_ell", "k_dia"):
+    for k in ("k_features_long", "k_features", "k_csr_scalar", "k_csr_vector", "k_hyb_tail", "k_hyb_fixup", "k_ell",
+              "k_dia"):
         if k in name:
             return k
     return name[:40]
@@ -75,8 +76,9 @@ def main():
         cfgsum = {}
         for i, r in enumerate(recs):
             k = short(r["kernel"])
-            var = {"k_features": "features", "k_csr_scalar": "csr_scalar", "k_csr_vector": "csr_vector",
-                   "k_dia": "dia", "k_hyb_tail": "hyb"}.get(k)
+            var = {"k_features": "features", "k_features_long": "features_long", "k_csr_scalar": "csr_scalar",
+                   "k_csr_vector": "csr_vector", "k_dia": "dia", "k_hyb_tail": "hyb",
+                   "k_hyb_fixup": "hyb_fixup"}.get(k)
             if k == "k_ell":
                 var = "ell" if seen_ell < 2 and cfg != "c2b" else "hyb_ell"
                 seen_ell += 1
