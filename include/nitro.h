@@ -245,6 +245,15 @@ nitro_status_t nitro_spmv_features_async(nitro_spmv *A);
 nitro_status_t nitro_spmv_allowed(nitro_spmv *A, int variant, int *out_allowed);
 /* budget for padded formats in bytes (default: 40% of free HBM at first use) */
 nitro_status_t nitro_spmv_set_budget(nitro_spmv *A, double bytes);
+/* Kernel implementation of the two CSR variants (DESIGN.md §6 K5/K6; the
+ * arithmetic, and so y, is identical across implementations):
+ * NITRO_CSR_IMPL_AUTO (default) = TMA row-tile pipeline when a mean tile fits
+ * the shared-memory stage, else the direct kernels; _DIRECT = direct kernels
+ * (loads from global memory); _STAGED = the tile pipeline for every matrix
+ * (tiles that do not fit are computed from global memory).  Returns
+ * NITRO_E_INVALID_ARG for any other value.  Takes effect at the next run. */
+enum { NITRO_CSR_IMPL_AUTO = 0, NITRO_CSR_IMPL_DIRECT = 1, NITRO_CSR_IMPL_STAGED = 2 };
+nitro_status_t nitro_spmv_set_csr_impl(nitro_spmv *A, int impl);
 /* Build the variant's format (cached; conversions are amortised). */
 nitro_status_t nitro_spmv_prepare(nitro_spmv *A, int variant);
 nitro_status_t nitro_spmv_format_info(nitro_spmv *A, int variant, nitro_format_info *out);

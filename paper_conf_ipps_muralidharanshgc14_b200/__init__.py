@@ -20,6 +20,7 @@ LIB_PATH = os.path.join(_HERE, "libnitro.so")
 
 CSR_SCALAR, CSR_VECTOR, ELL, DIA, HYB = range(5)
 NUM_VARIANTS = 5
+CSR_IMPL_AUTO, CSR_IMPL_DIRECT, CSR_IMPL_STAGED = range(3)
 VARIANT_NAMES = ("csr_scalar", "csr_vector", "ell", "dia", "hyb")
 FEATURE_NAMES = ("nnz", "rows", "mean", "sd", "max_dev", "dia_fill", "ell_fill")
 
@@ -138,6 +139,7 @@ _SIGS = {
     "nitro_spmv_features_async": ([_vp], _int),
     "nitro_spmv_allowed": ([_vp, _int, _P(_int)], _int),
     "nitro_spmv_set_budget": ([_vp, _dbl], _int),
+    "nitro_spmv_set_csr_impl": ([_vp, _int], _int),
     "nitro_spmv_prepare": ([_vp, _int], _int),
     "nitro_spmv_format_info": ([_vp, _int, _P(FormatInfo)], _int),
     "nitro_spmv_run": ([_vp, _int, _vp, _vp], _int),
@@ -260,6 +262,10 @@ class SpMV:
 
     def set_budget(self, nbytes: float):
         _check(_L.nitro_spmv_set_budget(self.h, float(nbytes)))
+
+    def set_csr_impl(self, impl: int):
+        """CSR_IMPL_AUTO / CSR_IMPL_DIRECT / CSR_IMPL_STAGED (nitro_spmv_set_csr_impl)."""
+        _check(_L.nitro_spmv_set_csr_impl(self.h, int(impl)))
 
     def prepare(self, v: int):
         _check(_L.nitro_spmv_prepare(self.h, v))

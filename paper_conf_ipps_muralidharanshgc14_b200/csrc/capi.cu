@@ -208,6 +208,12 @@ nitro_status_t nitro_spmv_set_budget(nitro_spmv *A, double bytes) {
   return NITRO_OK;
 }
 
+nitro_status_t nitro_spmv_set_csr_impl(nitro_spmv *A, int impl) {
+  if (!A || impl < NITRO_CSR_IMPL_AUTO || impl > NITRO_CSR_IMPL_STAGED) return fail(NITRO_E_INVALID_ARG, "bad argument");
+  A->csr_impl = impl;
+  return NITRO_OK;
+}
+
 nitro_status_t nitro_spmv_prepare(nitro_spmv *A, int variant) {
   NITRO_GUARD_BEGIN
   if (!A || !valid_variant(variant)) return fail(NITRO_E_INVALID_ARG, "bad argument");

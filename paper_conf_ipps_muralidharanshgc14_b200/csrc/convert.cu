@@ -447,7 +447,15 @@ nitro_status_t prepare_csrv(nitro_spmv *A) {
   cudaStream_t s = A->stream;
   const int64_t N = A->N;
   const int64_t q = N > 0 ? A->Z / N : 0;
-  int V = q <= 2 ? 2 : q <= 4 ? 4 : q <= 8 ? 8 : q <= 16 ? 16 : 32;
+  // ~2-4 entries per lane (B200 sweep: V = mean/4 beat CUSP's V = mean by
+  // 1.3-1.6x on stencils and sparse bands — more loads in flight per lane);
+  // NITRO_CSRV_RULE=cusp restores V = 2/4/8/16/32 for q <= 2/4/8/16/else
+  static const bool cusp = [] {
+    const char *e = getenv("NITRO_CSRV_RULE");
+    return e && std::string(e) == "cusp";
+  }();
+  int V = cusp ? (q <= 2 ? 2 : q <= 4 ? 4 : q <= 8 ? 8 : q <= 16 ? 16 : 32)
+               : (q <= 8 ? 2 : q <= 16 ? 4 : q <= 32 ? 8 : q <= 64 ? 16 : 32);
   // tuning hook: NITRO_CSRV_SHIFT=k divides V by 2^k (more entries per lane)
   static int shift = [] {
     const char *e = getenv("NITRO_CSRV_SHIFT");

@@ -264,27 +264,37 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
     if (maxL <= (unsigned)kRowCap && maxL * 32u <= 2u * sumL) {
       if (Ln > 0) {
         const bool full = *(volatile unsigned *)&s_full != 0;
+        // Per entry: strictly-increasing check (with prev = -1 it also gives
+        // c >= 0; c < M then follows from the last entry), and the offset's
+        // window bit rel = c - row + kWin/2 tested before it is set.  The
+        // bound checks sit outside the loop: the pass is issue-bound on
+        // stencils (ncu: SM throughput 74 %, IPC 3.2), so instructions per
+        // entry are what the loop is tuned for.
+        const uint32_t rbase = myrow - (kWin >> 1);
         int prev = -1;
-        // per-entry body; the staged / global source is hoisted out of the loop
+        bool inc = true;
         auto entry = [&](int c) {
-          if ((uint32_t)c >= M32) { bad |= 4; return; }
-          if (c <= prev) bad |= 2;
+          inc &= c > prev;
           prev = c;
-          const uint32_t idx = (uint32_t)c - myrow + G32;
-          const uint32_t rel = idx - win_lo;
+          const uint32_t rel = (uint32_t)c - rbase;
           if (rel < kWin) {
             const uint32_t bit = 1u << (rel & 31);
             if (!(s_win[rel >> 5] & bit)) atomicOr(&s_win[rel >> 5], bit);
-          } else {
-            lane_far(idx, full);
+          } else if ((uint32_t)c < M32) {
+            lane_far((uint32_t)c - myrow + G32, full);
           }
         };
         if (staged) {
           const int rel0 = (int)(a - E0);
+#pragma unroll 4
           for (int k = 0; k < (int)Ln; ++k) entry(buf[skew(rel0 + k)]);
         } else {
+#pragma unroll 4
           for (int k = 0; k < (int)Ln; ++k) entry(__ldg(col + a + k));
         }
+        const int first = staged ? buf[skew((int)(a - E0))] : __ldg(col + a);
+        if (first < 0 || (uint32_t)prev >= M32) bad |= 4;
+        else if (!inc) bad |= 2;
       }
     } else if (staged) {
       walk_span_warp<true>(buf, E0, E1, E0, a, L > 0, rowbase, G32, M32, win_lo, s_win, s_slot[wib], bitmap, lane,

@@ -104,6 +104,7 @@ struct nitro_spmv {
   cudaEvent_t feat_done = nullptr;
 
   double budget = -1.0;
+  int csr_impl = 0;  // NITRO_CSR_IMPL_*
 
   nitro::EllFmt ell;
   nitro::DiaFmt dia;

@@ -8,6 +8,7 @@
 // below ~21 u sum|a_ij x_j| (u = 2^-24) for any row length: inside the
 // 1e-5 bound of the north star, and exact on integer stencils.
 #include "nitro_internal.h"
+#include "tma.cuh"
 #include "util.cuh"
 
 #include <algorithm>
@@ -58,37 +59,51 @@ __device__ __forceinline__ void store4(VT *y, int64_t i0, int64_t N, const doubl
 }
 
 // ------------------------------------------------------------------ K5 CSR-scalar
-template <typename IT, typename VT>
+// Row arithmetic shared by every CSR-scalar implementation (R2):
+// fp32 (fp64) FFMA partials over 16-term chunks counted from the row start,
+// summed in fp64.  The first H entries of a row arrive as one predicated batch
+// (all loads issued before the first gather), so rows of <= H entries — this
+// variant's class — cost one load round trip; H only changes load batching,
+// never the result.
+template <int H, typename VT, typename LC, typename LV>
+__device__ __forceinline__ double csr_row(int64_t a, int64_t b, const VT *__restrict__ x, LC ldc, LV ldv) {
+  static_assert(H <= 16, "head batch must lie in the first 16-term chunk");
+  int c[H];
+  VT v[H];
+#pragma unroll
+  for (int k = 0; k < H; ++k) {
+    const bool in = a + k < b;
+    c[k] = in ? ldc(a + k) : -1;
+    v[k] = in ? ldv(a + k) : (VT)0;
+  }
+  VT xv[H];
+#pragma unroll
+  for (int k = 0; k < H; ++k) xv[k] = c[k] >= 0 ? __ldg(x + c[k]) : (VT)0;
+  VT part = 0;
+#pragma unroll
+  for (int k = 0; k < H; ++k) part = fma(v[k], xv[k], part);
+  const int64_t e0 = a + 16 < b ? a + 16 : b;
+  for (int64_t k = a + H; k < e0; ++k) part = fma(ldv(k), __ldg(x + ldc(k)), part);
+  double acc = (double)part;
+  for (int64_t k = a + 16; k < b; k += 16) {
+    const int64_t e = k + 16 < b ? k + 16 : b;
+    VT p2 = 0;
+#pragma unroll 4
+    for (int64_t j = k; j < e; ++j) p2 = fma(ldv(j), __ldg(x + ldc(j)), p2);
+    acc += (double)p2;
+  }
+  return acc;
+}
+
+template <int H, typename IT, typename VT>
 __global__ void __launch_bounds__(256) k_csr_scalar(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
                                                     const VT *__restrict__ val, const VT *__restrict__ x,
                                                     VT *__restrict__ y, int64_t N) {
-  // thread per row; the first kHead entries of the row are loaded as one
-  // predicated batch (short rows — this variant's class — then cost a single
-  // load round trip), longer rows continue sequentially in 16-term chunks
-  constexpr int kHead = 4;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < N; i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t a = (int64_t)rowptr[i], b = (int64_t)rowptr[i + 1];
-    int c[kHead];
-    VT v[kHead];
-#pragma unroll
-    for (int k = 0; k < kHead; ++k) {
-      const bool in = a + k < b;
-      c[k] = in ? __ldg(col + a + k) : -1;
-      v[k] = in ? __ldg(val + a + k) : (VT)0;
-    }
-    VT part = 0;
-#pragma unroll
-    for (int k = 0; k < kHead; ++k) part = fma(v[k], c[k] >= 0 ? __ldg(x + c[k]) : (VT)0, part);
-    double acc = (double)part;
-    for (int64_t k = a + kHead; k < b; k += 16) {
-      const int64_t e = k + 16 < b ? k + 16 : b;
-      VT p2 = 0;
-#pragma unroll 4
-      for (int64_t j = k; j < e; ++j) p2 = fma(__ldg(val + j), __ldg(x + __ldg(col + j)), p2);
-      acc += (double)p2;
-    }
-    y[i] = (VT)acc;
-  }
+  // thread per row ("CSR": one thread walks one row)
+  auto ldc = [&](int64_t e) { return __ldg(col + e); };
+  auto ldv = [&](int64_t e) { return __ldg(val + e); };
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < N; i += (int64_t)gridDim.x * blockDim.x)
+    y[i] = (VT)csr_row<H, VT>((int64_t)rowptr[i], (int64_t)rowptr[i + 1], x, ldc, ldv);
 }
 
 // Transposed reduction of R per-lane values (one per row) over groups of V
@@ -124,15 +139,12 @@ __device__ __forceinline__ VT reduce_transpose(VT (&p)[R], int li, int &ridx) {
 // warp first works through the segment list (grid-stride), then through row
 // tiles.  A multi-segment row's partials are summed in segment order by the
 // last warp to finish one of its segments (deterministic, no float atomics).
-template <int V, typename IT, typename VT>
-__global__ void __launch_bounds__(256, sizeof(VT) == 4 ? 4 : 3) k_csr_vector(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
-                                                    const VT *__restrict__ val, const VT *__restrict__ x,
-                                                    VT *__restrict__ y, int64_t N, int64_t nseg,
-                                                    const int32_t *__restrict__ seg_row,
-                                                    const int32_t *__restrict__ seg_k, double *seg_part,
-                                                    unsigned *seg_ctr, bool l2ef) {
-  constexpr int64_t T = 8 * V;
-  const uint64_t pol = l2_policy(l2ef);
+template <typename IT, typename VT>
+__device__ __forceinline__ void csrv_segments(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
+                                              const VT *__restrict__ val, const VT *__restrict__ x,
+                                              VT *__restrict__ y, int64_t nseg, const int32_t *__restrict__ seg_row,
+                                              const int32_t *__restrict__ seg_k, double *seg_part,
+                                              unsigned *seg_ctr, uint64_t pol) {
   {
     constexpr int64_t S = kCsrvSeg;
     const int lane = threadIdx.x & 31;
@@ -175,13 +187,25 @@ __global__ void __launch_bounds__(256, sizeof(VT) == 4 ? 4 : 3) k_csr_vector(con
       }
     }
   }
+}
+
+template <int V, int R, int kB, typename IT, typename VT>
+__global__ void __launch_bounds__(256, R * kB >= 16 ? 2 : R * kB >= 12 ? (sizeof(VT) == 4 ? 3 : 2) : (sizeof(VT) == 4 ? 4 : 3)) k_csr_vector(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
+                                                    const VT *__restrict__ val, const VT *__restrict__ x,
+                                                    VT *__restrict__ y, int64_t N, int64_t nseg,
+                                                    const int32_t *__restrict__ seg_row,
+                                                    const int32_t *__restrict__ seg_k, double *seg_part,
+                                                    unsigned *seg_ctr, bool l2ef) {
+  constexpr int64_t T = 8 * V;
+  const uint64_t pol = l2_policy(l2ef);
+  csrv_segments<IT, VT>(rowptr, col, val, x, y, nseg, seg_row, seg_k, seg_part, seg_ctr, pol);
   // Software-pipelined main path.  A "stage" is R rows of one lane group:
   // row starts/lengths come from the tile's rowptr registers by shuffle, and
   // the (col, val) loads of the NEXT stage are issued before the current
   // stage's x gathers and reduction, so loads stay in flight continuously;
   // the rowptr of the tile after the next is prefetched one tile ahead.
   constexpr int G = 32 / V;
-  constexpr int R = V >= 4 ? 4 : 2;
+  static_assert(R <= V && (R & (R - 1)) == 0, "R rows per stage: a power of two <= V");
   const int lane = threadIdx.x & 31, g = lane / V, li = lane % V;
   const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t stride = (((int64_t)gridDim.x * blockDim.x) >> 5) * 32;
@@ -221,9 +245,31 @@ __global__ void __launch_bounds__(256, sizeof(VT) == 4 ? 4 : 3) k_csr_vector(con
     VT part[R];
 #pragma unroll
     for (int u = 0; u < R; ++u) part[u] = st.c[u] >= 0 ? st.v[u] * __ldg(x + st.c[u]) : (VT)0;
+    // rows of V+1 .. 8V entries: <= 7 more terms per lane.  The next kB
+    // terms of all R rows are loaded as one predicated batch (every load
+    // before the first gather; kB = 3 covers rows of <= 4V entries, kB = 7
+    // all rows of the short path), further terms in a loop; summed in m order.
+    {
+      int cm[R][kB];
+      VT vm[R][kB];
+#pragma unroll
+      for (int u = 0; u < R; ++u)
+#pragma unroll
+        for (int q = 0; q < kB; ++q) {
+          const int m = V * (q + 1) + li;
+          const bool in = m < st.l[u];
+          cm[u][q] = in ? ld_stream_i(col + t.abase + st.s[u] + m, pol) : -1;
+          vm[u][q] = in ? ld_stream(val + t.abase + st.s[u] + m, pol) : (VT)0;
+        }
+#pragma unroll
+      for (int u = 0; u < R; ++u)
+#pragma unroll
+        for (int q = 0; q < kB; ++q)
+          if (cm[u][q] >= 0) part[u] = fma(vm[u][q], __ldg(x + cm[u][q]), part[u]);
+    }
 #pragma unroll
     for (int u = 0; u < R; ++u)
-      for (int m = V + li; m < st.l[u]; m += V)  // <= 7 more terms per lane
+      for (int m = V * (kB + 1) + li; m < st.l[u]; m += V)
         part[u] = fma(ld_stream(val + t.abase + st.s[u] + m, pol), __ldg(x + ld_stream_i(col + t.abase + st.s[u] + m, pol)),
                       part[u]);
     int ridx;
@@ -260,6 +306,177 @@ __global__ void __launch_bounds__(256, sizeof(VT) == 4 ? 4 : 3) k_csr_vector(con
     cur = nxt;
     t0 = nt0;
     tb = ntb;
+  }
+}
+
+// ------------------------------------------------------------------ K5/K6 staged: TMA row-tile pipeline
+// Persistent CTAs walk row tiles of TR rows round-robin.  For each tile one
+// elected thread issues three 1D bulk copies (cp.async.bulk, evict-first) of
+// the tile's rowptr slice and its contiguous colidx / value spans into a
+// kStgStages-deep shared-memory ring tracked by mbarriers, kStgStages - 1
+// tiles ahead of the compute; the spans are rounded out to the enclosing
+// 16-byte chunks (every chunk holds at least one byte of the span, so no read
+// leaves the arrays' pages).  Threads then run the same per-row arithmetic as
+// the direct kernels from shared memory: V = 1 is CSR-scalar (thread per
+// row, RPT rows per thread), V > 1 CSR-vector (V lanes per row, R rows per
+// transposed reduction, rows > 8V on the warp-segment path).  A tile whose
+// span exceeds the stage capacity is computed from global memory instead
+// (same arithmetic, so results are bit-identical either way).  Coalescing no
+// longer depends on the row length, and ~100 KB per SM of HBM traffic stays
+// in flight with a single issuing thread per CTA.
+constexpr int kStgThr = 256;
+constexpr int kStgStages = 3;
+constexpr int kStgBytes = 32768;  // colidx + value bytes per stage
+constexpr int kStgRpBytes = 4096; // rowptr slice bytes per stage (TR * sizeof(IT) <= this)
+template <typename VT> __host__ __device__ constexpr int stg_cap() { return (kStgBytes / (4 + (int)sizeof(VT))) & ~3; }
+template <typename VT> __host__ __device__ constexpr int stg_cb() { return stg_cap<VT>() * 4 + 32; }
+template <typename VT> __host__ __device__ constexpr int stg_vb() { return stg_cap<VT>() * (int)sizeof(VT) + 32; }
+__host__ __device__ constexpr int stg_rb() { return kStgRpBytes + 48; }
+template <typename VT> __host__ __device__ constexpr int stg_stage() { return stg_cb<VT>() + stg_vb<VT>() + stg_rb(); }
+template <typename VT> constexpr size_t stg_smem() { return (size_t)kStgStages * stg_stage<VT>(); }
+
+struct StgMeta {
+  int64_t cbase, vbase, rbase;  // global index held by slot 0 of the stage's colidx / value / rowptr region
+  int over;                     // span did not fit: compute from global memory
+};
+
+template <int V, int RPT, typename IT, typename VT>
+__global__ void __launch_bounds__(kStgThr, 2) k_csr_staged(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
+                                                           const VT *__restrict__ val, const VT *__restrict__ x,
+                                                           VT *__restrict__ y, int64_t N, int64_t ntiles, int rpg,
+                                                           int64_t nseg,
+                                                           const int32_t *__restrict__ seg_row,
+                                                           const int32_t *__restrict__ seg_k, double *seg_part,
+                                                           unsigned *seg_ctr, bool l2ef) {
+  // tile = TR rows: V = 1 -> RPT (template) rows per thread; V > 1 -> rpg (a
+  // multiple of R) rows per lane group of V lanes
+  constexpr int G = kStgThr / V;
+  const int TR = V == 1 ? kStgThr * RPT : G * rpg;
+  constexpr int CB = stg_cb<VT>(), VB = stg_vb<VT>(), RB = stg_rb(), SB = stg_stage<VT>();
+  extern __shared__ __align__(128) unsigned char smem[];
+  __shared__ __align__(8) uint64_t bar[kStgStages];
+  __shared__ StgMeta meta[kStgStages];
+  const int tid = threadIdx.x;
+  const uint64_t pol = l2_policy(l2ef);
+  if constexpr (V > 1) csrv_segments<IT, VT>(rowptr, col, val, x, y, nseg, seg_row, seg_k, seg_part, seg_ctr, pol);
+  const int64_t my = (int64_t)blockIdx.x < ntiles ? (ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+  if (my == 0) return;
+  if (tid == 0) {
+    for (int s = 0; s < kStgStages; ++s) mbar_init(&bar[s], 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+  auto tile_rows = [&](int64_t t, int64_t &r0, int64_t &r1) {
+    r0 = t * TR;
+    r1 = r0 + TR < N ? r0 + TR : N;
+  };
+  auto issue = [&](int64_t t, int st, int64_t a, int64_t b) {  // thread 0 only
+    int64_t r0, r1;
+    tile_rows(t, r0, r1);
+    unsigned char *base = smem + (size_t)st * SB;
+    const uintptr_t ra = reinterpret_cast<uintptr_t>(rowptr + r0) & ~(uintptr_t)15;
+    const uintptr_t re = (reinterpret_cast<uintptr_t>(rowptr + r1 + 1) + 15) & ~(uintptr_t)15;
+    const uintptr_t ca = reinterpret_cast<uintptr_t>(col + a) & ~(uintptr_t)15;
+    const uintptr_t ce = (reinterpret_cast<uintptr_t>(col + b) + 15) & ~(uintptr_t)15;
+    const uintptr_t va = reinterpret_cast<uintptr_t>(val + a) & ~(uintptr_t)15;
+    const uintptr_t ve = (reinterpret_cast<uintptr_t>(val + b) + 15) & ~(uintptr_t)15;
+    const bool any = b > a;
+    const bool fit = !any || ((ce - ca) <= (uintptr_t)CB && (ve - va) <= (uintptr_t)VB);
+    meta[st].rbase = r0 - (int64_t)((reinterpret_cast<uintptr_t>(rowptr + r0) - ra) / sizeof(IT));
+    meta[st].cbase = a - (int64_t)((reinterpret_cast<uintptr_t>(col + a) - ca) / 4);
+    meta[st].vbase = a - (int64_t)((reinterpret_cast<uintptr_t>(val + a) - va) / sizeof(VT));
+    meta[st].over = fit ? 0 : 1;
+    const bool cv = any && fit;
+    mbar_arrive_expect_tx(&bar[st], (uint32_t)((re - ra) + (cv ? (ce - ca) + (ve - va) : 0)));
+    bulk_g2s_evict_first(base + CB + VB, reinterpret_cast<const void *>(ra), (uint32_t)(re - ra), &bar[st], pol);
+    if (cv) {
+      bulk_g2s_evict_first(base, reinterpret_cast<const void *>(ca), (uint32_t)(ce - ca), &bar[st], pol);
+      bulk_g2s_evict_first(base + CB, reinterpret_cast<const void *>(va), (uint32_t)(ve - va), &bar[st], pol);
+    }
+  };
+  auto span = [&](int64_t t, int64_t &a, int64_t &b) {
+    int64_t r0, r1;
+    tile_rows(t, r0, r1);
+    a = (int64_t)rowptr[r0];
+    b = (int64_t)rowptr[r1];
+  };
+  if (tid == 0) {
+    for (int j = 0; j < kStgStages && j < my; ++j) {
+      int64_t a, b;
+      span(blockIdx.x + (int64_t)j * gridDim.x, a, b);
+      issue(blockIdx.x + (int64_t)j * gridDim.x, j, a, b);
+    }
+  }
+  for (int64_t j = 0; j < my; ++j) {
+    const int st = (int)(j % kStgStages);
+    const int64_t t = blockIdx.x + j * gridDim.x;
+    int64_t pa = 0, pb = 0;  // thread 0: span of the tile that refills this stage (loads overlap the compute)
+    const bool refill = tid == 0 && j + kStgStages < my;
+    if (refill) span(t + (int64_t)kStgStages * gridDim.x, pa, pb);
+    mbar_wait(&bar[st], (uint32_t)((j / kStgStages) & 1));
+    int64_t r0, r1;
+    tile_rows(t, r0, r1);
+    const unsigned char *base = smem + (size_t)st * SB;
+    const int32_t *scol = reinterpret_cast<const int32_t *>(base);
+    const VT *sval = reinterpret_cast<const VT *>(base + CB);
+    const IT *srp = reinterpret_cast<const IT *>(base + CB + VB);
+    const int64_t cb = meta[st].cbase, vb = meta[st].vbase, rb = meta[st].rbase;
+    const bool over = meta[st].over != 0;
+    // entry e of the tile's span: from shared memory, or global when the span did not fit
+    auto C = [&](int64_t e) -> int { return over ? ld_stream_i(col + e, pol) : scol[(int)(e - cb)]; };
+    auto W = [&](int64_t e) -> VT { return over ? ld_stream(val + e, pol) : sval[(int)(e - vb)]; };
+    if constexpr (V == 1) {
+      // CSR-scalar arithmetic of k_csr_scalar (csr_row), RPT rows per thread
+#pragma unroll
+      for (int q = 0; q < RPT; ++q) {
+        const int64_t r = r0 + tid + q * kStgThr;
+        if (r < r1) y[r] = (VT)csr_row<8, VT>((int64_t)srp[(int)(r - rb)], (int64_t)srp[(int)(r + 1 - rb)], x, C, W);
+      }
+    } else {
+      // CSR-vector arithmetic of k_csr_vector: lane li takes entries li, li + V, ...
+      // (<= 8 per lane; longer rows are segments), R rows per transposed reduction
+      constexpr int R = V >= 4 ? 4 : 2;
+      constexpr int64_t T = 8 * V;
+      const int g = tid / V, li = tid % V;
+#pragma unroll 1
+      for (int kb = 0; kb < rpg; kb += R) {
+        int64_t s[R];
+        int l[R];
+        unsigned longmask = 0;
+#pragma unroll
+        for (int u = 0; u < R; ++u) {
+          const int64_t r = r0 + g + G * (kb + u);
+          s[u] = 0;
+          l[u] = 0;
+          if (r < r1) {
+            s[u] = (int64_t)srp[(int)(r - rb)];
+            const int64_t L = (int64_t)srp[(int)(r + 1 - rb)] - s[u];
+            if (L > T) longmask |= 1u << u;
+            else l[u] = (int)L;
+          }
+        }
+        int cc[R];
+        VT vv[R];
+#pragma unroll
+        for (int u = 0; u < R; ++u) {
+          const bool in = li < l[u];
+          cc[u] = in ? C(s[u] + li) : -1;
+          vv[u] = in ? W(s[u] + li) : (VT)0;
+        }
+        VT part[R];
+#pragma unroll
+        for (int u = 0; u < R; ++u) part[u] = cc[u] >= 0 ? vv[u] * __ldg(x + cc[u]) : (VT)0;
+#pragma unroll
+        for (int u = 0; u < R; ++u)
+          for (int m = V + li; m < l[u]; m += V) part[u] = fma(W(s[u] + m), __ldg(x + C(s[u] + m)), part[u]);
+        int ridx;
+        const VT tot = reduce_transpose<V, R>(part, li, ridx);
+        const int64_t row = r0 + g + G * (kb + ridx);
+        if (li % (V / R) == 0 && row < r1 && !((longmask >> ridx) & 1u)) y[row] = tot;
+      }
+    }
+    __syncthreads();  // stage st consumed
+    if (refill) issue(t + (int64_t)kStgStages * gridDim.x, st, pa, pb);
   }
 }
 
@@ -766,6 +983,129 @@ unsigned grid_cap(int64_t blocks, int per_sm = 8) {
   return (unsigned)(blocks < 1 ? 1 : blocks);
 }
 
+// staged CSR kernels (TMA row-tile pipeline) under NITRO_CSR_IMPL_AUTO: off by
+// default (B200: slower than the direct kernels on every
+// class measured); NITRO_CSR_STAGED=1 turns them on for AUTO
+bool csr_staged_on() {
+  static bool v = [] {
+    const char *e = getenv("NITRO_CSR_STAGED");
+    return e ? atoi(e) != 0 : false;
+  }();
+  return v;
+}
+
+// CSR-vector rows per pipeline stage R: 2 (B200 sweep: R = 2 beat 4 and 8 on
+// every class — registers and resident warps beat rows in flight per lane);
+// NITRO_CSRV_R=4 overrides
+int csrv_rows(int V) {
+  static int env = [] {
+    const char *e = getenv("NITRO_CSRV_R");
+    return e ? atoi(e) : 0;
+  }();
+  return (env == 4 && V >= 4) ? 4 : 2;
+}
+
+// CSR-vector remainder batch kB = 3 (terms 2..4 of a lane in one batch;
+// longer rows loop); NITRO_CSRV_B=7 batches every term of the short path
+int csrv_batch(const nitro_spmv *A, int V) {
+  static int env = [] {
+    const char *e = getenv("NITRO_CSRV_B");
+    return e ? atoi(e) : 0;
+  }();
+  if (env == 3 || env == 7) return env;
+  (void)A;
+  (void)V;
+  return 3;  // B200 sweep: kB = 7 lost on every class (registers), even rows of > 4V entries
+}
+
+// CSR-scalar head batch H (entries loaded before the first gather): the
+// smallest of 4 / 8 / 16 covering the mean row length; NITRO_CSRS_HEAD overrides
+int csrs_head(const nitro_spmv *A) {
+  static int env = [] {
+    const char *e = getenv("NITRO_CSRS_HEAD");
+    return e ? atoi(e) : 0;
+  }();
+  if (env == 4 || env == 8 || env == 16) return env;
+  const double mean = A->N > 0 ? (double)A->Z / (double)A->N : 0.0;
+  return mean <= 8.0 ? 8 : 16;  // B200: H = 8 beat 4 on every short-row class measured
+}
+
+struct SegArgs {
+  int64_t nseg = 0;
+  int32_t *row = nullptr, *k = nullptr;
+  double *part = nullptr;
+  unsigned *ctr = nullptr;
+};
+
+template <int V, int RPT, typename IT, typename VT>
+nitro_status_t launch_staged_k(const IT *rp, const int32_t *col, const VT *val, const VT *x, VT *y, int64_t N,
+                               int rpg, const SegArgs &sg, bool l2ef, cudaStream_t s) {
+  constexpr size_t sm = stg_smem<VT>();
+  static int bps = -1;  // resident CTAs per SM at this shared-memory size
+  if (bps < 0) {
+    NITRO_CUDA(cudaFuncSetAttribute(k_csr_staged<V, RPT, IT, VT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+    int b = 0;
+    NITRO_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_csr_staged<V, RPT, IT, VT>, kStgThr, sm));
+    bps = std::max(b, 1);
+  }
+  const int64_t TR = V == 1 ? (int64_t)kStgThr * RPT : (int64_t)(kStgThr / V) * rpg;
+  const int64_t ntiles = (N + TR - 1) / TR;
+  const int64_t cap = (int64_t)num_sms() * bps;
+  int64_t grid = std::min<int64_t>(ntiles, cap);
+  if (V > 1) grid = std::max<int64_t>(grid, std::min<int64_t>((sg.nseg + 7) / 8, cap));
+  k_csr_staged<V, RPT, IT, VT><<<(unsigned)std::max<int64_t>(grid, 1), kStgThr, sm, s>>>(
+      rp, col, val, x, y, N, ntiles, rpg, sg.nseg, sg.row, sg.k, sg.part, sg.ctr, l2ef);
+  NITRO_CUDA(cudaGetLastError());
+  return NITRO_OK;
+}
+
+// Tile height: the largest that keeps a mean tile within half a stage (and the
+// rowptr slice within kStgRpBytes); matrices whose rows are too long for one
+// row (V = 1) or R rows per lane group (V > 1) per tile keep the direct kernels.
+template <typename IT, typename VT>
+nitro_status_t launch_staged(const nitro_spmv *A, int V, const IT *rp, const VT *val, const VT *x, VT *y, int64_t N,
+                             const SegArgs &sg, cudaStream_t s, bool &used) {
+  used = false;
+  const bool force = A->csr_impl == NITRO_CSR_IMPL_STAGED;
+  if (A->csr_impl == NITRO_CSR_IMPL_DIRECT || (!force && !csr_staged_on()) || N <= 0 || A->N <= 0) return NITRO_OK;
+  const double mean = (double)A->Z / (double)A->N;
+  constexpr double CAP = stg_cap<VT>();
+  constexpr int sp = (int)sizeof(IT);
+  const bool l2ef = l2_evict_first();
+  if (V == 1) {
+    int rpt = 0;
+    for (int c = 4; c >= 1 && !rpt; c /= 2)
+      if (c * kStgThr * sp <= kStgRpBytes && c * kStgThr * mean <= CAP / 2) rpt = c;
+    if (!rpt) {
+      if (kStgThr * mean > 0.75 * CAP && !force) return NITRO_OK;
+      rpt = 1;
+    }
+    used = true;
+    switch (rpt) {
+      case 4: return launch_staged_k<1, 4, IT, VT>(rp, A->col, val, x, y, N, 0, sg, l2ef, s);
+      case 2: return launch_staged_k<1, 2, IT, VT>(rp, A->col, val, x, y, N, 0, sg, l2ef, s);
+      default: return launch_staged_k<1, 1, IT, VT>(rp, A->col, val, x, y, N, 0, sg, l2ef, s);
+    }
+  }
+  const int R = V >= 4 ? 4 : 2, G = kStgThr / V;
+  int rpg = 0;
+  for (int c = 8 * R; c >= R && !rpg; c /= 2)
+    if (c * G * sp <= kStgRpBytes && c * G * mean <= CAP / 2) rpg = c;
+  if (!rpg) {
+    if (R * G * mean > 0.75 * CAP && !force) return NITRO_OK;
+    rpg = R;  // R * G * sp <= 2048 for every V
+  }
+  used = true;
+  const bool ef = l2ef && V >= 16;  // as the direct kernel: the hint hurts short rows
+  switch (V) {
+    case 2: return launch_staged_k<2, 0, IT, VT>(rp, A->col, val, x, y, N, rpg, sg, ef, s);
+    case 4: return launch_staged_k<4, 0, IT, VT>(rp, A->col, val, x, y, N, rpg, sg, ef, s);
+    case 8: return launch_staged_k<8, 0, IT, VT>(rp, A->col, val, x, y, N, rpg, sg, ef, s);
+    case 16: return launch_staged_k<16, 0, IT, VT>(rp, A->col, val, x, y, N, rpg, sg, ef, s);
+    default: return launch_staged_k<32, 0, IT, VT>(rp, A->col, val, x, y, N, rpg, sg, ef, s);
+  }
+}
+
 template <typename IT, typename VT>
 nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_t s, int64_t r0 = 0,
                      int64_t r1 = -1) {
@@ -779,7 +1119,18 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
   y += r0;
   switch (variant) {
     case NITRO_CSR_SCALAR:
-      if (N > 0) k_csr_scalar<IT, VT><<<grid_cap((N + 255) / 256, 16), 256, 0, s>>>(rp, A->col, val, x, y, N);
+      if (N > 0) {
+        bool used = false;
+        NITRO_TRY((launch_staged<IT, VT>)(A, 1, rp, val, x, y, N, SegArgs{}, s, used));
+        if (!used) {
+          const unsigned g = grid_cap((N + 255) / 256, 16);
+          switch (csrs_head(A)) {
+            case 4: k_csr_scalar<4, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N); break;
+            case 16: k_csr_scalar<16, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N); break;
+            default: k_csr_scalar<8, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N); break;
+          }
+        }
+      }
       break;
     case NITRO_CSR_VECTOR: {
       if (part) return fail(NITRO_E_INVALID_ARG, "CSR-vector has no row-range launch");
@@ -789,10 +1140,34 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
       int32_t *seg_k = seg_row + nseg;
       double *seg_part = reinterpret_cast<double *>(reinterpret_cast<char *>(A->csrv.long_rows.p) + nseg * 8);
       unsigned *seg_ctr = reinterpret_cast<unsigned *>(reinterpret_cast<char *>(A->csrv.long_rows.p) + nseg * 16);
+      {
+        SegArgs sg;
+        sg.nseg = nseg;
+        sg.row = seg_row;
+        sg.k = seg_k;
+        sg.part = seg_part;
+        sg.ctr = seg_ctr;
+        bool used = false;
+        NITRO_TRY((launch_staged<IT, VT>)(A, A->csrv.V, rp, val, x, y, N, sg, s, used));
+        if (used) break;
+      }
       // 8 warps x 32 rows per block-iteration; segments are spread over all warps
       const unsigned g = grid_cap(std::max<int64_t>((N + 255) / 256, (nseg + 7) / 8), 8);
 #define NITRO_CSRV(VV)                                                                                      \
-  k_csr_vector<VV, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, nseg, seg_row, seg_k, seg_part, seg_ctr, l2_evict_first() && VV >= 16)
+  do {                                                                                                      \
+    const bool ef_ = l2_evict_first() && VV >= 16;                                                          \
+    const bool b7_ = csrv_batch(A, VV) == 7;                                                                \
+    switch (csrv_rows(VV)) {                                                                                \
+      case 4:                                                                                               \
+        if (b7_) k_csr_vector<VV, (VV >= 4 ? 4 : 2), 7, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, nseg, seg_row, seg_k, seg_part, seg_ctr, ef_); \
+        else k_csr_vector<VV, (VV >= 4 ? 4 : 2), 3, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, nseg, seg_row, seg_k, seg_part, seg_ctr, ef_); \
+        break;                                                                                              \
+      default:                                                                                              \
+        if (b7_) k_csr_vector<VV, 2, 7, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, nseg, seg_row, seg_k, seg_part, seg_ctr, ef_); \
+        else k_csr_vector<VV, 2, 3, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, nseg, seg_row, seg_k, seg_part, seg_ctr, ef_); \
+        break;                                                                                              \
+    }                                                                                                       \
+  } while (0)
       switch (A->csrv.V) {
         case 2: NITRO_CSRV(2); break;
         case 4: NITRO_CSRV(4); break;

@@ -297,6 +297,69 @@ def test_spmv_long_row(cuda, fp64):
             assert np.array_equal(y, y2)
 
 
+def _csr_impls(A, x, cuda, rowptr32=None, shift=(0, 0, 0)):
+    """y of both CSR variants under every kernel implementation.  shift =
+    (rowptr, colidx, vals) element offsets of the arrays inside larger device
+    buffers, so the staged kernel's 16-byte chunk rounding sees misaligned spans."""
+    import torch
+    n = nitro()
+    Ad = synth.to_device(A, cuda, rowptr32=rowptr32)
+
+    def shifted(t, k):
+        if k == 0:
+            return t
+        buf = torch.zeros(t.numel() + k, dtype=t.dtype, device=cuda)
+        buf[k:] = t
+        return buf[k:]
+    rp, ci, vv = (shifted(t, k) for t, k in zip((Ad.rowptr, Ad.colidx, Ad.vals), shift))
+    M = n.SpMV(rp, ci, vv, A.rows, A.cols)
+    xd = torch.from_numpy(x).to(cuda)
+    out = {}
+    for v in (n.CSR_SCALAR, n.CSR_VECTOR):
+        for impl in (n.CSR_IMPL_AUTO, n.CSR_IMPL_DIRECT, n.CSR_IMPL_STAGED):
+            M.set_csr_impl(impl)
+            y = torch.full((A.rows,), float("nan"), dtype=xd.dtype, device=cuda)
+            M.run(v, xd, y)
+            torch.cuda.synchronize()
+            out[(v, impl)] = y.cpu().numpy()
+    M.close()
+    return out
+
+
+def _impl_mats():
+    yield from small_mats()
+    yield "long_row_fp32", long_row_matrix()
+    yield "long_row_fp64", long_row_matrix(fp64=True, seed=22)
+    yield "banded_b33_d01", synth.banded(40_000, 33, 0.1, seed=23)   # CSR-scalar's class in configs[3]
+    yield "uniform_var_k3", synth.uniform(50_001, 3, variable=True, seed=24)
+    yield "3d27_n40_fp64", synth.stencil("3d27", 40, mode=1, seed=25, fp64=True)
+
+
+@pytest.mark.parametrize("name,A", list(_impl_mats()))
+def test_csr_impls_bit_identical(cuda, name, A):
+    """The TMA row-tile pipeline (auto / forced, incl. tiles computed from
+    global memory when their span overflows a stage) and the direct kernels run
+    the same per-row arithmetic: y bit-identical, and within the oracle bound."""
+    x = synth.vector(A.cols, seed=41, mode=0, fp64=A.fp64)
+    y_ref, r = oracle.spmv(A, x)
+    for rp32 in ((True, False) if A.nnz < 2**31 else (False,)):
+        out = _csr_impls(A, x, cuda, rowptr32=rp32)
+        for (v, impl), y in out.items():
+            check_y(y, y_ref, r, A.fp64, f"{name} v{v} impl{impl} rp32={rp32}")
+            assert np.array_equal(y, out[(v, 1)]), (name, v, impl, rp32)
+
+
+@pytest.mark.parametrize("shift", [(1, 1, 1), (3, 2, 1), (2, 3, 3)])
+def test_csr_staged_misaligned_spans(cuda, shift):
+    A = synth.banded(30_011, 6, 0.7, seed=26)
+    x = synth.vector(A.cols, seed=42)
+    y_ref, r = oracle.spmv(A, x)
+    out = _csr_impls(A, x, cuda, rowptr32=True, shift=shift)
+    for (v, impl), y in out.items():
+        check_y(y, y_ref, r, False, f"shift {shift} v{v} impl{impl}")
+        assert np.array_equal(y, out[(v, 1)]), (shift, v, impl)
+
+
 def test_run_host_matches_device(cuda):
     n = nitro()
     A = synth.uniform(10000, 7, variable=True, seed=3)

@@ -26,6 +26,10 @@ def make(cfg, dev):
         return synth.rmat(23, 16, seed=7, fp64=True, device=dev)
     if cfg == "short":   # very short rows (CSR-scalar class): 1D 3-pt, 2^23 rows
         return synth.stencil("1d3", 1 << 23, mode=1, seed=3, device=dev)
+    if cfg == "band01":  # sparse band (b = 28, density 0.1): CSR-scalar wins these in configs[3]
+        return synth.banded(1 << 23, 28, 0.1, seed=4, device=dev)
+    if cfg == "uvar3":   # short random rows of variable length (k ~ U{1..4}): CSR-scalar class in configs[3]
+        return synth.uniform(1 << 23, 3, variable=True, seed=6, device=dev)
     raise SystemExit(f"unknown config {cfg}")
 
 
@@ -35,8 +39,9 @@ def main():
     import synth
     args = sys.argv[1:]
     timing = "--time" in args
-    args = [a for a in args if a != "--time"]
-    cfgs = [a for a in args if a in ("c0", "c1", "c1big", "c2a", "c2b", "short")] or ["c1"]
+    csr_ab = "--csr-ab" in args   # also time the CSR variants with the direct kernels
+    args = [a for a in args if a not in ("--time", "--csr-ab")]
+    cfgs = [a for a in args if a in ("c0", "c1", "c1big", "c2a", "c2b", "short", "band01", "uvar3")] or ["c1"]
     want = [] if "none" in args else ([nitro.VARIANT_NAMES.index(v) for v in args if v in nitro.VARIANT_NAMES] or list(range(5)))
     dev = torch.device("cuda:0")
     table = {}
@@ -72,6 +77,12 @@ def main():
                     "ms": med * 1e3, "GBps": info["compulsory_bytes"] / med / 1e9,
                     "GFLOPs": 2 * A.nnz / med / 1e9, "bytes": info["compulsory_bytes"], "width": info["width"],
                     "tail": info["tail"], "launches": M.launches(v)}
+                if csr_ab and v in (nitro.CSR_SCALAR, nitro.CSR_VECTOR):
+                    M.set_csr_impl(nitro.CSR_IMPL_DIRECT)
+                    med, _ = M.time(v, x, y, warmup=3, reps=20, flush_l2=True)
+                    M.set_csr_impl(nitro.CSR_IMPL_AUTO)
+                    row["variants"][nitro.VARIANT_NAMES[v] + "_direct"] = {
+                        "ms": med * 1e3, "GBps": info["compulsory_bytes"] / med / 1e9}
             else:
                 for _ in range(2):
                     M.flush_l2()
