@@ -64,6 +64,9 @@ def lib():
         L.oracle_spmv.restype = None
         L.oracle_features.argtypes = [i64, i64, vp, vp, ctypes.POINTER(Features), vp]
         L.oracle_is_canonical.argtypes = [i64, i64, i64, vp, vp]
+        L.oracle_finish_features.argtypes = [i64, i64, i64, ctypes.c_uint64, ctypes.c_uint64, i64, i64,
+                                             ctypes.POINTER(Features)]
+        L.oracle_finish_features.restype = None
         L.oracle_csr_to_ell.argtypes = [i64, vp, vp, vp, i64, i64, vp, vp]
         L.oracle_ell_to_csr.argtypes = [i64, i64, i64, vp, vp, vp, vp, vp]
         L.oracle_ell_to_csr.restype = i64
@@ -120,6 +123,15 @@ def features(A, with_offsets: bool = False):
     assert rc == 0
     if with_offsets:
         return f.as_dict(), offs[: f.ndiag].copy()
+    return f.as_dict()
+
+
+def finish_features(N: int, M: int, Z: int, s1: int, s2: int, lmax: int, D: int) -> dict:
+    """C4 finishing step alone, from exact integers (e.g. closed forms of a
+    matrix too large for the host); 'canonical' is reported as 1."""
+    f = Features()
+    f.canonical = 1
+    lib().oracle_finish_features(N, M, Z, s1, s2, lmax, D, ctypes.byref(f))
     return f.as_dict()
 
 

@@ -66,6 +66,31 @@ int oracle_is_canonical(int64_t N, int64_t M, int64_t Z, const int64_t *rowptr, 
   return 1;
 }
 
+/* The finishing step of C4 on given exact integers (also used alone where the
+ * integers come from closed forms, e.g. configs[4] whose CSR does not fit the
+ * host): fp64, round-to-nearest, no contraction; all doubles 0 when N = 0.
+ * Leaves canonical as it finds it. */
+void oracle_finish_features(int64_t N, int64_t M, int64_t Z, uint64_t s1, uint64_t s2, int64_t lmax, int64_t D,
+                            oracle_features_t *f) {
+  f->rows = N;
+  f->cols = M;
+  f->nnz = Z;
+  f->sum_len = s1;
+  f->sum_len2 = s2;
+  f->max_row = lmax;
+  f->ndiag = D;
+  f->mean = f->sd = f->max_dev = f->dia_fill = f->ell_fill = 0.0;
+  if (N == 0) return;
+  __int128 num = (__int128)N * (__int128)s2 - (__int128)s1 * (__int128)s1;
+  int64_t Zc = Z > 1 ? Z : 1;
+  f->mean = (double)s1 / (double)N;
+  double var = (double)num / ((double)N * (double)N);
+  f->sd = sqrt(var);
+  f->max_dev = (double)lmax - f->mean;
+  f->dia_fill = (double)D * (double)N / (double)Zc;
+  f->ell_fill = (double)lmax * (double)N / (double)Zc;
+}
+
 /* offsets_out (nullable, capacity N+M-1) receives the distinct diagonal offsets
  * d = col - row in ascending order.  Returns 0. */
 int oracle_features(int64_t N, int64_t M, const int64_t *rowptr, const int32_t *col,
@@ -101,19 +126,7 @@ int oracle_features(int64_t N, int64_t M, const int64_t *rowptr, const int32_t *
       ++D;
     }
   free(seen);
-  f->sum_len = s1;
-  f->sum_len2 = s2;
-  f->max_row = lmax;
-  f->ndiag = D;
-  /* finishing (fp64, round-to-nearest, no contraction) */
-  __int128 num = (__int128)N * (__int128)s2 - (__int128)s1 * (__int128)s1;
-  int64_t Zc = f->nnz > 1 ? f->nnz : 1;
-  f->mean = (double)s1 / (double)N;
-  double var = (double)num / ((double)N * (double)N);
-  f->sd = sqrt(var);
-  f->max_dev = (double)lmax - f->mean;
-  f->dia_fill = (double)D * (double)N / (double)Zc;
-  f->ell_fill = (double)lmax * (double)N / (double)Zc;
+  oracle_finish_features(N, M, f->nnz, s1, s2, lmax, D, f);
   return 0;
 }
 

@@ -173,6 +173,23 @@ def test_features_3d27_n128_golden():
     assert ulp_close(f["sd"], exact_sd(g["rows"], g["nnz"], g["sum_len2"]))
 
 
+def test_finish_features_matches_full_pass_and_n512_closed_form():
+    """The finishing step alone (used where the integers come from closed forms)
+    equals the full pass on a computed matrix, and at 512^3 (BASELINE configs[4],
+    whose CSR does not fit the host) gives the exact-rational sd within 2 ulp."""
+    A = synth.stencil("3d27", 12, mode=1, seed=4)
+    f = oracle.features(A)
+    g = oracle.finish_features(f["rows"], f["cols"], f["nnz"], f["sum_len"], f["sum_len2"], f["max_row"], f["ndiag"])
+    assert g == f
+    c = GOLDEN["3d27_n512"]
+    g = oracle.finish_features(c["rows"], c["rows"], c["nnz"], c["nnz"], c["sum_len2"], 27, 27)
+    assert ulp_close(g["sd"], exact_sd(c["rows"], c["nnz"], c["sum_len2"]))
+    assert g["mean"] == c["nnz"] / c["rows"] and g["max_dev"] == 27 - c["nnz"] / c["rows"]
+    assert g["dia_fill"] == g["ell_fill"] == 27 * c["rows"] / c["nnz"]
+    z = oracle.finish_features(0, 5, 0, 0, 0, 0, 0)
+    assert z["mean"] == z["sd"] == z["dia_fill"] == 0.0
+
+
 @pytest.mark.parametrize("n", [2, 5, 1000])
 def test_features_1d3(n):
     f = oracle.features(synth.stencil("1d3", n))
