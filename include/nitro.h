@@ -90,6 +90,14 @@ nitro_status_t nitro_cv_add_feature_group(nitro_cv *cv, const char *const *names
 /* add_constraint(&variant, &constraint).  Several may be
  * added per variant; all must hold. */
 nitro_status_t nitro_cv_add_constraint(nitro_cv *cv, int variant_id, nitro_constraint_fn fn, void *user);
+/* Feature transform of the model (R11; default none = libSVM's
+ * svm-scale): features j with bit j of log_mask set are replaced by
+ * log1p(x) (they must be >= 0) before the [-1, 1] min-max scaling; clip != 0
+ * clips scaled inputs to [-1, 1], so inputs beyond the training range are
+ * treated as the nearest training extreme instead of extrapolated by the RBF
+ * kernel.  Before training (NITRO_E_STATE after); saved in the model file.
+ * nitro_spmv_register sets log_mask = all seven features, clip = 1. */
+nitro_status_t nitro_cv_set_feature_transform(nitro_cv *cv, uint32_t log_mask, int clip);
 /* set_training_args.  `input` is borrowed until train returns. */
 nitro_status_t nitro_cv_add_training_input(nitro_cv *cv, void *input);
 

@@ -18,13 +18,13 @@ import math
 
 import numpy as np
 
-from .select import (ProbModel, bvsb_pick, exhaustive_best, grid_search, scale_apply, scale_fit, splitmix64,
-                     svc_fit, LOG2C, LOG2G)
+from .select import (ProbModel, bvsb_pick, exhaustive_best, feature_transform, grid_search, scale_apply, scale_fit,
+                     splitmix64, svc_fit, LOG2C, LOG2G)
 
 
 def itune(F_pool, label_fn, n_var, init=0, iters=0, acc=0.0, seed=0, prob_folds=5, test_feat=None,
-          test_cost=None, folds=5, tol=1e-6, log2c=LOG2C, log2g=LOG2G, default=1):
-    F_pool = np.asarray(F_pool, dtype=np.float64)
+          test_cost=None, folds=5, tol=1e-6, log2c=LOG2C, log2g=LOG2G, default=1, log_mask=0, clip=False):
+    F_pool = feature_transform(F_pool, log_mask)
     n = F_pool.shape[0]
     lo, hi = scale_fit(F_pool)
     Xall = scale_apply(F_pool, lo, hi)
@@ -55,7 +55,7 @@ def itune(F_pool, label_fn, n_var, init=0, iters=0, acc=0.0, seed=0, prob_folds=
         svc, const = svc_fit(X, y, C, g, tol)
         a = p = float("nan")
         if test_feat is not None:
-            Xt = scale_apply(np.asarray(test_feat, dtype=np.float64), lo, hi)
+            Xt = scale_apply(feature_transform(test_feat, log_mask), lo, hi, clip)
             pred = np.full(len(Xt), const) if svc is None else svc.predict(Xt)
             ok, ps, cnt = 0, 0.0, 0
             for t, v in enumerate(pred):

@@ -62,13 +62,29 @@ def nitro_percent(costs, selected) -> dict:
 
 
 # ---------------------------------------------------------------- C11 scaling
+# Reading R11 for the SpMV feature set: all seven features are >= 0
+# and heavy-tailed, so the model sees log1p(x), min-max scaled, and clips
+# scaled inputs to [-1, 1].  Other feature sets default to plain svm-scale.
+SPMV_LOG_MASK, SPMV_CLIP = 0x7F, True
+
+
+def feature_transform(X, log_mask: int = 0):
+    """log1p of the columns j with bit j of log_mask set (values must be >= 0)."""
+    X = np.array(X, dtype=np.float64, copy=True)
+    for j in range(X.shape[1]):
+        if (log_mask >> j) & 1:
+            X[:, j] = np.log1p(X[:, j])
+    return X
+
+
 def scale_fit(X):
     X = np.asarray(X, dtype=np.float64)
     return X.min(axis=0), X.max(axis=0)
 
 
-def scale_apply(X, lo, hi):
-    """x' = -1 + 2 (x - lo) / (hi - lo); a constant feature maps to 0; no clipping."""
+def scale_apply(X, lo, hi, clip: bool = False):
+    """x' = -1 + 2 (x - lo) / (hi - lo); a constant feature maps to 0; clipped
+    to [-1, 1] only if clip."""
     X = np.asarray(X, dtype=np.float64)
     out = np.zeros_like(X)
     for j in range(X.shape[1]):
@@ -76,7 +92,7 @@ def scale_apply(X, lo, hi):
             out[:, j] = 0.0
         else:
             out[:, j] = -1.0 + 2.0 * (X[:, j] - lo[j]) / (hi[j] - lo[j])
-    return out
+    return np.clip(out, -1.0, 1.0) if clip else out
 
 
 # ---------------------------------------------------------------- C12 SVM + CV
@@ -98,9 +114,10 @@ def fold_assign(y, k: int, seed: int = 0) -> np.ndarray:
 class Model:
     """Scaled-feature RBF C-SVC (one-vs-one), or a constant if one class."""
 
-    def __init__(self, lo, hi, C, gamma, svc=None, const_label=None):
+    def __init__(self, lo, hi, C, gamma, svc=None, const_label=None, log_mask=0, clip=False):
         self.lo, self.hi, self.C, self.gamma = lo, hi, C, gamma
         self.svc, self.const_label = svc, const_label
+        self.log_mask, self.clip = log_mask, clip
 
     def predict_scaled(self, Xs):
         Xs = np.asarray(Xs, dtype=np.float64)
@@ -109,7 +126,7 @@ class Model:
         return self.svc.predict(Xs).astype(np.int64)
 
     def predict(self, X):
-        return self.predict_scaled(scale_apply(X, self.lo, self.hi))
+        return self.predict_scaled(scale_apply(feature_transform(X, self.log_mask), self.lo, self.hi, self.clip))
 
 
 def svc_fit(Xs, y, C: float, gamma: float, tol: float = 1e-6):
@@ -151,14 +168,15 @@ def grid_search(Xs, y, folds: int = 5, seed: int = 0, tol: float = 1e-6, log2c=L
     return best, table
 
 
-def train(F, labels, folds: int = 5, seed: int = 0, tol: float = 1e-6, log2c=LOG2C, log2g=LOG2G) -> Model:
-    """Scale -> CV grid -> refit on all data."""
-    F = np.asarray(F, dtype=np.float64)
+def train(F, labels, folds: int = 5, seed: int = 0, tol: float = 1e-6, log2c=LOG2C, log2g=LOG2G,
+          log_mask: int = 0, clip: bool = False) -> Model:
+    """(Transform ->) scale -> CV grid -> refit on all data."""
+    F = feature_transform(F, log_mask)
     lo, hi = scale_fit(F)
     Xs = scale_apply(F, lo, hi)
     (acc, lc, lg), _ = grid_search(Xs, labels, folds, seed, tol, log2c, log2g)
     svc, const = svc_fit(Xs, labels, 2.0 ** lc, 2.0 ** lg, tol)
-    m = Model(lo, hi, 2.0 ** lc, 2.0 ** lg, svc, const)
+    m = Model(lo, hi, 2.0 ** lc, 2.0 ** lg, svc, const, log_mask, clip)
     m.cv_accuracy = acc
     return m
 

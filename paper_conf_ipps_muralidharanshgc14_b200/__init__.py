@@ -112,6 +112,7 @@ _SIGS = {
     "nitro_cv_model_info": ([_vp, _P(_dbl), _P(_dbl), _P(_dbl), _P(_int)], _int),
     "nitro_cv_save_model": ([_vp, ctypes.c_char_p], _int),
     "nitro_cv_load_model": ([_vp, ctypes.c_char_p], _int),
+    "nitro_cv_set_feature_transform": ([_vp, ctypes.c_uint32, _int], _int),
     "nitro_cv_num_features": ([_vp, _P(_int)], _int),
     "nitro_cv_num_variants": ([_vp, _P(_int)], _int),
     "nitro_cv_select": ([_vp, _vp, _P(_int), _vp], _int),
@@ -388,6 +389,10 @@ class CodeVariant:
 
     def register_spmv(self):
         _check(_L.nitro_spmv_register(self.h))
+
+    def set_feature_transform(self, log_mask: int, clip: bool):
+        """log1p of the features in log_mask, clip scaled inputs (nitro_cv_set_feature_transform)."""
+        _check(_L.nitro_cv_set_feature_transform(self.h, int(log_mask), int(bool(clip))))
 
     def train(self, **opts):
         o = train_opts(**opts)

@@ -49,6 +49,11 @@ struct nitro_cv {
   int n_in = 0;
   std::vector<double> t_feat, t_cost;
   std::vector<int> t_label;
+  // feature transform (nitro_cv_set_feature_transform): log1p of the features
+  // in flog (bit j = feature j) before min-max scaling; fclip clips scaled
+  // inputs to [-1, 1]
+  uint32_t flog = 0;
+  int fclip = 0;
   // model
   std::vector<double> lo, hi;
   double C = 1.0, gamma = 1.0, cv_acc = 0.0;
@@ -85,10 +90,19 @@ bool allowed(const nitro_cv *cv, int v, const void *input) {
   return true;
 }
 
+// feature j as the model sees it: log1p(x) for the features in flog (R11)
+inline double tf(const nitro_cv *cv, int j, double x) {
+  return (j < 32 && ((cv->flog >> j) & 1u)) ? std::log1p(x) : x;
+}
+
 void scale_row(const nitro_cv *cv, const double *f, double *out) {
-  // x' = -1 + 2 (x - lo) / (hi - lo); constant feature -> 0; no clipping (R11)
-  for (int j = 0; j < cv->n_feat; ++j)
-    out[j] = cv->hi[j] == cv->lo[j] ? 0.0 : -1.0 + 2.0 * (f[j] - cv->lo[j]) / (cv->hi[j] - cv->lo[j]);
+  // x' = -1 + 2 (t(x) - lo) / (hi - lo); constant feature -> 0; clipped to
+  // [-1, 1] when fclip (R11)
+  for (int j = 0; j < cv->n_feat; ++j) {
+    double v = cv->hi[j] == cv->lo[j] ? 0.0 : -1.0 + 2.0 * (tf(cv, j, f[j]) - cv->lo[j]) / (cv->hi[j] - cv->lo[j]);
+    if (cv->fclip) v = v < -1.0 ? -1.0 : (v > 1.0 ? 1.0 : v);
+    out[j] = v;
+  }
 }
 
 int predict_raw(const nitro_cv *cv, const double *f) {
@@ -103,8 +117,9 @@ void scale_from(nitro_cv *cv, const double *F, int n) {
   cv->hi.assign(d, -kInf);
   for (int i = 0; i < n; ++i)
     for (int j = 0; j < d; ++j) {
-      cv->lo[j] = std::min(cv->lo[j], F[(size_t)i * d + j]);
-      cv->hi[j] = std::max(cv->hi[j], F[(size_t)i * d + j]);
+      const double v = tf(cv, j, F[(size_t)i * d + j]);
+      cv->lo[j] = std::min(cv->lo[j], v);
+      cv->hi[j] = std::max(cv->hi[j], v);
     }
 }
 
@@ -212,6 +227,14 @@ nitro_status_t nitro_cv_add_variant(nitro_cv *cv, const char *name, nitro_varian
 nitro_status_t nitro_cv_set_default(nitro_cv *cv, int id) {
   if (!cv || id < 0 || id >= (int)cv->variants.size()) return fail(NITRO_E_INVALID_ARG, "bad variant id");
   cv->default_id = id;
+  return NITRO_OK;
+}
+
+nitro_status_t nitro_cv_set_feature_transform(nitro_cv *cv, uint32_t log_mask, int clip) {
+  if (!cv) return fail(NITRO_E_INVALID_ARG, "NULL argument");
+  if (cv->frozen) return fail(NITRO_E_STATE, "code variant already trained");
+  cv->flog = log_mask;
+  cv->fclip = clip ? 1 : 0;
   return NITRO_OK;
 }
 
@@ -529,7 +552,8 @@ nitro_status_t nitro_cv_save_model(const nitro_cv *cv, const char *path) {
   FILE *f = std::fopen(path, "w");
   if (!f) return fail(NITRO_E_IO, std::string("cannot write ") + path);
   const SvmModel &m = cv->svm;
-  std::fprintf(f, "NITRO_MODEL 1\n%d %d %d\n", cv->n_feat, (int)cv->variants.size(), cv->default_id);
+  std::fprintf(f, "NITRO_MODEL 2\n%d %d %d\n%u %d\n", cv->n_feat, (int)cv->variants.size(), cv->default_id,
+               (unsigned)cv->flog, cv->fclip);
   for (int j = 0; j < cv->n_feat; ++j) std::fprintf(f, "%.17g %.17g\n", cv->lo[j], cv->hi[j]);
   std::fprintf(f, "%.17g %.17g %.17g\n", cv->C, cv->gamma, cv->cv_acc);
   std::fprintf(f, "%d %d %d %zu\n", m.d, m.n_train, m.const_label, m.classes.size());
@@ -552,9 +576,15 @@ nitro_status_t nitro_cv_load_model(nitro_cv *cv, const char *path) {
   if (!f) return fail(NITRO_E_IO, std::string("cannot read ") + path);
   auto bad = [&](const char *why) { std::fclose(f); return fail(NITRO_E_IO, std::string("bad model file: ") + why); };
   int ver = 0, nf = 0, nv = 0, def = 0;
-  if (std::fscanf(f, "NITRO_MODEL %d\n%d %d %d", &ver, &nf, &nv, &def) != 4 || ver != 1) return bad("header");
+  if (std::fscanf(f, "NITRO_MODEL %d\n%d %d %d", &ver, &nf, &nv, &def) != 4 || (ver != 1 && ver != 2))
+    return bad("header");
+  unsigned flog = 0;
+  int fclip = 0;
+  if (ver >= 2 && std::fscanf(f, "%u %d", &flog, &fclip) != 2) return bad("feature transform");
   if (cv->n_feat && nf != cv->n_feat) return bad("feature count differs from this code variant");
   if (!cv->variants.empty() && nv != (int)cv->variants.size()) return bad("variant count differs");
+  cv->flog = flog;
+  cv->fclip = fclip;
   cv->lo.assign(nf, 0.0);
   cv->hi.assign(nf, 0.0);
   for (int j = 0; j < nf; ++j)
@@ -666,6 +696,10 @@ nitro_status_t nitro_spmv_register(nitro_cv *cv) {
   NITRO_TRY(nitro_cv_add_feature_group(cv, fn, 7, spmv_feature_group, nullptr));
   NITRO_TRY(nitro_cv_add_constraint(cv, NITRO_DIA, spmv_constraint, (void *)(intptr_t)NITRO_DIA));
   NITRO_TRY(nitro_cv_add_constraint(cv, NITRO_ELL, spmv_constraint, (void *)(intptr_t)NITRO_ELL));
+  // the seven SpMV features are >= 0 and heavy-tailed (nnz and rows span
+  // decades, fills up to 1e4): log1p before scaling, and inputs beyond the
+  // training range clipped to it (R11)
+  NITRO_TRY(nitro_cv_set_feature_transform(cv, 0x7fu, 1));
   return nitro_cv_set_default(cv, NITRO_CSR_VECTOR);
   GUARD_END
 }

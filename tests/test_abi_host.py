@@ -179,10 +179,41 @@ def test_train_from_table_equals_oracle():
     cv = n.CodeVariant(ctx, "t")
     cv.register_spmv()
     cv.train_from_table(F, costs, log2c_lo=-5, log2c_hi=15, log2g_lo=-15, log2g_hi=3)
-    m = S.train(F, S.exhaustive_best(costs.tolist()))
+    # register_spmv sets the SpMV feature transform (R11: log1p of all seven, clipping)
+    m = S.train(F, S.exhaustive_best(costs.tolist()), log_mask=S.SPMV_LOG_MASK, clip=S.SPMV_CLIP)
     info = cv.model_info()
     assert (info["C"], info["gamma"]) == (m.C, m.gamma)
     assert info["cv_accuracy"] == pytest.approx(m.cv_accuracy)
+    # predictions agree, including inputs far outside the training range (clipped)
+    T = np.abs(rng.normal(0, 1, (30, 7))) * np.array([1e6, 1e5, 10, 3, 50, 2, 2])
+    T[:10] *= 1e3
+    ours = [cv.predict(t) for t in T]
+    ref = m.predict(T).tolist()
+    assert sum(a == b for a, b in zip(ours, ref)) >= len(T) - 1
+
+
+def test_feature_transform_clips_to_training_extremes():
+    """With clipping, an input beyond the training range predicts like the
+    training extreme it is clipped to; without it the RBF model extrapolates."""
+    n = nitro()
+    F = np.array([[1.0, 10.0], [2.0, 20.0], [3.0, 30.0], [4.0, 40.0], [5.0, 50.0], [6.0, 60.0]])
+    costs = np.array([[1, 2], [1, 2], [1, 2], [2, 1], [2, 1], [2, 1]], float)
+    for clip in (False, True):
+        ctx = n.Context()
+        cv = n.CodeVariant(ctx, f"clip{clip}")
+        for v in range(2):
+            cv.add_variant(f"v{v}", lambda inp: 0.0)
+        for j in range(2):
+            cv.add_feature(f"f{j}", lambda inp: 0.0)
+        cv.set_feature_transform(0b11, clip)
+        cv.train_from_table(F, costs, log2c_lo=1, log2c_hi=1, log2g_lo=1, log2g_hi=1)
+        m = S.train(F, S.exhaustive_best(costs.tolist()), log2c=[1], log2g=[1], log_mask=0b11, clip=clip)
+        far = np.array([[6.0e6, 6.0e7]])
+        assert cv.predict(far[0]) == m.predict(far)[0]
+        if clip:
+            assert cv.predict(far[0]) == cv.predict(F[-1]) == 1
+    with pytest.raises(n.NitroError):
+        cv.set_feature_transform(0, False)   # after training: NITRO_E_STATE
 
 
 def test_dist_partition_nnz_balanced():

@@ -51,7 +51,7 @@ def test_library_training_matches_oracle():
     t, rep = _load()
     F = np.array([r["features"] for r in t["train"]])
     lab = S.exhaustive_best(_costs(t["train"]))
-    m = S.train(F, lab)
+    m = S.train(F, lab, log_mask=S.SPMV_LOG_MASK, clip=S.SPMV_CLIP)   # nitro_spmv_register's transform
     assert (rep["model"]["C"], rep["model"]["gamma"]) == (m.C, m.gamma)
     assert rep["model"]["cv_accuracy"] == pytest.approx(m.cv_accuracy, abs=1e-12)
     # the committed model file selects like the oracle model on the held-out set

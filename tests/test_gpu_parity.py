@@ -160,6 +160,31 @@ def test_features_mixed_walks(cuda, rp32):
         assert f[k] == f_ref[k], k
 
 
+@pytest.mark.parametrize("rows", [[1000], [1024], [1055], [1023, 1024], [2000, 2001, 2002], [64 * 64 - 1]])
+def test_features_single_row_pattern_change(cuda, rows):
+    """The feature pass skips rows whose offset pattern equals the previous
+    row's: a single interior row of a 2D 5-pt stencil whose last column moves
+    one to the right (lane 0 / lane 31 of a 32-row block, runs of changed rows,
+    the last row) brings one new diagonal, which must be counted."""
+    n = nitro()
+    A = synth.stencil("2d5", 64)
+    rp = np.asarray(A.rowptr, np.int64)
+    ci = A.colidx.copy()
+    for r in rows:
+        e = rp[r + 1] - 1
+        if r + 1 < A.rows and ci[e] + 1 < A.cols:
+            ci[e] += 1
+        else:                       # last row: move its first column left instead
+            ci[rp[r]] -= 1
+    B = Csr(A.rows, A.cols, rp, ci, A.vals, A.fp64)
+    assert oracle.is_canonical(B)
+    f_ref = oracle.features(B)
+    assert f_ref["ndiag"] > 5
+    M, _ = handle(B, cuda)
+    f = M.features()
+    assert f["ndiag"] == f_ref["ndiag"] and f["dia_fill"] == f_ref["dia_fill"]
+
+
 @pytest.mark.parametrize("where", ["long_chunk_boundary", "long_dup", "medium", "short_var", "short_equal"])
 def test_non_canonical_in_every_walk(cuda, where):
     """A broken row is caught whichever walk of the feature pass visits it."""

@@ -55,6 +55,7 @@ def ablation(table, nitro):
         for f in feats:
             cv.add_feature(f, lambda i: 0.0)
         cv.set_default(nitro.CSR_VECTOR)
+        cv.set_feature_transform((1 << len(cols)) - 1, True)   # as nitro_spmv_register (R11)
         cv.train_from_table(Ftr[:, cols], Ctr)
         ratios = []
         for r in table["test"]:

@@ -34,6 +34,7 @@ def main():
     for v in (nitro.ELL, nitro.DIA):
         cv.add_constraint(v, lambda i, v=v: math.isfinite(Cp[i, v]))
     cv.set_default(nitro.CSR_VECTOR)
+    cv.set_feature_transform(0x7F, True)   # as nitro_spmv_register (R11)
     for i in range(len(Fp)):
         cv.add_training_input(i)
     seeds = [0, 1, 2, 3, 4]
@@ -48,6 +49,7 @@ def main():
         for v in (nitro.ELL, nitro.DIA):
             cvi.add_constraint(v, lambda i, v=v: math.isfinite(Cp[i, v]))
         cvi.set_default(nitro.CSR_VECTOR)
+        cvi.set_feature_transform(0x7F, True)
         for i in range(len(Fp)):
             cvi.add_training_input(i)
         h = cvi.itune(init=len(nitro.VARIANT_NAMES), iters=0, seed=sd, test_feat=Ft, test_cost=Ct)
