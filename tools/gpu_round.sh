@@ -17,6 +17,10 @@ if want c3; then
   timeout 1200 python tools/feature_study.py --gpu > gpurun_out/feature_study.log 2>&1; echo "fstudy rc=$?"; tail -4 gpurun_out/feature_study.log
   mkdir -p gpurun_out/artifacts; cp artifacts/* gpurun_out/artifacts/
 fi
+if want fstudy; then
+  timeout 1200 python tools/feature_study.py --gpu > gpurun_out/feature_study.log 2>&1; echo "fstudy rc=$?"; tail -4 gpurun_out/feature_study.log
+  mkdir -p gpurun_out/artifacts; cp artifacts/feature_study.json gpurun_out/artifacts/
+fi
 if want bench; then
   timeout 600 python bench.py --steps 20 --warmup 5 > gpurun_out/bench.json 2> gpurun_out/bench.err; echo "bench rc=$?"
   cat gpurun_out/bench.json; tail -3 gpurun_out/bench.err
@@ -26,6 +30,9 @@ if want table; then
   echo "table rc=$?"; python -c "
 import json; t=json.load(open('gpurun_out/variant_table.json'))
 for c,r in t.items(): print(c, round(r['feature_ms'],3), {k: round(v['GBps']) for k,v in r['variants'].items()})"
+fi
+if want prof; then
+  bash tools/gpu_check.sh prof
 fi
 if want c4; then
   timeout 1200 python tools/c4_probe.py --out gpurun_out/c4_probe.json > gpurun_out/c4_probe.log 2>&1; echo "c4 rc=$?"; tail -12 gpurun_out/c4_probe.log
