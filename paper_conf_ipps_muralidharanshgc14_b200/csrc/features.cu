@@ -38,6 +38,7 @@ constexpr uint32_t kWin = 1u << 16;     // per-block bitmap of offsets in [-2^15
 constexpr uint32_t kEmpty = 0xffffffffu;
 constexpr int kStage = 1024;            // per-warp staging buffer (entries)
 constexpr int kRowCap = 64;             // lane-per-row walk only for rows up to this length
+constexpr int kQ = 4;                   // 32-row blocks per super-block (one staging round trip for short rows)
 constexpr int64_t kLong = 4096;         // rows longer than this go to k_features_long
 constexpr int64_t kChunk = 4096;        // entries per task of k_features_long
 
@@ -219,11 +220,44 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
   unsigned long long s1 = 0, s2 = 0, lmax = 0;
   const int64_t nblk = (N + 31) / 32;
   const int64_t gw = (int64_t)blockIdx.x * kWarps + wib, nw = (int64_t)gridDim.x * kWarps;
-  for (int64_t rb = gw; rb < nblk; rb += nw) {
+  // Lane-per-row walk of one row of L entries (staged at buf slots rel0.., or
+  // from global memory at entry a).  Per entry: strictly-increasing check
+  // (with prev = -1 it also gives c >= 0; c < M then follows from the last
+  // entry), and the offset's window bit rel = c - row + kWin/2 tested before
+  // it is set.  The bound checks sit outside the loop: the pass is issue-bound
+  // on stencils (ncu: SM throughput 74 %, IPC 3.2), so instructions per entry
+  // are what the loop is tuned for.
+  auto lane_walk_core = [&](auto ld, int L, uint32_t myrow, bool full) {
+    const uint32_t rbase = myrow - (kWin >> 1);
+    int prev = -1;
+    bool inc = true;
+#pragma unroll 4
+    for (int k = 0; k < L; ++k) {
+      const int c = ld(k);
+      inc &= c > prev;
+      prev = c;
+      const uint32_t rel = (uint32_t)c - rbase;
+      if (rel < kWin) {
+        const uint32_t bit = 1u << (rel & 31);
+        if (!(s_win[rel >> 5] & bit)) atomicOr(&s_win[rel >> 5], bit);
+      } else if ((uint32_t)c < M32) {
+        lane_far((uint32_t)c - myrow + G32, full);
+      }
+    }
+    const int first = ld(0);
+    if (first < 0 || (uint32_t)prev >= M32) bad |= 4;
+    else if (!inc) bad |= 2;
+  };
+  auto lane_walk_staged = [&](const int *buf, int rel0, int L, uint32_t myrow, bool full) {
+    lane_walk_core([&](int k) { return buf[skew(rel0 + k)]; }, L, myrow, full);
+  };
+  auto lane_walk_global = [&](int64_t a, int L, uint32_t myrow, bool full) {
+    lane_walk_core([&](int k) { return __ldg(col + a + k); }, L, myrow, full);
+  };
+
+  // One block of 32 rows (lane j <-> row rb*32 + j) with its row bounds a, b.
+  auto process_block = [&](int64_t rb, int64_t a, int64_t b) {
     const int64_t r = rb * 32 + lane;
-    int64_t a, b;
-    if (r < N) { a = (int64_t)rowptr[r]; b = (int64_t)rowptr[r + 1]; }
-    else { a = b = (int64_t)rowptr[N]; }
     const int64_t L = b - a;
     if (L > 0) {
       s1 += (unsigned long long)L;
@@ -232,7 +266,7 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
     }
     // a block of rows with a broken rowptr is not walked (flagged)
     const bool brk = L < 0 || a < 0 || b > Z;
-    if (__any_sync(kFull, brk)) { bad |= brk ? 1u : 0u; continue; }
+    if (__any_sync(kFull, brk)) { bad |= brk ? 1u : 0u; return; }
     const int64_t E0 = __shfl_sync(kFull, a, 0), E1 = __shfl_sync(kFull, b, 31);
     const uint32_t rowbase = (uint32_t)(row0 + rb * 32), myrow = rowbase + (uint32_t)lane;
     // long rows: their kChunk-entry chunks become tasks of k_features_long
@@ -264,37 +298,8 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
     if (maxL <= (unsigned)kRowCap && maxL * 32u <= 2u * sumL) {
       if (Ln > 0) {
         const bool full = *(volatile unsigned *)&s_full != 0;
-        // Per entry: strictly-increasing check (with prev = -1 it also gives
-        // c >= 0; c < M then follows from the last entry), and the offset's
-        // window bit rel = c - row + kWin/2 tested before it is set.  The
-        // bound checks sit outside the loop: the pass is issue-bound on
-        // stencils (ncu: SM throughput 74 %, IPC 3.2), so instructions per
-        // entry are what the loop is tuned for.
-        const uint32_t rbase = myrow - (kWin >> 1);
-        int prev = -1;
-        bool inc = true;
-        auto entry = [&](int c) {
-          inc &= c > prev;
-          prev = c;
-          const uint32_t rel = (uint32_t)c - rbase;
-          if (rel < kWin) {
-            const uint32_t bit = 1u << (rel & 31);
-            if (!(s_win[rel >> 5] & bit)) atomicOr(&s_win[rel >> 5], bit);
-          } else if ((uint32_t)c < M32) {
-            lane_far((uint32_t)c - myrow + G32, full);
-          }
-        };
-        if (staged) {
-          const int rel0 = (int)(a - E0);
-#pragma unroll 4
-          for (int k = 0; k < (int)Ln; ++k) entry(buf[skew(rel0 + k)]);
-        } else {
-#pragma unroll 4
-          for (int k = 0; k < (int)Ln; ++k) entry(__ldg(col + a + k));
-        }
-        const int first = staged ? buf[skew((int)(a - E0))] : __ldg(col + a);
-        if (first < 0 || (uint32_t)prev >= M32) bad |= 4;
-        else if (!inc) bad |= 2;
+        if (staged) lane_walk_staged(buf, (int)(a - E0), (int)Ln, myrow, full);
+        else lane_walk_global(a, (int)Ln, myrow, full);
       }
     } else if (staged) {
       walk_span_warp<true>(buf, E0, E1, E0, a, L > 0, rowbase, G32, M32, win_lo, s_win, s_slot[wib], bitmap, lane,
@@ -316,6 +321,88 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
       }
     }
     __syncwarp();  // the staging buffer is reused by the next block of rows
+  };
+  // Super-blocks of kQ consecutive 32-row blocks: the rowptr loads of all kQ
+  // blocks are issued together, and when every block takes the lane-per-row
+  // walk and their joint colidx span fits the staging buffer (short rows:
+  // stencils of low order, sparse bands, short random rows) that span is
+  // staged by ONE cp.async round trip — the walk of short rows is latency-
+  // bound per iteration, so kQ blocks per round trip is up to kQ x faster.
+  // Otherwise each block goes through process_block as before.
+  const int64_t nsb = (nblk + kQ - 1) / kQ;
+  // register array element j < kQ for a runtime j (no local-memory indexing)
+  auto pick = [](const int64_t (&v)[kQ], int j) {
+    int64_t r = v[0];
+#pragma unroll
+    for (int t = 1; t < kQ; ++t) r = j == t ? v[t] : r;
+    return r;
+  };
+  for (int64_t sb = gw; sb < nsb; sb += nw) {
+    int64_t a[kQ], b[kQ];
+#pragma unroll
+    for (int j = 0; j < kQ; ++j) {
+      const int64_t r = (sb * kQ + j) * 32 + lane;
+      if (r < N) { a[j] = (int64_t)rowptr[r]; b[j] = (int64_t)rowptr[r + 1]; }
+      else { a[j] = b[j] = -1; }
+    }
+    const bool full_sb = (sb + 1) * kQ <= nblk;
+    bool fast = full_sb;
+    unsigned mx[kQ];
+    if (fast) {
+#pragma unroll
+      for (int j = 0; j < kQ; ++j) {
+        const int64_t L = b[j] - a[j];
+        const bool brk = L < 0 || a[j] < 0 || b[j] > Z;
+        const unsigned Lc = brk ? (unsigned)(kRowCap + 1) : (unsigned)(L > kRowCap ? kRowCap + 1 : L);
+        mx[j] = __reduce_max_sync(kFull, Lc);
+        const unsigned sm = __reduce_add_sync(kFull, Lc);
+        fast = fast && mx[j] <= (unsigned)kRowCap && mx[j] * 32u <= 2u * sm;
+      }
+      // contiguous blocks: block j ends where block j + 1 starts (else rowptr is broken)
+      if (fast) {
+        const int64_t A0 = __shfl_sync(kFull, a[0], 0), B1 = __shfl_sync(kFull, b[kQ - 1], 31);
+        bool cont = true;
+#pragma unroll
+        for (int j = 0; j + 1 < kQ; ++j) cont = cont && __shfl_sync(kFull, b[j], 31) == __shfl_sync(kFull, a[j + 1], 0);
+        fast = cont && B1 - A0 <= kStage / 2 && B1 >= A0;  // short rows only (band01-like spans: slower)
+      }
+    }
+    if (!fast) {
+#pragma unroll 1
+      for (int j = 0; j < kQ; ++j) {
+        const int64_t rb = sb * kQ + j;
+        if (rb >= nblk) break;
+        const int64_t r = rb * 32 + lane;
+        int64_t aa = pick(a, j), bb = pick(b, j);
+        if (r >= N) aa = bb = (int64_t)rowptr[N];
+        process_block(rb, aa, bb);
+      }
+      continue;
+    }
+    const int64_t E0 = __shfl_sync(kFull, a[0], 0), E1 = __shfl_sync(kFull, b[kQ - 1], 31);
+    int *buf = s_stage[wib];
+    {
+      const int span = (int)(E1 - E0);
+      for (int e = lane; e < span; e += 32)
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"((uint32_t)__cvta_generic_to_shared(buf + skew(e))),
+                     "l"(col + E0 + e)
+                     : "memory");
+      asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
+      __syncwarp();
+    }
+    const bool full = *(volatile unsigned *)&s_full != 0;
+#pragma unroll 1
+    for (int j = 0; j < kQ; ++j) {
+      const int64_t aj = pick(a, j), L = pick(b, j) - aj;
+      if (L > 0) {
+        s1 += (unsigned long long)L;
+        s2 += (unsigned long long)L * (unsigned long long)L;
+        if ((unsigned long long)L > lmax) lmax = (unsigned long long)L;
+        const uint32_t myrow = (uint32_t)(row0 + (sb * kQ + j) * 32 + lane);
+        lane_walk_staged(buf, (int)(aj - E0), (int)L, myrow, full);
+      }
+    }
+    __syncwarp();  // the staging buffer is reused by the next iteration
   }
   // reduce s1, s2 (sum) and lmax (max) over the block
 #pragma unroll

@@ -189,8 +189,16 @@ __device__ __forceinline__ void csrv_segments(const IT *__restrict__ rowptr, con
   }
 }
 
+// Resident CTAs per SM (launch bounds): occupancy beat per-lane depth in every
+// B200 sweep (issuing the remainder batch a stage ahead: c1 4041 -> 3539 GB/s);
+// fp64 R = 2: 5 CTAs (c2b 1257 -> 1568 GB/s; fp32 loses with 5: c1 4036 -> 3140)
+template <int V, int R, int kB, typename VT>
+constexpr int csrv_min_blocks() {
+  return R * kB >= 16 ? 2 : R * kB >= 12 ? (sizeof(VT) == 4 ? 3 : 2) : (sizeof(VT) == 4 ? 4 : 5);
+}
+
 template <int V, int R, int kB, typename IT, typename VT>
-__global__ void __launch_bounds__(256, R * kB >= 16 ? 2 : R * kB >= 12 ? (sizeof(VT) == 4 ? 3 : 2) : (sizeof(VT) == 4 ? 4 : 3)) k_csr_vector(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
+__global__ void __launch_bounds__(256, csrv_min_blocks<V, R, kB, VT>()) k_csr_vector(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
                                                     const VT *__restrict__ val, const VT *__restrict__ x,
                                                     VT *__restrict__ y, int64_t N, int64_t nseg,
                                                     const int32_t *__restrict__ seg_row,
@@ -1153,6 +1161,7 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
       }
       // 8 warps x 32 rows per block-iteration; segments are spread over all warps
       const unsigned g = grid_cap(std::max<int64_t>((N + 255) / 256, (nseg + 7) / 8), 8);
+      const unsigned gw_ = grid_cap(std::max<int64_t>((N + 255) / 256, (nseg + 7) / 8), 12);
 #define NITRO_CSRV(VV)                                                                                      \
   do {                                                                                                      \
     const bool ef_ = l2_evict_first() && VV >= 16;                                                          \
@@ -1164,6 +1173,7 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
         break;                                                                                              \
       default:                                                                                              \
         if (b7_) k_csr_vector<VV, 2, 7, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, nseg, seg_row, seg_k, seg_part, seg_ctr, ef_); \
+        else if (sizeof(VT) == 8) k_csr_vector<VV, 2, 3, IT, VT><<<gw_, 256, 0, s>>>(rp, A->col, val, x, y, N, nseg, seg_row, seg_k, seg_part, seg_ctr, ef_); \
         else k_csr_vector<VV, 2, 3, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, nseg, seg_row, seg_k, seg_part, seg_ctr, ef_); \
         break;                                                                                              \
     }                                                                                                       \
