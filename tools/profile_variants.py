@@ -30,6 +30,10 @@ def make(cfg, dev):
         return synth.banded(1 << 23, 28, 0.1, seed=4, device=dev)
     if cfg == "uvar3":   # short random rows of variable length (k ~ U{1..4}): CSR-scalar class in configs[3]
         return synth.uniform(1 << 23, 3, variable=True, seed=6, device=dev)
+    if cfg == "band48":  # dense band (b = 48): 97-entry local rows, the long-row CSR-vector class
+        return synth.banded(1 << 21, 48, 1.0, seed=8, device=dev)
+    if cfg == "band96h": # half-dense wide band (b = 96, density 0.5): ~97 local entries per row, uneven lengths
+        return synth.banded(1 << 21, 96, 0.5, seed=9, device=dev)
     raise SystemExit(f"unknown config {cfg}")
 
 
@@ -41,7 +45,7 @@ def main():
     timing = "--time" in args
     csr_ab = "--csr-ab" in args   # also time the CSR variants with the direct kernels
     args = [a for a in args if a not in ("--time", "--csr-ab")]
-    cfgs = [a for a in args if a in ("c0", "c1", "c1big", "c2a", "c2b", "short", "band01", "uvar3")] or ["c1"]
+    cfgs = [a for a in args if a in ("c0", "c1", "c1big", "c2a", "c2b", "short", "band01", "uvar3", "band48", "band96h")] or ["c1"]
     want = [] if "none" in args else ([nitro.VARIANT_NAMES.index(v) for v in args if v in nitro.VARIANT_NAMES] or list(range(5)))
     dev = torch.device("cuda:0")
     table = {}
