@@ -497,14 +497,32 @@ __global__ void __launch_bounds__(kStgThr, 2) k_csr_staged(const IT *__restrict_
 template <typename VT, int U>  // U <= 16: terms per fp32 partial
 __global__ void __launch_bounds__(256) k_ell(const int32_t *__restrict__ ecol, const VT *__restrict__ eval,
                                              const VT *__restrict__ x, VT *__restrict__ y, int64_t N, int64_t K,
-                                             int64_t ld, int64_t nr, bool l2ef) {
+                                             int64_t ld, int64_t nr, bool l2ef, int pf, bool pfh) {
   // rows [0, nr) (nr <= ld: ld for a whole multiply incl. padding, less for a row chunk)
   const uint64_t pol = l2_policy(l2ef);
   const int64_t nq = (nr + 3) >> 2;
+  // pf > 0: thread 0 keeps the block's (col, val) slot segments pf batches
+  // ahead in L2 (cp.async.bulk prefetch; see k_dia).  Whole-multiply launches
+  // only (pf = 0 for row chunks), so B0 and nr are multiples of 32 rows.
+  auto prefetch = [&](int64_t k, int64_t B0, uint32_t rows) {
+    if (pfh) {
+      bulk_prefetch_l2(ecol + k * ld + B0, rows * 4u, pol);
+      bulk_prefetch_l2(eval + k * ld + B0, rows * (uint32_t)sizeof(VT), pol);
+    } else {
+      bulk_prefetch_l2(ecol + k * ld + B0, rows * 4u);
+      bulk_prefetch_l2(eval + k * ld + B0, rows * (uint32_t)sizeof(VT));
+    }
+  };
   for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < nq; q += (int64_t)gridDim.x * blockDim.x) {
     const int64_t i0 = q << 2;
+    const int64_t B0 = (q - threadIdx.x) << 2;  // block's first row this iteration
+    const uint32_t pr = (uint32_t)((B0 + 4 * (int64_t)blockDim.x < nr ? B0 + 4 * (int64_t)blockDim.x : nr) - B0);
+    if (pf > 0 && threadIdx.x == 0)
+      for (int64_t k = 0; k < (int64_t)pf * U && k < K; ++k) prefetch(k, B0, pr);
     double acc[4] = {0.0, 0.0, 0.0, 0.0};
     for (int64_t k0 = 0; k0 < K; k0 += U) {
+      if (pf > 0 && threadIdx.x == 0)
+        for (int64_t k = k0 + (int64_t)pf * U; k < k0 + (int64_t)(pf + 1) * U && k < K; ++k) prefetch(k, B0, pr);
       int4 c[U];
       V4<VT> v[U];
 #pragma unroll
@@ -552,10 +570,14 @@ __global__ void __launch_bounds__(256, (U == 1 && DS == 1 && sizeof(VT) == 4) ? 
     k_dia(const int32_t *__restrict__ offs, const VT *__restrict__ dval,
                                              const VT *__restrict__ x, VT *__restrict__ y, int64_t N, int64_t M,
                                              int64_t D, int64_t ld, int64_t nr, int64_t row0, int64_t off_min,
-                                             int64_t off_max, bool x_aligned, bool l2ef) {
+                                             int64_t off_max, bool x_aligned, bool l2ef, int pf, bool pfh) {
   constexpr int64_t RB = 1024 / DS;  // rows per block iteration
   const uint64_t pol = l2_policy(l2ef);
   extern __shared__ int s_off[];
+  // pf > 0: thread 0 keeps the block's value segments pf diagonals ahead in L2
+  // (one cp.async.bulk L2 prefetch per diagonal, no registers or shared
+  // memory): the per-thread chain of dependent value loads then waits on L2,
+  // not HBM, and the HBM stream has pf x 4 KB per CTA in flight.
   for (int64_t d = threadIdx.x; d < D; d += blockDim.x) s_off[d] = offs[d];
   __syncthreads();
   const int q = (int)(threadIdx.x % DS);
@@ -564,6 +586,11 @@ __global__ void __launch_bounds__(256, (U == 1 && DS == 1 && sizeof(VT) == 4) ? 
     const int64_t B0 = blk * RB;
     const int64_t i0 = B0 + 4 * (threadIdx.x / DS);
     const bool active = i0 < nr;  // whole DS groups share i0: uniform within a group
+    // segment bytes of one diagonal of this block (16-byte multiple: B0 and ld are multiples of 32 rows)
+    const uint32_t pfb = (uint32_t)(((B0 + RB < nr ? B0 + RB : nr) - B0) * (int64_t)sizeof(VT)) & ~15u;
+    if (pf > 0 && threadIdx.x == 0)
+      for (int64_t d = 0; d < pf && d < D; ++d)
+        pfh ? bulk_prefetch_l2(dval + d * ld + B0, pfb, pol) : bulk_prefetch_l2(dval + d * ld + B0, pfb);
     if constexpr (DS == 1) {
       if (!active) continue;      // no cross-lane combine needed
     }
@@ -573,6 +600,9 @@ __global__ void __launch_bounds__(256, (U == 1 && DS == 1 && sizeof(VT) == 4) ? 
     const bool xvec = x_aligned && row0 + B0 + off_min - 3 >= 0 && row0 + Bend + off_max + 4 < M;
     double acc[4] = {0.0, 0.0, 0.0, 0.0};
     for (int64_t d0 = (int64_t)q * U; (DS == 1 || active) && d0 < D; d0 += (int64_t)DS * U) {
+      if (pf > 0 && threadIdx.x == 0)
+        for (int64_t d = d0 + pf; d < d0 + pf + DS * U && d < D; ++d)
+          pfh ? bulk_prefetch_l2(dval + d * ld + B0, pfb, pol) : bulk_prefetch_l2(dval + d * ld + B0, pfb);
       V4<VT> v[U];
       VT xv[U][4];
 #pragma unroll
@@ -925,6 +955,37 @@ int dia_split(int64_t D) {
   return 1;
 }
 
+// DIA L2 prefetch distance in diagonals: NITRO_DIA_PF overrides; default 1.
+// B200, 3 interleaved repeats (GB/s): configs[1] 128^3 PF=0 5133, 1 5357,
+// 2 5367; 256^3 PF=0 6355, 1 6796, 2 6731.
+int dia_prefetch() {
+  static int env = [] {
+    const char *e = getenv("NITRO_DIA_PF");
+    return e ? atoi(e) : -1;
+  }();
+  return env >= 0 ? env : 1;
+}
+
+// bulk L2 prefetches carry the evict-first policy: NITRO_PF_HINT=0 disables; default on
+bool prefetch_hint() {
+  static int env = [] {
+    const char *e = getenv("NITRO_PF_HINT");
+    return e ? atoi(e) : 1;
+  }();
+  return env != 0;
+}
+
+// ELL L2 prefetch distance in slot batches: NITRO_ELL_PF overrides; default 1.
+// B200 (GB/s, PF 0 -> 1, same box): configs[1] 6035 -> 6369 and 5732 -> 5815,
+// dense band b = 48 6527 -> 6921, 256^3 stencil 5894 -> 6331
+int ell_prefetch() {
+  static int env = [] {
+    const char *e = getenv("NITRO_ELL_PF");
+    return e ? atoi(e) : -1;
+  }();
+  return env >= 0 ? env : 1;
+}
+
 // DIA grid cap in blocks per SM: NITRO_DIA_GRID overrides; default 16
 // (one wave-free launch of every 1024-row block at configs[1])
 int dia_blocks_per_sm() {
@@ -959,16 +1020,28 @@ int ell_batch(size_t sv) {
 
 unsigned grid_cap(int64_t blocks, int per_sm);
 
+// columns on few diagonals (the DIA fill test of C9: D * N <= 3 Z)
+bool diag_local(const nitro_spmv *A) {
+  return A->feat_ready && (double)A->feat.ndiag * (double)A->N <= 3.0 * (double)std::max<int64_t>(A->Z, 1);
+}
+
 template <typename VT>
 void launch_ell(const int32_t *col, const VT *val, const VT *x, VT *y, int64_t N, int64_t K, int64_t ld,
-                cudaStream_t s, int64_t nr = -1) {
+                cudaStream_t s, int64_t nr = -1, bool local = false) {
+  // L2 prefetch of the slot stream: whole multiplies (nr < 0) of matrices whose
+  // columns lie on few diagonals (x gathers hit L1/L2 lines shared by
+  // neighbouring rows).  Random-column matrices are bound by the L2 sector
+  // traffic of the gathers, and the prefetched lines compete with them
+  // (B200, configs[2] uniform ELL: 2110 -> 2060 GB/s with, 1873 without the
+  // evict-first hint), so they run without.
+  const int pf = nr < 0 && local ? ell_prefetch() : 0;
   if (nr < 0) nr = ld;
   const unsigned g = grid_cap(((nr + 3) / 4 + 255) / 256, 16);
   switch (ell_batch(sizeof(VT))) {
-    case 1: k_ell<VT, 1><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first()); break;
-    case 2: k_ell<VT, 2><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first()); break;
-    case 4: k_ell<VT, 4><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first()); break;
-    default: k_ell<VT, 8><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first()); break;
+    case 1: k_ell<VT, 1><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first(), pf, prefetch_hint()); break;
+    case 2: k_ell<VT, 2><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first(), pf, prefetch_hint()); break;
+    case 4: k_ell<VT, 4><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first(), pf, prefetch_hint()); break;
+    default: k_ell<VT, 8><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first(), pf, prefetch_hint()); break;
   }
 }
 
@@ -1191,7 +1264,7 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
     case NITRO_ELL:
       if (N > 0)
         launch_ell<VT>(A->ell.col.as<int32_t>() + r0, A->ell.val.as<VT>() + r0, x, y, N, A->ell.K, A->ell.ld, s,
-                       part ? round_up(N, 32) : A->ell.ld);
+                       part ? round_up(N, 32) : -1, diag_local(A));
       break;
     case NITRO_DIA:
       if (N > 0 && A->dia.D > 0 && dia_use_tma() && !part) return launch_dia_tma(A, x, y, s);
@@ -1204,7 +1277,7 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
 #define NITRO_DIA_LAUNCH(UU, SS)                                                                                   \
   k_dia<VT, UU, SS><<<g, 256, sm, s>>>(A->dia.off.as<int32_t>(), A->dia.val.as<VT>() + r0, x, y, N, A->M,         \
                                        A->dia.D, A->dia.ld, nr, row0, A->dia.off_min, A->dia.off_max, x_al,      \
-                                       l2_evict_first())
+                                       l2_evict_first(), part ? 0 : dia_prefetch(), prefetch_hint())
 #define NITRO_DIA_U(SS)                      \
   switch (U) {                               \
     case 2: NITRO_DIA_LAUNCH(2, SS); break;  \
@@ -1223,7 +1296,8 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
     case NITRO_HYB:
       if (part) return fail(NITRO_E_INVALID_ARG, "HYB has no row-range launch");
       if (N > 0) {
-        launch_ell<VT>(A->hyb.col.as<int32_t>(), A->hyb.val.as<VT>(), x, y, N, A->hyb.K, A->hyb.ld, s);
+        launch_ell<VT>(A->hyb.col.as<int32_t>(), A->hyb.val.as<VT>(), x, y, N, A->hyb.K, A->hyb.ld, s, -1,
+                       diag_local(A));
         if (A->hyb.Zt > 0) {
           const unsigned gt = grid_cap((A->hyb.nchunks + 7) / 8, 16);
 #define NITRO_TAIL(WW)                                                                                        \

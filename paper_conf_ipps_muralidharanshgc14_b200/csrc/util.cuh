@@ -97,6 +97,16 @@ __device__ __forceinline__ double ld_stream(const double *p) {
 // L2 eviction policies (createpolicy) and streaming loads carrying one: the
 // matrix streams are read once; marking them evict-first keeps the reused x
 // vector resident in L2 next to gigabytes of streamed values/indices.
+// bulk L2 prefetch (TMA unit): [p, p + bytes) into L2, p and bytes 16-byte multiples
+__device__ __forceinline__ void bulk_prefetch_l2(const void *p, uint32_t bytes) {
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
+}
+// same, the lines inserted with an L2 eviction policy (createpolicy)
+__device__ __forceinline__ void bulk_prefetch_l2(const void *p, uint32_t bytes, uint64_t pol) {
+  asm volatile("cp.async.bulk.prefetch.L2.global.L2::cache_hint [%0], %1, %2;" ::"l"(p), "r"(bytes), "l"(pol)
+               : "memory");
+}
+
 __device__ __forceinline__ uint64_t l2_policy(bool evict_first) {
   uint64_t p;
   if (evict_first) asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));

@@ -563,3 +563,47 @@ def test_features_async_then_select(cuda):
     for k in FEAT_KEYS:
         assert f[k] == f_ref[k], k
     assert torch.isfinite(z)
+
+
+_PF_CHILD = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, sys.argv[1])
+import synth, paper_conf_ipps_muralidharanshgc14_b200 as n
+dev = torch.device("cuda:0")
+out = {}
+for name, A in (("3d27", synth.stencil("3d27", 40, mode=1, seed=31)),
+                ("band", synth.banded(70_001, 12, 0.6, seed=32)),
+                ("3d7_fp64", synth.stencil("3d7", 33, mode=1, seed=33, fp64=True))):
+    M = n.SpMV.from_csr(synth.to_device(A, dev))
+    M.features()
+    x = torch.from_numpy(synth.vector(A.cols, seed=34, fp64=A.fp64)).to(dev)
+    for v in (n.ELL, n.DIA, n.HYB):
+        if M.allowed(v):
+            y = M.run(v, x)
+            torch.cuda.synchronize()
+            out[f"{name}_{v}"] = y.cpu().numpy()
+    M.close()
+np.savez(sys.argv[2], **out)
+"""
+
+
+def test_l2_prefetch_is_result_neutral(cuda, tmp_path):
+    """The cp.async.bulk L2 prefetches of the DIA / ELL streams are
+    pure performance hints: y with them off (NITRO_DIA_PF=0, NITRO_ELL_PF=0) is
+    bit-identical to y with the defaults (on)."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    script = tmp_path / "pf_child.py"
+    script.write_text(_PF_CHILD)
+    res = {}
+    for tag, env in (("on", {}), ("off", {"NITRO_DIA_PF": "0", "NITRO_ELL_PF": "0"})):
+        out = tmp_path / f"{tag}.npz"
+        r = subprocess.run([sys.executable, str(script), root, str(out)], env={**os.environ, **env},
+                           capture_output=True, text=True, timeout=600)
+        assert r.returncode == 0, r.stderr[-2000:]
+        res[tag] = dict(np.load(out))
+    assert res["on"].keys() == res["off"].keys() and len(res["on"]) >= 6
+    for k in res["on"]:
+        assert np.array_equal(res["on"][k], res["off"][k]), k

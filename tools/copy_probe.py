@@ -21,6 +21,17 @@ def main():
         ts.sort()
         t = ts[len(ts) // 2]
         print(f"copy {mb} MB moved: {t*1e6:.1f} us  {(mb << 20) / t / 1e9:.0f} GB/s", flush=True)
+        c = torch.ones((mb << 20) // 4, dtype=torch.float32, device=dev)   # read-only: a sum over mb MB
+        ts = []
+        for r in range(23):
+            flush.fill_(r & 255)
+            s.record(); c.sum(); e.record(); torch.cuda.synchronize()
+            if r >= 3:
+                ts.append(s.elapsed_time(e) * 1e-3)
+        ts.sort()
+        t = ts[len(ts) // 2]
+        print(f"read {mb} MB (torch sum): {t*1e6:.1f} us  {(mb << 20) / t / 1e9:.0f} GB/s", flush=True)
+        del c
         del a, b
 
 if __name__ == "__main__":
