@@ -374,6 +374,59 @@ nitro_status_t nitro_dist_init_local(int rank, int nranks, int device, nitro_dis
  * union of diagonal offsets): identical to the single-GPU features. */
 nitro_status_t nitro_dist_features(nitro_dist *D, nitro_spmv *A_local, nitro_spmv_feat *out);
 
+/* ========================================================================
+ * 4. Histogram code-variant family: a second workload
+ *    through the same generic layer.  PAPER.md P:L216-217 (Fig. 4 row
+ *    "Histogram": Sort-ES / Sort-Dynamic, Shared-Atomic-ES /
+ *    Shared-Atomic-Dynamic; features N, N/#bins, SubSampleSD), P:L226 (the
+ *    CUB variants: "three variants and two grid-mapping strategies thus giving
+ *    rise to six code variants"), P:L254 (results), P:L269 (sub-sample size).
+ * ======================================================================== */
+typedef enum {
+  NITRO_HIST_SORT_ES = 0,      /* per tile: sort bin ids in shared memory, run-length -> atomics (default) */
+  NITRO_HIST_SORT_DYN = 1,     /* same, tiles from a global atomic queue */
+  NITRO_HIST_SHARED_ES = 2,    /* per-CTA shared-memory histogram, merged at the end */
+  NITRO_HIST_SHARED_DYN = 3,
+  NITRO_HIST_GLOBAL_ES = 4,    /* one global atomic per sample */
+  NITRO_HIST_GLOBAL_DYN = 5
+} nitro_hist_variant;
+#define NITRO_HIST_NUM_VARIANTS 6
+typedef struct nitro_hist nitro_hist;
+/* An even histogram of n uint32 samples (device array, borrowed; 16-byte
+ * alignment enables 128-bit loads):
+ *   h[b] = #{ i : s_i < range, floor(s_i * nbins / range) = b },  b < nbins,
+ * 1 <= nbins <= 65536, 1 <= range <= 2^32; samples >= range are not counted.
+ * All work is enqueued on `stream`. */
+nitro_status_t nitro_hist_create(int device, void *stream, int64_t n, const uint32_t *d_samples, int32_t nbins,
+                                 uint64_t range, nitro_hist **out);
+void nitro_hist_destroy(nitro_hist *H);
+/* out3 = {N, N / nbins, SubSampleSD}: SubSampleSD = population standard
+ * deviation of s[floor(j*N/k)], j < k, k = min(ceil(N/4), 10000),
+ * from exact integer moments: sqrt((double)(k*S2 - S1^2) / ((double)k*k)),
+ * 0 for N = 0.  Syncs the stream; cached. */
+nitro_status_t nitro_hist_features(nitro_hist *H, double *out3);
+/* Constraint: the shared-atomic variants need nbins <= 49152 (192 KB of
+ * shared counters per CTA); the others are always allowed. */
+nitro_status_t nitro_hist_allowed(nitro_hist *H, int variant, int *out_allowed);
+/* d_hist (uint32[nbins], device) = the histogram; async on the stream.
+ * NITRO_E_CONSTRAINT for a shared-atomic variant with nbins > 49152. */
+nitro_status_t nitro_hist_run(nitro_hist *H, int variant, uint32_t *d_hist);
+/* Median of reps CUDA-event timings of nitro_hist_run (L2 flushed before
+ * each when flush_l2), after warmup untimed runs.  Syncs. */
+nitro_status_t nitro_hist_time(nitro_hist *H, int variant, uint32_t *d_hist, int warmup, int reps, int flush_l2,
+                               double *out_median_s);
+/* Input record of the registered histogram variants. */
+typedef struct {
+  nitro_hist *H;
+  uint32_t *d_hist;
+  int warmup, reps, flush_l2;
+} nitro_hist_input;
+/* Register on a fresh cv: the 6 variants (ids = nitro_hist_variant), the
+ * feature group {n, n_per_bin, subsample_sd} (log1p + clip transform), the
+ * shared-memory constraints, default = SORT_ES (always allowed; robust to
+ * skewed inputs, where atomics contend). */
+nitro_status_t nitro_hist_register(nitro_cv *cv);
+
 #ifdef __cplusplus
 }
 #endif

@@ -15,6 +15,7 @@ Parts (PAPER.md line cites, readings in SURVEY.md §8(c) / DESIGN.md):
   dia_allowed /
   ell_allowed    C9
   select.*       C10-C13
+  hist.*         §8(f) f4 histogram family: counts + features (DESIGN R17)
 Parity status of each part is listed in DESIGN.md; the held-out "Nitro %"
 value (C13) is parity-unpinned (no reference GPU timings exist).
 """

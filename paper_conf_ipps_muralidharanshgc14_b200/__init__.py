@@ -29,6 +29,13 @@ PART_ELL_COL, PART_ELL_VAL, PART_DIA_OFF, PART_DIA_VAL = 0, 1, 2, 3
 PART_HYB_COL, PART_HYB_VAL, PART_HYB_TROW, PART_HYB_TCOL, PART_HYB_TVAL = 4, 5, 6, 7, 8
 PART_OFFSETS = 9
 
+# histogram family (include/nitro.h §4)
+HIST_SORT_ES, HIST_SORT_DYN, HIST_SHARED_ES, HIST_SHARED_DYN, HIST_GLOBAL_ES, HIST_GLOBAL_DYN = range(6)
+HIST_NUM_VARIANTS = 6
+HIST_VARIANT_NAMES = ("sort_es", "sort_dynamic", "shared_atomic_es", "shared_atomic_dynamic",
+                      "global_atomic_es", "global_atomic_dynamic")
+HIST_FEATURE_NAMES = ("n", "n_per_bin", "subsample_sd")
+
 STATUS = {0: "OK", 1: "INVALID_ARG", 2: "BAD_MATRIX", 3: "STATE", 4: "CONSTRAINT", 5: "OOM", 6: "CUDA",
           7: "NCCL", 8: "IO", 9: "UNSUPPORTED"}
 
@@ -80,6 +87,11 @@ class ItuneOpts(ctypes.Structure):
 
 class SpmvInput(ctypes.Structure):
     _fields_ = [("A", ctypes.c_void_p), ("d_x", ctypes.c_void_p), ("d_y", ctypes.c_void_p),
+                ("warmup", ctypes.c_int), ("reps", ctypes.c_int), ("flush_l2", ctypes.c_int)]
+
+
+class HistInput(ctypes.Structure):
+    _fields_ = [("H", ctypes.c_void_p), ("d_hist", ctypes.c_void_p),
                 ("warmup", ctypes.c_int), ("reps", ctypes.c_int), ("flush_l2", ctypes.c_int)]
 
 
@@ -168,6 +180,14 @@ _SIGS = {
     "nitro_dist_exchange_info": ([_vp, _P(_int), _P(_i64), _P(_i64), _P(_i64)], _int),
     "nitro_dist_halo_cols": ([_vp, _vp], _int),
     "nitro_dist_x_local": ([_vp, _P(_vp)], _int),
+    # histogram family
+    "nitro_hist_create": ([_int, _vp, _i64, _vp, ctypes.c_int32, _u64, _P(_vp)], _int),
+    "nitro_hist_destroy": ([_vp], None),
+    "nitro_hist_features": ([_vp, _P(_dbl)], _int),
+    "nitro_hist_allowed": ([_vp, _int, _P(_int)], _int),
+    "nitro_hist_run": ([_vp, _int, _vp], _int),
+    "nitro_hist_time": ([_vp, _int, _vp, _int, _int, _int, _P(_dbl)], _int),
+    "nitro_hist_register": ([_vp], _int),
 }
 for _name, (_args, _res) in _SIGS.items():
     _f = getattr(_L, _name)
@@ -390,6 +410,10 @@ class CodeVariant:
     def register_spmv(self):
         _check(_L.nitro_spmv_register(self.h))
 
+    def register_hist(self):
+        """The six histogram variants, their features and constraints (nitro_hist_register)."""
+        _check(_L.nitro_hist_register(self.h))
+
     def set_feature_transform(self, log_mask: int, clip: bool):
         """log1p of the features in log_mask, clip scaled inputs (nitro_cv_set_feature_transform)."""
         _check(_L.nitro_cv_set_feature_transform(self.h, int(log_mask), int(bool(clip))))
@@ -480,6 +504,64 @@ def spmv_input(A: SpMV, x, y, warmup=3, reps=20, flush_l2=True) -> SpmvInput:
     """Input record for the registered SpMV variants (keep it alive while used)."""
     rec = SpmvInput(A.h.value, _ptr(x), _ptr(y), warmup, reps, int(flush_l2))
     rec._keep = (A, x, y)
+    return rec
+
+
+class Hist:
+    """An even histogram of borrowed device uint32 samples (include/nitro.h §4):
+    h[b] = #{i : s_i < range, floor(s_i * nbins / range) = b}."""
+
+    def __init__(self, samples, nbins: int, value_range: int, stream=None):
+        import torch
+        assert samples.is_cuda and samples.dtype in (torch.int32, torch.uint32), "uint32 CUDA samples"
+        self._keep = samples
+        self.n, self.nbins, self.range = int(samples.numel()), int(nbins), int(value_range)
+        self.device = samples.device.index
+        if stream is None:
+            stream = torch.cuda.current_stream(self.device).cuda_stream
+        h = ctypes.c_void_p()
+        _check(_L.nitro_hist_create(self.device, stream, self.n, _ptr(samples), self.nbins, self.range,
+                                    ctypes.byref(h)))
+        self.h = h
+
+    def close(self):
+        if getattr(self, "h", None):
+            _L.nitro_hist_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def features(self) -> dict:
+        out = (ctypes.c_double * 3)()
+        _check(_L.nitro_hist_features(self.h, out))
+        return dict(zip(HIST_FEATURE_NAMES, list(out)))
+
+    def allowed(self, v: int) -> bool:
+        ok = ctypes.c_int()
+        _check(_L.nitro_hist_allowed(self.h, v, ctypes.byref(ok)))
+        return bool(ok.value)
+
+    def run(self, v: int, hist=None):
+        import torch
+        if hist is None:
+            hist = torch.empty(self.nbins, dtype=torch.int32, device=self._keep.device)
+        _check(_L.nitro_hist_run(self.h, v, _ptr(hist)))
+        return hist
+
+    def time(self, v: int, hist, warmup=3, reps=20, flush_l2=True) -> float:
+        t = ctypes.c_double()
+        _check(_L.nitro_hist_time(self.h, v, _ptr(hist), warmup, reps, int(flush_l2), ctypes.byref(t)))
+        return t.value
+
+
+def hist_input(H: Hist, hist, warmup=3, reps=20, flush_l2=True) -> HistInput:
+    """Input record for the registered histogram variants (keep it alive while used)."""
+    rec = HistInput(H.h.value, _ptr(hist), warmup, reps, int(flush_l2))
+    rec._keep = (H, hist)
     return rec
 
 

@@ -239,3 +239,32 @@ def checksum(A: Csr) -> tuple:
     v = np.asarray(A.vals)
     return (A.rows, A.cols, A.nnz, int(rp.sum() % (1 << 61)), int(ci.astype(np.int64).sum()),
             v.view(np.uint32 if v.dtype == np.float32 else np.uint64).astype(np.uint64).sum(dtype=np.uint64).item())
+
+
+# ---------------------------------------------------------------- histogram samples
+HIST_DISTS = ("uniform", "normal", "exponential", "spike", "sorted")
+
+
+def hist_samples(n: int, dist: str, value_range: int, seed: int = 0, param: float = 0.1) -> np.ndarray:
+    """Seeded uint32 histogram inputs over [0, value_range) (host numpy; no
+    method arithmetic).  dist: uniform; normal (mean range/2, sd = param *
+    range, clipped); exponential (scale = param * range, clipped); spike (a
+    fraction param of the samples equal to one value, the rest uniform);
+    sorted (uniform, sorted ascending — the paper's "almost sorted" style
+    input, P:L229)."""
+    rng = np.random.default_rng(seed)
+    hi = value_range - 1
+    if dist == "uniform":
+        v = rng.integers(0, value_range, n, dtype=np.uint64)
+    elif dist == "normal":
+        v = np.clip(np.rint(rng.normal(value_range / 2, param * value_range, n)), 0, hi)
+    elif dist == "exponential":
+        v = np.clip(np.floor(rng.exponential(param * value_range, n)), 0, hi)
+    elif dist == "spike":
+        v = rng.integers(0, value_range, n, dtype=np.uint64)
+        v[rng.random(n) < param] = int(rng.integers(0, value_range))
+    elif dist == "sorted":
+        v = np.sort(rng.integers(0, value_range, n, dtype=np.uint64))
+    else:
+        raise ValueError(dist)
+    return np.asarray(v, dtype=np.uint64).astype(np.uint32)
