@@ -38,13 +38,13 @@ constexpr uint32_t kNoBin = 0xffffffffu;
 constexpr int kSubMax = 10000;                     // sub-sample cap
 constexpr uint32_t kMaxSharedBins = 49152;         // 192 KB of shared counters
 
+// general even binning: floor(s * nbins / range) by an fp64 reciprocal and an
+// exact integer correction
 struct BinMap {
   uint64_t nbins, range;
   double rinv;  // nbins / range (rounded); corrected below to the exact floor
-  int shift;    // >= 0 when range / nbins is a power of two 2^shift: bin = s >> shift
   __device__ __forceinline__ uint32_t operator()(uint32_t s) const {
     if ((uint64_t)s >= range) return kNoBin;
-    if (shift >= 0) return shift >= 32 ? 0u : s >> shift;
     const uint64_t a = (uint64_t)s * nbins;  // < 2^48
     uint64_t q = (uint64_t)((double)s * rinv);
     // |q - a/range| <= 1 before correction: make q = floor(a / range) exactly
@@ -53,6 +53,19 @@ struct BinMap {
     return (uint32_t)q;
   }
 };
+// range / nbins = 2^sh (equal power-of-two bin widths, e.g. 8/16-bit data):
+// the same floor is s >> sh; lim = range - 1 (< 2^32)
+struct BinShift {
+  uint32_t lim, sh;  // sh <= 32
+  __device__ __forceinline__ uint32_t operator()(uint32_t s) const {
+    if (s > lim) return kNoBin;
+    return sh >= 32 ? 0u : s >> sh;
+  }
+};
+
+__device__ __forceinline__ void red_shared_inc(uint32_t saddr) {
+  asm volatile("red.shared.add.u32 [%0], 1;" ::"r"(saddr) : "memory");
+}
 
 __device__ __forceinline__ int64_t next_tile(unsigned long long *queue, int64_t *s_t) {
   if (threadIdx.x == 0) *s_t = (int64_t)atomicAdd(queue, 1ull);
@@ -87,19 +100,19 @@ __device__ __forceinline__ void for_tile_samples(const uint32_t *__restrict__ s,
 // same-bin contention of concentrated inputs over R addresses; the copies
 // are summed per bin at the end and merged with one global atomic per
 // non-zero bin.
-template <int T, bool DYN>
-__global__ void __launch_bounds__(T) k_hist_shared(const uint32_t *__restrict__ s, int64_t n, BinMap bm,
+template <int T, bool DYN, typename BM>
+__global__ void __launch_bounds__(T) k_hist_shared(const uint32_t *__restrict__ s, int64_t n, BM bm, uint32_t nb,
                                                    uint32_t *__restrict__ hist, int64_t tiles,
                                                    unsigned long long *queue, bool vec, int R) {
   extern __shared__ uint32_t sh[];
   __shared__ int64_t s_t;
-  const uint32_t nb = (uint32_t)bm.nbins;
   for (uint32_t i = threadIdx.x; i < nb * (uint32_t)R; i += T) sh[i] = 0;
   __syncthreads();
-  uint32_t *mine = sh + (uint32_t)((threadIdx.x >> 5) % R) * nb;
+  // this warp's counter copy as a 32-bit shared-window address (red.shared per sample)
+  const uint32_t mine = (uint32_t)__cvta_generic_to_shared(sh + (uint32_t)((threadIdx.x >> 5) % R) * nb);
   auto add = [&](uint32_t v) {
     const uint32_t b = bm(v);
-    if (b != kNoBin) atomicAdd(mine + b, 1u);
+    if (b != kNoBin) red_shared_inc(mine + 4u * b);
   };
   if (DYN) {
     for (int64_t t = next_tile(queue, &s_t); t < tiles; t = next_tile(queue, &s_t))
@@ -116,8 +129,8 @@ __global__ void __launch_bounds__(T) k_hist_shared(const uint32_t *__restrict__ 
   }
 }
 
-template <bool DYN>
-__global__ void __launch_bounds__(kHThr) k_hist_global(const uint32_t *__restrict__ s, int64_t n, BinMap bm,
+template <bool DYN, typename BM>
+__global__ void __launch_bounds__(kHThr) k_hist_global(const uint32_t *__restrict__ s, int64_t n, BM bm,
                                                        uint32_t *__restrict__ hist, int64_t tiles,
                                                        unsigned long long *queue, bool vec) {
   __shared__ int64_t s_t;
@@ -136,7 +149,8 @@ __global__ void __launch_bounds__(kHThr) k_hist_global(const uint32_t *__restric
 
 // one sort tile: load + bin, bitonic sort of kSortTile keys in shared memory,
 // run detection with the (tail + 1) - head atomics
-__device__ __forceinline__ void sort_tile(const uint32_t *__restrict__ s, int64_t n, const BinMap &bm,
+template <typename BM>
+__device__ __forceinline__ void sort_tile(const uint32_t *__restrict__ s, int64_t n, const BM &bm,
                                           uint32_t *__restrict__ hist, int64_t t, uint32_t *key) {
   const int64_t base = t * kSortTile;
 #pragma unroll
@@ -169,8 +183,8 @@ __device__ __forceinline__ void sort_tile(const uint32_t *__restrict__ s, int64_
   __syncthreads();
 }
 
-template <bool DYN>
-__global__ void __launch_bounds__(kHThr) k_hist_sort(const uint32_t *__restrict__ s, int64_t n, BinMap bm,
+template <bool DYN, typename BM>
+__global__ void __launch_bounds__(kHThr) k_hist_sort(const uint32_t *__restrict__ s, int64_t n, BM bm,
                                                      uint32_t *__restrict__ hist, int64_t tiles,
                                                      unsigned long long *queue) {
   __shared__ uint32_t key[kSortTile];
@@ -260,6 +274,52 @@ int blocks_per_sm(const void *fn, size_t smem) {
   return b;
 }
 
+template <typename BM>
+nitro_status_t hist_kernels(nitro_hist *H, int v, uint32_t *hist, cudaStream_t st, const BM &bm,
+                            unsigned long long *q, bool dyn) {
+  const bool vec = (reinterpret_cast<uintptr_t>(H->s) & 15) == 0;
+  const int sms = num_sms();
+  if (v == NITRO_HIST_SORT_ES || v == NITRO_HIST_SORT_DYN) {
+    const int64_t tiles = (H->n + kSortTile - 1) / kSortTile;
+    const void *fn = dyn ? (const void *)k_hist_sort<true, BM> : (const void *)k_hist_sort<false, BM>;
+    const int64_t g = std::min<int64_t>(tiles, (int64_t)sms * blocks_per_sm(fn, 0));
+    if (dyn) k_hist_sort<true, BM><<<(unsigned)g, kHThr, 0, st>>>(H->s, H->n, bm, hist, tiles, q);
+    else k_hist_sort<false, BM><<<(unsigned)g, kHThr, 0, st>>>(H->s, H->n, bm, hist, tiles, q);
+  } else if (hist_is_shared(v)) {
+    if (H->nbins > kMaxSharedBins) return fail(NITRO_E_CONSTRAINT, "shared-atomic histogram: nbins > 49152");
+    // counter copies: up to 8 while they fit 48 KB (several CTAs per SM)
+    int R = 1;
+    while (R < 8 && (size_t)(2 * R) * H->nbins * 4 <= 48 * 1024) R *= 2;
+    const size_t smem = (size_t)R * H->nbins * 4;
+    const bool big = smem > 76 * 1024;  // at most two CTAs per SM: 1024 threads each
+    const uint32_t nb = H->nbins;
+#define HIST_SHARED_LAUNCH(TT)                                                                                    \
+  do {                                                                                                            \
+    const void *fn = dyn ? (const void *)k_hist_shared<TT, true, BM> : (const void *)k_hist_shared<TT, false, BM>; \
+    NITRO_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));                 \
+    int b = 0;                                                                                                    \
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fn, TT, smem) != cudaSuccess || b < 1) b = 1;           \
+    const int64_t tiles = (H->n + (int64_t)TT * 16 - 1) / ((int64_t)TT * 16);                                   \
+    const int64_t g = std::min<int64_t>(tiles, (int64_t)sms * b);                                                 \
+    if (dyn)                                                                                                      \
+      k_hist_shared<TT, true, BM><<<(unsigned)g, TT, smem, st>>>(H->s, H->n, bm, nb, hist, tiles, q, vec, R);     \
+    else                                                                                                          \
+      k_hist_shared<TT, false, BM><<<(unsigned)g, TT, smem, st>>>(H->s, H->n, bm, nb, hist, tiles, q, vec, R);    \
+  } while (0)
+    if (big) HIST_SHARED_LAUNCH(1024);
+    else HIST_SHARED_LAUNCH(256);
+#undef HIST_SHARED_LAUNCH
+  } else {
+    const int64_t tiles = (H->n + kHTile - 1) / kHTile;
+    const void *fn = dyn ? (const void *)k_hist_global<true, BM> : (const void *)k_hist_global<false, BM>;
+    const int64_t g = std::min<int64_t>(tiles, (int64_t)sms * blocks_per_sm(fn, 0));
+    if (dyn) k_hist_global<true, BM><<<(unsigned)g, kHThr, 0, st>>>(H->s, H->n, bm, hist, tiles, q, vec);
+    else k_hist_global<false, BM><<<(unsigned)g, kHThr, 0, st>>>(H->s, H->n, bm, hist, tiles, q, vec);
+  }
+  NITRO_CUDA(cudaGetLastError());
+  return NITRO_OK;
+}
+
 nitro_status_t hist_launch(nitro_hist *H, int v, uint32_t *hist, cudaStream_t st) {
   NITRO_CUDA(cudaMemsetAsync(hist, 0, (size_t)H->nbins * 4, st));
   if (H->n == 0) return NITRO_OK;
@@ -270,52 +330,15 @@ nitro_status_t hist_launch(nitro_hist *H, int v, uint32_t *hist, cudaStream_t st
     q = H->queue.as<unsigned long long>();
     NITRO_CUDA(cudaMemsetAsync(q, 0, 8, st));
   }
-  BinMap bm{H->nbins, H->range, (double)H->nbins / (double)H->range, -1};
   if (H->range % H->nbins == 0) {  // equal integer bins of width w = range / nbins; a power of two -> shift
     const uint64_t w = H->range / H->nbins;
     if ((w & (w - 1)) == 0) {
-      bm.shift = 0;
-      while ((1ull << bm.shift) < w) ++bm.shift;
+      uint32_t sh = 0;
+      while ((1ull << sh) < w) ++sh;
+      return hist_kernels(H, v, hist, st, BinShift{(uint32_t)(H->range - 1), sh}, q, dyn);
     }
   }
-  const bool vec = (reinterpret_cast<uintptr_t>(H->s) & 15) == 0;
-  const int sms = num_sms();
-  if (v == NITRO_HIST_SORT_ES || v == NITRO_HIST_SORT_DYN) {
-    const int64_t tiles = (H->n + kSortTile - 1) / kSortTile;
-    const void *fn = dyn ? (const void *)k_hist_sort<true> : (const void *)k_hist_sort<false>;
-    const int64_t g = std::min<int64_t>(tiles, (int64_t)sms * blocks_per_sm(fn, 0));
-    if (dyn) k_hist_sort<true><<<(unsigned)g, kHThr, 0, st>>>(H->s, H->n, bm, hist, tiles, q);
-    else k_hist_sort<false><<<(unsigned)g, kHThr, 0, st>>>(H->s, H->n, bm, hist, tiles, q);
-  } else if (hist_is_shared(v)) {
-    if (H->nbins > kMaxSharedBins) return fail(NITRO_E_CONSTRAINT, "shared-atomic histogram: nbins > 49152");
-    // counter copies: up to 8 while they fit 48 KB (several CTAs per SM)
-    int R = 1;
-    while (R < 8 && (size_t)(2 * R) * H->nbins * 4 <= 48 * 1024) R *= 2;
-    const size_t smem = (size_t)R * H->nbins * 4;
-    const bool big = smem > 76 * 1024;  // at most two CTAs per SM: 1024 threads each
-#define HIST_SHARED_LAUNCH(TT)                                                                                \
-  do {                                                                                                        \
-    const void *fn = dyn ? (const void *)k_hist_shared<TT, true> : (const void *)k_hist_shared<TT, false>;    \
-    NITRO_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));             \
-    int b = 0;                                                                                                \
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fn, TT, smem) != cudaSuccess || b < 1) b = 1;       \
-    const int64_t tiles = (H->n + (int64_t)TT * 16 - 1) / ((int64_t)TT * 16);                               \
-    const int64_t g = std::min<int64_t>(tiles, (int64_t)sms * b);                                             \
-    if (dyn) k_hist_shared<TT, true><<<(unsigned)g, TT, smem, st>>>(H->s, H->n, bm, hist, tiles, q, vec, R);  \
-    else k_hist_shared<TT, false><<<(unsigned)g, TT, smem, st>>>(H->s, H->n, bm, hist, tiles, q, vec, R);     \
-  } while (0)
-    if (big) HIST_SHARED_LAUNCH(1024);
-    else HIST_SHARED_LAUNCH(256);
-#undef HIST_SHARED_LAUNCH
-  } else {
-    const int64_t tiles = (H->n + kHTile - 1) / kHTile;
-    const void *fn = dyn ? (const void *)k_hist_global<true> : (const void *)k_hist_global<false>;
-    const int64_t g = std::min<int64_t>(tiles, (int64_t)sms * blocks_per_sm(fn, 0));
-    if (dyn) k_hist_global<true><<<(unsigned)g, kHThr, 0, st>>>(H->s, H->n, bm, hist, tiles, q, vec);
-    else k_hist_global<false><<<(unsigned)g, kHThr, 0, st>>>(H->s, H->n, bm, hist, tiles, q, vec);
-  }
-  NITRO_CUDA(cudaGetLastError());
-  return NITRO_OK;
+  return hist_kernels(H, v, hist, st, BinMap{H->nbins, H->range, (double)H->nbins / (double)H->range}, q, dyn);
 }
 
 nitro_status_t hist_flush(nitro_hist *H, cudaStream_t st) {
