@@ -67,12 +67,42 @@ __device__ __forceinline__ void red_shared_inc(uint32_t saddr) {
   asm volatile("red.shared.add.u32 [%0], 1;" ::"r"(saddr) : "memory");
 }
 
-__device__ __forceinline__ int64_t next_tile(unsigned long long *queue, int64_t *s_t) {
-  if (threadIdx.x == 0) *s_t = (int64_t)atomicAdd(queue, 1ull);
+// Per-handle control words (no per-call memsets): p[0] = dynamic tile queue,
+// p[1] = "output zeroed" flag.  Both only grow: a call with epoch e takes
+// tiles as (p[0] value - qbase) and waits for p[1] >= e; the host advances
+// qbase by tiles + gridDim after each dynamic call (every CTA makes exactly
+// one failing fetch) and e by one per call.  Launched cooperatively, so every
+// CTA is resident and the wait on CTA 0's zeroing cannot deadlock.
+struct Ctl {
+  unsigned long long *p;
+  unsigned long long epoch, qbase;
+};
+
+__device__ __forceinline__ int64_t next_tile(const Ctl &c, int64_t *s_t) {
+  if (threadIdx.x == 0) *s_t = (int64_t)(atomicAdd(c.p, 1ull) - c.qbase);
   __syncthreads();
   const int64_t t = *s_t;
   __syncthreads();
   return t;
+}
+
+// CTA 0 zeroes the output and publishes epoch in p[1]
+__device__ __forceinline__ void zero_output(uint32_t *__restrict__ hist, uint32_t nb, const Ctl &c) {
+  if (blockIdx.x != 0) return;
+  for (uint32_t i = threadIdx.x; i < nb; i += blockDim.x) hist[i] = 0;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    atomicExch(c.p + 1, c.epoch);
+  }
+}
+// every CTA, before its first update of the output
+__device__ __forceinline__ void wait_zeroed(const Ctl &c) {
+  if (threadIdx.x == 0) {
+    while (*((volatile unsigned long long *)(c.p + 1)) < c.epoch) __nanosleep(64);
+    __threadfence();
+  }
+  __syncthreads();
 }
 
 // samples of tile t handled by this thread (T threads, T * 16 samples per
@@ -102,10 +132,11 @@ __device__ __forceinline__ void for_tile_samples(const uint32_t *__restrict__ s,
 // non-zero bin.
 template <int T, bool DYN, typename BM>
 __global__ void __launch_bounds__(T) k_hist_shared(const uint32_t *__restrict__ s, int64_t n, BM bm, uint32_t nb,
-                                                   uint32_t *__restrict__ hist, int64_t tiles,
-                                                   unsigned long long *queue, bool vec, int R) {
+                                                   uint32_t *__restrict__ hist, int64_t tiles, Ctl ctl, bool vec,
+                                                   int R) {
   extern __shared__ uint32_t sh[];
   __shared__ int64_t s_t;
+  zero_output(hist, nb, ctl);
   for (uint32_t i = threadIdx.x; i < nb * (uint32_t)R; i += T) sh[i] = 0;
   __syncthreads();
   // this warp's counter copy as a 32-bit shared-window address (red.shared per sample)
@@ -115,13 +146,14 @@ __global__ void __launch_bounds__(T) k_hist_shared(const uint32_t *__restrict__ 
     if (b != kNoBin) red_shared_inc(mine + 4u * b);
   };
   if (DYN) {
-    for (int64_t t = next_tile(queue, &s_t); t < tiles; t = next_tile(queue, &s_t))
+    for (int64_t t = next_tile(ctl, &s_t); t < tiles; t = next_tile(ctl, &s_t))
       for_tile_samples<T>(s, n, t, vec, add);
   } else {
     const int64_t t0 = blockIdx.x * tiles / gridDim.x, t1 = (blockIdx.x + 1) * tiles / gridDim.x;
     for (int64_t t = t0; t < t1; ++t) for_tile_samples<T>(s, n, t, vec, add);
   }
   __syncthreads();
+  wait_zeroed(ctl);
   for (uint32_t i = threadIdx.x; i < nb; i += T) {
     uint32_t c = 0;
     for (int r = 0; r < R; ++r) c += sh[(uint32_t)r * nb + i];
@@ -131,15 +163,17 @@ __global__ void __launch_bounds__(T) k_hist_shared(const uint32_t *__restrict__ 
 
 template <bool DYN, typename BM>
 __global__ void __launch_bounds__(kHThr) k_hist_global(const uint32_t *__restrict__ s, int64_t n, BM bm,
-                                                       uint32_t *__restrict__ hist, int64_t tiles,
-                                                       unsigned long long *queue, bool vec) {
+                                                       uint32_t nb, uint32_t *__restrict__ hist, int64_t tiles,
+                                                       Ctl ctl, bool vec) {
   __shared__ int64_t s_t;
+  zero_output(hist, nb, ctl);
+  wait_zeroed(ctl);
   auto add = [&](uint32_t v) {
     const uint32_t b = bm(v);
     if (b != kNoBin) atomicAdd(hist + b, 1u);
   };
   if (DYN) {
-    for (int64_t t = next_tile(queue, &s_t); t < tiles; t = next_tile(queue, &s_t))
+    for (int64_t t = next_tile(ctl, &s_t); t < tiles; t = next_tile(ctl, &s_t))
       for_tile_samples<kHThr>(s, n, t, vec, add);
   } else {
     const int64_t t0 = blockIdx.x * tiles / gridDim.x, t1 = (blockIdx.x + 1) * tiles / gridDim.x;
@@ -185,12 +219,14 @@ __device__ __forceinline__ void sort_tile(const uint32_t *__restrict__ s, int64_
 
 template <bool DYN, typename BM>
 __global__ void __launch_bounds__(kHThr) k_hist_sort(const uint32_t *__restrict__ s, int64_t n, BM bm,
-                                                     uint32_t *__restrict__ hist, int64_t tiles,
-                                                     unsigned long long *queue) {
+                                                     uint32_t nb, uint32_t *__restrict__ hist, int64_t tiles,
+                                                     Ctl ctl) {
   __shared__ uint32_t key[kSortTile];
   __shared__ int64_t s_t;
+  zero_output(hist, nb, ctl);
+  wait_zeroed(ctl);
   if (DYN) {
-    for (int64_t t = next_tile(queue, &s_t); t < tiles; t = next_tile(queue, &s_t)) sort_tile(s, n, bm, hist, t, key);
+    for (int64_t t = next_tile(ctl, &s_t); t < tiles; t = next_tile(ctl, &s_t)) sort_tile(s, n, bm, hist, t, key);
   } else {
     const int64_t t0 = blockIdx.x * tiles / gridDim.x, t1 = (blockIdx.x + 1) * tiles / gridDim.x;
     for (int64_t t = t0; t < t1; ++t) sort_tile(s, n, bm, hist, t, key);
@@ -258,7 +294,8 @@ struct nitro_hist {
   uint64_t range = 1;
   bool feat_ready = false;
   double feat[3] = {0, 0, 0};
-  nitro::DevBuf queue, moments, flush;
+  nitro::DevBuf ctl, moments, flush;  // ctl: 2 x u64 control words (see Ctl)
+  unsigned long long epoch = 0, qbase = 0;
 };
 
 using namespace nitro;
@@ -274,71 +311,71 @@ int blocks_per_sm(const void *fn, size_t smem) {
   return b;
 }
 
+// cooperative launch (all CTAs co-resident: required by the zeroing wait)
+template <typename... Args>
+nitro_status_t coop(void (*k)(Args...), int64_t g, int threads, size_t smem, cudaStream_t st, Args... args) {
+  void *argv[] = {(void *)&args...};
+  NITRO_CUDA(cudaLaunchCooperativeKernel((const void *)k, dim3((unsigned)g), dim3((unsigned)threads), argv, smem, st));
+  return NITRO_OK;
+}
+
 template <typename BM>
-nitro_status_t hist_kernels(nitro_hist *H, int v, uint32_t *hist, cudaStream_t st, const BM &bm,
-                            unsigned long long *q, bool dyn) {
+nitro_status_t hist_kernels(nitro_hist *H, int v, uint32_t *hist, cudaStream_t st, const BM &bm, bool dyn) {
   const bool vec = (reinterpret_cast<uintptr_t>(H->s) & 15) == 0;
   const int sms = num_sms();
+  const uint32_t nb = H->nbins;
+  Ctl ctl{H->ctl.as<unsigned long long>(), ++H->epoch, H->qbase};
+  int64_t tiles = 0, g = 0;
   if (v == NITRO_HIST_SORT_ES || v == NITRO_HIST_SORT_DYN) {
-    const int64_t tiles = (H->n + kSortTile - 1) / kSortTile;
-    const void *fn = dyn ? (const void *)k_hist_sort<true, BM> : (const void *)k_hist_sort<false, BM>;
-    const int64_t g = std::min<int64_t>(tiles, (int64_t)sms * blocks_per_sm(fn, 0));
-    if (dyn) k_hist_sort<true, BM><<<(unsigned)g, kHThr, 0, st>>>(H->s, H->n, bm, hist, tiles, q);
-    else k_hist_sort<false, BM><<<(unsigned)g, kHThr, 0, st>>>(H->s, H->n, bm, hist, tiles, q);
+    tiles = (H->n + kSortTile - 1) / kSortTile;
+    auto k = dyn ? k_hist_sort<true, BM> : k_hist_sort<false, BM>;
+    g = std::min<int64_t>(tiles, (int64_t)sms * blocks_per_sm((const void *)k, 0));
+    NITRO_TRY(coop(k, g, kHThr, 0, st, H->s, H->n, bm, nb, hist, tiles, ctl));
   } else if (hist_is_shared(v)) {
-    if (H->nbins > kMaxSharedBins) return fail(NITRO_E_CONSTRAINT, "shared-atomic histogram: nbins > 49152");
+    if (nb > kMaxSharedBins) return fail(NITRO_E_CONSTRAINT, "shared-atomic histogram: nbins > 49152");
     // counter copies: up to 8 while they fit 48 KB (several CTAs per SM)
     int R = 1;
-    while (R < 8 && (size_t)(2 * R) * H->nbins * 4 <= 48 * 1024) R *= 2;
-    const size_t smem = (size_t)R * H->nbins * 4;
+    while (R < 8 && (size_t)(2 * R) * nb * 4 <= 48 * 1024) R *= 2;
+    const size_t smem = (size_t)R * nb * 4;
     const bool big = smem > 76 * 1024;  // at most two CTAs per SM: 1024 threads each
-    const uint32_t nb = H->nbins;
-#define HIST_SHARED_LAUNCH(TT)                                                                                    \
-  do {                                                                                                            \
-    const void *fn = dyn ? (const void *)k_hist_shared<TT, true, BM> : (const void *)k_hist_shared<TT, false, BM>; \
-    NITRO_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));                 \
-    int b = 0;                                                                                                    \
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fn, TT, smem) != cudaSuccess || b < 1) b = 1;           \
-    const int64_t tiles = (H->n + (int64_t)TT * 16 - 1) / ((int64_t)TT * 16);                                   \
-    const int64_t g = std::min<int64_t>(tiles, (int64_t)sms * b);                                                 \
-    if (dyn)                                                                                                      \
-      k_hist_shared<TT, true, BM><<<(unsigned)g, TT, smem, st>>>(H->s, H->n, bm, nb, hist, tiles, q, vec, R);     \
-    else                                                                                                          \
-      k_hist_shared<TT, false, BM><<<(unsigned)g, TT, smem, st>>>(H->s, H->n, bm, nb, hist, tiles, q, vec, R);    \
-  } while (0)
-    if (big) HIST_SHARED_LAUNCH(1024);
-    else HIST_SHARED_LAUNCH(256);
-#undef HIST_SHARED_LAUNCH
+    auto k = big ? (dyn ? k_hist_shared<1024, true, BM> : k_hist_shared<1024, false, BM>)
+                 : (dyn ? k_hist_shared<256, true, BM> : k_hist_shared<256, false, BM>);
+    const int T = big ? 1024 : 256;
+    NITRO_CUDA(cudaFuncSetAttribute((const void *)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    int b = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, (const void *)k, T, smem) != cudaSuccess || b < 1) b = 1;
+    tiles = (H->n + (int64_t)T * 16 - 1) / ((int64_t)T * 16);
+    g = std::min<int64_t>(tiles, (int64_t)sms * b);
+    NITRO_TRY(coop(k, g, T, smem, st, H->s, H->n, bm, nb, hist, tiles, ctl, vec, R));
   } else {
-    const int64_t tiles = (H->n + kHTile - 1) / kHTile;
-    const void *fn = dyn ? (const void *)k_hist_global<true, BM> : (const void *)k_hist_global<false, BM>;
-    const int64_t g = std::min<int64_t>(tiles, (int64_t)sms * blocks_per_sm(fn, 0));
-    if (dyn) k_hist_global<true, BM><<<(unsigned)g, kHThr, 0, st>>>(H->s, H->n, bm, hist, tiles, q, vec);
-    else k_hist_global<false, BM><<<(unsigned)g, kHThr, 0, st>>>(H->s, H->n, bm, hist, tiles, q, vec);
+    tiles = (H->n + kHTile - 1) / kHTile;
+    auto k = dyn ? k_hist_global<true, BM> : k_hist_global<false, BM>;
+    g = std::min<int64_t>(tiles, (int64_t)sms * blocks_per_sm((const void *)k, 0));
+    NITRO_TRY(coop(k, g, kHThr, 0, st, H->s, H->n, bm, nb, hist, tiles, ctl, vec));
   }
-  NITRO_CUDA(cudaGetLastError());
+  if (dyn) H->qbase += (unsigned long long)(tiles + g);  // every CTA made exactly one failing fetch
   return NITRO_OK;
 }
 
 nitro_status_t hist_launch(nitro_hist *H, int v, uint32_t *hist, cudaStream_t st) {
-  NITRO_CUDA(cudaMemsetAsync(hist, 0, (size_t)H->nbins * 4, st));
-  if (H->n == 0) return NITRO_OK;
-  const bool dyn = v == NITRO_HIST_SORT_DYN || v == NITRO_HIST_SHARED_DYN || v == NITRO_HIST_GLOBAL_DYN;
-  unsigned long long *q = nullptr;
-  if (dyn) {
-    NITRO_TRY(H->queue.alloc(16));
-    q = H->queue.as<unsigned long long>();
-    NITRO_CUDA(cudaMemsetAsync(q, 0, 8, st));
+  if (H->n == 0) {
+    NITRO_CUDA(cudaMemsetAsync(hist, 0, (size_t)H->nbins * 4, st));
+    return NITRO_OK;
   }
+  if (!H->ctl.p) {
+    NITRO_TRY(H->ctl.alloc(16));
+    NITRO_CUDA(cudaMemsetAsync(H->ctl.p, 0, 16, st));  // once per handle
+  }
+  const bool dyn = v == NITRO_HIST_SORT_DYN || v == NITRO_HIST_SHARED_DYN || v == NITRO_HIST_GLOBAL_DYN;
   if (H->range % H->nbins == 0) {  // equal integer bins of width w = range / nbins; a power of two -> shift
     const uint64_t w = H->range / H->nbins;
     if ((w & (w - 1)) == 0) {
       uint32_t sh = 0;
       while ((1ull << sh) < w) ++sh;
-      return hist_kernels(H, v, hist, st, BinShift{(uint32_t)(H->range - 1), sh}, q, dyn);
+      return hist_kernels(H, v, hist, st, BinShift{(uint32_t)(H->range - 1), sh}, dyn);
     }
   }
-  return hist_kernels(H, v, hist, st, BinMap{H->nbins, H->range, (double)H->nbins / (double)H->range}, q, dyn);
+  return hist_kernels(H, v, hist, st, BinMap{H->nbins, H->range, (double)H->nbins / (double)H->range}, dyn);
 }
 
 nitro_status_t hist_flush(nitro_hist *H, cudaStream_t st) {
