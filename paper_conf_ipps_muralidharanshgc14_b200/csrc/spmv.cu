@@ -210,8 +210,8 @@ constexpr int csrv_min_blocks() {
   return R * kB >= 16 ? 2 : R * kB >= 12 ? (sizeof(VT) == 4 ? 3 : 2) : (sizeof(VT) == 4 ? 4 : 5);
 }
 
-template <int V, int R, int kB, typename IT, typename VT, int MB = 0>
-__global__ void __launch_bounds__(256, MB ? MB : csrv_min_blocks<V, R, kB, VT>()) k_csr_vector(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
+template <int V, int R, int kB, typename IT, typename VT>
+__global__ void __launch_bounds__(256, csrv_min_blocks<V, R, kB, VT>()) k_csr_vector(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
                                                     const VT *__restrict__ val, const VT *__restrict__ x,
                                                     VT *__restrict__ y, int64_t N, int64_t nseg,
                                                     const int32_t *__restrict__ seg_row,
@@ -1004,16 +1004,6 @@ bool prefetch_hint() {
   return env != 0;
 }
 
-// CSR-vector fp32 occupancy bound: NITRO_CSRV_MB=3 builds the R = 2 path for
-// 3 CTAs/SM (80 registers) instead of 4 (64); A/B knob, default 4
-int csrv_mb() {
-  static int env = [] {
-    const char *e = getenv("NITRO_CSRV_MB");
-    return e ? atoi(e) : 0;
-  }();
-  return env;
-}
-
 // ELL L2 prefetch distance in slot batches: NITRO_ELL_PF overrides; default 1.
 // B200 (GB/s, PF 0 -> 1, same box): configs[1] 6035 -> 6369 and 5732 -> 5815,
 // dense band b = 48 6527 -> 6921, 256^3 stencil 5894 -> 6331
@@ -1286,7 +1276,6 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
       default:                                                                                              \
         if (b7_) k_csr_vector<VV, 2, 7, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, nseg, seg_row, seg_k, seg_part, seg_ctr, ef_); \
         else if (sizeof(VT) == 8) k_csr_vector<VV, 2, 3, IT, VT><<<gw_, 256, 0, s>>>(rp, A->col, val, x, y, N, nseg, seg_row, seg_k, seg_part, seg_ctr, ef_); \
-        else if (csrv_mb() == 3) k_csr_vector<VV, 2, 3, IT, VT, 3><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, nseg, seg_row, seg_k, seg_part, seg_ctr, ef_); \
         else k_csr_vector<VV, 2, 3, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, nseg, seg_row, seg_k, seg_part, seg_ctr, ef_); \
         break;                                                                                              \
     }                                                                                                       \
