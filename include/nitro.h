@@ -409,7 +409,10 @@ nitro_status_t nitro_hist_features(nitro_hist *H, double *out3);
  * shared counters per CTA); the others are always allowed. */
 nitro_status_t nitro_hist_allowed(nitro_hist *H, int variant, int *out_allowed);
 /* d_hist (uint32[nbins], device) = the histogram; async on the stream.
- * NITRO_E_CONSTRAINT for a shared-atomic variant with nbins > 49152. */
+ * NITRO_E_CONSTRAINT for a shared-atomic variant with nbins > 49152.
+ * Kernels are launched cooperatively (all CTAs resident: CTA 0 zeroes d_hist
+ * and the others wait on a per-handle epoch flag), so the calls of one handle
+ * must stay ordered on its stream (no concurrent calls on one handle). */
 nitro_status_t nitro_hist_run(nitro_hist *H, int variant, uint32_t *d_hist);
 /* Median of reps CUDA-event timings of nitro_hist_run (L2 flushed before
  * each when flush_l2), after warmup untimed runs.  Syncs. */
