@@ -398,7 +398,7 @@ def test_run_host_matches_device(cuda):
 
 @pytest.mark.parametrize("kind", ["3d27_n64", "banded_300k", "uniform_300k_rect"])
 def test_run_host_pipelined_bit_identical(cuda, kind):
-    """>= 2^18 rows: CSR-scalar / ELL / DIA host-buffer calls run as 8 row chunks
+    """>= 2^17 rows: CSR-scalar / ELL / DIA host-buffer calls run as 4 row chunks
     (x in column pieces, y out per chunk on separate streams); every row must be
     bit-identical to the single-launch device multiply (same kernels, same
     per-row order) and within tolerance of the oracle."""

@@ -1,2 +1,1 @@
-timeout 900 python -m pytest tests/test_gpu_hist.py -x -q 2>&1 | tail -3
-timeout 1500 python tools/hist_select.py --out gpurun_out/artifacts > gpurun_out/hist_select.log 2>&1; echo "hist rc=$?"
+for g in 1 0; do for c in 1 2 4 8 16; do echo "GRAPH=$g CHUNKS=$c"; NITRO_RUN_HOST_GRAPH=$g NITRO_RUN_HOST_CHUNKS=$c timeout 300 python tools/e2e_probe.py 2>&1 | tail -4; done; done
