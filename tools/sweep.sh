@@ -1,3 +1,4 @@
-t() { timeout 300 python tools/profile_variants.py --time $1 $2 2>/dev/null | python -c "import json,sys; t=json.load(sys.stdin); print({c: {k: (round(v['GBps']), round(v['ms'],4)) for k,v in r['variants'].items()} for c,r in t.items()})"; }
-for rep in 1 2; do for pf in 0 1 2 4; do echo "HYB_PF=$pf"; NITRO_HYB_PF=$pf t "c2b uvar3 band01" "hyb"; done; done
-NITRO_HYB_PF=2 timeout 900 python -m pytest tests/test_gpu_parity.py -q -x -k "tolerance or long_row or c2b or integer" 2>&1 | tail -2
+python tools/hist_probe.py --time uniform; python tools/hist_probe.py --time spike; python tools/hist_probe.py --time normal
+timeout 900 ncu --set full --clock-control none -k 'regex:k_hist_(shared|global|sort)' -c 12 -o /tmp/prof_hist -f python tools/hist_probe.py uniform > gpurun_out/prof_hist.log 2>&1; echo "ncu rc=$?"
+ncu -i /tmp/prof_hist.ncu-rep --page raw --csv > gpurun_out/prof_hist_raw.csv 2>/dev/null
+ls -la gpurun_out/prof_hist_raw.csv
