@@ -1,4 +1,5 @@
+timeout 600 python -m pytest tests/test_gpu_hist.py -x -q 2>&1 | tail -2
 python tools/hist_probe.py --time uniform; python tools/hist_probe.py --time spike; python tools/hist_probe.py --time normal
-timeout 900 ncu --set full --clock-control none -k 'regex:k_hist_(shared|global|sort)' -c 12 -o /tmp/prof_hist -f python tools/hist_probe.py uniform > gpurun_out/prof_hist.log 2>&1; echo "ncu rc=$?"
-ncu -i /tmp/prof_hist.ncu-rep --page raw --csv > gpurun_out/prof_hist_raw.csv 2>/dev/null
-ls -la gpurun_out/prof_hist_raw.csv
+timeout 1500 python tools/hist_select.py --out gpurun_out/artifacts > gpurun_out/hist_select.log 2>&1; echo "hist rc=$?"
+python -c "
+import json; r=json.load(open('gpurun_out/artifacts/hist_report.json')); print({k:v for k,v in r.items() if k in ('nitro_pct_mean','share_ge_90','best_gbps_median','best_gbps_max','train_label_counts','always_variant_mean')})"
