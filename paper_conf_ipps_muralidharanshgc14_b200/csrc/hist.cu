@@ -544,6 +544,10 @@ static int hist_constraint(const void *input, void *user) {
 nitro_status_t nitro_hist_register(nitro_cv *cv) {
   HIST_GUARD_BEGIN
   if (!cv) return fail(NITRO_E_INVALID_ARG, "NULL cv");
+  int nv = 0, nf = 0;
+  NITRO_TRY(nitro_cv_num_variants(cv, &nv));
+  NITRO_TRY(nitro_cv_num_features(cv, &nf));
+  if (nv != 0 || nf != 0) return fail(NITRO_E_STATE, "register on a fresh code variant");
   static const char *vn[NITRO_HIST_NUM_VARIANTS] = {"sort_es", "sort_dynamic", "shared_atomic_es",
                                                      "shared_atomic_dynamic", "global_atomic_es",
                                                      "global_atomic_dynamic"};
