@@ -1037,14 +1037,18 @@ bool l2_evict_first() {
 // ELL slot batch width: NITRO_ELL_U overrides (1/2/4/8); default 2.  B200 sweep
 // on configs[1] (fp32): U=2 6372, U=4 5461, U=8 4681 GB/s — fewer registers and
 // more resident warps beat deeper per-thread batches for this gather pattern.
-int ell_batch(size_t sv) {
+// With the L2 prefetch on (few-diagonal matrices) U = 1 is best: the prefetch
+// keeps the stream in flight and the fewer registers buy occupancy (B200,
+// U=1 vs 2 at PF=1, 2 repeats: c1 6458 vs 5817 GB/s, dense band b=48 6965 vs
+// 6197, 256^3 6540 vs 6810); random-column matrices keep U = 2 (c2a 2127 vs 2102).
+int ell_batch(size_t sv, bool local) {
   static int env = [] {
     const char *e = getenv("NITRO_ELL_U");
     return e ? atoi(e) : 0;
   }();
   (void)sv;
   if (env == 1 || env == 2 || env == 4 || env == 8) return env;
-  return 2;
+  return local ? 1 : 2;
 }
 
 unsigned grid_cap(int64_t blocks, int per_sm);
@@ -1066,7 +1070,9 @@ void launch_ell(const int32_t *col, const VT *val, const VT *x, VT *y, int64_t N
   const int pf = nr < 0 && local ? ell_prefetch() : 0;
   if (nr < 0) nr = ld;
   const unsigned g = grid_cap(((nr + 3) / 4 + 255) / 256, 16);
-  switch (ell_batch(sizeof(VT))) {
+  // U from the matrix class only (not from pf), so row-chunk launches (pf = 0)
+  // and NITRO_ELL_PF=0 sum a row exactly like the default whole multiply
+  switch (ell_batch(sizeof(VT), local)) {
     case 1: k_ell<VT, 1><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first(), pf, prefetch_hint()); break;
     case 2: k_ell<VT, 2><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first(), pf, prefetch_hint()); break;
     case 4: k_ell<VT, 4><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first(), pf, prefetch_hint()); break;
