@@ -1072,7 +1072,11 @@ void launch_ell(const int32_t *col, const VT *val, const VT *x, VT *y, int64_t N
   const unsigned g = grid_cap(((nr + 3) / 4 + 255) / 256, 16);
   // U from the matrix class only (not from pf), so row-chunk launches (pf = 0)
   // and NITRO_ELL_PF=0 sum a row exactly like the default whole multiply
-  switch (ell_batch(sizeof(VT), local)) {
+  // (the U = 1 gain holds up to ~2 GB of slot arrays: c1 0.47 GB and a dense
+  // band 1.6 GB gain 11-12 %, a 256^3 stencil 3.6 GB loses 4 % and 512^3 30 GB
+  // loses 14 % — 6585 vs 5642 GB/s — so larger ELL formats keep U = 2)
+  const bool small = (double)K * (double)ld * (double)(sizeof(VT) + 4) <= 2.0 * 1073741824.0;
+  switch (ell_batch(sizeof(VT), local && small)) {
     case 1: k_ell<VT, 1><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first(), pf, prefetch_hint()); break;
     case 2: k_ell<VT, 2><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first(), pf, prefetch_hint()); break;
     case 4: k_ell<VT, 4><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first(), pf, prefetch_hint()); break;
