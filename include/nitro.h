@@ -90,13 +90,14 @@ nitro_status_t nitro_cv_add_feature_group(nitro_cv *cv, const char *const *names
 /* add_constraint(&variant, &constraint).  Several may be
  * added per variant; all must hold. */
 nitro_status_t nitro_cv_add_constraint(nitro_cv *cv, int variant_id, nitro_constraint_fn fn, void *user);
-/* Feature transform of the model (R11; default none = libSVM's
- * svm-scale): features j with bit j of log_mask set are replaced by
+/* Feature transform of the model.  Default (and the paper's reading):
+ * none = libSVM's svm-scale min-max to [-1, 1].  EXTENSION (R11x,
+ * not from the paper): features j with bit j of log_mask set are replaced by
  * log1p(x) (they must be >= 0) before the [-1, 1] min-max scaling; clip != 0
  * clips scaled inputs to [-1, 1], so inputs beyond the training range are
  * treated as the nearest training extreme instead of extrapolated by the RBF
  * kernel.  Before training (NITRO_E_STATE after); saved in the model file.
- * nitro_spmv_register sets log_mask = all seven features, clip = 1. */
+ * The registration helpers leave the paper's plain scaling in place. */
 nitro_status_t nitro_cv_set_feature_transform(nitro_cv *cv, uint32_t log_mask, int clip);
 /* set_training_args.  `input` is borrowed until train returns. */
 nitro_status_t nitro_cv_add_training_input(nitro_cv *cv, void *input);
@@ -255,10 +256,12 @@ nitro_status_t nitro_spmv_allowed(nitro_spmv *A, int variant, int *out_allowed);
 nitro_status_t nitro_spmv_set_budget(nitro_spmv *A, double bytes);
 /* Kernel implementation of the two CSR variants (DESIGN.md §6 K5/K6; the
  * arithmetic, and so y, is identical across implementations):
- * NITRO_CSR_IMPL_AUTO (default) = TMA row-tile pipeline when a mean tile fits
- * the shared-memory stage, else the direct kernels; _DIRECT = direct kernels
- * (loads from global memory); _STAGED = the tile pipeline for every matrix
- * (tiles that do not fit are computed from global memory).  Returns
+ * NITRO_CSR_IMPL_AUTO (default) = the direct kernels (loads from global
+ * memory; the TMA row-tile pipeline measured slower on every class, so AUTO
+ * uses it only when the environment sets NITRO_CSR_STAGED=1); _DIRECT = the
+ * direct kernels; _STAGED = the TMA row-tile pipeline for every matrix
+ * (tiles that do not fit the shared-memory stage are computed from global
+ * memory).  Returns
  * NITRO_E_INVALID_ARG for any other value.  Takes effect at the next run. */
 enum { NITRO_CSR_IMPL_AUTO = 0, NITRO_CSR_IMPL_DIRECT = 1, NITRO_CSR_IMPL_STAGED = 2 };
 nitro_status_t nitro_spmv_set_csr_impl(nitro_spmv *A, int impl);
@@ -272,12 +275,13 @@ nitro_status_t nitro_spmv_run(nitro_spmv *A, int variant, const void *d_x, void 
  * synchronises.  h_x / h_y should be pinned for full speed. */
 nitro_status_t nitro_spmv_run_host(nitro_spmv *A, int variant, const void *h_x, void *h_y);
 /* Timing (a variant's cost is its elapsed time): warmup runs, then
- * `reps` runs each preceded (if flush_l2) by an L2-evicting write, CUDA events
+ * `reps` runs each preceded (if flush_l2) by an L2-evicting read of 3x the L2 size, CUDA events
  * around the SpMV kernels only; returns the median in seconds.  out_all
  * (nullable) receives all reps. */
 nitro_status_t nitro_spmv_time(nitro_spmv *A, int variant, const void *d_x, void *d_y, int warmup, int reps,
                                int flush_l2, double *out_median_s, double *out_all);
-/* Write >= 2x L2 bytes to a scratch buffer on the handle's stream. */
+/* Evict L2: a streaming read of a scratch buffer of 3x the L2 size (clean
+ * lines, so no write-back lands in the next timed region), on the handle's stream. */
 nitro_status_t nitro_spmv_flush_l2(nitro_spmv *A);
 /* Number of kernel launches one nitro_spmv_run of `variant` issues. */
 nitro_status_t nitro_spmv_launches(nitro_spmv *A, int variant, int *out);
@@ -425,7 +429,7 @@ typedef struct {
   int warmup, reps, flush_l2;
 } nitro_hist_input;
 /* Register on a fresh cv: the 6 variants (ids = nitro_hist_variant), the
- * feature group {n, n_per_bin, subsample_sd} (log1p + clip transform), the
+ * feature group {n, n_per_bin, subsample_sd} (plain [-1, 1] scaling), the
  * shared-memory constraints, default = SORT_ES (always allowed; robust to
  * skewed inputs, where atomics contend). */
 nitro_status_t nitro_hist_register(nitro_cv *cv);

@@ -62,14 +62,20 @@ def nitro_percent(costs, selected) -> dict:
 
 
 # ---------------------------------------------------------------- C11 scaling
-# Reading R11 for the SpMV feature set: all seven features are >= 0
-# and heavy-tailed, so the model sees log1p(x), min-max scaled, and clips
-# scaled inputs to [-1, 1].  Other feature sets default to plain svm-scale.
-SPMV_LOG_MASK, SPMV_CLIP = 0x7F, True
+# The paper's reading ("features are scaled to the range [-1, 1]"):
+# libSVM svm-scale min-max with the training min/max, test inputs not clipped.
+# That is the default of every function below (log_mask = 0, clip = False).
+#
+# EXTENSION (not from the paper; R11x): the SpMV features are >= 0 and
+# heavy-tailed, so a variant of the model sees log1p(x) before the min-max
+# scaling and clips scaled inputs to [-1, 1].  It is reported next to the
+# paper-faithful model, never instead of it.
+R11X_LOG_MASK, R11X_CLIP = 0x7F, True
 
 
 def feature_transform(X, log_mask: int = 0):
-    """log1p of the columns j with bit j of log_mask set (values must be >= 0)."""
+    """log1p of the columns j with bit j of log_mask set (values must be >= 0).
+    log_mask = 0 (the paper's reading) is the identity."""
     X = np.array(X, dtype=np.float64, copy=True)
     for j in range(X.shape[1]):
         if (log_mask >> j) & 1:
@@ -179,6 +185,47 @@ def train(F, labels, folds: int = 5, seed: int = 0, tol: float = 1e-6, log2c=LOG
     m = Model(lo, hi, 2.0 ** lc, 2.0 ** lg, svc, const, log_mask, clip)
     m.cv_accuracy = acc
     return m
+
+
+def decisions(model: Model, X):
+    """One-vs-one decision values [n, n_pairs] of raw feature rows (after the
+    model's transform and scaling); None for a single-class model."""
+    if model.svc is None:
+        return None
+    Xs = scale_apply(feature_transform(X, model.log_mask), model.lo, model.hi, model.clip)
+    D = model.svc.decision_function(Xs)
+    return D[:, None] if D.ndim == 1 else D
+
+
+def decided(model: Model, X, eps: float = 1e-6):
+    """Reading C12: two solvers of the same convex QP (to tolerance) may flip
+    the sign of an OvO decision value within eps of 0, so a prediction is only
+    required to agree where it is decided by the firm signs: every assignment
+    of signs to the pairs with |decision| <= eps gives the same OvO vote
+    winner (votes: dec > 0 -> the pair's first class, else the second; vote
+    ties -> lowest label, as libSVM).  Boolean mask over the rows of X."""
+    D = decisions(model, X)
+    if D is None:
+        return np.ones(len(X), dtype=bool)
+    cls = list(model.svc.classes_)
+    k = len(cls)
+    pairs = [(a, b) for a in range(k) for b in range(a + 1, k)]
+    out = np.zeros(len(X), dtype=bool)
+    for i, row in enumerate(D):
+        soft = [p for p in range(len(pairs)) if abs(row[p]) <= eps]
+        if len(soft) > 12:
+            continue
+        winners = set()
+        for mask in range(1 << len(soft)):
+            sign = [row[p] > 0 for p in range(len(pairs))]
+            for t, p in enumerate(soft):
+                sign[p] = bool((mask >> t) & 1)
+            votes = [0] * k
+            for p, (a, b) in enumerate(pairs):
+                votes[a if sign[p] else b] += 1
+            winners.add(max(range(k), key=lambda c: (votes[c], -c)))
+        out[i] = len(winners) == 1
+    return out
 
 
 def select(model: Model, feat_vec, allowed, default: int = 1) -> int:

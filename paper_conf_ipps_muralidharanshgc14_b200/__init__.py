@@ -214,6 +214,20 @@ def _ptr(t):
     return t.data_ptr()
 
 
+def _dev_vec(t, n: int, dtype, device: int, name: str):
+    """A device array argument of the C ABI: contiguous, right dtype and
+    device, at least n elements (the library reads n elements behind the pointer)."""
+    if not t.is_cuda or t.device.index != device:
+        raise ValueError(f"{name}: expected a tensor on cuda:{device}, got {t.device}")
+    if t.dtype != dtype:
+        raise ValueError(f"{name}: expected {dtype}, got {t.dtype}")
+    if not t.is_contiguous():
+        raise ValueError(f"{name}: must be contiguous")
+    if t.numel() < n:
+        raise ValueError(f"{name}: {t.numel()} elements, need {n}")
+    return t.data_ptr()
+
+
 def _np(a, dtype):
     return np.ascontiguousarray(np.asarray(a, dtype=dtype))
 
@@ -226,14 +240,18 @@ class SpMV:
 
     def __init__(self, rowptr, colidx, vals, rows: int, cols: int, stream=None, device: int | None = None):
         import torch
-        assert rowptr.is_cuda and colidx.is_cuda and vals.is_cuda, "SpMV needs CUDA tensors"
-        assert colidx.dtype == torch.int32 and rowptr.dtype in (torch.int32, torch.int64)
-        assert vals.dtype in (torch.float32, torch.float64)
+        if not (rowptr.is_cuda and colidx.is_cuda and vals.is_cuda):
+            raise ValueError("SpMV needs CUDA tensors")
+        if rowptr.dtype not in (torch.int32, torch.int64) or vals.dtype not in (torch.float32, torch.float64):
+            raise ValueError("rowptr must be int32/int64 and vals fp32/fp64")
         self._keep = (rowptr, colidx, vals)
         self.rows, self.cols, self.nnz = int(rows), int(cols), int(colidx.numel())
         self.fp64 = vals.dtype == torch.float64
         self.dtype = vals.dtype
         self.device = rowptr.device.index if device is None else device
+        _dev_vec(rowptr, self.rows + 1, rowptr.dtype, self.device, "rowptr")
+        _dev_vec(colidx, self.nnz, torch.int32, self.device, "colidx")
+        _dev_vec(vals, self.nnz, vals.dtype, self.device, "vals")
         if stream is None:
             stream = torch.cuda.current_stream(self.device).cuda_stream
         self.stream = stream
@@ -300,21 +318,30 @@ class SpMV:
         import torch
         if y is None:
             y = torch.empty(self.rows, dtype=self.dtype, device=x.device)
-        _check(_L.nitro_spmv_run(self.h, v, _ptr(x), _ptr(y)))
+        _check(_L.nitro_spmv_run(self.h, v, self._x(x), self._y(y)))
         return y
+
+    def _x(self, x):
+        return _dev_vec(x, self.cols, self.dtype, self.device, "x")
+
+    def _y(self, y):
+        return _dev_vec(y, self.rows, self.dtype, self.device, "y")
 
     def run_host(self, v: int, x_host: np.ndarray, y_host: np.ndarray | None = None) -> np.ndarray:
         dt = np.float64 if self.fp64 else np.float32
-        assert x_host.dtype == dt and x_host.flags.c_contiguous
+        if x_host.dtype != dt or not x_host.flags.c_contiguous or x_host.size < self.cols:
+            raise ValueError(f"x_host: need a contiguous {np.dtype(dt)} array of >= {self.cols} elements")
         if y_host is None:
             y_host = np.empty(self.rows, dtype=dt)
+        if y_host.dtype != dt or not y_host.flags.c_contiguous or y_host.size < self.rows:
+            raise ValueError(f"y_host: need a contiguous {np.dtype(dt)} array of >= {self.rows} elements")
         _check(_L.nitro_spmv_run_host(self.h, v, _ptr(x_host), _ptr(y_host)))
         return y_host
 
     def time(self, v: int, x, y, warmup: int = 3, reps: int = 20, flush_l2: bool = True):
         med = ctypes.c_double()
         allt = np.empty(reps, dtype=np.float64)
-        _check(_L.nitro_spmv_time(self.h, v, _ptr(x), _ptr(y), warmup, reps, int(flush_l2), ctypes.byref(med),
+        _check(_L.nitro_spmv_time(self.h, v, self._x(x), self._y(y), warmup, reps, int(flush_l2), ctypes.byref(med),
                                   _ptr(allt)))
         return med.value, allt
 
@@ -502,7 +529,7 @@ class CodeVariant:
 
 def spmv_input(A: SpMV, x, y, warmup=3, reps=20, flush_l2=True) -> SpmvInput:
     """Input record for the registered SpMV variants (keep it alive while used)."""
-    rec = SpmvInput(A.h.value, _ptr(x), _ptr(y), warmup, reps, int(flush_l2))
+    rec = SpmvInput(A.h.value, A._x(x), A._y(y), warmup, reps, int(flush_l2))
     rec._keep = (A, x, y)
     return rec
 
@@ -513,7 +540,9 @@ class Hist:
 
     def __init__(self, samples, nbins: int, value_range: int, stream=None):
         import torch
-        assert samples.is_cuda and samples.dtype in (torch.int32, torch.uint32), "uint32 CUDA samples"
+        if samples.dtype not in (torch.int32, torch.uint32):
+            raise ValueError("samples: uint32 (or int32 bit pattern) CUDA tensor expected")
+        _dev_vec(samples, samples.numel(), samples.dtype, samples.device.index if samples.is_cuda else -1, "samples")
         self._keep = samples
         self.n, self.nbins, self.range = int(samples.numel()), int(nbins), int(value_range)
         self.device = samples.device.index
@@ -549,13 +578,19 @@ class Hist:
         import torch
         if hist is None:
             hist = torch.empty(self.nbins, dtype=torch.int32, device=self._keep.device)
-        _check(_L.nitro_hist_run(self.h, v, _ptr(hist)))
+        _check(_L.nitro_hist_run(self.h, v, self._h(hist)))
         return hist
 
     def time(self, v: int, hist, warmup=3, reps=20, flush_l2=True) -> float:
         t = ctypes.c_double()
-        _check(_L.nitro_hist_time(self.h, v, _ptr(hist), warmup, reps, int(flush_l2), ctypes.byref(t)))
+        _check(_L.nitro_hist_time(self.h, v, self._h(hist), warmup, reps, int(flush_l2), ctypes.byref(t)))
         return t.value
+
+    def _h(self, hist):
+        import torch
+        if hist.dtype not in (torch.int32, torch.uint32):
+            raise ValueError("hist: int32/uint32 tensor expected")
+        return _dev_vec(hist, self.nbins, hist.dtype, self.device, "hist")
 
 
 def hist_input(H: Hist, hist, warmup=3, reps=20, flush_l2=True) -> HistInput:

@@ -267,7 +267,6 @@ int run_host_chunks(const nitro_spmv *A, int variant) {
     return e ? atoi(e) : 0;
   }();
   if (variant != NITRO_CSR_SCALAR && variant != NITRO_ELL && variant != NITRO_DIA) return 1;
-  if (variant == NITRO_DIA && nitro::dia_use_tma()) return 1;
   // 4: B200 host wall time of the configs[1] DIA call, pinned buffers (ms):
   // 1 chunk 0.372, 2 0.320, 4 0.313, 8 0.340, 16 0.410 (smaller copies lose
   // more to per-copy setup than the finer overlap gains); a CUDA-graph

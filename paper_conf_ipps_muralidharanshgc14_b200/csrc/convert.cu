@@ -315,7 +315,7 @@ int hyb_windows(size_t sv) {
     const char *e = getenv("NITRO_HYB_W");
     return e ? atoi(e) : 0;
   }();
-  if (env == 2 || env == 4 || env == 8) return env;
+  if (env == 4 || env == 8) return env;
   return sv == 8 ? 4 : 8;
 }
 

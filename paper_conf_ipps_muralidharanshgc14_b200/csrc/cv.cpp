@@ -41,6 +41,7 @@ struct nitro_cv {
   std::string name;
   std::vector<Variant> variants;
   int default_id = 0;
+  int model_nv = 0;  // variant count of a loaded model (a cv without registered variants)
   std::vector<FeatureEntry> feats;
   int n_feat = 0;
   std::vector<void *> inputs;
@@ -581,6 +582,7 @@ nitro_status_t nitro_cv_load_model(nitro_cv *cv, const char *path) {
   unsigned flog = 0;
   int fclip = 0;
   if (ver >= 2 && std::fscanf(f, "%u %d", &flog, &fclip) != 2) return bad("feature transform");
+  if (nf <= 0 || nf > 4096 || nv <= 0 || nv > 4096) return bad("feature / variant count");
   if (cv->n_feat && nf != cv->n_feat) return bad("feature count differs from this code variant");
   if (!cv->variants.empty() && nv != (int)cv->variants.size()) return bad("variant count differs");
   cv->flog = flog;
@@ -593,9 +595,14 @@ nitro_status_t nitro_cv_load_model(nitro_cv *cv, const char *path) {
   SvmModel m;
   size_t ncls = 0;
   if (std::fscanf(f, "%d %d %d %zu", &m.d, &m.n_train, &m.const_label, &ncls) != 4) return bad("svm header");
+  // every index the predictor follows is validated here (a stale or corrupted
+  // file must give NITRO_E_IO, not out-of-bounds reads at predict time)
+  if (m.d != nf) return bad("SVM dimension differs from the feature count");
+  if (m.n_train < 0 || m.n_train > (1 << 24) || ncls > (size_t)nv) return bad("svm sizes");
+  if (m.const_label >= nv || (m.const_label < 0 && ncls == 0)) return bad("constant label");
   m.classes.resize(ncls);
   for (auto &c : m.classes)
-    if (std::fscanf(f, "%d", &c) != 1) return bad("classes");
+    if (std::fscanf(f, "%d", &c) != 1 || c < 0 || c >= nv) return bad("classes");
   m.X.resize((size_t)m.d * m.n_train);
   for (auto &x : m.X)
     if (std::fscanf(f, "%lg", &x) != 1) return bad("points");
@@ -605,16 +612,20 @@ nitro_status_t nitro_cv_load_model(nitro_cv *cv, const char *path) {
   for (auto &p : m.pairs) {
     size_t ns = 0;
     if (std::fscanf(f, "%d %d %lg %zu", &p.ca, &p.cb, &p.rho, &ns) != 4) return bad("pair");
+    if (p.ca < 0 || p.cb < 0 || (size_t)p.ca >= ncls || (size_t)p.cb >= ncls || ns > (size_t)m.n_train)
+      return bad("pair classes");
     p.sv.resize(ns);
     p.coef.resize(ns);
     for (size_t t = 0; t < ns; ++t)
-      if (std::fscanf(f, "%d %lg", &p.sv[t], &p.coef[t]) != 2) return bad("sv");
+      if (std::fscanf(f, "%d %lg", &p.sv[t], &p.coef[t]) != 2 || p.sv[t] < 0 || p.sv[t] >= m.n_train)
+        return bad("sv");
   }
   std::fclose(f);
   m.gamma = cv->gamma;
   cv->svm = std::move(m);
   cv->n_feat = nf;
   if (def >= 0 && def < nv && (int)cv->variants.size() == nv) cv->default_id = def;
+  cv->model_nv = nv;
   cv->trained = true;
   cv->frozen = true;
   return NITRO_OK;
@@ -626,7 +637,8 @@ nitro_status_t nitro_cv_predict(nitro_cv *cv, const double *feat, const int *all
   if (!cv || !feat || !out_variant) return fail(NITRO_E_INVALID_ARG, "NULL argument");
   if (!cv->trained) return fail(NITRO_E_STATE, "select before train/load");
   int v = predict_raw(cv, feat);
-  if (allowed_mask && (v < 0 || !allowed_mask[v])) v = cv->default_id;
+  const int nvar = cv->variants.empty() ? cv->model_nv : (int)cv->variants.size();
+  if (v < 0 || v >= nvar || (allowed_mask && !allowed_mask[v])) v = cv->default_id;
   *out_variant = v;
   return NITRO_OK;
   GUARD_END
@@ -696,10 +708,8 @@ nitro_status_t nitro_spmv_register(nitro_cv *cv) {
   NITRO_TRY(nitro_cv_add_feature_group(cv, fn, 7, spmv_feature_group, nullptr));
   NITRO_TRY(nitro_cv_add_constraint(cv, NITRO_DIA, spmv_constraint, (void *)(intptr_t)NITRO_DIA));
   NITRO_TRY(nitro_cv_add_constraint(cv, NITRO_ELL, spmv_constraint, (void *)(intptr_t)NITRO_ELL));
-  // the seven SpMV features are >= 0 and heavy-tailed (nnz and rows span
-  // decades, fills up to 1e4): log1p before scaling, and inputs beyond the
-  // training range clipped to it (R11)
-  NITRO_TRY(nitro_cv_set_feature_transform(cv, 0x7fu, 1));
+  // features scaled to [-1, 1] as the paper states; the log1p + clip
+  // extension (R11x) is opt-in: nitro_cv_set_feature_transform
   return nitro_cv_set_default(cv, NITRO_CSR_VECTOR);
   GUARD_END
 }

@@ -177,7 +177,7 @@ template <typename IT>
 __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
                                                         int64_t N, int64_t M, int64_t Z, int64_t row0, int64_t G,
                                                         FeatAcc *__restrict__ acc, uint32_t *__restrict__ bitmap,
-                                                        int2 *__restrict__ tasks) {
+                                                        int2 *__restrict__ tasks, int64_t cap_tasks) {
   __shared__ int s_stage[kWarps][kStage + kStage / 32];
   __shared__ int8_t s_slot[kWarps][32];
   __shared__ uint32_t s_seen[kCache];
@@ -274,7 +274,11 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
     if (is_long) {
       const int nc = (int)((L + kChunk - 1) / kChunk);
       const unsigned t0 = atomicAdd(&acc->nlong, (unsigned)nc);
-      for (int j = 0; j < nc; ++j) tasks[t0 + j] = make_int2((int)r, j);
+      // a malformed rowptr (rows overlapping, each within [0, Z]) can list more
+      // chunks than a monotone one: flag it instead of writing past the list
+      if ((int64_t)t0 + nc > cap_tasks) bad |= 1;
+      else
+        for (int j = 0; j < nc; ++j) tasks[t0 + j] = make_int2((int)r, j);
     }
     const unsigned long_mask = __ballot_sync(kFull, is_long);
     const bool staged = E1 - E0 <= kStage;  // implies no long row
@@ -439,14 +443,15 @@ __global__ void __launch_bounds__(kThreads) k_features_long(const IT *__restrict
                                                              const int32_t *__restrict__ col, int64_t M, int64_t row0,
                                                              int64_t G, FeatAcc *__restrict__ acc,
                                                              uint32_t *__restrict__ bitmap,
-                                                             const int2 *__restrict__ tasks) {
-  const unsigned n = *(volatile unsigned *)&acc->nlong;
+                                                             const int2 *__restrict__ tasks, int64_t cap_tasks) {
+  const int64_t n0 = (int64_t)*(volatile unsigned *)&acc->nlong;
+  const int64_t n = n0 < cap_tasks ? n0 : cap_tasks;  // more = malformed rowptr (flagged by k_features)
   const int lane = threadIdx.x & 31;
   const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const uint32_t G32 = (uint32_t)G, M32 = (uint32_t)M;
   unsigned bad = 0;
-  for (int64_t t = gw; t < (int64_t)n; t += nw) {
+  for (int64_t t = gw; t < n; t += nw) {
     const int2 tk = tasks[t];
     const int64_t a = (int64_t)rowptr[tk.x], b = (int64_t)rowptr[tk.x + 1];
     const int64_t st = a + (int64_t)tk.y * kChunk, en = st + kChunk < b ? st + kChunk : b;
@@ -552,16 +557,16 @@ nitro_status_t features_launch(nitro_spmv *A) {
                                                                            (A->Z / kChunk + kWarps - 1) / kWarps));
   if (A->rp64) {
     k_features<int64_t><<<(unsigned)grid, kThreads, 0, s>>>((const int64_t *)A->rowptr, A->col, A->N, A->M, A->Z,
-                                                            A->row0, G, acc, A->bitmap.as<uint32_t>(), tasks);
+                                                            A->row0, G, acc, A->bitmap.as<uint32_t>(), tasks, cap_tasks);
     if (A->Z > kLong)
       k_features_long<int64_t><<<glong, kThreads, 0, s>>>((const int64_t *)A->rowptr, A->col, A->M, A->row0, G, acc,
-                                                          A->bitmap.as<uint32_t>(), tasks);
+                                                          A->bitmap.as<uint32_t>(), tasks, cap_tasks);
   } else {
     k_features<int32_t><<<(unsigned)grid, kThreads, 0, s>>>((const int32_t *)A->rowptr, A->col, A->N, A->M, A->Z,
-                                                            A->row0, G, acc, A->bitmap.as<uint32_t>(), tasks);
+                                                            A->row0, G, acc, A->bitmap.as<uint32_t>(), tasks, cap_tasks);
     if (A->Z > kLong)
       k_features_long<int32_t><<<glong, kThreads, 0, s>>>((const int32_t *)A->rowptr, A->col, A->M, A->row0, G, acc,
-                                                          A->bitmap.as<uint32_t>(), tasks);
+                                                          A->bitmap.as<uint32_t>(), tasks, cap_tasks);
   }
   if (nwords) {
     int64_t g2 = (nwords + 255) / 256;

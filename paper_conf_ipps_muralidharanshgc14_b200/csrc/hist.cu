@@ -558,8 +558,7 @@ nitro_status_t nitro_hist_register(nitro_cv *cv) {
   NITRO_TRY(nitro_cv_add_constraint(cv, NITRO_HIST_SHARED_ES, hist_constraint, (void *)(intptr_t)NITRO_HIST_SHARED_ES));
   NITRO_TRY(nitro_cv_add_constraint(cv, NITRO_HIST_SHARED_DYN, hist_constraint,
                                     (void *)(intptr_t)NITRO_HIST_SHARED_DYN));
-  // N and N/#bins span decades, the SD up to 2^31: log1p + clip as for SpMV (R11)
-  NITRO_TRY(nitro_cv_set_feature_transform(cv, 0x7u, 1));
+  // plain [-1, 1] scaling; log1p + clip is the opt-in extension R11x
   // default: always allowed (the shared variants are not) and robust to skew
   return nitro_cv_set_default(cv, NITRO_HIST_SORT_ES);
   HIST_GUARD_END

@@ -151,8 +151,6 @@ nitro_status_t csr_chunk_xhi(nitro_spmv *A, const std::vector<int64_t> &ends, st
 int launches_of(const nitro_spmv *A, int variant);
 nitro_status_t launch_flush(nitro_spmv *A, cudaStream_t s);
 // spmv_dia_tma.cu: DIA with TMA-streamed diagonal slabs
-nitro_status_t launch_dia_tma(nitro_spmv *A, const void *x, void *y, cudaStream_t s);
-bool dia_use_tma();
 double compulsory_bytes(const nitro_spmv *A, int variant);
 
 // scan.cu: exclusive scan of int64 counts; out[n] = total.  scratch grows.

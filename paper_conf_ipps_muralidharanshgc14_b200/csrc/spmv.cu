@@ -585,218 +585,98 @@ __global__ void __launch_bounds__(256) k_ell(const int32_t *__restrict__ ecol, c
 }
 
 // ------------------------------------------------------------------ K8 DIA
-// Thread per 4 consecutive rows, block = 1024 rows; offsets in shared memory.
-// Blocks whose rows see every diagonal in range skip all bounds checks.
-// U diagonals per batch (all value and x loads of a batch issued before the
-// FMAs): larger U = more bytes in flight per thread but more registers, i.e.
-// fewer resident warps; chosen per launch (dia_batch()).
-// DS ("diagonal split") adjacent lanes share one 4-row quad, lane q taking the
-// diagonals d = q, q + DS, ...: each thread's serial chain of dependent
-// (value, x) loads is DS times shorter; the DS partial sums are combined by a
-// fixed xor butterfly (deterministic).
-template <typename VT, int U, int DS>
-__global__ void __launch_bounds__(256, (U == 1 && DS == 1 && sizeof(VT) == 4) ? 8 : 1)  // U=1 fp32: <= 32 regs, full occupancy
-    k_dia(const int32_t *__restrict__ offs, const VT *__restrict__ dval,
-                                             const VT *__restrict__ x, VT *__restrict__ y, int64_t N, int64_t M,
-                                             int64_t D, int64_t ld, int64_t nr, int64_t row0, int64_t off_min,
-                                             int64_t off_max, bool x_aligned, bool l2ef, int pf, bool pfh) {
-  constexpr int64_t RB = 1024 / DS;  // rows per block iteration
+// Thread per 4 consecutive rows, block = 1024 rows; offsets in shared memory
+// (the first kDiaSmemOffs; larger D reads the rest through L1).  Blocks whose
+// rows see every diagonal in range skip all bounds checks.  One diagonal per
+// step and <= 32 registers (full occupancy): B200 sweeps on configs[1] put
+// more diagonals per batch (U = 2/4/8: 4916/4561/3033 vs 5373 GB/s) and a
+// diagonal split across lanes (DS = 2/4: 4076/3115) behind — resident warps
+// matter more than per-thread bytes in flight.
+constexpr int kDiaSmemOffs = 12288;  // 48 KB of offsets: no dynamic-smem opt-in needed
+template <typename VT>
+__global__ void __launch_bounds__(256, sizeof(VT) == 4 ? 8 : 1)
+    k_dia(const int32_t *__restrict__ offs, const VT *__restrict__ dval, const VT *__restrict__ x,
+          VT *__restrict__ y, int64_t N, int64_t M, int64_t D, int64_t ld, int64_t nr, int64_t row0,
+          int64_t off_min, int64_t off_max, bool x_aligned, bool l2ef, int pf, bool pfh) {
+  constexpr int64_t RB = 1024;  // rows per block iteration
   const uint64_t pol = l2_policy(l2ef);
   extern __shared__ int s_off[];
+  const int64_t Ds = D < kDiaSmemOffs ? D : kDiaSmemOffs;
+  auto off_of = [&](int64_t d) -> int { return d < kDiaSmemOffs ? s_off[d] : __ldg(offs + d); };
   // pf > 0: thread 0 keeps the block's value segments pf diagonals ahead in L2
   // (one cp.async.bulk L2 prefetch per diagonal, no registers or shared
   // memory): the per-thread chain of dependent value loads then waits on L2,
   // not HBM, and the HBM stream has pf x 4 KB per CTA in flight.
-  for (int64_t d = threadIdx.x; d < D; d += blockDim.x) s_off[d] = offs[d];
+  for (int64_t d = threadIdx.x; d < Ds; d += blockDim.x) s_off[d] = offs[d];
   __syncthreads();
-  const int q = (int)(threadIdx.x % DS);
   const int64_t nb = (nr + RB - 1) / RB;  // rows [0, nr), nr <= ld (a row chunk: less)
   for (int64_t blk = blockIdx.x; blk < nb; blk += gridDim.x) {
     const int64_t B0 = blk * RB;
-    const int64_t i0 = B0 + 4 * (threadIdx.x / DS);
-    const bool active = i0 < nr;  // whole DS groups share i0: uniform within a group
+    const int64_t i0 = B0 + 4 * threadIdx.x;
     // segment bytes of one diagonal of this block (16-byte multiple: B0 and ld are multiples of 32 rows)
     const uint32_t pfb = (uint32_t)(((B0 + RB < nr ? B0 + RB : nr) - B0) * (int64_t)sizeof(VT)) & ~15u;
     if (pf > 0 && threadIdx.x == 0)
       for (int64_t d = 0; d < pf && d < D; ++d)
         pfh ? bulk_prefetch_l2(dval + d * ld + B0, pfb, pol) : bulk_prefetch_l2(dval + d * ld + B0, pfb);
-    if constexpr (DS == 1) {
-      if (!active) continue;      // no cross-lane combine needed
-    }
+    if (i0 >= nr) continue;
     const int64_t Bend = (B0 + RB < nr ? B0 + RB : nr) - 1;
     const bool interior = row0 + B0 + off_min >= 0 && row0 + Bend + off_max < M;
     // vector x path: aligned windows may reach 3 floats left / 4 right of the needed ones
     const bool xvec = x_aligned && row0 + B0 + off_min - 3 >= 0 && row0 + Bend + off_max + 4 < M;
     double acc[4] = {0.0, 0.0, 0.0, 0.0};
-    for (int64_t d0 = (int64_t)q * U; (DS == 1 || active) && d0 < D; d0 += (int64_t)DS * U) {
-      if (pf > 0 && threadIdx.x == 0)
-        for (int64_t d = d0 + pf; d < d0 + pf + DS * U && d < D; ++d)
-          pfh ? bulk_prefetch_l2(dval + d * ld + B0, pfb, pol) : bulk_prefetch_l2(dval + d * ld + B0, pfb);
-      V4<VT> v[U];
-      VT xv[U][4];
-#pragma unroll
-      for (int u = 0; u < U; ++u) {
-        if (d0 + u < D) v[u].load(dval + (d0 + u) * ld + i0, pol);
-        else v[u].v[0] = v[u].v[1] = v[u].v[2] = v[u].v[3] = (VT)0;
-      }
+    for (int64_t d = 0; d < D; ++d) {
+      if (pf > 0 && threadIdx.x == 0 && d + pf < D)
+        pfh ? bulk_prefetch_l2(dval + (d + pf) * ld + B0, pfb, pol) : bulk_prefetch_l2(dval + (d + pf) * ld + B0, pfb);
+      V4<VT> v;
+      v.load(dval + d * ld + i0, pol);
+      const int off = off_of(d);
+      VT xv[4];
       if (sizeof(VT) == 4 && xvec) {
         // fp32, x 16-byte aligned at row0: the 4 values x[j..j+3] (j = row0 + i0 +
         // off) come from the aligned 8-float window at j - (off & 3): two 128-bit
         // loads instead of four 32-bit ones (half the L1 wavefronts); off & 3 is
         // uniform across the warp (i0 is a multiple of 4)
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-          const bool live = d0 + u < D;
-          const int off = live ? s_off[d0 + u] : 0;
-          const int r = off & 3;
-          const float *xb = reinterpret_cast<const float *>(x) + (row0 + i0 + off - r);
-          float4 lo = make_float4(0.f, 0.f, 0.f, 0.f), hi = lo;
-          if (live) {
-            lo = __ldg(reinterpret_cast<const float4 *>(xb));
-            if (r) hi = __ldg(reinterpret_cast<const float4 *>(xb) + 1);
-          }
-          float w[4];
-          switch (r) {
-            case 0: w[0] = lo.x; w[1] = lo.y; w[2] = lo.z; w[3] = lo.w; break;
-            case 1: w[0] = lo.y; w[1] = lo.z; w[2] = lo.w; w[3] = hi.x; break;
-            case 2: w[0] = lo.z; w[1] = lo.w; w[2] = hi.x; w[3] = hi.y; break;
-            default: w[0] = lo.w; w[1] = hi.x; w[2] = hi.y; w[3] = hi.z; break;
-          }
-#pragma unroll
-          for (int t = 0; t < 4; ++t) xv[u][t] = (VT)w[t];
+        const int r = off & 3;
+        const float *xb = reinterpret_cast<const float *>(x) + (row0 + i0 + off - r);
+        const float4 lo = __ldg(reinterpret_cast<const float4 *>(xb));
+        float4 hi = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (r) hi = __ldg(reinterpret_cast<const float4 *>(xb) + 1);
+        float w[4];
+        switch (r) {
+          case 0: w[0] = lo.x; w[1] = lo.y; w[2] = lo.z; w[3] = lo.w; break;
+          case 1: w[0] = lo.y; w[1] = lo.z; w[2] = lo.w; w[3] = hi.x; break;
+          case 2: w[0] = lo.z; w[1] = lo.w; w[2] = hi.x; w[3] = hi.y; break;
+          default: w[0] = lo.w; w[1] = hi.x; w[2] = hi.y; w[3] = hi.z; break;
         }
+#pragma unroll
+        for (int t = 0; t < 4; ++t) xv[t] = (VT)w[t];
       } else if (interior) {
+        const VT *xp = x + (row0 + i0 + off);
 #pragma unroll
-        for (int u = 0; u < U; ++u) {
-          const bool live = d0 + u < D;  // uniform
-          const VT *xp = x + (row0 + i0 + (live ? s_off[d0 + u] : 0));
-#pragma unroll
-          for (int t = 0; t < 4; ++t) xv[u][t] = live ? __ldg(xp + t) : (VT)0;
-        }
+        for (int t = 0; t < 4; ++t) xv[t] = __ldg(xp + t);
       } else {
+        const int64_t j = row0 + i0 + off;
 #pragma unroll
-        for (int u = 0; u < U; ++u) {
-          const bool live = d0 + u < D;
-          const int64_t j = row0 + i0 + (live ? s_off[d0 + u] : 0);
-#pragma unroll
-          for (int t = 0; t < 4; ++t) xv[u][t] = (live && j + t >= 0 && j + t < M) ? __ldg(x + j + t) : (VT)0;
-        }
+        for (int t = 0; t < 4; ++t) xv[t] = (j + t >= 0 && j + t < M) ? __ldg(x + j + t) : (VT)0;
       }
-      VT part[4] = {0, 0, 0, 0};
 #pragma unroll
-      for (int u = 0; u < U; ++u)
-#pragma unroll
-        for (int t = 0; t < 4; ++t) part[t] = fma(v[u].v[t], xv[u][t], part[t]);
-#pragma unroll
-      for (int t = 0; t < 4; ++t) acc[t] += (double)part[t];
+      for (int t = 0; t < 4; ++t) acc[t] += (double)fma(v.v[t], xv[t], (VT)0);
     }
-#pragma unroll
-    for (int o = 1; o < DS; o <<= 1)
-#pragma unroll
-      for (int t = 0; t < 4; ++t) acc[t] += __shfl_xor_sync(kFull, acc[t], o);
-    if (active && q == 0) store4<VT>(y, i0, N, acc);
+    store4<VT>(y, i0, N, acc);
   }
 }
 
 // ------------------------------------------------------------------ K9b HYB COO tail
-// Warp per chunk of 32*W row-sorted tail entries: W coalesced windows loaded up
-// front, then a segmented inclusive scan per window (rows sorted => equal row
-// ids are contiguous).  Rows wholly inside the chunk are added to y directly
-// (single owner); the chunk's first and last rows go to two carry slots that
-// k_hyb_fixup_seg applies per row in slot order.  No atomics; deterministic.
-template <typename VT, int W>
-__global__ void __launch_bounds__(256) k_hyb_tail(const int32_t *__restrict__ trow, const int32_t *__restrict__ tcol,
-                                                  const VT *__restrict__ tval, const VT *__restrict__ x,
-                                                  VT *__restrict__ y, int64_t Zt, int64_t nch,
-                                                  int32_t *__restrict__ carry_row, double *__restrict__ carry_val) {
-  constexpr int64_t CH = 32 * W;  // chunk = W windows of 32 entries
-  const int lane = threadIdx.x & 31;
-  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  // software pipeline over the warp's chunks: the next chunk's (row, col, val)
-  // loads are issued right after the current chunk's x gathers, so they are in
-  // flight while the current chunk's segmented scans run
-  int rr[W], cc[W];
-  VT vv[W];
-  auto load_chunk = [&](int64_t c0, int64_t cend) {
-#pragma unroll
-    for (int w = 0; w < W; ++w) {
-      const int64_t e = c0 + w * 32 + lane;
-      const bool ok = e < cend;
-      rr[w] = ok ? ld_stream_i(trow + e) : -2;
-      cc[w] = ok ? ld_stream_i(tcol + e) : 0;
-      vv[w] = ok ? ld_stream(tval + e) : (VT)0;
-    }
-  };
-  if (warp < nch) load_chunk(warp * CH, warp * CH + CH < Zt ? warp * CH + CH : Zt);
-  for (int64_t ch = warp; ch < nch; ch += nw) {
-    const int64_t c0 = ch * CH, cend = c0 + CH < Zt ? c0 + CH : Zt;
-    const int first_row = __shfl_sync(kFull, rr[0], 0);
-    const int wl = (int)((cend - 1 - c0) >> 5), ll = (int)((cend - 1 - c0) & 31);
-    int last_row = 0;
-#pragma unroll
-    for (int w = 0; w < W; ++w) {
-      const int t = __shfl_sync(kFull, rr[w], ll);
-      if (w == wl) last_row = t;
-    }
-    double p[W];
-    int rcur[W];
-#pragma unroll
-    for (int w = 0; w < W; ++w) {
-      p[w] = (double)vv[w] * (double)__ldg(x + cc[w]);
-      rcur[w] = rr[w];
-    }
-    {
-      const int64_t n0 = ch + nw;
-      if (n0 < nch) load_chunk(n0 * CH, n0 * CH + CH < Zt ? n0 * CH + CH : Zt);
-    }
-    if (lane == 0) { carry_row[2 * ch] = -1; carry_row[2 * ch + 1] = -1; }
-    __syncwarp();
-    int carry_r = -3;
-    double carry_v = 0.0;
-#pragma unroll
-    for (int w = 0; w < W; ++w) {
-      const int64_t w0 = c0 + w * 32;
-      if (w0 >= cend) break;
-      double q = p[w];
-      const int r = rcur[w];
-      // a segment left open at the previous window's last lane ended exactly
-      // at the window boundary if this window starts a new row: emit it now
-      const int r_first = __shfl_sync(kFull, r, 0);
-      if (carry_r >= 0 && r_first != carry_r && lane == 0) {
-        if (carry_r == first_row) { carry_row[2 * ch] = carry_r; carry_val[2 * ch] = carry_v; }
-        else if (carry_r == last_row) { carry_row[2 * ch + 1] = carry_r; carry_val[2 * ch + 1] = carry_v; }
-        else y[carry_r] = (VT)((double)y[carry_r] + carry_v);
-      }
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const double t = __shfl_up_sync(kFull, q, o);
-        const int rt = __shfl_up_sync(kFull, r, o);
-        if (lane >= o && rt == r) q += t;
-      }
-      if (r == carry_r) q += carry_v;
-      const int nr = __shfl_down_sync(kFull, r, 1);
-      const int lvl = (int)(cend - 1 - w0 < 31 ? cend - 1 - w0 : 31);  // last valid lane
-      const bool more = w0 + 32 < cend;
-      const bool is_end = r >= 0 && (lane == lvl || nr != r);
-      const bool open = lane == lvl && more;
-      if (is_end && !open) {
-        if (r == first_row) { carry_row[2 * ch] = r; carry_val[2 * ch] = q; }
-        else if (r == last_row) { carry_row[2 * ch + 1] = r; carry_val[2 * ch + 1] = q; }
-        else y[r] = (VT)((double)y[r] + q);
-      }
-      carry_r = __shfl_sync(kFull, r, lvl);
-      carry_v = __shfl_sync(kFull, q, lvl);
-    }
-  }
-}
-
-// K9b' (default): lane-sequential variant.  Lane l of a chunk owns the EP
+// Rows sorted => equal row ids are contiguous.  Rows wholly inside a chunk are
+// added to y directly (single owner); the chunk's first and last rows go to
+// two carry slots that k_hyb_fixup_seg applies per row in slot order.  No
+// atomics; deterministic.
+// Lane-sequential layout: lane l of a chunk owns the EP
 // consecutive entries [c0 + l*EP, c0 + (l+1)*EP) (128-bit vector loads of
 // row/col ids), sums them sequentially per row, writes rows that start and end
 // inside the lane directly, and one segmented scan ACROSS LANES (5 steps)
 // joins the runs that cross lane boundaries — 1 scan per 32*EP entries
-// instead of one per 32.  Same chunk-level ownership/carry rule as k_hyb_tail.
+// instead of one per 32.
 template <typename VT, int EP>
 __global__ void __launch_bounds__(256) k_hyb_tail_ls(const int32_t *__restrict__ trow, const int32_t *__restrict__ tcol,
                                                      const VT *__restrict__ tval, const VT *__restrict__ x,
@@ -957,33 +837,6 @@ __global__ void __launch_bounds__(256) k_flush(const int4 *__restrict__ buf, int
   if (acc == 0x7fffffff) *sink = acc;
 }
 
-// DIA batch width: NITRO_DIA_U overrides (1/2/4); default 1.  B200 sweep on
-// configs[1] with vectorised x loads: U=1 5373, 2 4916, 4 4561, 8 3033 GB/s —
-// registers (resident warps) matter more than per-thread bytes in flight.
-int dia_batch(int64_t D, size_t sv) {
-  static int env = [] {
-    const char *e = getenv("NITRO_DIA_U");
-    return e ? atoi(e) : 0;
-  }();
-  if (env == 1 || env == 2 || env == 4) return env;
-  (void)D;
-  (void)sv;
-  return 1;
-}
-
-// DIA diagonal split: NITRO_DIA_DS overrides (1/2/4); default 1 (B200 sweep on
-// configs[1]: DS=2 4076, DS=4 3115 GB/s — the extra registers and butterfly
-// cost more than the shorter per-thread chains gain)
-int dia_split(int64_t D) {
-  static int env = [] {
-    const char *e = getenv("NITRO_DIA_DS");
-    return e ? atoi(e) : 0;
-  }();
-  (void)D;
-  if (env == 1 || env == 2 || env == 4) return env;
-  return 1;
-}
-
 // DIA L2 prefetch distance in diagonals: NITRO_DIA_PF overrides; default 1.
 // B200, 3 interleaved repeats (GB/s): configs[1] 128^3 PF=0 5133, 1 5357,
 // 2 5367; 256^3 PF=0 6355, 1 6796, 2 6731.
@@ -1034,7 +887,7 @@ bool l2_evict_first() {
   return v;
 }
 
-// ELL slot batch width: NITRO_ELL_U overrides (1/2/4/8); default 2.  B200 sweep
+// ELL slot batch width: NITRO_ELL_U overrides (1/2); default 2.  B200 sweep
 // on configs[1] (fp32): U=2 6372, U=4 5461, U=8 4681 GB/s — fewer registers and
 // more resident warps beat deeper per-thread batches for this gather pattern.
 // With the L2 prefetch on (few-diagonal matrices) U = 1 is best: the prefetch
@@ -1047,7 +900,7 @@ int ell_batch(size_t sv, bool local) {
     return e ? atoi(e) : 0;
   }();
   (void)sv;
-  if (env == 1 || env == 2 || env == 4 || env == 8) return env;
+  if (env == 1 || env == 2) return env;
   return local ? 1 : 2;
 }
 
@@ -1076,26 +929,11 @@ void launch_ell(const int32_t *col, const VT *val, const VT *x, VT *y, int64_t N
   // band 1.6 GB gain 11-12 %, a 256^3 stencil 3.6 GB loses 4 % and 512^3 30 GB
   // loses 14 % — 6585 vs 5642 GB/s — so larger ELL formats keep U = 2)
   const bool small = (double)K * (double)ld * (double)(sizeof(VT) + 4) <= 2.0 * 1073741824.0;
-  switch (ell_batch(sizeof(VT), local && small)) {
-    case 1: k_ell<VT, 1><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first(), pf, prefetch_hint()); break;
-    case 2: k_ell<VT, 2><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first(), pf, prefetch_hint()); break;
-    case 4: k_ell<VT, 4><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first(), pf, prefetch_hint()); break;
-    default: k_ell<VT, 8><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first(), pf, prefetch_hint()); break;
-  }
+  if (ell_batch(sizeof(VT), local && small) == 1)
+    k_ell<VT, 1><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first(), pf, prefetch_hint());
+  else
+    k_ell<VT, 2><<<g, 256, 0, s>>>(col, val, x, y, N, K, ld, nr, l2_evict_first(), pf, prefetch_hint());
 }
-
-}  // namespace
-
-// DIA implementation: NITRO_DIA_TMA=1 selects the TMA-streamed kernel
-bool dia_use_tma() {
-  static int v = [] {
-    const char *e = getenv("NITRO_DIA_TMA");
-    return e ? atoi(e) : 0;
-  }();
-  return v != 0;
-}
-
-namespace {
 
 unsigned grid_cap(int64_t blocks, int per_sm = 8) {
   int64_t cap = (int64_t)num_sms() * per_sm;
@@ -1306,30 +1144,14 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
                        part ? round_up(N, 32) : -1, diag_local(A));
       break;
     case NITRO_DIA:
-      if (N > 0 && A->dia.D > 0 && dia_use_tma() && !part) return launch_dia_tma(A, x, y, s);
       if (N > 0) {
-        const size_t sm = (size_t)std::max<int64_t>(A->dia.D, 1) * 4;
+        const size_t sm = (size_t)std::min<int64_t>(std::max<int64_t>(A->dia.D, 1), kDiaSmemOffs) * 4;
         const int64_t row0 = A->row0 + r0, nr = part ? round_up(N, 32) : A->dia.ld;
         const bool x_al = ((reinterpret_cast<uintptr_t>(x) & 15) == 0) && (row0 % 4 == 0);
-        const int U = dia_batch(A->dia.D, sizeof(VT)), DS = dia_split(A->dia.D);
-        const unsigned g = grid_cap((nr + 1024 / DS - 1) / (1024 / DS), dia_blocks_per_sm());
-#define NITRO_DIA_LAUNCH(UU, SS)                                                                                   \
-  k_dia<VT, UU, SS><<<g, 256, sm, s>>>(A->dia.off.as<int32_t>(), A->dia.val.as<VT>() + r0, x, y, N, A->M,         \
-                                       A->dia.D, A->dia.ld, nr, row0, A->dia.off_min, A->dia.off_max, x_al,      \
-                                       l2_evict_first(), part ? 0 : dia_prefetch(), prefetch_hint())
-#define NITRO_DIA_U(SS)                      \
-  switch (U) {                               \
-    case 2: NITRO_DIA_LAUNCH(2, SS); break;  \
-    case 4: NITRO_DIA_LAUNCH(4, SS); break;  \
-    default: NITRO_DIA_LAUNCH(1, SS); break; \
-  }
-        switch (DS) {
-          case 2: NITRO_DIA_U(2); break;
-          case 4: NITRO_DIA_U(4); break;
-          default: NITRO_DIA_U(1); break;
-        }
-#undef NITRO_DIA_U
-#undef NITRO_DIA_LAUNCH
+        const unsigned g = grid_cap((nr + 1023) / 1024, dia_blocks_per_sm());
+        k_dia<VT><<<g, 256, sm, s>>>(A->dia.off.as<int32_t>(), A->dia.val.as<VT>() + r0, x, y, N, A->M, A->dia.D,
+                                     A->dia.ld, nr, row0, A->dia.off_min, A->dia.off_max, x_al, l2_evict_first(),
+                                     part ? 0 : dia_prefetch(), prefetch_hint());
       }
       break;
     case NITRO_HYB:
@@ -1339,26 +1161,16 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
                        diag_local(A));
         if (A->hyb.Zt > 0) {
           const unsigned gt = grid_cap((A->hyb.nchunks + 7) / 8, 16);
-#define NITRO_TAIL(WW)                                                                                        \
-  k_hyb_tail<VT, WW><<<gt, 256, 0, s>>>(A->hyb.trow.as<int32_t>(), A->hyb.tcol.as<int32_t>(), A->hyb.tval.as<VT>(), \
-                                        x, y, A->hyb.Zt, A->hyb.nchunks, A->hyb.carry_row.as<int32_t>(),          \
-                                        A->hyb.carry_val.as<double>())
-#define NITRO_TAIL_LS(WW)                                                                                      \
-  k_hyb_tail_ls<VT, WW><<<gt, 256, 0, s>>>(A->hyb.trow.as<int32_t>(), A->hyb.tcol.as<int32_t>(),                \
-                                           A->hyb.tval.as<VT>(), x, y, A->hyb.Zt, A->hyb.nchunks,               \
-                                           A->hyb.carry_row.as<int32_t>(), A->hyb.carry_val.as<double>(),     \
-                                           l2_evict_first())
-          static const bool ls = [] {
-            const char *e = getenv("NITRO_HYB_LS");
-            return e ? atoi(e) != 0 : true;
-          }();
-          switch (A->hyb.W) {
-            case 2: NITRO_TAIL(2); break;
-            case 4: if (ls) NITRO_TAIL_LS(4); else NITRO_TAIL(4); break;
-            default: if (ls) NITRO_TAIL_LS(8); else NITRO_TAIL(8); break;
-          }
-#undef NITRO_TAIL_LS
-#undef NITRO_TAIL
+          if (A->hyb.W == 4)
+            k_hyb_tail_ls<VT, 4><<<gt, 256, 0, s>>>(A->hyb.trow.as<int32_t>(), A->hyb.tcol.as<int32_t>(),
+                                                   A->hyb.tval.as<VT>(), x, y, A->hyb.Zt, A->hyb.nchunks,
+                                                   A->hyb.carry_row.as<int32_t>(), A->hyb.carry_val.as<double>(),
+                                                   l2_evict_first());
+          else
+            k_hyb_tail_ls<VT, 8><<<gt, 256, 0, s>>>(A->hyb.trow.as<int32_t>(), A->hyb.tcol.as<int32_t>(),
+                                                   A->hyb.tval.as<VT>(), x, y, A->hyb.Zt, A->hyb.nchunks,
+                                                   A->hyb.carry_row.as<int32_t>(), A->hyb.carry_val.as<double>(),
+                                                   l2_evict_first());
           const unsigned nshort = grid_cap((A->hyb.fix_S + 255) / 256, 8);
           const unsigned nlong_blk =
               A->hyb.fix_nlong > 0 ? (unsigned)std::min<int64_t>((A->hyb.fix_nlong + 7) / 8, (int64_t)num_sms() * 4) : 0;

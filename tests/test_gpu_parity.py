@@ -607,3 +607,70 @@ def test_l2_prefetch_is_result_neutral(cuda, tmp_path):
     assert res["on"].keys() == res["off"].keys() and len(res["on"]) >= 6
     for k in res["on"]:
         assert np.array_equal(res["on"][k], res["off"][k]), k
+
+
+# ------------------------------------------------------------------ round-2 robustness cases
+def test_dia_more_diagonals_than_shared_offsets(cuda):
+    """D > 12288 (the offsets kept in shared memory): a dense 32 x 14000 block
+    has 14031 diagonals at fill 1.0, so DIA is allowed and must run correctly
+    (offsets past the shared window are read through L1)."""
+    n = nitro()
+    import torch
+    N, M = 32, 14000
+    rp = np.arange(N + 1, dtype=np.int64) * M
+    ci = np.tile(np.arange(M, dtype=np.int32), N)
+    rng = np.random.default_rng(5)
+    va = (rng.integers(1, 9, N * M) * rng.choice([-1, 1], N * M)).astype(np.float32)
+    A = Csr(N, M, rp, ci, va, False)
+    f = oracle.features(A)
+    assert f["ndiag"] == N + M - 1 and f["dia_fill"] <= 3.0
+    M_, _ = handle(A, cuda)
+    assert M_.allowed(n.DIA)
+    x = synth.vector(M, seed=1, mode=1)
+    y_ref, _ = oracle.spmv(A, x)
+    y = M_.run(n.DIA, torch.from_numpy(x).to(cuda))
+    torch.cuda.synchronize()
+    assert np.array_equal(y.cpu().numpy().astype(np.float64), y_ref)   # integer data: exact
+
+
+def test_malformed_rowptr_with_long_rows_is_rejected(cuda):
+    """Overlapping rows that each lie inside [0, Z] (rowptr not monotone) and
+    are long enough for the long-row task list must give NITRO_E_BAD_MATRIX,
+    not a write past the task list."""
+    n = nitro()
+    Z, N = 20000, 96
+    rp = np.zeros(N + 1, np.int64)
+    rp[1:32] = Z          # block 0: row 0 has Z entries, the rest are empty
+    rp[32] = Z
+    rp[33:64] = 0         # block 1: row 32 goes Z -> 0 (negative; flagged)
+    rp[64] = 0
+    rp[65:N] = Z          # block 2: row 64 again has Z entries
+    rp[N] = Z
+    ci = np.arange(Z, dtype=np.int32)
+    A = Csr(N, Z, rp, ci, np.ones(Z, np.float32), False)
+    M, _ = handle(A, cuda)
+    with pytest.raises(n.NitroError) as e:
+        M.features()
+    assert e.value.code == 2
+    import torch
+    torch.cuda.synchronize()            # no sticky CUDA error left behind
+    assert torch.ones(4, device=cuda).sum().item() == 4
+
+
+def test_binding_rejects_bad_vectors(cuda):
+    """The Python binding checks dtype / contiguity / length / device before
+    passing a pointer to the C ABI."""
+    n = nitro()
+    import torch
+    A = synth.stencil("2d5", 16)
+    M, _ = handle(A, cuda)
+    good = torch.zeros(A.cols, dtype=torch.float32, device=cuda)
+    for bad in (torch.zeros(A.cols, dtype=torch.float64, device=cuda),
+                torch.zeros(2 * A.cols, dtype=torch.float32, device=cuda)[::2],
+                torch.zeros(A.cols - 1, dtype=torch.float32, device=cuda),
+                torch.zeros(A.cols, dtype=torch.float32)):
+        with pytest.raises(ValueError):
+            M.run(n.CSR_SCALAR, bad)
+        with pytest.raises(ValueError):
+            M.run(n.CSR_SCALAR, good, bad[: A.rows] if bad.numel() >= A.rows else bad)
+    M.run(n.CSR_SCALAR, good)
