@@ -367,6 +367,12 @@ nitro_status_t nitro_dist_spmv_run(nitro_dist *D, nitro_spmv *A_local, int varia
  * into the next x), and to check every rank's part on one GPU. */
 nitro_status_t nitro_dist_spmv_run_gathered(nitro_dist *D, nitro_spmv *A_local, int variant,
                                             const void *d_x_gathered, void *d_y_local);
+/* Format facts of this rank's multiply (prepares the parts' formats):
+ * bytes / tail summed over the rank's row parts, width / ld their maximum,
+ * compulsory_bytes = the parts' matrix + y bytes (DESIGN.md §6 formulas) + the
+ * exchanged x layout read once.  A part whose constraint rules the variant
+ * out is counted with the default (CSR-vector), as nitro_dist_spmv_run runs it. */
+nitro_status_t nitro_dist_format_info(nitro_spmv *A_local, int variant, nitro_format_info *out);
 /* Padded block size B and this rank's [i0, i1) interior row run (rows that
  * read only local x and overlap the all-gather). */
 nitro_status_t nitro_dist_layout(nitro_spmv *A_local, int64_t *B, int64_t *i0, int64_t *i1);
@@ -374,9 +380,27 @@ nitro_status_t nitro_dist_layout(nitro_spmv *A_local, int64_t *B, int64_t *i0, i
  * calls works (partition, remap, parts, run_gathered); run/features with
  * nranks > 1 return NITRO_E_STATE.  For single-GPU checks of multi-rank logic. */
 nitro_status_t nitro_dist_init_local(int rank, int nranks, int device, nitro_dist **out);
-/* Global features from per-rank feature passes (sum / max all-reduce and a
- * union of diagonal offsets): identical to the single-GPU features. */
+/* Global features from per-rank feature passes: S1, S2 all-reduced (sum),
+ * Lmax and the non-canonical flag all-reduced (max), and D = |union of the
+ * ranks' occupied diagonals|, each rank contributing its compacted sorted
+ * offset list through one all-gather.  Identical (bit for bit)
+ * to the single-GPU features of the whole matrix.  Collective; syncs. */
 nitro_status_t nitro_dist_features(nitro_dist *D, nitro_spmv *A_local, nitro_spmv_feat *out);
+
+/* LOOPBACK transport: P rank handles inside ONE process on ONE GPU, each
+ * driven by its own host thread.  Every collective of nitro_dist_* (the
+ * exchange-plan all-gather and send/recv in create, the per-multiply x
+ * all-gather or halo send/recv, the feature reductions) meets at a host
+ * barrier and moves data with device copies ordered on the callers' streams
+ * — the same pack / send-list / receive-offset / layout code as NCCL, so the
+ * P > 1 paths run (and are tested) on a single GPU.  Each rank's thread calls
+ * nitro_dist_init_loopback(L, rank) and then the ordinary nitro_dist_* calls
+ * in the same order as the other ranks (as with NCCL).  The group object must
+ * outlive its rank handles. */
+typedef struct nitro_loopback nitro_loopback;
+nitro_status_t nitro_dist_loopback_create(int nranks, int device, nitro_loopback **out);
+void nitro_dist_loopback_destroy(nitro_loopback *L);
+nitro_status_t nitro_dist_init_loopback(nitro_loopback *L, int rank, nitro_dist **out);
 
 /* ========================================================================
  * 4. Histogram code-variant family: a second workload

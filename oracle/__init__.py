@@ -35,8 +35,8 @@ _SRC = os.path.join(_HERE, "oracle.c")
 def build(force: bool = False) -> str:
     if not force and os.path.exists(_SO) and os.path.getmtime(_SO) >= os.path.getmtime(_SRC):
         return _SO
-    subprocess.check_call(["gcc", "-O2", "-std=c11", "-ffp-contract=off", "-fno-fast-math", "-shared", "-fPIC",
-                           "-o", _SO, _SRC, "-lm"], cwd=_HERE)
+    subprocess.check_call(["gcc", "-O2", "-std=c11", "-ffp-contract=off", "-fno-fast-math", "-fopenmp", "-shared",
+                           "-fPIC", "-o", _SO, _SRC, "-lm"], cwd=_HERE)
     return _SO
 
 
@@ -63,6 +63,8 @@ def lib():
         vp, i64 = ctypes.c_void_p, ctypes.c_int64
         L.oracle_spmv.argtypes = [i64, vp, vp, vp, vp, vp, vp]
         L.oracle_spmv.restype = None
+        L.oracle_spmv_threads.argtypes = [i64, vp, vp, vp, vp, vp, vp, ctypes.c_int]
+        L.oracle_spmv_threads.restype = ctypes.c_int
         L.oracle_features.argtypes = [i64, i64, vp, vp, ctypes.POINTER(Features), vp]
         L.oracle_is_canonical.argtypes = [i64, i64, i64, vp, vp]
         L.oracle_finish_features.argtypes = [i64, i64, i64, ctypes.c_uint64, ctypes.c_uint64, i64, i64,
@@ -113,6 +115,19 @@ def spmv(A, x):
     r = np.empty(N, dtype=np.float64)
     lib().oracle_spmv(N, _p(rp), _p(ci), _p(v), _p(xd), _p(y), _p(r))
     return y, r
+
+
+def spmv_threads(A, x, nthreads: int | None = None):
+    """C1 with the rows split over host threads (bit-identical to spmv);
+    returns (y, r, threads used).  bench.py's all-core CPU baseline only."""
+    N, M, rp, ci, v = _csr(A)
+    xd = np.ascontiguousarray(np.asarray(x), dtype=np.float64)
+    assert xd.shape[0] >= M
+    y = np.empty(N, dtype=np.float64)
+    r = np.empty(N, dtype=np.float64)
+    used = lib().oracle_spmv_threads(N, _p(rp), _p(ci), _p(v), _p(xd), _p(y), _p(r),
+                                     int(nthreads or os.cpu_count() or 1))
+    return y, r, used
 
 
 def features(A, with_offsets: bool = False):

@@ -14,6 +14,7 @@
  * silent (also listed in DESIGN.md "Readings").
  */
 #include <math.h>
+#include <omp.h>
 #include <stdint.h>
 #include <stdlib.h>
 #include <string.h>
@@ -35,6 +36,33 @@ void oracle_spmv(int64_t N, const int64_t *rowptr, const int32_t *col, const dou
     y[i] = s;
     if (r) r[i] = a;
   }
+}
+
+/* The same loop with the rows split over host threads (OpenMP, static
+ * schedule): every row is still summed sequentially in storage order, so y and
+ * r are bit-identical to oracle_spmv.  Used only by bench.py's all-core CPU
+ * baseline leg (the north star asks for the oracle timed on the box's host
+ * cores).  Returns the number of threads that ran. */
+int oracle_spmv_threads(int64_t N, const int64_t *rowptr, const int32_t *col, const double *val,
+                        const double *x, double *y, double *r, int nthreads) {
+  int used = 1;
+#pragma omp parallel num_threads(nthreads > 0 ? nthreads : 1)
+  {
+#pragma omp single
+    used = omp_get_num_threads();
+#pragma omp for schedule(static)
+    for (int64_t i = 0; i < N; ++i) {
+      double s = 0.0, a = 0.0;
+      for (int64_t k = rowptr[i]; k < rowptr[i + 1]; ++k) {
+        double p = val[k] * x[col[k]];
+        s = s + p;
+        a = a + fabs(p);
+      }
+      y[i] = s;
+      if (r) r[i] = a;
+    }
+  }
+  return used;
 }
 
 /* ------------------------------------------------------------------ C4 features

@@ -176,6 +176,10 @@ _SIGS = {
     "nitro_dist_spmv_run_gathered": ([_vp, _vp, _int, _vp, _vp], _int),
     "nitro_dist_layout": ([_vp, _P(_i64), _P(_i64), _P(_i64)], _int),
     "nitro_dist_init_local": ([_int, _int, _int, _P(_vp)], _int),
+    "nitro_dist_loopback_create": ([_int, _int, _P(_vp)], _int),
+    "nitro_dist_format_info": ([_vp, _int, _P(FormatInfo)], _int),
+    "nitro_dist_loopback_destroy": ([_vp], None),
+    "nitro_dist_init_loopback": ([_vp, _int, _P(_vp)], _int),
     "nitro_dist_spmv_create_ex": ([_vp, _i64, _vp, _i64, _vp, _int, _vp, _vp, _int, _int, _P(_vp)], _int),
     "nitro_dist_exchange_info": ([_vp, _P(_int), _P(_i64), _P(_i64), _P(_i64)], _int),
     "nitro_dist_halo_cols": ([_vp, _vp], _int),
@@ -698,15 +702,40 @@ def dist_unique_id() -> bytes:
     return buf.raw
 
 
+class Loopback:
+    """A loopback transport group (nitro_dist_loopback_create): P ranks in one
+    process on one GPU, one host thread per rank (``Dist.loopback``)."""
+
+    def __init__(self, nranks: int, device: int = 0):
+        h = ctypes.c_void_p()
+        _check(_L.nitro_dist_loopback_create(int(nranks), int(device), ctypes.byref(h)))
+        self.h, self.nranks, self.device = h, int(nranks), int(device)
+
+    def close(self):
+        if getattr(self, "h", None):
+            _L.nitro_dist_loopback_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
 class Dist:
     """One rank of the row-partitioned multi-GPU SpMV (NCCL communicator).
 
     ``Dist.local(rank, nranks, device)`` builds a communicator-less handle whose
-    ``run_gathered`` computes that rank's rows from an already gathered x."""
+    ``run_gathered`` computes that rank's rows from an already gathered x;
+    ``Dist.loopback(group, rank)`` a rank of a single-GPU loopback group."""
 
-    def __init__(self, uid: bytes | None, rank: int, nranks: int, device: int):
+    def __init__(self, uid: bytes | None, rank: int, nranks: int, device: int, loopback: "Loopback | None" = None):
         h = ctypes.c_void_p()
-        if uid is None:
+        self._group = loopback
+        if loopback is not None:
+            _check(_L.nitro_dist_init_loopback(loopback.h, rank, ctypes.byref(h)))
+        elif uid is None:
             _check(_L.nitro_dist_init_local(rank, nranks, device, ctypes.byref(h)))
         else:
             buf = ctypes.create_string_buffer(uid, 128)
@@ -716,6 +745,10 @@ class Dist:
     @classmethod
     def local(cls, rank: int, nranks: int, device: int = 0):
         return cls(None, rank, nranks, device)
+
+    @classmethod
+    def loopback(cls, group: Loopback, rank: int):
+        return cls(None, rank, group.nranks, group.device, loopback=group)
 
     def run_gathered(self, A: "SpMV", v: int, x_gathered, y_local):
         _check(_L.nitro_dist_spmv_run_gathered(self.h, A.h, v, _ptr(x_gathered), _ptr(y_local)))
@@ -743,6 +776,13 @@ class Dist:
         p = ctypes.c_void_p()
         _check(_L.nitro_dist_x_local(A.h, ctypes.byref(p)))
         return _wrap_device(p.value, A.rows, A.dtype, A.device)
+
+    @staticmethod
+    def format_info(A: "SpMV", v: int) -> dict:
+        """nitro_dist_format_info: this rank's multiply (all row parts + the exchanged x)."""
+        fi = FormatInfo()
+        _check(_L.nitro_dist_format_info(A.h, v, ctypes.byref(fi)))
+        return fi.as_dict()
 
     @staticmethod
     def layout(A: "SpMV"):

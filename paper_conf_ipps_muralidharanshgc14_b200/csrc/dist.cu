@@ -17,20 +17,70 @@
 // is an ordinary nitro_spmv over a rebased CSR slice, so every variant (and
 // its constraint) works unchanged.  Global features: per-rank K1 over a
 // global-offset bitmap, integer moments all-reduced (sum / max), occupied
-// diagonals unioned (max over u8 flags).
+// diagonals as each rank's compacted sorted offset list, all-gathered and
+// unioned.
+//
+// Transport: every exchange goes through four operations (all-gather,
+// u64 all-reduce, grouped send/recv) implemented either with NCCL (one
+// process per GPU) or with the LOOPBACK transport: P rank handles of one
+// process on one GPU (one host thread each) whose collectives meet at a host
+// barrier and move data with stream-ordered device copies.  The loopback runs
+// the same pack / send-list / receive-offset / layout code as NCCL for any P
+// on a single GPU, so the P > 1 paths are testable without a second device.
 #include <nccl.h>
 
 #include <algorithm>
+#include <condition_variable>
+#include <mutex>
 #include <vector>
 
 #include "nitro_internal.h"
 #include "util.cuh"
 
+namespace {
+struct Msg {
+  int peer;
+  const void *src;  // send: source; recv: unused
+  void *dst;        // recv: destination; send: unused
+  size_t bytes;
+};
+}  // namespace
+
+struct nitro_loopback {
+  int nranks = 1, device = 0;
+  std::mutex mu;
+  std::condition_variable cv;
+  int arrived = 0;
+  uint64_t gen = 0;
+  struct Slot {
+    const void *send = nullptr;
+    void *recv = nullptr;
+    size_t bytes = 0;
+    cudaEvent_t ready = nullptr, done = nullptr;
+    std::vector<Msg> sends;
+    std::vector<unsigned long long> host;
+  };
+  std::vector<Slot> slot;
+  void barrier() {
+    std::unique_lock<std::mutex> lk(mu);
+    const uint64_t g = gen;
+    if (++arrived == nranks) {
+      arrived = 0;
+      ++gen;
+      cv.notify_all();
+    } else {
+      cv.wait(lk, [&] { return gen != g; });
+    }
+  }
+};
+
 struct nitro_dist {
   ncclComm_t comm = nullptr;
+  nitro_loopback *lb = nullptr;  // loopback transport (one process, one GPU)
   int rank = 0, nranks = 1, device = 0;
   cudaStream_t comm_stream = nullptr;
   cudaEvent_t ev_x = nullptr, ev_g = nullptr;
+  bool has_transport() const { return comm != nullptr || lb != nullptr; }
 };
 
 namespace nitro {
@@ -41,6 +91,100 @@ namespace {
     ncclResult_t r_ = (call);                                                                                    \
     if (r_ != ncclSuccess) return fail(NITRO_E_NCCL, std::string("NCCL: ") + ncclGetErrorString(r_) + " at " #call); \
   } while (0)
+
+// ---------------------------------------------------------------- transport
+// All four are collective: every rank of the handle's group calls them in the
+// same order.  Work is ordered on stream s.
+nitro_status_t t_allgather(nitro_dist *D, const void *send, void *recv, size_t bytes, cudaStream_t s) {
+  if (D->nranks == 1) {
+    if (send != recv && bytes) NITRO_CUDA(cudaMemcpyAsync(recv, send, bytes, cudaMemcpyDeviceToDevice, s));
+    return NITRO_OK;
+  }
+  if (D->comm) {
+    NITRO_NCCL(ncclAllGather(send, recv, bytes, ncclInt8, D->comm, s));
+    return NITRO_OK;
+  }
+  nitro_loopback *L = D->lb;
+  auto &me = L->slot[D->rank];
+  me.send = send;
+  me.recv = recv;
+  me.bytes = bytes;
+  NITRO_CUDA(cudaEventRecord(me.ready, s));
+  L->barrier();
+  char *rb = (char *)recv;
+  for (int q = 0; q < D->nranks; ++q) {
+    const void *src = q == D->rank ? send : L->slot[q].send;
+    char *dst = rb + (size_t)q * bytes;
+    if (q != D->rank) NITRO_CUDA(cudaStreamWaitEvent(s, L->slot[q].ready, 0));
+    if (src != dst && bytes) NITRO_CUDA(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDeviceToDevice, s));
+  }
+  NITRO_CUDA(cudaEventRecord(me.done, s));
+  L->barrier();
+  for (int q = 0; q < D->nranks; ++q)  // nobody reuses its send buffer before every copy of it is done
+    if (q != D->rank) NITRO_CUDA(cudaStreamWaitEvent(s, L->slot[q].done, 0));
+  L->barrier();  // slots may be re-posted
+  return NITRO_OK;
+}
+
+// in-place u64 all-reduce (sum or max) of a small device array; syncs s
+nitro_status_t t_allreduce_u64(nitro_dist *D, unsigned long long *dbuf, int n, bool is_max, cudaStream_t s) {
+  if (D->nranks == 1) return NITRO_OK;
+  if (D->comm) {
+    NITRO_NCCL(ncclAllReduce(dbuf, dbuf, n, ncclUint64, is_max ? ncclMax : ncclSum, D->comm, s));
+    NITRO_CUDA(cudaStreamSynchronize(s));
+    return NITRO_OK;
+  }
+  nitro_loopback *L = D->lb;
+  auto &me = L->slot[D->rank];
+  me.host.assign(n, 0ull);
+  NITRO_CUDA(cudaMemcpyAsync(me.host.data(), dbuf, (size_t)n * 8, cudaMemcpyDeviceToHost, s));
+  NITRO_CUDA(cudaStreamSynchronize(s));
+  L->barrier();
+  std::vector<unsigned long long> r(L->slot[0].host);
+  for (int q = 1; q < D->nranks; ++q)
+    for (int i = 0; i < n; ++i) r[i] = is_max ? std::max(r[i], L->slot[q].host[i]) : r[i] + L->slot[q].host[i];
+  L->barrier();
+  NITRO_CUDA(cudaMemcpyAsync(dbuf, r.data(), (size_t)n * 8, cudaMemcpyHostToDevice, s));
+  NITRO_CUDA(cudaStreamSynchronize(s));
+  return NITRO_OK;
+}
+
+// grouped point-to-point: the k-th send to q pairs with q's k-th receive from me
+nitro_status_t t_sendrecv(nitro_dist *D, const std::vector<Msg> &sends, const std::vector<Msg> &recvs,
+                          cudaStream_t s) {
+  if (D->nranks == 1) return NITRO_OK;
+  if (D->comm) {
+    NITRO_NCCL(ncclGroupStart());
+    for (const Msg &m : sends)
+      if (m.bytes) NITRO_NCCL(ncclSend(m.src, m.bytes, ncclInt8, m.peer, D->comm, s));
+    for (const Msg &m : recvs)
+      if (m.bytes) NITRO_NCCL(ncclRecv(m.dst, m.bytes, ncclInt8, m.peer, D->comm, s));
+    NITRO_NCCL(ncclGroupEnd());
+    return NITRO_OK;
+  }
+  nitro_loopback *L = D->lb;
+  auto &me = L->slot[D->rank];
+  me.sends = sends;
+  NITRO_CUDA(cudaEventRecord(me.ready, s));
+  L->barrier();
+  std::vector<int> used(D->nranks, 0);
+  for (const Msg &m : recvs) {
+    const auto &ps = L->slot[m.peer].sends;
+    int k = used[m.peer]++, seen = 0;
+    const Msg *src = nullptr;
+    for (const Msg &t : ps)
+      if (t.peer == D->rank && seen++ == k) { src = &t; break; }
+    if (!src || src->bytes != m.bytes) return fail(NITRO_E_STATE, "loopback send/recv mismatch");
+    NITRO_CUDA(cudaStreamWaitEvent(s, L->slot[m.peer].ready, 0));
+    if (m.bytes) NITRO_CUDA(cudaMemcpyAsync(m.dst, src->src, m.bytes, cudaMemcpyDeviceToDevice, s));
+  }
+  NITRO_CUDA(cudaEventRecord(me.done, s));
+  L->barrier();
+  for (int q = 0; q < D->nranks; ++q)
+    if (q != D->rank) NITRO_CUDA(cudaStreamWaitEvent(s, L->slot[q].done, 0));
+  L->barrier();
+  return NITRO_OK;
+}
 
 enum { kAllGather = 0, kHalo = 1 };
 
@@ -179,17 +323,19 @@ __global__ void k_pack(const VT *__restrict__ xl, const int32_t *__restrict__ id
     out[i] = xl[idx[i]];
 }
 
-__global__ void k_bits_to_flags(const uint32_t *__restrict__ bm, int64_t nbits, uint8_t *__restrict__ f) {
-  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < nbits; t += (int64_t)gridDim.x * blockDim.x)
-    f[t] = (bm[t >> 5] >> (t & 31)) & 1u;
+__global__ void k_set_bits(const int32_t *__restrict__ idx, int64_t n, uint32_t *__restrict__ bm) {
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < n; t += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t i = (uint32_t)idx[t];
+    atomicOr(bm + (i >> 5), 1u << (i & 31));
+  }
 }
-__global__ void k_count_flags(const uint8_t *__restrict__ f, int64_t n, unsigned long long *out) {
-  unsigned long long s = 0;
-  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < n; t += (int64_t)gridDim.x * blockDim.x)
-    s += f[t] != 0;
+__global__ void k_popc_sum(const uint32_t *__restrict__ bm, int64_t nwords, unsigned long long *out) {
+  unsigned long long c = 0;
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < nwords; t += (int64_t)gridDim.x * blockDim.x)
+    c += __popc(bm[t]);
 #pragma unroll
-  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-  if ((threadIdx.x & 31) == 0 && s) atomicAdd(out, s);
+  for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+  if ((threadIdx.x & 31) == 0 && c) atomicAdd(out, c);
 }
 __global__ void k_pack_acc(const FeatAcc *a, unsigned long long *sum2, unsigned long long *max2) {
   sum2[0] = a->s1; sum2[1] = a->s2; max2[0] = a->lmax; max2[1] = a->bad;
@@ -232,29 +378,29 @@ nitro_status_t halo_plan(DistState *st) {
   st->nb = st->recv_off[me];  // halo entries owned by lower ranks (columns < lo)
   st->send_off.assign(P + 1, 0);
   st->ns = 0;
-  if (!D->comm || P == 1) return NITRO_OK;  // communicator-less: the caller supplies the layout
+  if (!D->has_transport() || P == 1) return NITRO_OK;  // communicator-less: the caller supplies the layout
   // need matrix: row r = counts rank r receives from each owner
   DevBuf need;
   NITRO_TRY(need.alloc((size_t)P * P * 8));
   std::vector<int64_t> mine(P), all((size_t)P * P);
   for (int q = 0; q < P; ++q) mine[q] = st->recv_off[q + 1] - st->recv_off[q];
   NITRO_CUDA(cudaMemcpy(need.as<int64_t>() + (size_t)me * P, mine.data(), P * 8, cudaMemcpyHostToDevice));
-  NITRO_NCCL(ncclAllGather(need.as<int64_t>() + (size_t)me * P, need.p, P, ncclInt64, D->comm, D->comm_stream));
+  NITRO_TRY(t_allgather(D, need.as<int64_t>() + (size_t)me * P, need.p, (size_t)P * 8, D->comm_stream));
   NITRO_CUDA(cudaStreamSynchronize(D->comm_stream));
   NITRO_CUDA(cudaMemcpy(all.data(), need.p, (size_t)P * P * 8, cudaMemcpyDeviceToHost));
   for (int r = 0; r < P; ++r) st->send_off[r + 1] = st->send_off[r] + all[(size_t)r * P + me];
   st->ns = st->send_off[P];
   NITRO_TRY(st->send_idx.alloc((size_t)std::max<int64_t>(st->ns, 1) * 4));
   // requesters send me the global ids they need from me
-  NITRO_NCCL(ncclGroupStart());
+  std::vector<Msg> sends, recvs;
   for (int q = 0; q < P; ++q) {
     if (q == me) continue;
     const int64_t rc = st->recv_off[q + 1] - st->recv_off[q];
     const int64_t sc = st->send_off[q + 1] - st->send_off[q];
-    if (rc > 0) NITRO_NCCL(ncclSend(st->halo_cols.as<int32_t>() + st->recv_off[q], rc, ncclInt32, q, D->comm, D->comm_stream));
-    if (sc > 0) NITRO_NCCL(ncclRecv(st->send_idx.as<int32_t>() + st->send_off[q], sc, ncclInt32, q, D->comm, D->comm_stream));
+    if (rc > 0) sends.push_back({q, st->halo_cols.as<int32_t>() + st->recv_off[q], nullptr, (size_t)rc * 4});
+    if (sc > 0) recvs.push_back({q, nullptr, st->send_idx.as<int32_t>() + st->send_off[q], (size_t)sc * 4});
   }
-  NITRO_NCCL(ncclGroupEnd());
+  NITRO_TRY(t_sendrecv(D, sends, recvs, D->comm_stream));
   NITRO_CUDA(cudaStreamSynchronize(D->comm_stream));
   if (st->ns > 0) k_to_local<<<grid_n(st->ns), 256>>>(st->send_idx.as<int32_t>(), st->ns, st->bounds[me]);
   NITRO_CUDA(cudaDeviceSynchronize());
@@ -376,12 +522,11 @@ nitro_status_t nitro_dist_spmv_create_ex(nitro_dist *D, int64_t global_rows, con
     // ---- exchange mode: halo when the largest halo is < 1/4 of the all-gather volume
     if ((rc = halo_list(st, d_colidx, local_nnz, st->halo_cols, st->nh))) return bail(rc);
     int64_t max_nh = st->nh;
-    if (D->comm && P > 1) {
+    if (D->has_transport() && P > 1) {
       DevBuf t;
       if ((rc = t.alloc(8))) return bail(rc);
       NITRO_CUDA(cudaMemcpy(t.p, &max_nh, 8, cudaMemcpyHostToDevice));
-      NITRO_NCCL(ncclAllReduce(t.p, t.p, 1, ncclInt64, ncclMax, D->comm, D->comm_stream));
-      NITRO_CUDA(cudaStreamSynchronize(D->comm_stream));
+      if ((rc = t_allreduce_u64(D, t.as<unsigned long long>(), 1, true, D->comm_stream))) return bail(rc);
       NITRO_CUDA(cudaMemcpy(&max_nh, t.p, 8, cudaMemcpyDeviceToHost));
     }
     st->mode = exchange == -1 ? (4 * max_nh < (int64_t)(P - 1) * st->B || P == 1 ? kHalo : kAllGather) : exchange;
@@ -487,7 +632,7 @@ nitro_status_t nitro_dist_spmv_create(nitro_dist *D, int64_t global_rows, const 
 nitro_status_t nitro_dist_spmv_run(nitro_dist *D, nitro_spmv *A, int variant, const void *d_x_local, void *d_y_local) {
   if (!D || !A || !A->dist_state || variant < 0 || variant >= NITRO_NUM_VARIANTS)
     return fail(NITRO_E_INVALID_ARG, "bad argument");
-  if (!D->comm && D->nranks > 1) return fail(NITRO_E_STATE, "communicator-less handle: use run_gathered");
+  if (!D->has_transport() && D->nranks > 1) return fail(NITRO_E_STATE, "communicator-less handle: use run_gathered");
   DistState *st = (DistState *)A->dist_state;
   NITRO_CUDA(cudaSetDevice(D->device));
   const size_t sv = A->fp64 ? 8 : 4;
@@ -496,7 +641,6 @@ nitro_status_t nitro_dist_spmv_run(nitro_dist *D, nitro_spmv *A, int variant, co
   char *mine = xb + (size_t)st->x_offset() * sv;
   if (st->n > 0 && d_x_local != mine)  // callers that write x in place (nitro_dist_x_local) skip this copy
     NITRO_CUDA(cudaMemcpyAsync(mine, d_x_local, st->n * sv, cudaMemcpyDeviceToDevice, s));
-  const ncclDataType_t dt = A->fp64 ? ncclFloat64 : ncclFloat32;
   if (st->mode == kHalo && st->ns > 0) {
     if (A->fp64) k_pack<double><<<grid_n(st->ns), 256, 0, s>>>((const double *)mine, st->send_idx.as<int32_t>(), st->ns, st->sendbuf.as<double>());
     else k_pack<float><<<grid_n(st->ns), 256, 0, s>>>((const float *)mine, st->send_idx.as<int32_t>(), st->ns, st->sendbuf.as<float>());
@@ -506,17 +650,16 @@ nitro_status_t nitro_dist_spmv_run(nitro_dist *D, nitro_spmv *A, int variant, co
   NITRO_CUDA(cudaStreamWaitEvent(D->comm_stream, D->ev_x, 0));
   if (D->nranks > 1) {
     if (st->mode == kAllGather) {
-      NITRO_NCCL(ncclAllGather(mine, xb, (size_t)st->B, dt, D->comm, D->comm_stream));
+      NITRO_TRY(t_allgather(D, mine, xb, (size_t)st->B * sv, D->comm_stream));
     } else {
-      NITRO_NCCL(ncclGroupStart());
+      std::vector<Msg> sends, recvs;
       for (int q = 0; q < D->nranks; ++q) {
         if (q == D->rank) continue;
         const int64_t sc = st->send_off[q + 1] - st->send_off[q], rc = st->recv_off[q + 1] - st->recv_off[q];
-        if (sc > 0) NITRO_NCCL(ncclSend(st->sendbuf.as<char>() + (size_t)st->send_off[q] * sv, sc, dt, q, D->comm, D->comm_stream));
-        if (rc > 0)
-          NITRO_NCCL(ncclRecv(xb + (size_t)st->halo_dest(st->recv_off[q]) * sv, rc, dt, q, D->comm, D->comm_stream));
+        if (sc > 0) sends.push_back({q, st->sendbuf.as<char>() + (size_t)st->send_off[q] * sv, nullptr, (size_t)sc * sv});
+        if (rc > 0) recvs.push_back({q, nullptr, xb + (size_t)st->halo_dest(st->recv_off[q]) * sv, (size_t)rc * sv});
       }
-      NITRO_NCCL(ncclGroupEnd());
+      NITRO_TRY(t_sendrecv(D, sends, recvs, D->comm_stream));
     }
   }
   NITRO_CUDA(cudaEventRecord(D->ev_g, D->comm_stream));
@@ -535,6 +678,30 @@ nitro_status_t nitro_dist_spmv_run_gathered(nitro_dist *D, nitro_spmv *A, int va
   NITRO_CUDA(cudaSetDevice(D->device));
   const size_t sv = A->fp64 ? 8 : 4;
   for (int k = 0; k < 3; ++k) NITRO_TRY(run_part(st, k, variant, A->stream, d_xg, d_y_local, sv));
+  return NITRO_OK;
+}
+
+nitro_status_t nitro_dist_format_info(nitro_spmv *A, int variant, nitro_format_info *out) {
+  if (!A || !A->dist_state || !out || variant < 0 || variant >= NITRO_NUM_VARIANTS)
+    return fail(NITRO_E_INVALID_ARG, "bad argument");
+  DistState *st = (DistState *)A->dist_state;
+  const double sv = A->fp64 ? 8 : 4;
+  memset(out, 0, sizeof(*out));
+  double cb = (double)st->layout_len() * sv;  // the exchanged x layout, read once
+  for (nitro_spmv *P : st->part) {
+    if (!P) continue;
+    int ok = 0, v = variant;
+    NITRO_TRY(nitro_spmv_allowed(P, v, &ok));
+    if (!ok) v = NITRO_CSR_VECTOR;  // as run_part
+    nitro_format_info fi;
+    NITRO_TRY(nitro_spmv_format_info(P, v, &fi));
+    cb += fi.compulsory_bytes - (double)P->M * sv;  // each part's matrix + y bytes
+    out->bytes += fi.bytes;
+    out->tail += fi.tail;
+    out->width = std::max(out->width, fi.width);
+    out->ld = std::max(out->ld, fi.ld);
+  }
+  out->compulsory_bytes = cb;
   return NITRO_OK;
 }
 
@@ -574,12 +741,13 @@ nitro_status_t nitro_dist_x_local(nitro_spmv *A, void **ptr) {
 
 nitro_status_t nitro_dist_features(nitro_dist *D, nitro_spmv *A, nitro_spmv_feat *out) {
   if (!D || !A || !A->dist_state || !out) return fail(NITRO_E_INVALID_ARG, "bad argument");
-  if (!D->comm && D->nranks > 1) return fail(NITRO_E_STATE, "communicator-less handle");
+  if (!D->has_transport() && D->nranks > 1) return fail(NITRO_E_STATE, "communicator-less handle");
   DistState *st = (DistState *)A->dist_state;
   NITRO_CUDA(cudaSetDevice(D->device));
   nitro_spmv *F = st->feat;
   F->stream = A->stream;
   cudaStream_t s = A->stream;
+  const int P = D->nranks;
   if (!F->feat_pending && !F->feat_ready) NITRO_TRY(features_launch(F));
   NITRO_CUDA(cudaEventSynchronize(F->feat_done));
   // integer moments: sum (s1, s2), max (lmax, bad)
@@ -587,29 +755,94 @@ nitro_status_t nitro_dist_features(nitro_dist *D, nitro_spmv *A, nitro_spmv_feat
   NITRO_TRY(red.alloc(5 * 8));
   unsigned long long *sum2 = red.as<unsigned long long>(), *max2 = sum2 + 2, *dcnt = sum2 + 4;
   k_pack_acc<<<1, 1, 0, s>>>(F->feat_acc.as<FeatAcc>(), sum2, max2);
-  // occupied diagonals: union of the per-rank bitmaps over the global offset range
-  const int64_t span = st->global_rows > 0 ? st->global_rows - 1 + F->M : 0;
-  NITRO_TRY(st->flags.alloc(std::max<int64_t>(span, 1)));
-  if (span > 0 && F->N > 0)
-    k_bits_to_flags<<<grid_n(span), 256, 0, s>>>(F->bitmap.as<uint32_t>(), span, st->flags.as<uint8_t>());
-  else if (span > 0)
-    NITRO_CUDA(cudaMemsetAsync(st->flags.p, 0, span, s));  // empty block: contributes no diagonal
   NITRO_CUDA(cudaGetLastError());
-  if (D->nranks > 1) {
-    NITRO_NCCL(ncclGroupStart());
-    NITRO_NCCL(ncclAllReduce(sum2, sum2, 2, ncclUint64, ncclSum, D->comm, s));
-    NITRO_NCCL(ncclAllReduce(max2, max2, 2, ncclUint64, ncclMax, D->comm, s));
-    if (span > 0) NITRO_NCCL(ncclAllReduce(st->flags.p, st->flags.p, span, ncclUint8, ncclMax, D->comm, s));
-    NITRO_NCCL(ncclGroupEnd());
+  NITRO_TRY(t_allreduce_u64(D, sum2, 2, false, s));
+  NITRO_TRY(t_allreduce_u64(D, max2, 2, true, s));
+  // occupied diagonals: this rank's sorted distinct offsets,
+  // compacted from its bitmap over the global offset range [0, span), are
+  // all-gathered (padded to the largest count) and unioned into one bitmap
+  const int64_t span = st->global_rows > 0 ? st->global_rows - 1 + F->M : 0;
+  const int64_t nwords = (span + 31) / 32, nt = (nwords + 1023) / 1024;
+  int64_t cnt = 0;
+  DevBuf tiles, scratch, mylist;
+  if (nt > 0 && F->N > 0) {
+    NITRO_TRY(tiles.alloc((size_t)(2 * nt + 2) * 8));
+    int64_t *tc = tiles.as<int64_t>(), *to = tc + nt + 1;
+    k_bm_tile_counts<<<(unsigned)nt, 256, 0, s>>>(F->bitmap.as<uint32_t>(), nwords, tc);
+    NITRO_TRY(exclusive_scan_i64(tc, to, nt, scratch, s));
+    NITRO_CUDA(cudaMemcpyAsync(&cnt, to + nt, 8, cudaMemcpyDeviceToHost, s));
+    NITRO_CUDA(cudaStreamSynchronize(s));
+    NITRO_TRY(mylist.alloc((size_t)std::max<int64_t>(cnt, 1) * 4));
+    if (cnt > 0) k_bm_emit<<<(unsigned)nt, 256, 0, s>>>(F->bitmap.as<uint32_t>(), nwords, to, mylist.as<int32_t>());
+    NITRO_CUDA(cudaGetLastError());
   }
-  NITRO_CUDA(cudaMemsetAsync(dcnt, 0, 8, s));
-  if (span > 0) k_count_flags<<<grid_n(span), 256, 0, s>>>(st->flags.as<uint8_t>(), span, dcnt);
-  unsigned long long h[5];
-  NITRO_CUDA(cudaMemcpyAsync(h, sum2, 5 * 8, cudaMemcpyDeviceToHost, s));
+  DevBuf counts;
+  NITRO_TRY(counts.alloc((size_t)P * 8));
+  NITRO_CUDA(cudaMemcpyAsync(counts.as<int64_t>() + D->rank, &cnt, 8, cudaMemcpyHostToDevice, s));
+  NITRO_TRY(t_allgather(D, counts.as<int64_t>() + D->rank, counts.p, 8, s));
+  std::vector<int64_t> hc(P);
+  NITRO_CUDA(cudaMemcpyAsync(hc.data(), counts.p, (size_t)P * 8, cudaMemcpyDeviceToHost, s));
   NITRO_CUDA(cudaStreamSynchronize(s));
-  finish_features(st->global_rows, F->M, (int64_t)h[0], h[0], h[1], (int64_t)h[2], (int64_t)h[4], out);
-  out->canonical = h[3] == 0;
+  const int64_t maxc = *std::max_element(hc.begin(), hc.end());
+  NITRO_CUDA(cudaMemsetAsync(dcnt, 0, 8, s));
+  if (maxc > 0) {
+    DevBuf all, bm;
+    NITRO_TRY(all.alloc((size_t)P * maxc * 4));
+    int32_t *mine = all.as<int32_t>() + (size_t)D->rank * maxc;
+    if (cnt > 0) NITRO_CUDA(cudaMemcpyAsync(mine, mylist.p, (size_t)cnt * 4, cudaMemcpyDeviceToDevice, s));
+    NITRO_TRY(t_allgather(D, mine, all.p, (size_t)maxc * 4, s));
+    NITRO_TRY(bm.alloc((size_t)nwords * 4));
+    NITRO_CUDA(cudaMemsetAsync(bm.p, 0, (size_t)nwords * 4, s));
+    for (int q = 0; q < P; ++q)
+      if (hc[q] > 0)
+        k_set_bits<<<grid_n(hc[q]), 256, 0, s>>>(all.as<int32_t>() + (size_t)q * maxc, hc[q], bm.as<uint32_t>());
+    k_popc_sum<<<grid_n(nwords), 256, 0, s>>>(bm.as<uint32_t>(), nwords, dcnt);
+    NITRO_CUDA(cudaGetLastError());
+    unsigned long long h[5];
+    NITRO_CUDA(cudaMemcpyAsync(h, sum2, 5 * 8, cudaMemcpyDeviceToHost, s));
+    NITRO_CUDA(cudaStreamSynchronize(s));
+    finish_features(st->global_rows, F->M, (int64_t)h[0], h[0], h[1], (int64_t)h[2], (int64_t)h[4], out);
+    out->canonical = h[3] == 0;
+  } else {
+    unsigned long long h[5];
+    NITRO_CUDA(cudaMemcpyAsync(h, sum2, 5 * 8, cudaMemcpyDeviceToHost, s));
+    NITRO_CUDA(cudaStreamSynchronize(s));
+    finish_features(st->global_rows, F->M, (int64_t)h[0], h[0], h[1], (int64_t)h[2], 0, out);
+    out->canonical = h[3] == 0;
+  }
   return out->canonical ? NITRO_OK : fail(NITRO_E_BAD_MATRIX, "non-canonical CSR on some rank");
+}
+
+nitro_status_t nitro_dist_loopback_create(int nranks, int device, nitro_loopback **out) {
+  if (!out || nranks < 1) return fail(NITRO_E_INVALID_ARG, "bad argument");
+  NITRO_CUDA(cudaSetDevice(device));
+  nitro_loopback *L = new nitro_loopback();
+  L->nranks = nranks;
+  L->device = device;
+  L->slot.resize(nranks);
+  for (auto &sl : L->slot) {
+    NITRO_CUDA(cudaEventCreateWithFlags(&sl.ready, cudaEventDisableTiming));
+    NITRO_CUDA(cudaEventCreateWithFlags(&sl.done, cudaEventDisableTiming));
+  }
+  *out = L;
+  return NITRO_OK;
+}
+
+void nitro_dist_loopback_destroy(nitro_loopback *L) {
+  if (!L) return;
+  cudaSetDevice(L->device);
+  for (auto &sl : L->slot) {
+    if (sl.ready) cudaEventDestroy(sl.ready);
+    if (sl.done) cudaEventDestroy(sl.done);
+  }
+  delete L;
+}
+
+nitro_status_t nitro_dist_init_loopback(nitro_loopback *L, int rank, nitro_dist **out) {
+  if (!L || !out || rank < 0 || rank >= L->nranks) return fail(NITRO_E_INVALID_ARG, "bad argument");
+  NITRO_TRY(nitro_dist_init_local(rank, L->nranks, L->device, out));
+  (*out)->lb = L;
+  return NITRO_OK;
 }
 
 }  // extern "C"

@@ -586,83 +586,118 @@ __global__ void __launch_bounds__(256) k_ell(const int32_t *__restrict__ ecol, c
 
 // ------------------------------------------------------------------ K8 DIA
 // Thread per 4 consecutive rows, block = 1024 rows; offsets in shared memory
-// (the first kDiaSmemOffs; larger D reads the rest through L1).  Blocks whose
-// rows see every diagonal in range skip all bounds checks.  One diagonal per
-// step and <= 32 registers (full occupancy): B200 sweeps on configs[1] put
-// more diagonals per batch (U = 2/4/8: 4916/4561/3033 vs 5373 GB/s) and a
-// diagonal split across lanes (DS = 2/4: 4076/3115) behind — resident warps
-// matter more than per-thread bytes in flight.
-constexpr int kDiaSmemOffs = 12288;  // 48 KB of offsets: no dynamic-smem opt-in needed
-template <typename VT>
-__global__ void __launch_bounds__(256, sizeof(VT) == 4 ? 8 : 1)
-    k_dia(const int32_t *__restrict__ offs, const VT *__restrict__ dval, const VT *__restrict__ x,
-          VT *__restrict__ y, int64_t N, int64_t M, int64_t D, int64_t ld, int64_t nr, int64_t row0,
-          int64_t off_min, int64_t off_max, bool x_aligned, bool l2ef, int pf, bool pfh) {
-  constexpr int64_t RB = 1024;  // rows per block iteration
+// (D <= kDiaSmemOffs = 48 KB; more diagonals read them through L1, GOFF).
+// Blocks whose rows see every diagonal in range skip all bounds checks.  One
+// diagonal per step, <= 32 registers (full occupancy): B200 sweeps on
+// configs[1] put more diagonals per batch (U = 2/4/8: 4916/4561/3033 vs 5373
+// GB/s) and a diagonal split across lanes (DS = 2/4: 4076/3115) behind —
+// resident warps matter more than per-thread bytes in flight.  (U and DS stay
+// template parameters fixed at 1: the loop below is written for them.)
+constexpr int kDiaSmemOffs = 12288;
+template <typename VT, bool GOFF, int U = 1, int DS = 1>  // GOFF: offsets read through L1 (D > kDiaSmemOffs)
+__global__ void __launch_bounds__(256, sizeof(VT) == 4 ? 8 : 1)  // fp32: <= 32 regs, full occupancy
+    k_dia(const int32_t *__restrict__ offs, const VT *__restrict__ dval,
+                                             const VT *__restrict__ x, VT *__restrict__ y, int64_t N, int64_t M,
+                                             int64_t D, int64_t ld, int64_t nr, int64_t row0, int64_t off_min,
+                                             int64_t off_max, bool x_aligned, bool l2ef, int pf, bool pfh) {
+  constexpr int64_t RB = 1024 / DS;  // rows per block iteration
   const uint64_t pol = l2_policy(l2ef);
   extern __shared__ int s_off[];
-  const int64_t Ds = D < kDiaSmemOffs ? D : kDiaSmemOffs;
-  auto off_of = [&](int64_t d) -> int { return d < kDiaSmemOffs ? s_off[d] : __ldg(offs + d); };
   // pf > 0: thread 0 keeps the block's value segments pf diagonals ahead in L2
   // (one cp.async.bulk L2 prefetch per diagonal, no registers or shared
   // memory): the per-thread chain of dependent value loads then waits on L2,
   // not HBM, and the HBM stream has pf x 4 KB per CTA in flight.
-  for (int64_t d = threadIdx.x; d < Ds; d += blockDim.x) s_off[d] = offs[d];
-  __syncthreads();
+  if constexpr (!GOFF) {
+    for (int64_t d = threadIdx.x; d < D; d += blockDim.x) s_off[d] = offs[d];
+    __syncthreads();
+  }
+  auto off_of = [&](int64_t d) -> int { if constexpr (GOFF) return __ldg(offs + d); else return s_off[d]; };
+  const int q = (int)(threadIdx.x % DS);
   const int64_t nb = (nr + RB - 1) / RB;  // rows [0, nr), nr <= ld (a row chunk: less)
   for (int64_t blk = blockIdx.x; blk < nb; blk += gridDim.x) {
     const int64_t B0 = blk * RB;
-    const int64_t i0 = B0 + 4 * threadIdx.x;
+    const int64_t i0 = B0 + 4 * (threadIdx.x / DS);
+    const bool active = i0 < nr;  // whole DS groups share i0: uniform within a group
     // segment bytes of one diagonal of this block (16-byte multiple: B0 and ld are multiples of 32 rows)
     const uint32_t pfb = (uint32_t)(((B0 + RB < nr ? B0 + RB : nr) - B0) * (int64_t)sizeof(VT)) & ~15u;
     if (pf > 0 && threadIdx.x == 0)
       for (int64_t d = 0; d < pf && d < D; ++d)
         pfh ? bulk_prefetch_l2(dval + d * ld + B0, pfb, pol) : bulk_prefetch_l2(dval + d * ld + B0, pfb);
-    if (i0 >= nr) continue;
+    if constexpr (DS == 1) {
+      if (!active) continue;      // no cross-lane combine needed
+    }
     const int64_t Bend = (B0 + RB < nr ? B0 + RB : nr) - 1;
     const bool interior = row0 + B0 + off_min >= 0 && row0 + Bend + off_max < M;
     // vector x path: aligned windows may reach 3 floats left / 4 right of the needed ones
     const bool xvec = x_aligned && row0 + B0 + off_min - 3 >= 0 && row0 + Bend + off_max + 4 < M;
     double acc[4] = {0.0, 0.0, 0.0, 0.0};
-    for (int64_t d = 0; d < D; ++d) {
-      if (pf > 0 && threadIdx.x == 0 && d + pf < D)
-        pfh ? bulk_prefetch_l2(dval + (d + pf) * ld + B0, pfb, pol) : bulk_prefetch_l2(dval + (d + pf) * ld + B0, pfb);
-      V4<VT> v;
-      v.load(dval + d * ld + i0, pol);
-      const int off = off_of(d);
-      VT xv[4];
+    for (int64_t d0 = (int64_t)q * U; (DS == 1 || active) && d0 < D; d0 += (int64_t)DS * U) {
+      if (pf > 0 && threadIdx.x == 0)
+        for (int64_t d = d0 + pf; d < d0 + pf + DS * U && d < D; ++d)
+          pfh ? bulk_prefetch_l2(dval + d * ld + B0, pfb, pol) : bulk_prefetch_l2(dval + d * ld + B0, pfb);
+      V4<VT> v[U];
+      VT xv[U][4];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (d0 + u < D) v[u].load(dval + (d0 + u) * ld + i0, pol);
+        else v[u].v[0] = v[u].v[1] = v[u].v[2] = v[u].v[3] = (VT)0;
+      }
       if (sizeof(VT) == 4 && xvec) {
         // fp32, x 16-byte aligned at row0: the 4 values x[j..j+3] (j = row0 + i0 +
         // off) come from the aligned 8-float window at j - (off & 3): two 128-bit
         // loads instead of four 32-bit ones (half the L1 wavefronts); off & 3 is
         // uniform across the warp (i0 is a multiple of 4)
-        const int r = off & 3;
-        const float *xb = reinterpret_cast<const float *>(x) + (row0 + i0 + off - r);
-        const float4 lo = __ldg(reinterpret_cast<const float4 *>(xb));
-        float4 hi = make_float4(0.f, 0.f, 0.f, 0.f);
-        if (r) hi = __ldg(reinterpret_cast<const float4 *>(xb) + 1);
-        float w[4];
-        switch (r) {
-          case 0: w[0] = lo.x; w[1] = lo.y; w[2] = lo.z; w[3] = lo.w; break;
-          case 1: w[0] = lo.y; w[1] = lo.z; w[2] = lo.w; w[3] = hi.x; break;
-          case 2: w[0] = lo.z; w[1] = lo.w; w[2] = hi.x; w[3] = hi.y; break;
-          default: w[0] = lo.w; w[1] = hi.x; w[2] = hi.y; w[3] = hi.z; break;
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          const bool live = d0 + u < D;
+          const int off = live ? off_of(d0 + u) : 0;
+          const int r = off & 3;
+          const float *xb = reinterpret_cast<const float *>(x) + (row0 + i0 + off - r);
+          float4 lo = make_float4(0.f, 0.f, 0.f, 0.f), hi = lo;
+          if (live) {
+            lo = __ldg(reinterpret_cast<const float4 *>(xb));
+            if (r) hi = __ldg(reinterpret_cast<const float4 *>(xb) + 1);
+          }
+          float w[4];
+          switch (r) {
+            case 0: w[0] = lo.x; w[1] = lo.y; w[2] = lo.z; w[3] = lo.w; break;
+            case 1: w[0] = lo.y; w[1] = lo.z; w[2] = lo.w; w[3] = hi.x; break;
+            case 2: w[0] = lo.z; w[1] = lo.w; w[2] = hi.x; w[3] = hi.y; break;
+            default: w[0] = lo.w; w[1] = hi.x; w[2] = hi.y; w[3] = hi.z; break;
+          }
+#pragma unroll
+          for (int t = 0; t < 4; ++t) xv[u][t] = (VT)w[t];
         }
-#pragma unroll
-        for (int t = 0; t < 4; ++t) xv[t] = (VT)w[t];
       } else if (interior) {
-        const VT *xp = x + (row0 + i0 + off);
 #pragma unroll
-        for (int t = 0; t < 4; ++t) xv[t] = __ldg(xp + t);
+        for (int u = 0; u < U; ++u) {
+          const bool live = d0 + u < D;  // uniform
+          const VT *xp = x + (row0 + i0 + (live ? off_of(d0 + u) : 0));
+#pragma unroll
+          for (int t = 0; t < 4; ++t) xv[u][t] = live ? __ldg(xp + t) : (VT)0;
+        }
       } else {
-        const int64_t j = row0 + i0 + off;
 #pragma unroll
-        for (int t = 0; t < 4; ++t) xv[t] = (j + t >= 0 && j + t < M) ? __ldg(x + j + t) : (VT)0;
+        for (int u = 0; u < U; ++u) {
+          const bool live = d0 + u < D;
+          const int64_t j = row0 + i0 + (live ? off_of(d0 + u) : 0);
+#pragma unroll
+          for (int t = 0; t < 4; ++t) xv[u][t] = (live && j + t >= 0 && j + t < M) ? __ldg(x + j + t) : (VT)0;
+        }
       }
+      VT part[4] = {0, 0, 0, 0};
 #pragma unroll
-      for (int t = 0; t < 4; ++t) acc[t] += (double)fma(v.v[t], xv[t], (VT)0);
+      for (int u = 0; u < U; ++u)
+#pragma unroll
+        for (int t = 0; t < 4; ++t) part[t] = fma(v[u].v[t], xv[u][t], part[t]);
+#pragma unroll
+      for (int t = 0; t < 4; ++t) acc[t] += (double)part[t];
     }
-    store4<VT>(y, i0, N, acc);
+#pragma unroll
+    for (int o = 1; o < DS; o <<= 1)
+#pragma unroll
+      for (int t = 0; t < 4; ++t) acc[t] += __shfl_xor_sync(kFull, acc[t], o);
+    if (active && q == 0) store4<VT>(y, i0, N, acc);
   }
 }
 
@@ -1145,13 +1180,18 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
       break;
     case NITRO_DIA:
       if (N > 0) {
-        const size_t sm = (size_t)std::min<int64_t>(std::max<int64_t>(A->dia.D, 1), kDiaSmemOffs) * 4;
+        const size_t sm = (size_t)std::max<int64_t>(A->dia.D, 1) * 4;
         const int64_t row0 = A->row0 + r0, nr = part ? round_up(N, 32) : A->dia.ld;
         const bool x_al = ((reinterpret_cast<uintptr_t>(x) & 15) == 0) && (row0 % 4 == 0);
         const unsigned g = grid_cap((nr + 1023) / 1024, dia_blocks_per_sm());
-        k_dia<VT><<<g, 256, sm, s>>>(A->dia.off.as<int32_t>(), A->dia.val.as<VT>() + r0, x, y, N, A->M, A->dia.D,
-                                     A->dia.ld, nr, row0, A->dia.off_min, A->dia.off_max, x_al, l2_evict_first(),
-                                     part ? 0 : dia_prefetch(), prefetch_hint());
+        if (A->dia.D <= kDiaSmemOffs)
+          k_dia<VT, false><<<g, 256, sm, s>>>(A->dia.off.as<int32_t>(), A->dia.val.as<VT>() + r0, x, y, N, A->M,
+                                              A->dia.D, A->dia.ld, nr, row0, A->dia.off_min, A->dia.off_max, x_al,
+                                              l2_evict_first(), part ? 0 : dia_prefetch(), prefetch_hint());
+        else
+          k_dia<VT, true><<<g, 256, 0, s>>>(A->dia.off.as<int32_t>(), A->dia.val.as<VT>() + r0, x, y, N, A->M,
+                                            A->dia.D, A->dia.ld, nr, row0, A->dia.off_min, A->dia.off_max, x_al,
+                                            l2_evict_first(), part ? 0 : dia_prefetch(), prefetch_hint());
       }
       break;
     case NITRO_HYB:

@@ -86,6 +86,18 @@ def test_spmv_bit_identical_to_scipy(seed):
     assert np.array_equal(y, S @ x)
 
 
+@pytest.mark.parametrize("threads", [1, 3, 8])
+def test_spmv_threads_bit_identical(threads):
+    """The all-core baseline loop (rows split over threads, bench.py only) is
+    the same per-row sequential sum: y and r bit-identical to oracle.spmv."""
+    A = synth.rmat(12, 8, seed=5, fp64=True)
+    x = synth.vector(A.cols, seed=3, fp64=True)
+    y, r = oracle.spmv(A, x)
+    y2, r2, used = oracle.spmv_threads(A, x, threads)
+    assert used == threads
+    assert np.array_equal(y, y2) and np.array_equal(r, r2)
+
+
 def test_spmv_identity_and_permutation():
     N = 1000
     x = np.random.default_rng(1).uniform(-1, 1, N)

@@ -13,7 +13,8 @@ The 60 training rows train the model through the library
 held-out matrices are selected with nitro_cv_predict (constraint fallback to
 CSR-vector) and scored against their exhaustive best.
 
-Writes artifacts/c3_table.json, artifacts/spmv_model.txt, artifacts/c3_report.json.
+Writes artifacts/c3_table.json, artifacts/spmv_model.txt (paper scaling), artifacts/spmv_model_r11x.txt
+(R11x extension) and artifacts/c3_report.json (both, side by side).
 """
 from __future__ import annotations
 
@@ -29,6 +30,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
 CLASSES = ("stencil", "banded", "uniform", "powerlaw")
+R11X_LOG_MASK = 0x7F   # DESIGN.md R11x: log1p of all seven SpMV features (extension, not the paper's reading)
 
 
 def params_for(cls: str, seed: int) -> dict:
@@ -129,49 +131,69 @@ def main():
     if not args.from_table:
         json.dump(rows, open(os.path.join(args.out, "c3_table.json"), "w"), indent=1)
 
-    # ---- train through the library (exhaustive labels -> scale -> CV grid -> SVM)
-    ctx = nitro.Context()
-    cv = nitro.CodeVariant(ctx, "spmv")
-    cv.register_spmv()
-    F = np.array([r["features"] for r in rows["train"]])
-    Cst = np.array([r["cost"] for r in rows["train"]])
-    cv.train_from_table(F, Cst)
-    cv.save(os.path.join(args.out, "spmv_model.txt"))
-    info = cv.model_info()
-    _, _, labels = cv.training_table()
+    # ---- train through the library (exhaustive labels -> scale -> CV grid -> SVM), twice:
+    # the paper's plain [-1, 1] scaling (the deployed default, spmv_model.txt) and the
+    # R11x extension (log1p + clip, not from the paper; spmv_model_r11x.txt), reported side by side
+    def fit(ext: bool):
+        ctx = nitro.Context()
+        cv = nitro.CodeVariant(ctx, "spmv")
+        cv.register_spmv()
+        if ext:
+            cv.set_feature_transform(R11X_LOG_MASK, True)
+        F = np.array([r["features"] for r in rows["train"]])
+        Cst = np.array([r["cost"] for r in rows["train"]])
+        cv.train_from_table(F, Cst)
+        cv.save(os.path.join(args.out, "spmv_model_r11x.txt" if ext else "spmv_model.txt"))
+        return ctx, cv
 
-    # ---- held-out selection
-    sel, ratios = [], []
-    always = {v: [] for v in nitro.VARIANT_NAMES}
+    def score(cv):
+        sel, ratios = [], []
+        for r in rows["test"]:
+            v = cv.predict(r["features"], r["allowed"])
+            sel.append(v)
+            c = r["cost"]
+            ratios.append(min(c) / c[v] if math.isfinite(c[v]) else 0.0)
+        n = len(ratios)
+        test_best = [int(np.argmin(r["cost"])) for r in rows["test"]]
+        return {
+            "nitro_pct_mean": sum(ratios) / n, "share_ge_70": sum(x >= 0.7 for x in ratios) / n,
+            "share_ge_90": sum(x >= 0.9 for x in ratios) / n,
+            "selected": [nitro.VARIANT_NAMES[v] for v in sel], "ratios": ratios,
+            "exact_pick_rate": sum(int(s_ == b_) for s_, b_ in zip(sel, test_best)) / n,
+            "model": cv.model_info(),
+            "mispredictions_below_70": [
+                {"params": r["params"], "selected": nitro.VARIANT_NAMES[s_], "best": nitro.VARIANT_NAMES[b_],
+                 "ratio": q, "features": dict(zip(nitro.FEATURE_NAMES, r["features"]))}
+                for r, s_, b_, q in zip(rows["test"], sel, test_best, ratios) if q < 0.7]}
+
+    ctx_p, cv_p = fit(False)
+    ctx_x, cv_x = fit(True)
+    _, _, labels = cv_p.training_table()
+    n = len(rows["test"])
+    always = {name: [] for name in nitro.VARIANT_NAMES}
     for r in rows["test"]:
-        v = cv.predict(r["features"], r["allowed"])
-        sel.append(v)
         c = r["cost"]
-        b = min(c)
-        ratios.append(b / c[v] if math.isfinite(c[v]) else 0.0)
         for k, name in enumerate(nitro.VARIANT_NAMES):
-            always[name].append(b / c[k] if math.isfinite(c[k]) else 0.0)
-    n = len(ratios)
+            always[name].append(min(c) / c[k] if math.isfinite(c[k]) else 0.0)
     test_best = [int(np.argmin(r["cost"])) for r in rows["test"]]
-    report = {
-        "nitro_pct_mean": sum(ratios) / n, "share_ge_70": sum(x >= 0.7 for x in ratios) / n,
-        "share_ge_90": sum(x >= 0.9 for x in ratios) / n, "n_test": n, "n_train": len(rows["train"]),
-        "selected": [nitro.VARIANT_NAMES[v] for v in sel], "ratios": ratios,
-        "exact_pick_rate": sum(int(s == b) for s, b in zip(sel, test_best)) / n,
+    paper, ext = score(cv_p), score(cv_x)
+    report = dict(paper)
+    report.update({
+        "scaling": "paper: libSVM svm-scale to [-1, 1] with the training min/max, no clipping (P:L179)",
+        "n_test": n, "n_train": len(rows["train"]),
         "always_variant_mean": {k: sum(v) / n for k, v in always.items()},
-        "train_label_counts": {nitro.VARIANT_NAMES[k]: int((labels == k).sum()) for k in range(5)},
-        "test_best_counts": {nitro.VARIANT_NAMES[k]: test_best.count(k) for k in range(5)},
-        "model": info,
-        "mispredictions_below_70": [
-            {"params": r["params"], "selected": nitro.VARIANT_NAMES[s], "best": nitro.VARIANT_NAMES[b], "ratio": q,
-             "features": dict(zip(nitro.FEATURE_NAMES, r["features"]))}
-            for r, s, b, q in zip(rows["test"], sel, test_best, ratios) if q < 0.7],
+        "train_label_counts": {nitro.VARIANT_NAMES[k]: int((labels == k).sum()) for k in range(nitro.NUM_VARIANTS)},
+        "test_best_counts": {nitro.VARIANT_NAMES[k]: test_best.count(k) for k in range(nitro.NUM_VARIANTS)},
+        "extension_r11x": dict(ext, scaling="EXTENSION (not from the paper, DESIGN.md R11x): log1p of all seven "
+                               "features before the [-1, 1] min-max scaling, scaled inputs clipped to [-1, 1]"),
         "paper_context": "P:L243 reports 93.74% on a Tesla C2050 (context, not the target)",
         "wall_s": time.time() - t0,
-    }
+    })
     json.dump(report, open(os.path.join(args.out, "c3_report.json"), "w"), indent=1)
-    print(json.dumps({k: report[k] for k in ("nitro_pct_mean", "share_ge_70", "share_ge_90", "exact_pick_rate",
-                                             "always_variant_mean", "train_label_counts", "model")}, indent=1))
+    keys = ("nitro_pct_mean", "share_ge_70", "share_ge_90", "exact_pick_rate", "model")
+    print(json.dumps({"paper": {k: report[k] for k in keys},
+                      "r11x": {k: report["extension_r11x"][k] for k in keys},
+                      "always": report["always_variant_mean"], "labels": report["train_label_counts"]}, indent=1))
 
 
 if __name__ == "__main__":
