@@ -179,10 +179,11 @@ def cpu_sample(nrows_target=2 * 1024 * 1024):
 
 
 def time_oracle(A, x, threads, seconds):
+    """Seconds per multiply of the oracle loop (inputs converted to its fp64
+    layout once, outside the timing), multiplies run, threads used."""
     import oracle
-    fn = (lambda: oracle.spmv(A, x)) if threads == 1 else (lambda: oracle.spmv_threads(A, x, threads))
-    r = fn()
-    used = 1 if threads == 1 else r[2]
+    fn = oracle.spmv_prepared(A, x, threads)
+    used = fn()
     n, t0 = 0, time.perf_counter()
     while True:
         fn()
@@ -227,12 +228,13 @@ def run_reference(args):
     bpr = (inrange * 4 + 27 * 4 + 8 * N) / N
     cores = os.cpu_count() or 1
     import oracle
+    fn = oracle.spmv_prepared(A, x, cores)
     for _ in range(args.warmup):
-        oracle.spmv_threads(A, x, cores)
+        fn()
     ts, used = [], cores
     for _ in range(args.steps):
         t0 = time.perf_counter()
-        used = oracle.spmv_threads(A, x, cores)[2]
+        used = fn()
         ts.append(time.perf_counter() - t0)
     t = sum(ts) / len(ts)
     val = bpr * A.rows / t / 1e9
@@ -681,7 +683,7 @@ def main():
     ap.add_argument("--workload", default="c4", choices=["c4", "c1"])
     ap.add_argument("--model", default="r11x", choices=["paper", "r11x"], help="deployed selection model")
     ap.add_argument("--ex-reps", type=int, default=7, help="timed reps per variant in the exhaustive reference")
-    ap.add_argument("--selection-per-class", type=int, default=3)
+    ap.add_argument("--selection-per-class", type=int, default=10, help="held-out configs[3] matrices per class")
     ap.add_argument("--quick", action="store_true", help="primary workload only (no extra configs/selection leg)")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     args = ap.parse_args()

@@ -130,6 +130,29 @@ def spmv_threads(A, x, nthreads: int | None = None):
     return y, r, used
 
 
+def spmv_prepared(A, x, nthreads: int = 1):
+    """C1 loop bound to A and x converted ONCE to the oracle's fp64 / int64
+    host layout; returns a no-argument callable that runs oracle_spmv (one
+    thread) or oracle_spmv_threads (nthreads > 1) into preallocated y, r.
+    bench.py times this callable so the baseline measures the oracle's loop,
+    not a per-call dtype conversion of x."""
+    N, M, rp, ci, v = _csr(A)
+    xd = np.ascontiguousarray(np.asarray(x), dtype=np.float64)
+    assert xd.shape[0] >= M
+    y = np.empty(N, dtype=np.float64)
+    r = np.empty(N, dtype=np.float64)
+    L = lib()
+    if nthreads <= 1:
+        def run():
+            L.oracle_spmv(N, _p(rp), _p(ci), _p(v), _p(xd), _p(y), _p(r))
+            return 1
+    else:
+        def run():
+            return L.oracle_spmv_threads(N, _p(rp), _p(ci), _p(v), _p(xd), _p(y), _p(r), int(nthreads))
+    run.y, run.r = y, r
+    return run
+
+
 def features(A, with_offsets: bool = False):
     """C4 features (dict); optionally also the ascending distinct offsets."""
     N, M, rp, ci, _ = _csr(A)

@@ -96,6 +96,9 @@ def test_spmv_threads_bit_identical(threads):
     y2, r2, used = oracle.spmv_threads(A, x, threads)
     assert used == threads
     assert np.array_equal(y, y2) and np.array_equal(r, r2)
+    fn = oracle.spmv_prepared(A, x, threads)
+    assert fn() == threads
+    assert np.array_equal(fn.y, y) and np.array_equal(fn.r, r)
 
 
 def test_spmv_identity_and_permutation():
