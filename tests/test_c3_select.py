@@ -20,6 +20,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 TABLE = os.path.join(ROOT, "artifacts", "c3_table.json")
 REPORT = os.path.join(ROOT, "artifacts", "c3_report.json")
 MODEL = os.path.join(ROOT, "artifacts", "spmv_model.txt")
+MODEL_R11X = os.path.join(ROOT, "artifacts", "spmv_model_r11x.txt")
 
 pytestmark = pytest.mark.skipif(not os.path.exists(TABLE), reason="configs[3] experiment not run yet")
 
@@ -46,31 +47,39 @@ def test_labels_are_exhaustive_argmin_and_constraints_infinite():
     assert counts == rep["train_label_counts"]
 
 
-def test_library_training_matches_oracle():
+@pytest.mark.parametrize("ext", [False, True], ids=["paper_scaling", "r11x"])
+def test_library_training_matches_oracle(ext):
+    """Both committed models: the paper's plain [-1, 1] scaling (spmv_model.txt,
+    the c3 report's top level) and the R11x extension (spmv_model_r11x.txt,
+    report["extension_r11x"]).  Same (C, gamma) and CV accuracy as the oracle's
+    re-derivation; held-out picks agree wherever the oracle model's decision is
+    firm (reading C12)."""
     import paper_conf_ipps_muralidharanshgc14_b200 as nitro
     t, rep = _load()
-    F = np.array([r["features"] for r in t["train"]])
+    r = rep["extension_r11x"] if ext else rep
+    F = np.array([row["features"] for row in t["train"]])
     lab = S.exhaustive_best(_costs(t["train"]))
-    m = S.train(F, lab, log_mask=S.R11X_LOG_MASK, clip=S.R11X_CLIP)   # the committed model's transform
-    assert (rep["model"]["C"], rep["model"]["gamma"]) == (m.C, m.gamma)
-    assert rep["model"]["cv_accuracy"] == pytest.approx(m.cv_accuracy, abs=1e-12)
-    # the committed model file selects like the oracle model on the held-out set
+    m = S.train(F, lab, log_mask=S.R11X_LOG_MASK, clip=S.R11X_CLIP) if ext else S.train(F, lab)
+    assert (r["model"]["C"], r["model"]["gamma"]) == (m.C, m.gamma)
+    assert r["model"]["cv_accuracy"] == pytest.approx(m.cv_accuracy, abs=1e-12)
     ctx = nitro.Context()
     cv = nitro.CodeVariant(ctx, "spmv")
     cv.register_spmv()
-    cv.load(MODEL)
-    sel_lib = [cv.predict(r["features"], r["allowed"]) for r in t["test"]]
-    sel_or = [S.select(m, r["features"], r["allowed"], default=1) for r in t["test"]]
-    firm = S.decided(m, np.array([r["features"] for r in t["test"]]))
-    assert all(a == b for a, b, f in zip(sel_lib, sel_or, firm) if f), (sel_lib, sel_or, firm)   # C12
-    names = ("csr_scalar", "csr_vector", "ell", "dia", "hyb")
-    assert [names[v] for v in sel_lib] == rep["selected"]
+    cv.load(MODEL_R11X if ext else MODEL)
+    sel_lib = [cv.predict(row["features"], row["allowed"]) for row in t["test"]]
+    sel_or = [S.select(m, row["features"], row["allowed"], default=1) for row in t["test"]]
+    firm = S.decided(m, np.array([row["features"] for row in t["test"]]))
+    assert firm.sum() >= len(firm) - 4
+    assert all(a_ == b_ for a_, b_, f in zip(sel_lib, sel_or, firm) if f), (sel_lib, sel_or, firm)   # C12
+    assert [nitro.VARIANT_NAMES[v] for v in sel_lib] == r["selected"]
 
 
-def test_nitro_percent_recomputed():
+@pytest.mark.parametrize("ext", [False, True], ids=["paper_scaling", "r11x"])
+def test_nitro_percent_recomputed(ext):
     t, rep = _load()
+    r_ = rep["extension_r11x"] if ext else rep
     names = ("csr_scalar", "csr_vector", "ell", "dia", "hyb")
-    sel = [names.index(s) for s in rep["selected"]]
+    sel = [names.index(s) for s in r_["selected"]]
     r = S.nitro_percent(_costs(t["test"]), sel)
-    assert r["mean"] == pytest.approx(rep["nitro_pct_mean"], abs=1e-12)
-    assert r["ge70"] == pytest.approx(rep["share_ge_70"]) and r["ge90"] == pytest.approx(rep["share_ge_90"])
+    assert r["mean"] == pytest.approx(r_["nitro_pct_mean"], abs=1e-12)
+    assert r["ge70"] == pytest.approx(r_["share_ge_70"]) and r["ge90"] == pytest.approx(r_["share_ge_90"])
