@@ -111,8 +111,17 @@ typedef struct {
   int log2c_lo, log2c_hi, log2c_step; /* default -5, 15, 2   (libSVM grid.py) */
   int log2g_lo, log2g_hi, log2g_step; /* default -15, 3, 2 */
   int verbose;                    /* 0 = silent */
+  double timeout_factor;          /* training timeout: while an input is labelled, a
+                                     variant may stop timing once its cost exceeds this factor x the
+                                     best cost seen so far on that input (default 20; <= 0 = off) */
 } nitro_train_opts;
 void nitro_train_opts_default(nitro_train_opts *o);
+/* For variant functions: the cost above which the input's exhaustive search
+ * no longer needs an exact value (timeout_factor x the best cost so far on
+ * the input being labelled); +INFINITY outside training or when off.  A
+ * variant may stop measuring once it is sure to exceed it and return the
+ * cost measured so far (the SpMV variants stop their reps, >= 3 run). */
+double nitro_cv_cost_cutoff(void);
 
 /* Offline training: for every training input evaluate features,
  * run every variant (constraint false => cost +INF), label = argmin

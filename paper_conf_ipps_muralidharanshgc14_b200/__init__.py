@@ -76,7 +76,7 @@ class TrainOpts(ctypes.Structure):
     _fields_ = [("folds", ctypes.c_int), ("seed", ctypes.c_uint64), ("tol", ctypes.c_double),
                 ("log2c_lo", ctypes.c_int), ("log2c_hi", ctypes.c_int), ("log2c_step", ctypes.c_int),
                 ("log2g_lo", ctypes.c_int), ("log2g_hi", ctypes.c_int), ("log2g_step", ctypes.c_int),
-                ("verbose", ctypes.c_int)]
+                ("verbose", ctypes.c_int), ("timeout_factor", ctypes.c_double)]
 
 
 class ItuneOpts(ctypes.Structure):
@@ -118,6 +118,7 @@ _SIGS = {
     "nitro_cv_add_constraint": ([_vp, _int, CONSTRAINT_FN, _vp], _int),
     "nitro_cv_add_training_input": ([_vp, _vp], _int),
     "nitro_train_opts_default": ([_P(TrainOpts)], None),
+    "nitro_cv_cost_cutoff": ([], _dbl),
     "nitro_cv_train": ([_vp, _P(TrainOpts)], _int),
     "nitro_cv_train_from_table": ([_vp, _int, _vp, _vp, _P(TrainOpts)], _int),
     "nitro_cv_training_table": ([_vp, _P(_int), _vp, _vp, _vp], _int),

@@ -375,35 +375,7 @@ nitro_status_t nitro_spmv_time(nitro_spmv *A, int variant, const void *d_x, void
   NITRO_GUARD_BEGIN
   if (!A || !valid_variant(variant) || reps < 1 || warmup < 0 || !out_median_s)
     return fail(NITRO_E_INVALID_ARG, "bad argument");
-  DeviceGuard g(A->device);
-  if (!is_ready(A, variant)) NITRO_TRY(prepare_impl(A, variant));
-  cudaStream_t s = A->stream;
-  for (int w = 0; w < warmup; ++w) NITRO_TRY(launch_spmv(A, variant, d_x, d_y, s));
-  std::vector<cudaEvent_t> ev(2 * reps, nullptr);
-  for (auto &e : ev) NITRO_CUDA(cudaEventCreate(&e));
-  nitro_status_t st = NITRO_OK;
-  for (int r = 0; r < reps && st == NITRO_OK; ++r) {
-    if (flush_l2) st = launch_flush(A, s);
-    if (st == NITRO_OK) {
-      cudaEventRecord(ev[2 * r], s);
-      st = launch_spmv(A, variant, d_x, d_y, s);
-      cudaEventRecord(ev[2 * r + 1], s);
-    }
-  }
-  std::vector<double> t(reps, 0.0);
-  cudaError_t e = cudaStreamSynchronize(s);
-  if (st == NITRO_OK && e != cudaSuccess) st = cuda_fail(e, "cudaStreamSynchronize");
-  for (int r = 0; r < reps && st == NITRO_OK; ++r) {
-    float ms = 0.f;
-    cudaEventElapsedTime(&ms, ev[2 * r], ev[2 * r + 1]);
-    t[r] = ms * 1e-3;
-  }
-  for (auto &x : ev) cudaEventDestroy(x);
-  if (st != NITRO_OK) return st;
-  if (out_all) std::copy(t.begin(), t.end(), out_all);
-  std::sort(t.begin(), t.end());
-  *out_median_s = reps % 2 ? t[reps / 2] : 0.5 * (t[reps / 2 - 1] + t[reps / 2]);
-  return NITRO_OK;
+  return nitro::time_variant(A, variant, d_x, d_y, warmup, reps, flush_l2, INFINITY, out_median_s, out_all, nullptr);
   NITRO_GUARD_END
 }
 
@@ -514,3 +486,61 @@ void nitro_spmv_destroy(nitro_spmv *A) {
 }
 
 }  // extern "C"
+
+namespace nitro {
+// Median of `reps` CUDA-event timings (L2 flushed before each when flush_l2).
+// cutoff_s finite (the training timeout of SURVEY §5): after every rep from
+// the third on, stop once the median so far exceeds cutoff_s — a variant 20x
+// slower than the input's current best is ranked by the reps it has run.
+nitro_status_t time_variant(nitro_spmv *A, int variant, const void *d_x, void *d_y, int warmup, int reps,
+                            int flush_l2, double cutoff_s, double *out_median_s, double *out_all, int *out_reps) {
+  DeviceGuard g(A->device);
+  if (!is_ready(A, variant)) NITRO_TRY(prepare_impl(A, variant));
+  cudaStream_t s = A->stream;
+  for (int w = 0; w < warmup; ++w) NITRO_TRY(launch_spmv(A, variant, d_x, d_y, s));
+  const bool early = std::isfinite(cutoff_s);
+  std::vector<cudaEvent_t> ev(2 * reps, nullptr);
+  for (auto &e : ev) NITRO_CUDA(cudaEventCreate(&e));
+  std::vector<double> t;
+  nitro_status_t st = NITRO_OK;
+  auto collect = [&](int upto) {  // rep times [t.size(), upto)
+    cudaError_t e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaStreamSynchronize");
+    for (int r = (int)t.size(); r < upto; ++r) {
+      float ms = 0.f;
+      cudaEventElapsedTime(&ms, ev[2 * r], ev[2 * r + 1]);
+      t.push_back(ms * 1e-3);
+    }
+    return (nitro_status_t)NITRO_OK;
+  };
+  auto median = [](std::vector<double> v) {
+    std::sort(v.begin(), v.end());
+    const size_t n = v.size();
+    return n % 2 ? v[n / 2] : 0.5 * (v[n / 2 - 1] + v[n / 2]);
+  };
+  int done = 0;
+  for (int r = 0; r < reps && st == NITRO_OK; ++r) {
+    if (flush_l2) st = launch_flush(A, s);
+    if (st == NITRO_OK) {
+      cudaEventRecord(ev[2 * r], s);
+      st = launch_spmv(A, variant, d_x, d_y, s);
+      cudaEventRecord(ev[2 * r + 1], s);
+    }
+    done = r + 1;
+    if (st == NITRO_OK && early && done >= 3 && done < reps) {
+      st = collect(done);
+      if (st == NITRO_OK && median(t) > cutoff_s) break;
+    }
+  }
+  if (st == NITRO_OK) st = collect(done);
+  for (auto &x : ev) cudaEventDestroy(x);
+  if (st != NITRO_OK) return st;
+  if (out_all) {
+    std::copy(t.begin(), t.end(), out_all);
+    std::fill(out_all + t.size(), out_all + reps, std::numeric_limits<double>::quiet_NaN());
+  }
+  *out_median_s = median(t);
+  if (out_reps) *out_reps = (int)t.size();
+  return NITRO_OK;
+}
+}  // namespace nitro

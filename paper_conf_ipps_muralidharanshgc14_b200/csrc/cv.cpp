@@ -70,6 +70,15 @@ namespace {
 
 constexpr double kInf = std::numeric_limits<double>::infinity();
 
+// Training timeout: while an input is labelled, the variant being
+// timed may stop early once its cost exceeds timeout_factor x the best cost
+// seen so far on that input (nitro_cv_cost_cutoff).
+thread_local double g_cost_cutoff = kInf;
+struct CutoffScope {
+  CutoffScope(double best, double factor) { g_cost_cutoff = (factor > 0 && best < kInf) ? factor * best : kInf; }
+  ~CutoffScope() { g_cost_cutoff = kInf; }
+};
+
 nitro_status_t eval_features(nitro_cv *cv, const void *input, double *out) {
   int k = 0;
   for (auto &f : cv->feats) {
@@ -180,6 +189,8 @@ nitro_status_t fit_scaled(nitro_cv *cv, const nitro_train_opts &o) {
 
 extern "C" {
 
+double nitro_cv_cost_cutoff(void) { return g_cost_cutoff; }
+
 void nitro_train_opts_default(nitro_train_opts *o) {
   if (!o) return;
   o->folds = 5;
@@ -188,6 +199,7 @@ void nitro_train_opts_default(nitro_train_opts *o) {
   o->log2c_lo = -5; o->log2c_hi = 15; o->log2c_step = 2;
   o->log2g_lo = -15; o->log2g_hi = 3; o->log2g_step = 2;
   o->verbose = 0;
+  o->timeout_factor = 20.0;
 }
 
 nitro_status_t nitro_context_create(nitro_context **out) {
@@ -304,7 +316,11 @@ nitro_status_t nitro_cv_train(nitro_cv *cv, const nitro_train_opts *opts) {
     double best = kInf;
     for (int v = 0; v < V; ++v) {
       // exhaustive search; a failed constraint makes the cost infinite
-      double c = allowed(cv, v, in) ? cv->variants[v].fn(in, cv->variants[v].user) : kInf;
+      double c = kInf;
+      if (allowed(cv, v, in)) {
+        const CutoffScope cs(best, o.timeout_factor);
+        c = cv->variants[v].fn(in, cv->variants[v].user);
+      }
       if (std::isnan(c)) c = kInf;
       cv->t_cost[(size_t)i * V + v] = c;
       if (c < best) { best = c; cv->t_label[i] = v; }  // ties -> lowest id
@@ -389,7 +405,11 @@ nitro_status_t nitro_cv_itune(nitro_cv *cv, const nitro_train_opts *topts, const
     void *in = cv->inputs[i];
     double best = kInf;
     for (int v = 0; v < V; ++v) {
-      double c = allowed(cv, v, in) ? cv->variants[v].fn(in, cv->variants[v].user) : kInf;
+      double c = kInf;
+      if (allowed(cv, v, in)) {
+        const CutoffScope cs(best, o.timeout_factor);
+        c = cv->variants[v].fn(in, cv->variants[v].user);
+      }
       if (std::isnan(c)) c = kInf;
       cost[(size_t)i * V + v] = c;
       if (c < best) { best = c; label_of[i] = v; }
@@ -674,9 +694,10 @@ static double spmv_variant_fn(void *input, void *user) {
   nitro_spmv_input *in = (nitro_spmv_input *)input;
   const int v = (int)(intptr_t)user;
   double t = kInf;
-  if (!in || !in->A) return kInf;
-  if (nitro_spmv_time(in->A, v, in->d_x, in->d_y, in->warmup, in->reps > 0 ? in->reps : 1, in->flush_l2, &t,
-                      nullptr) != NITRO_OK)
+  if (!in || !in->A || !in->d_x || !in->d_y) return kInf;
+  // training timeout: stop the reps once the median passes the cv's cutoff
+  if (nitro::time_variant(in->A, v, in->d_x, in->d_y, std::max(in->warmup, 0), in->reps > 0 ? in->reps : 1,
+                          in->flush_l2, nitro_cv_cost_cutoff(), &t, nullptr, nullptr) != NITRO_OK)
     return kInf;
   return t;
 }

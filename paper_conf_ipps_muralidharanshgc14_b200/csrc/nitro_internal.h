@@ -154,6 +154,8 @@ nitro_status_t launch_flush(nitro_spmv *A, cudaStream_t s);
 double compulsory_bytes(const nitro_spmv *A, int variant);
 
 // scan.cu: exclusive scan of int64 counts; out[n] = total.  scratch grows.
+nitro_status_t time_variant(nitro_spmv *A, int variant, const void *d_x, void *d_y, int warmup, int reps,
+                            int flush_l2, double cutoff_s, double *out_median_s, double *out_all, int *out_reps);
 nitro_status_t exclusive_scan_i64(const int64_t *in, int64_t *out, int64_t n, DevBuf &scratch, cudaStream_t s);
 
 inline int64_t round_up(int64_t n, int64_t m) { return (n + m - 1) / m * m; }

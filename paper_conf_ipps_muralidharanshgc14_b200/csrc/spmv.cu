@@ -1099,64 +1099,9 @@ nitro_status_t launch_staged(const nitro_spmv *A, int V, const IT *rp, const VT 
   }
 }
 
-// x residency in L2 for the gather-heavy launches (CSR-scalar, CSR-vector,
-// ELL, HYB on matrices whose columns are NOT on few diagonals): the x range is
-// given an L2 access-policy window with the PERSISTING property for the
-// launch, so the streamed matrix arrays (evict-first) cannot push the reused x
-// out of L2 (round 1 ncu, configs[2] R-MAT fp64: 1.87x the algorithmic DRAM
-// bytes, x re-read).  The set-aside is the device's maximum persisting size;
-// an x larger than it gets hitRatio = set-aside / x bytes.  The stream's
-// previous window is restored after the launch, and launch_flush demotes all
-// persisting lines first (cudaCtxResetPersistingL2Cache), so L2-flushed
-// timings still read x from HBM.  NITRO_L2_PERSIST=0 disables.
-bool l2_persist_on() {
-  static bool v = [] {
-    const char *e = getenv("NITRO_L2_PERSIST");
-    return e ? atoi(e) != 0 : true;
-  }();
-  return v;
-}
-
-struct XWindow {
-  cudaStream_t s = nullptr;
-  bool on = false;
-  cudaStreamAttrValue prev{};
-  XWindow(const nitro_spmv *A, int variant, const void *x, size_t xbytes, cudaStream_t s_) : s(s_) {
-    if (!l2_persist_on() || variant == NITRO_DIA || diag_local(A) || xbytes < (8u << 20)) return;
-    static int maxp = -1, maxw = 0;
-    if (maxp < 0) {
-      maxp = 0;
-      if (cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, A->device) != cudaSuccess ||
-          cudaDeviceGetAttribute(&maxw, cudaDevAttrMaxAccessPolicyWindowSize, A->device) != cudaSuccess ||
-          cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)maxp) != cudaSuccess) {
-        maxp = 0;
-        cudaGetLastError();
-      }
-    }
-    if (maxp <= 0 || maxw <= 0) return;
-    if (cudaStreamGetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &prev) != cudaSuccess) {
-      cudaGetLastError();
-      return;
-    }
-    cudaStreamAttrValue v{};
-    const size_t nb = std::min(xbytes, (size_t)maxw);
-    v.accessPolicyWindow.base_ptr = const_cast<void *>(x);
-    v.accessPolicyWindow.num_bytes = nb;
-    v.accessPolicyWindow.hitRatio = (float)std::min(1.0, (double)maxp / (double)nb);
-    v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
-    v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
-    on = cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &v) == cudaSuccess;
-    if (!on) cudaGetLastError();
-  }
-  ~XWindow() {
-    if (on) cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &prev);
-  }
-};
-
 template <typename IT, typename VT>
 nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_t s, int64_t r0 = 0,
                      int64_t r1 = -1) {
-  const XWindow xw(A, variant, x, (size_t)A->M * sizeof(VT), s);
   // rows [r0, r1) (default: all).  Partial ranges only for the row-separable
   // CSR-scalar / ELL / DIA launches (launch_spmv_rows); r0 % 32 == 0.
   const bool part = r1 >= 0;
@@ -1347,12 +1292,6 @@ nitro_status_t csr_chunk_xhi(nitro_spmv *A, const std::vector<int64_t> &ends, st
 }
 
 nitro_status_t launch_flush(nitro_spmv *A, cudaStream_t s) {
-  // persisting lines (XWindow) would survive a plain streaming read: demote
-  // them first, so a flushed run reads x from HBM like every other variant
-  if (l2_persist_on()) {
-    NITRO_CUDA(cudaStreamSynchronize(s));
-    NITRO_CUDA(cudaCtxResetPersistingL2Cache());
-  }
   if (!A->flush.p) {
     int l2 = 0;
     NITRO_CUDA(cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, A->device));
