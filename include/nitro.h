@@ -263,16 +263,21 @@ nitro_status_t nitro_spmv_features_async(nitro_spmv *A);
 nitro_status_t nitro_spmv_allowed(nitro_spmv *A, int variant, int *out_allowed);
 /* budget for padded formats in bytes (default: 40% of free HBM at first use) */
 nitro_status_t nitro_spmv_set_budget(nitro_spmv *A, double bytes);
-/* Kernel implementation of the two CSR variants (DESIGN.md §6 K5/K6; the
- * arithmetic, and so y, is identical across implementations):
- * NITRO_CSR_IMPL_AUTO (default) = the direct kernels (loads from global
- * memory; the TMA row-tile pipeline measured slower on every class, so AUTO
- * uses it only when the environment sets NITRO_CSR_STAGED=1); _DIRECT = the
- * direct kernels; _STAGED = the TMA row-tile pipeline for every matrix
- * (tiles that do not fit the shared-memory stage are computed from global
- * memory).  Returns
- * NITRO_E_INVALID_ARG for any other value.  Takes effect at the next run. */
-enum { NITRO_CSR_IMPL_AUTO = 0, NITRO_CSR_IMPL_DIRECT = 1, NITRO_CSR_IMPL_STAGED = 2 };
+/* Kernel implementation of the two CSR variants (DESIGN.md §6 K5/K6/K6s):
+ * NITRO_CSR_IMPL_AUTO (default) = the direct kernels, and for CSR-vector the
+ * nnz-split stream kernel (K6s) when the row lengths are skewed (row-length
+ * SD > mean: power-law rows); the TMA row-tile pipeline measured slower on
+ * every class, so AUTO uses it only when the environment sets
+ * NITRO_CSR_STAGED=1.  _DIRECT = the direct row-oriented kernels; _STAGED =
+ * the TMA row-tile pipeline for every matrix (tiles that do not fit the
+ * shared-memory stage are computed from global memory); _STREAM = the
+ * nnz-split stream kernel for CSR-vector (CSR-scalar keeps the direct
+ * kernel).  Within a mode the result is deterministic; the row-oriented
+ * implementations are bit-identical to each other, the stream mode sums each
+ * row in fp64 in a different association (within the R2 tolerance).
+ * Returns NITRO_E_INVALID_ARG for any other value.  Takes effect at the next
+ * run (the CSR-vector format is rebuilt if its mode changes). */
+enum { NITRO_CSR_IMPL_AUTO = 0, NITRO_CSR_IMPL_DIRECT = 1, NITRO_CSR_IMPL_STAGED = 2, NITRO_CSR_IMPL_STREAM = 3 };
 nitro_status_t nitro_spmv_set_csr_impl(nitro_spmv *A, int impl);
 /* Build the variant's format (cached; conversions are amortised). */
 nitro_status_t nitro_spmv_prepare(nitro_spmv *A, int variant);

@@ -209,8 +209,10 @@ nitro_status_t nitro_spmv_set_budget(nitro_spmv *A, double bytes) {
 }
 
 nitro_status_t nitro_spmv_set_csr_impl(nitro_spmv *A, int impl) {
-  if (!A || impl < NITRO_CSR_IMPL_AUTO || impl > NITRO_CSR_IMPL_STAGED) return fail(NITRO_E_INVALID_ARG, "bad argument");
+  if (!A || impl < NITRO_CSR_IMPL_AUTO || impl > NITRO_CSR_IMPL_STREAM) return fail(NITRO_E_INVALID_ARG, "bad argument");
   A->csr_impl = impl;
+  // the CSR-vector format depends on the mode (stream chunks vs long-row segments)
+  if (A->csrv.ready && A->csrv.stream != csrv_stream_mode(A)) A->csrv.ready = false;
   return NITRO_OK;
 }
 
@@ -231,7 +233,12 @@ nitro_status_t nitro_spmv_format_info(nitro_spmv *A, int variant, nitro_format_i
   memset(out, 0, sizeof(*out));
   switch (variant) {
     case NITRO_CSR_SCALAR: out->width = 1; break;
-    case NITRO_CSR_VECTOR: out->width = A->csrv.V; out->tail = A->csrv.n_long; out->bytes = (int64_t)A->csrv.long_rows.bytes; break;
+    case NITRO_CSR_VECTOR:
+      out->width = A->csrv.stream ? 0 : A->csrv.V;  // 0: nnz-split stream mode (K6s)
+      out->tail = A->csrv.stream ? A->csrv.nch : A->csrv.n_long;
+      out->bytes = (int64_t)(A->csrv.long_rows.bytes + A->csrv.chunk_row.bytes + A->csrv.carry_row.bytes +
+                             A->csrv.carry_val.bytes + A->csrv.fix_seg.bytes + A->csrv.fix_long.bytes);
+      break;
     case NITRO_ELL: out->ld = A->ell.ld; out->width = A->ell.K; out->bytes = (int64_t)(A->ell.col.bytes + A->ell.val.bytes); break;
     case NITRO_DIA: out->ld = A->dia.ld; out->width = A->dia.D; out->bytes = (int64_t)(A->dia.off.bytes + A->dia.val.bytes); break;
     case NITRO_HYB:
@@ -463,7 +470,12 @@ nitro_status_t nitro_spmv_release(nitro_spmv *A, int variant) {
     A->hyb.tval.release(); A->hyb.carry_row.release(); A->hyb.carry_val.release();
     A->hyb.fix_seg.release(); A->hyb.fix_long.release(); A->hyb.ready = false;
   }
-  if (variant == -1 || variant == NITRO_CSR_VECTOR) { A->csrv.long_rows.release(); A->csrv.ready = false; }
+  if (variant == -1 || variant == NITRO_CSR_VECTOR) {
+    A->csrv.long_rows.release();
+    A->csrv.chunk_row.release(); A->csrv.carry_row.release(); A->csrv.carry_val.release();
+    A->csrv.fix_seg.release(); A->csrv.fix_long.release();
+    A->csrv.ready = false;
+  }
   return NITRO_OK;
 }
 

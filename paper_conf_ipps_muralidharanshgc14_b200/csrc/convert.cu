@@ -438,6 +438,42 @@ nitro_status_t prepare_hyb(nitro_spmv *A) {
   return NITRO_OK;
 }
 
+bool csrv_stream_mode(const nitro_spmv *A) {
+  static int env = [] {
+    const char *e = getenv("NITRO_CSRV_STREAM");
+    return e ? atoi(e) : -1;
+  }();
+  if (A->csr_impl == NITRO_CSR_IMPL_STREAM) return true;
+  if (A->csr_impl != NITRO_CSR_IMPL_AUTO) return false;
+  if (env == 0 || env == 1) return env == 1;
+  return A->feat_ready && A->feat.sd > A->feat.mean;
+}
+
+// ------------------------------------------------------------------ CSR-vector stream mode (K6s)
+// chunk_row[c] = the row holding entry c*CH (the last row whose start <= c*CH),
+// chunk_row[nch] = N; eff[2c] / eff[2c+1] = rows of the chunk's first / last
+// entry (the carry slots' rows, grouped into the fixup plan like HYB's)
+template <typename IT>
+__global__ void k_stream_rows(const IT *__restrict__ rowptr, int64_t N, int64_t Z, int64_t CH, int64_t nch,
+                              int32_t *__restrict__ chunk_row, int32_t *__restrict__ eff) {
+  auto row_of = [&](int64_t e) {  // last r with rowptr[r] <= e
+    int64_t lo = 0, hi = N;        // rowptr[lo] <= e < rowptr[hi] (rowptr[N] = Z > e)
+    while (hi - lo > 1) {
+      const int64_t m = (lo + hi) >> 1;
+      if ((int64_t)rowptr[m] <= e) lo = m; else hi = m;
+    }
+    return (int32_t)lo;
+  };
+  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c <= nch; c += (int64_t)gridDim.x * blockDim.x) {
+    if (c == nch) { chunk_row[c] = (int32_t)N; continue; }
+    const int64_t s0 = c * CH, e1 = (s0 + CH < Z ? s0 + CH : Z) - 1;
+    const int32_t r0 = row_of(s0);
+    chunk_row[c] = r0;
+    eff[2 * c] = r0;
+    eff[2 * c + 1] = row_of(e1);
+  }
+}
+
 // ------------------------------------------------------------------ CSR-vector (C8)
 // V = lanes per row from the mean row length; rows longer than 8V are split
 // into segments of kCsrvSeg entries, each reduced by one warp (see spmv.cu).
@@ -463,6 +499,44 @@ nitro_status_t prepare_csrv(nitro_spmv *A) {
   }();
   for (int k = 0; k < shift && V > 2; ++k) V >>= 1;
   A->csrv.V = V;
+  A->csrv.stream = csrv_stream_mode(A);
+  if (A->csrv.stream && A->Z > 0) {
+    const int EP = A->fp64 ? 4 : 8;
+    const int64_t CH = 32LL * EP, nch = (A->Z + CH - 1) / CH, nslot = 2 * nch;
+    A->csrv.EP = EP;
+    A->csrv.nch = nch;
+    NITRO_TRY(A->csrv.chunk_row.alloc((size_t)(nch + 1) * 4));
+    NITRO_TRY(A->csrv.carry_row.alloc((size_t)nslot * 4));
+    NITRO_TRY(A->csrv.carry_val.alloc((size_t)nslot * 8));
+    DevBuf fx;
+    NITRO_TRY(fx.alloc((size_t)nslot * 4 + (size_t)(2 * nslot + 2) * 8 + 8));
+    int32_t *eff = fx.as<int32_t>();
+    int64_t *hd = reinterpret_cast<int64_t *>(fx.as<char>() + round_up(nslot * 4, 8)), *pos = hd + nslot + 1;
+    if (A->rp64) k_stream_rows<int64_t><<<grid_of(nch + 1), 256, 0, s>>>((const int64_t *)A->rowptr, N, A->Z, CH, nch, A->csrv.chunk_row.as<int32_t>(), eff);
+    else k_stream_rows<int32_t><<<grid_of(nch + 1), 256, 0, s>>>((const int32_t *)A->rowptr, N, A->Z, CH, nch, A->csrv.chunk_row.as<int32_t>(), eff);
+    k_fix_heads<<<grid_of(nslot), 256, 0, s>>>(eff, nslot, hd);
+    NITRO_TRY(exclusive_scan_i64(hd, pos, nslot, A->scratch, s));
+    int64_t S = 0;
+    NITRO_CUDA(cudaMemcpyAsync(&S, pos + nslot, 8, cudaMemcpyDeviceToHost, s));
+    NITRO_CUDA(cudaStreamSynchronize(s));
+    NITRO_TRY(A->csrv.fix_seg.alloc((size_t)(S + 1) * 4));
+    NITRO_TRY(A->csrv.fix_long.alloc((size_t)std::max<int64_t>(S, 1) * 4));
+    k_fix_emit<<<grid_of(nslot), 256, 0, s>>>(eff, pos, nslot, A->csrv.fix_seg.as<int32_t>());
+    DevBuf lc;
+    NITRO_TRY(lc.alloc(8));
+    NITRO_CUDA(cudaMemsetAsync(lc.p, 0, 8, s));
+    k_fix_long<<<grid_of(S), 256, 0, s>>>(A->csrv.fix_seg.as<int32_t>(), S, A->csrv.fix_long.as<int32_t>(),
+                                          lc.as<unsigned long long>());
+    NITRO_CUDA(cudaGetLastError());
+    unsigned long long nl = 0;
+    NITRO_CUDA(cudaMemcpyAsync(&nl, lc.p, 8, cudaMemcpyDeviceToHost, s));
+    NITRO_CUDA(cudaStreamSynchronize(s));
+    A->csrv.fix_S = S;
+    A->csrv.fix_nlong = (int64_t)nl;
+    A->csrv.n_long = 0;
+    A->csrv.ready = true;
+    return NITRO_OK;
+  }
   const int64_t T = 8LL * V, S = kCsrvSeg;
   A->csrv.n_long = 0;
   if (A->feat.max_row > T) {

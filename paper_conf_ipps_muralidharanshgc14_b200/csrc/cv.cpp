@@ -314,8 +314,11 @@ nitro_status_t nitro_cv_train(nitro_cv *cv, const nitro_train_opts *opts) {
     void *in = cv->inputs[i];
     NITRO_TRY(eval_features(cv, in, &cv->t_feat[(size_t)i * d]));
     double best = kInf;
-    for (int v = 0; v < V; ++v) {
-      // exhaustive search; a failed constraint makes the cost infinite
+    for (int q = 0; q < V; ++q) {
+      // exhaustive search; a failed constraint makes the cost infinite.
+      // The default variant is timed first, so the training timeout has a
+      // reference cost early; the label is the argmin whatever the order.
+      const int v = q == 0 ? cv->default_id : (q <= cv->default_id ? q - 1 : q);
       double c = kInf;
       if (allowed(cv, v, in)) {
         const CutoffScope cs(best, o.timeout_factor);
@@ -323,8 +326,12 @@ nitro_status_t nitro_cv_train(nitro_cv *cv, const nitro_train_opts *opts) {
       }
       if (std::isnan(c)) c = kInf;
       cv->t_cost[(size_t)i * V + v] = c;
-      if (c < best) { best = c; cv->t_label[i] = v; }  // ties -> lowest id
+      best = std::min(best, c);
     }
+    for (int v = 0; v < V; ++v)  // label = argmin, ties -> lowest id
+      if (cv->t_label[i] < 0 ? cv->t_cost[(size_t)i * V + v] < kInf
+                             : cv->t_cost[(size_t)i * V + v] < cv->t_cost[(size_t)i * V + cv->t_label[i]])
+        cv->t_label[i] = v;
     if (o.verbose)
       std::fprintf(stderr, "nitro: input %d/%d label %d\n", i + 1, n, cv->t_label[i]);
   }
@@ -404,7 +411,8 @@ nitro_status_t nitro_cv_itune(nitro_cv *cv, const nitro_train_opts *topts, const
   auto label_input = [&](int i) {  // exhaustive search on one input
     void *in = cv->inputs[i];
     double best = kInf;
-    for (int v = 0; v < V; ++v) {
+    for (int q = 0; q < V; ++q) {  // default first (training timeout reference), as nitro_cv_train
+      const int v = q == 0 ? cv->default_id : (q <= cv->default_id ? q - 1 : q);
       double c = kInf;
       if (allowed(cv, v, in)) {
         const CutoffScope cs(best, o.timeout_factor);
@@ -412,8 +420,12 @@ nitro_status_t nitro_cv_itune(nitro_cv *cv, const nitro_train_opts *topts, const
       }
       if (std::isnan(c)) c = kInf;
       cost[(size_t)i * V + v] = c;
-      if (c < best) { best = c; label_of[i] = v; }
+      best = std::min(best, c);
     }
+    for (int v = 0; v < V; ++v)  // label = argmin, ties -> lowest id
+      if (cost[(size_t)i * V + v] < kInf &&
+          (label_of[i] < 0 || cost[(size_t)i * V + v] < cost[(size_t)i * V + label_of[i]]))
+        label_of[i] = v;
     done[i] = 1;
     labelled.push_back(i);
   };

@@ -77,6 +77,14 @@ struct CsrvFmt {
   int V = 32;
   int64_t n_long = 0;
   DevBuf long_rows;
+  // nnz-split stream mode (skewed row lengths, K6s): chunks of
+  // 32*EP entries, chunk_row[c] = row holding entry c*32*EP (chunk_row[nch] = N),
+  // two carry slots per chunk and the static fixup plan (as HybFmt)
+  bool stream = false;
+  int EP = 8;
+  int64_t nch = 0;
+  DevBuf chunk_row, carry_row, carry_val, fix_seg, fix_long;
+  int64_t fix_S = 0, fix_nlong = 0;
 };
 
 }  // namespace nitro
@@ -163,6 +171,9 @@ constexpr int64_t kCsrvSeg = 256;  // CSR-vector long-row segment (one warp, 8 e
 // HYB tail chunk = 32 * W entries per warp; W = 8 (fp32) / 4 (fp64: registers),
 // NITRO_HYB_W overrides (2/4/8).  Fixed per matrix at prepare time.
 int hyb_windows(size_t sv);
+// CSR-vector mode: the nnz-split stream kernel (K6s) for skewed row lengths
+// (row-length SD above the mean); NITRO_CSRV_STREAM=0/1 forces it off/on.
+bool csrv_stream_mode(const nitro_spmv *A);
 // bitmap index of diagonal offset d is d + G; the bitmap spans G + M bits
 inline int64_t diag_shift(const nitro_spmv *A) { return A->feat_G >= 0 ? A->feat_G : A->row0 + A->N - 1; }
 int num_sms();

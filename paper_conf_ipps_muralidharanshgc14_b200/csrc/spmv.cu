@@ -821,12 +821,150 @@ __global__ void __launch_bounds__(256) k_hyb_tail_ls(const int32_t *__restrict__
   }
 }
 
+// ------------------------------------------------------------------ K6s CSR-vector, nnz-split stream mode
+// For skewed row-length distributions (power-law rows, many empty rows) the
+// row-oriented K6 wastes lane groups on empty and short rows and serialises
+// hub rows; here every warp takes a fixed chunk of 32*EP nonzeros (EP = 8
+// fp32 / 4 fp64 consecutive entries per lane, 128-bit loads), so the work is
+// balanced by nnz.  The row of each entry is found from rowptr: the chunk's
+// rows [chunk_row[c], chunk_row[c+1]] are walked in windows of 32 row starts
+// held one per lane, and each entry binary-searches the window by shuffles
+// (5 steps, starts rebased to the chunk as 32-bit values).  Products are
+// formed and summed in fp64 (R2), lane-sequentially per row, with one
+// segmented scan across lanes (as K9b).  Rows wholly inside a chunk are
+// written directly; a chunk's first and last rows go to two carry slots that
+// k_hyb_fixup_seg<.., false> sums per row in slot order and STORES; empty
+// rows between a chunk's rows are zeroed by that chunk (rows before the first
+// nonempty row by chunk 0).  No atomics; deterministic.
+template <typename IT, typename VT, int EP>
+__global__ void __launch_bounds__(256) k_csr_stream(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
+                                                    const VT *__restrict__ val, const VT *__restrict__ x,
+                                                    VT *__restrict__ y, int64_t N, int64_t Z, int64_t nch,
+                                                    const int32_t *__restrict__ chunk_row,
+                                                    int32_t *__restrict__ carry_row, double *__restrict__ carry_val,
+                                                    bool vec, bool l2ef) {
+  static_assert(EP == 4 || EP == 8, "EP");
+  constexpr int64_t CH = 32 * EP;
+  const uint64_t pol = l2_policy(l2ef);
+  const int lane = threadIdx.x & 31;
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  if (warp == 0) {  // rows before the first nonempty row (chunk_row[0] = last row starting at 0)
+    const int r0 = nch > 0 ? chunk_row[0] : (int)N;
+    for (int r = lane; r < r0; r += 32) y[r] = (VT)0;
+  }
+  for (int64_t ch = warp; ch < nch; ch += nw) {
+    const int64_t c0 = ch * CH, cend = c0 + CH < Z ? c0 + CH : Z;
+    const int64_t e0 = c0 + (int64_t)lane * EP;
+    const int nv = e0 >= cend ? 0 : (cend - e0 < EP ? (int)(cend - e0) : EP);
+    int c[EP];
+    VT v[EP];
+    if (nv == EP && vec) {
+#pragma unroll
+      for (int k = 0; k < EP; k += 4) {
+        const int4 cc = ld_stream_i4(reinterpret_cast<const int4 *>(col + e0 + k), pol);
+        c[k] = cc.x; c[k + 1] = cc.y; c[k + 2] = cc.z; c[k + 3] = cc.w;
+        V4<VT> vv;
+        vv.load(val + e0 + k, pol);
+        v[k] = vv.v[0]; v[k + 1] = vv.v[1]; v[k + 2] = vv.v[2]; v[k + 3] = vv.v[3];
+      }
+    } else {
+#pragma unroll
+      for (int k = 0; k < EP; ++k) {
+        const bool ok = k < nv;
+        c[k] = ok ? ld_stream_i(col + e0 + k, pol) : 0;
+        v[k] = ok ? ld_stream(val + e0 + k, pol) : (VT)0;
+      }
+    }
+    double p[EP];
+#pragma unroll
+    for (int k = 0; k < EP; ++k) p[k] = k < nv ? (double)v[k] * (double)__ldg(x + c[k]) : 0.0;
+    // rows of the entries: windows of 32 row starts over [r_lo, r_hi]
+    const int r_lo = chunk_row[ch], r_nx = chunk_row[ch + 1];
+    const int r_hi = r_nx < (int)N ? r_nx : (int)N - 1;
+    int r[EP];
+#pragma unroll
+    for (int k = 0; k < EP; ++k) r[k] = k < nv ? r_lo : -2;
+    for (int w0 = r_lo; w0 <= r_hi; w0 += 32) {  // warp-uniform
+      const int rr = w0 + lane;
+      int rel = CH;  // row start rebased to the chunk, clamped to [-1, CH]
+      if (rr <= r_hi) {
+        const int64_t rs = (int64_t)rowptr[rr];
+        rel = rs < c0 ? -1 : (rs - c0 > CH ? (int)CH : (int)(rs - c0));
+        // an empty row strictly inside the chunk's row range: nobody else writes it
+        if (rr > r_lo && rr < r_nx && (int64_t)rowptr[rr + 1] == rs) y[rr] = (VT)0;
+      }
+      const int ws0 = __shfl_sync(kFull, rel, 0);
+#pragma unroll
+      for (int k = 0; k < EP; ++k) {
+        const int e = (int)(e0 - c0) + k;  // < CH
+        int pos = 0;
+#pragma unroll
+        for (int step = 16; step > 0; step >>= 1) {
+          const int t = __shfl_sync(kFull, rel, pos + step);
+          if (t <= e) pos += step;
+        }
+        if (k < nv && ws0 <= e) r[k] = w0 + pos;
+      }
+    }
+    const int first_row = r_lo;
+    const int lastl = (int)((cend - 1 - c0) / EP), lastk = (int)((cend - 1 - c0) % EP);
+    int my_last_k = 0;
+#pragma unroll
+    for (int k = 0; k < EP; ++k) my_last_k = k == lastk ? r[k] : my_last_k;
+    const int last_row = __shfl_sync(kFull, my_last_k, lastl);
+    if (lane == 0) { carry_row[2 * ch] = -1; carry_row[2 * ch + 1] = -1; }
+    __syncwarp();
+    auto emit = [&](int row, double s_) {  // a completed row segment (chunk ownership rule)
+      if (row == first_row) { carry_row[2 * ch] = row; carry_val[2 * ch] = s_; }
+      else if (row == last_row) { carry_row[2 * ch + 1] = row; carry_val[2 * ch + 1] = s_; }
+      else y[row] = (VT)s_;
+    };
+    const int fr = nv > 0 ? r[0] : -2;
+    int cur = fr;
+    double acc = 0.0, pf = 0.0;
+    bool boundary = false;
+#pragma unroll
+    for (int k = 0; k < EP; ++k) {
+      if (k < nv) {
+        if (r[k] != cur) {
+          if (!boundary) { pf = acc; boundary = true; }
+          else emit(cur, acc);
+          cur = r[k];
+          acc = 0.0;
+        }
+        acc += p[k];
+      }
+    }
+    const int lr = cur;
+    double s = acc;
+    const int prev_lr = __shfl_up_sync(kFull, lr, 1);
+    bool f = boundary || lane == 0 || fr != prev_lr;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const double t = __shfl_up_sync(kFull, s, o);
+      const bool tf = __shfl_up_sync(kFull, f, o);
+      if (lane >= o) {
+        if (!f) s += t;
+        f = f || tf;
+      }
+    }
+    const double prev_s = __shfl_up_sync(kFull, s, 1);
+    const int next_fr = __shfl_down_sync(kFull, fr, 1);
+    const bool next_valid = __shfl_down_sync(kFull, nv, 1) > 0 && lane < 31;
+    if (nv > 0) {
+      if (boundary) emit(fr, pf + ((lane > 0 && prev_lr == fr) ? prev_s : 0.0));
+      if (!(next_valid && next_fr == lr)) emit(lr, s);
+    }
+  }
+}
+
 // Carry fixup by the static plan of prepare_hyb: segment s = the carry slots
 // [seg[s], seg[s+1]) of one row, summed in slot order (slots left empty by the
 // tail kernel, row -1, skipped) and added to y once.  Segments of <= 32 slots:
 // a thread each (blocks [0, nshort)); longer ones (rows spanning many chunks,
 // e.g. R-MAT hubs): a warp each, lane-strided partial sums + a fixed xor tree.
-template <typename VT>
+template <typename VT, bool ADD = true>  // ADD: y[r] += carries (HYB); else y[r] = carries (K6s)
 __global__ void __launch_bounds__(256) k_hyb_fixup_seg(const int32_t *__restrict__ carry_row,
                                                        const double *__restrict__ carry_val,
                                                        const int32_t *__restrict__ seg, int64_t S,
@@ -840,7 +978,7 @@ __global__ void __launch_bounds__(256) k_hyb_fixup_seg(const int32_t *__restrict
       for (int j = j0; j < j1; ++j)
         if (carry_row[j] >= 0) tot += carry_val[j];
       const int r = carry_row[j0];
-      y[r] = (VT)((double)y[r] + tot);
+      y[r] = ADD ? (VT)((double)y[r] + tot) : (VT)tot;
     }
     return;
   }
@@ -857,7 +995,7 @@ __global__ void __launch_bounds__(256) k_hyb_fixup_seg(const int32_t *__restrict
     for (int o = 16; o > 0; o >>= 1) t += __shfl_xor_sync(kFull, t, o);
     if (lane == 0) {
       const int r = carry_row[j0];
-      y[r] = (VT)((double)y[r] + t);
+      y[r] = ADD ? (VT)((double)y[r] + t) : (VT)t;
     }
   }
 }
@@ -1128,6 +1266,29 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
     case NITRO_CSR_VECTOR: {
       if (part) return fail(NITRO_E_INVALID_ARG, "CSR-vector has no row-range launch");
       if (N == 0) break;
+      if (A->csrv.stream) {  // K6s: nnz-split chunks + carry fixup
+        const int64_t nch = A->csrv.nch;
+        const bool vec = ((reinterpret_cast<uintptr_t>(A->col) | reinterpret_cast<uintptr_t>(val)) & 15) == 0;
+        const unsigned gs = grid_cap(std::max<int64_t>((nch + 7) / 8, 1), 16);
+        if (A->csrv.EP == 4)
+          k_csr_stream<IT, VT, 4><<<gs, 256, 0, s>>>(rp, A->col, val, x, y, N, A->Z, nch,
+                                                     A->csrv.chunk_row.as<int32_t>(), A->csrv.carry_row.as<int32_t>(),
+                                                     A->csrv.carry_val.as<double>(), vec, l2_evict_first());
+        else
+          k_csr_stream<IT, VT, 8><<<gs, 256, 0, s>>>(rp, A->col, val, x, y, N, A->Z, nch,
+                                                     A->csrv.chunk_row.as<int32_t>(), A->csrv.carry_row.as<int32_t>(),
+                                                     A->csrv.carry_val.as<double>(), vec, l2_evict_first());
+        if (nch > 0) {
+          const unsigned nshort = grid_cap((A->csrv.fix_S + 255) / 256, 8);
+          const unsigned nlong_blk = A->csrv.fix_nlong > 0
+                                         ? (unsigned)std::min<int64_t>((A->csrv.fix_nlong + 7) / 8, (int64_t)num_sms() * 4)
+                                         : 0;
+          k_hyb_fixup_seg<VT, false><<<nshort + nlong_blk, 256, 0, s>>>(
+              A->csrv.carry_row.as<int32_t>(), A->csrv.carry_val.as<double>(), A->csrv.fix_seg.as<int32_t>(),
+              A->csrv.fix_S, A->csrv.fix_long.as<int32_t>(), A->csrv.fix_nlong, nshort, y);
+        }
+        break;
+      }
       const int64_t nseg = A->csrv.n_long;
       int32_t *seg_row = A->csrv.long_rows.as<int32_t>();
       int32_t *seg_k = seg_row + nseg;
@@ -1307,6 +1468,7 @@ nitro_status_t launch_flush(nitro_spmv *A, cudaStream_t s) {
 
 int launches_of(const nitro_spmv *A, int variant) {
   if (A->N == 0) return 0;
+  if (variant == NITRO_CSR_VECTOR && A->csrv.stream) return A->csrv.nch > 0 ? 2 : 1;
   if (variant == NITRO_HYB) return A->hyb.Zt > 0 ? 3 : 1;
   return 1;
 }

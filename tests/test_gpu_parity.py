@@ -341,7 +341,7 @@ def _csr_impls(A, x, cuda, rowptr32=None, shift=(0, 0, 0)):
     xd = torch.from_numpy(x).to(cuda)
     out = {}
     for v in (n.CSR_SCALAR, n.CSR_VECTOR):
-        for impl in (n.CSR_IMPL_AUTO, n.CSR_IMPL_DIRECT, n.CSR_IMPL_STAGED):
+        for impl in (n.CSR_IMPL_AUTO, n.CSR_IMPL_DIRECT, n.CSR_IMPL_STAGED, n.CSR_IMPL_STREAM):
             M.set_csr_impl(impl)
             y = torch.full((A.rows,), float("nan"), dtype=xd.dtype, device=cuda)
             M.run(v, xd, y)
@@ -364,14 +364,21 @@ def _impl_mats():
 def test_csr_impls_bit_identical(cuda, name, A):
     """The TMA row-tile pipeline (auto / forced, incl. tiles computed from
     global memory when their span overflows a stage) and the direct kernels run
-    the same per-row arithmetic: y bit-identical, and within the oracle bound."""
+    the same per-row arithmetic: y bit-identical, and within the oracle bound.
+    The nnz-split stream mode of CSR-vector (K6s; AUTO picks it when the
+    row-length SD exceeds the mean) sums in another association: within the
+    bound, deterministic, and AUTO equals it exactly when it is picked."""
+    n = nitro()
     x = synth.vector(A.cols, seed=41, mode=0, fp64=A.fp64)
     y_ref, r = oracle.spmv(A, x)
+    skewed = oracle.features(A)["sd"] > oracle.features(A)["mean"]
     for rp32 in ((True, False) if A.nnz < 2**31 else (False,)):
         out = _csr_impls(A, x, cuda, rowptr32=rp32)
         for (v, impl), y in out.items():
             check_y(y, y_ref, r, A.fp64, f"{name} v{v} impl{impl} rp32={rp32}")
-            assert np.array_equal(y, out[(v, 1)]), (name, v, impl, rp32)
+            stream = v == n.CSR_VECTOR and (impl == n.CSR_IMPL_STREAM or (impl == n.CSR_IMPL_AUTO and skewed))
+            want = out[(v, n.CSR_IMPL_STREAM)] if stream else out[(v, n.CSR_IMPL_DIRECT)]
+            assert np.array_equal(y, want), (name, v, impl, rp32)
 
 
 @pytest.mark.parametrize("shift", [(1, 1, 1), (3, 2, 1), (2, 3, 3)])
@@ -380,9 +387,11 @@ def test_csr_staged_misaligned_spans(cuda, shift):
     x = synth.vector(A.cols, seed=42)
     y_ref, r = oracle.spmv(A, x)
     out = _csr_impls(A, x, cuda, rowptr32=True, shift=shift)
+    n = nitro()
     for (v, impl), y in out.items():
         check_y(y, y_ref, r, False, f"shift {shift} v{v} impl{impl}")
-        assert np.array_equal(y, out[(v, 1)]), (shift, v, impl)
+        if not (v == n.CSR_VECTOR and impl == n.CSR_IMPL_STREAM):   # misaligned arrays: the scalar-load path of K6s
+            assert np.array_equal(y, out[(v, 1)]), (shift, v, impl)
 
 
 def test_run_host_matches_device(cuda):
@@ -674,3 +683,43 @@ def test_binding_rejects_bad_vectors(cuda):
         with pytest.raises(ValueError):
             M.run(n.CSR_SCALAR, good, bad[: A.rows] if bad.numel() >= A.rows else bad)
     M.run(n.CSR_SCALAR, good)
+
+
+def _stream_mats():
+    yield "rmat14_fp32", synth.rmat(14, 16, seed=31, fp64=False)
+    yield "rmat13_fp64", synth.rmat(13, 8, seed=32, fp64=True)
+    yield "long_row", long_row_matrix(L=60_000, N=4000)
+    yield "empty_runs", Csr(300, 300, np.array([0] * 100 + [1] * 150 + [40] * 51, np.int64),
+                            np.concatenate([[5], np.arange(39)]).astype(np.int32),
+                            np.linspace(1, 2, 40).astype(np.float32), False)
+    yield "uniform_k1", synth.uniform(5000, 1, seed=33)          # chunks spanning many rows (windows)
+    yield "2d5_int", synth.stencil("2d5", 70)
+
+
+@pytest.mark.parametrize("name,A", list(_stream_mats()))
+def test_csr_stream_mode(cuda, name, A):
+    """K6s (nnz-split chunks, rows from rowptr by warp binary search, carry
+    fixup that stores): within the bound on skewed, long-row, empty-run and
+    one-entry-per-row matrices; exact on integer data; empty rows written 0
+    (y starts as NaN); deterministic across runs."""
+    import torch
+    n = nitro()
+    exact = name.endswith("_int")
+    x = synth.vector(A.cols, seed=7, mode=1 if exact else 0, fp64=A.fp64)
+    y_ref, r = oracle.spmv(A, x)
+    M, _ = handle(A, cuda)
+    M.set_csr_impl(n.CSR_IMPL_STREAM)
+    xd = torch.from_numpy(x).to(cuda)
+    ys = []
+    for _ in range(2):
+        y = torch.full((A.rows,), float("nan"), dtype=xd.dtype, device=cuda)
+        M.run(n.CSR_VECTOR, xd, y)
+        torch.cuda.synchronize()
+        ys.append(y.cpu().numpy())
+    assert M.format_info(n.CSR_VECTOR)["width"] == 0          # stream mode active
+    assert np.all(np.isfinite(ys[0]))                          # every row written (empty rows = 0)
+    if exact:
+        assert np.array_equal(ys[0].astype(np.float64), y_ref)
+    else:
+        check_y(ys[0], y_ref, r, A.fp64, name)
+    assert np.array_equal(ys[0], ys[1])
