@@ -401,6 +401,30 @@ nitro_status_t nitro_dist_init_local(int rank, int nranks, int device, nitro_dis
  * to the single-GPU features of the whole matrix.  Collective; syncs. */
 nitro_status_t nitro_dist_features(nitro_dist *D, nitro_spmv *A_local, nitro_spmv_feat *out);
 
+/* Solver-loop mode: in loops where the y of one
+ * multiply is the x of the next (power iteration, Krylov-type methods), the
+ * SpMV epilogue stores every y_i straight into EVERY rank's next x layout
+ * (all-gather layout, block r at r*B): through NCCL symmetric-memory windows
+ * (ncclMemAlloc + ncclCommWindowRegister, peer addresses from the NCCL device
+ * API, one LSA barrier per step) on NCCL ranks, through the group's buffers
+ * on the loopback transport.  No separate all-gather runs: the exchange is
+ * spread over the multiply.  Two layouts alternate (x_k is read from one,
+ * x_{k+1} written into the other).  CSR-scalar, ELL and DIA have the fused
+ * epilogue; other variants compute the rank's block and push it with a copy
+ * kernel.  Requires a handle created with the all-gather exchange
+ * (NITRO_E_UNSUPPORTED otherwise) and, on NCCL, every rank in one NVLink
+ * domain.  create / start / step are collective (all ranks, same order). */
+typedef struct nitro_dist_loop nitro_dist_loop;
+nitro_status_t nitro_dist_loop_create(nitro_dist *D, nitro_spmv *A_local, nitro_dist_loop **out);
+void nitro_dist_loop_destroy(nitro_dist_loop *L);
+/* Device address of this rank's block of the CURRENT x (write x_0 here before start). */
+nitro_status_t nitro_dist_loop_x(nitro_dist_loop *L, void **d_x_local);
+/* Exchange x_0 once (all-gather into every rank's current layout). */
+nitro_status_t nitro_dist_loop_start(nitro_dist_loop *L);
+/* One multiply y = A x_k; x_{k+1} = y on every rank (fused epilogue +
+ * barrier); d_y_local (nullable) also receives this rank's y block. */
+nitro_status_t nitro_dist_loop_step(nitro_dist_loop *L, int variant, void *d_y_local);
+
 /* LOOPBACK transport: P rank handles inside ONE process on ONE GPU, each
  * driven by its own host thread.  Every collective of nitro_dist_* (the
  * exchange-plan all-gather and send/recv in create, the per-multiply x

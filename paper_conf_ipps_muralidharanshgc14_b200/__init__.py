@@ -179,6 +179,11 @@ _SIGS = {
     "nitro_dist_init_local": ([_int, _int, _int, _P(_vp)], _int),
     "nitro_dist_loopback_create": ([_int, _int, _P(_vp)], _int),
     "nitro_dist_format_info": ([_vp, _int, _P(FormatInfo)], _int),
+    "nitro_dist_loop_create": ([_vp, _vp, _P(_vp)], _int),
+    "nitro_dist_loop_destroy": ([_vp], None),
+    "nitro_dist_loop_x": ([_vp, _P(_vp)], _int),
+    "nitro_dist_loop_start": ([_vp], _int),
+    "nitro_dist_loop_step": ([_vp, _int, _vp], _int),
     "nitro_dist_loopback_destroy": ([_vp], None),
     "nitro_dist_init_loopback": ([_vp, _int, _P(_vp)], _int),
     "nitro_dist_spmv_create_ex": ([_vp, _i64, _vp, _i64, _vp, _int, _vp, _vp, _int, _int, _P(_vp)], _int),
@@ -826,3 +831,35 @@ class Dist:
         f = Feat()
         _check(_L.nitro_dist_features(self.h, A.h, ctypes.byref(f)))
         return f.as_dict()
+
+    def loop(self, A: SpMV) -> "DistLoop":
+        """Solver-loop mode (nitro_dist_loop_*, f3 (ii)): y -> next x fused into the epilogue."""
+        return DistLoop(self, A)
+
+
+class DistLoop:
+    """nitro_dist_loop: x_{k+1} = A x_k with the exchange fused into the SpMV epilogue."""
+
+    def __init__(self, D: "Dist", A: SpMV):
+        h = ctypes.c_void_p()
+        _check(_L.nitro_dist_loop_create(D.h, A.h, ctypes.byref(h)))
+        self.h, self.D, self.A = h, D, A
+
+    def x(self):
+        """torch view of this rank's block of the current x (write x_0 here, then start())."""
+        p = ctypes.c_void_p()
+        _check(_L.nitro_dist_loop_x(self.h, ctypes.byref(p)))
+        return _wrap_device(p.value, self.A.rows, self.A.dtype, self.A.device)
+
+    def start(self):
+        _check(_L.nitro_dist_loop_start(self.h))
+
+    def step(self, v: int, y_local=None):
+        _check(_L.nitro_dist_loop_step(self.h, v, None if y_local is None else
+                                       _dev_vec(y_local, self.A.rows, self.A.dtype, self.A.device, "y_local")))
+        return y_local
+
+    def close(self):
+        if getattr(self, "h", None):
+            _L.nitro_dist_loop_destroy(self.h)
+            self.h = None

@@ -151,6 +151,20 @@ nitro_status_t prepare_csrv(nitro_spmv *A);
 
 // spmv.cu
 nitro_status_t launch_spmv(nitro_spmv *A, int variant, const void *x, void *y, cudaStream_t s);
+// Fused y -> x epilogue of the solver-loop mode: every
+// computed y_i (local row i of this launch) is also stored at element
+// row_off + i of each of the n destination arrays dst[q] (device array of
+// device pointers: each rank's next-x layout at this rank's block; peer
+// memory through NCCL symmetric windows, or loopback buffers).
+struct PeerOut {
+  void *const *dst = nullptr;
+  int n = 0;
+  int64_t row_off = 0;
+};
+// CSR-scalar, ELL and DIA only (NITRO_E_UNSUPPORTED otherwise); y may be NULL
+// (peer stores only).
+nitro_status_t launch_spmv_fused(nitro_spmv *A, int variant, const void *x, void *y, const PeerOut &po,
+                                 cudaStream_t s);
 // rows [r0, r1) only (CSR-scalar, ELL, DIA: row-separable launches; r0 a multiple of 32)
 nitro_status_t launch_spmv_rows(nitro_spmv *A, int variant, const void *x, void *y, cudaStream_t s, int64_t r0,
                                 int64_t r1);

@@ -58,6 +58,21 @@ __device__ __forceinline__ void store4(VT *y, int64_t i0, int64_t N, const doubl
   }
 }
 
+// y stores of a launch, optionally fused with the f3 (ii) peer stores (FUSED:
+// each value also goes to element row_off + i of every dst[q]; y may be NULL)
+template <bool FUSED, typename VT>
+__device__ __forceinline__ void out1(VT *y, const PeerOut &po, int64_t i, VT v) {
+  if (!FUSED || y) y[i] = v;
+  if constexpr (FUSED)
+    for (int q = 0; q < po.n; ++q) reinterpret_cast<VT *>(po.dst[q])[po.row_off + i] = v;
+}
+template <bool FUSED, typename VT>
+__device__ __forceinline__ void out4(VT *y, const PeerOut &po, int64_t i0, int64_t N, const double *acc) {
+  if (!FUSED || y) store4<VT>(y, i0, N, acc);
+  if constexpr (FUSED)
+    for (int q = 0; q < po.n; ++q) store4<VT>(reinterpret_cast<VT *>(po.dst[q]) + po.row_off, i0, N, acc);
+}
+
 // ------------------------------------------------------------------ K5 CSR-scalar
 // Row arithmetic shared by every CSR-scalar implementation (R2):
 // fp32 (fp64) FFMA partials over 16-term chunks counted from the row start,
@@ -95,10 +110,10 @@ __device__ __forceinline__ double csr_row(XI a, XI b, const VT *__restrict__ x, 
   return acc;
 }
 
-template <int H, typename IT, typename VT>
+template <int H, typename IT, typename VT, bool FUSED = false>
 __global__ void __launch_bounds__(256) k_csr_scalar(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
                                                     const VT *__restrict__ val, const VT *__restrict__ x,
-                                                    VT *__restrict__ y, int64_t N) {
+                                                    VT *__restrict__ y, int64_t N, const PeerOut po = PeerOut{}) {
   // thread per row ("CSR": one thread walks one row)
   if constexpr (sizeof(VT) == 4) {
     // fp32: row-rebased pointers and 32-bit offsets (the kernel is issue-bound;
@@ -109,13 +124,13 @@ __global__ void __launch_bounds__(256) k_csr_scalar(const IT *__restrict__ rowpt
       const VT *vp = val + a;
       auto ldc = [&](int e) { return __ldg(cp + e); };
       auto ldv = [&](int e) { return __ldg(vp + e); };
-      y[i] = (VT)csr_row<H, VT, int>(0, (int)((int64_t)rowptr[i + 1] - a), x, ldc, ldv);
+      out1<FUSED, VT>(y, po, i, (VT)csr_row<H, VT, int>(0, (int)((int64_t)rowptr[i + 1] - a), x, ldc, ldv));
     }
   } else {
     auto ldc = [&](int64_t e) { return __ldg(col + e); };
     auto ldv = [&](int64_t e) { return __ldg(val + e); };
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < N; i += (int64_t)gridDim.x * blockDim.x)
-      y[i] = (VT)csr_row<H, VT>((int64_t)rowptr[i], (int64_t)rowptr[i + 1], x, ldc, ldv);
+      out1<FUSED, VT>(y, po, i, (VT)csr_row<H, VT>((int64_t)rowptr[i], (int64_t)rowptr[i + 1], x, ldc, ldv));
   }
 }
 
@@ -523,10 +538,11 @@ __global__ void __launch_bounds__(kStgThr, 2) k_csr_staged(const IT *__restrict_
 // slots are all issued before the first FMA (explicit register batches: the
 // compiler otherwise reuses one register quad and serialises the slots), so
 // each thread keeps U x (16 + 16|32) bytes of HBM traffic in flight.
-template <typename VT, int U>  // U <= 16: terms per fp32 partial
+template <typename VT, int U, bool FUSED = false>  // U <= 16: terms per fp32 partial
 __global__ void __launch_bounds__(256) k_ell(const int32_t *__restrict__ ecol, const VT *__restrict__ eval,
                                              const VT *__restrict__ x, VT *__restrict__ y, int64_t N, int64_t K,
-                                             int64_t ld, int64_t nr, bool l2ef, int pf, bool pfh) {
+                                             int64_t ld, int64_t nr, bool l2ef, int pf, bool pfh,
+                                             const PeerOut po = PeerOut{}) {
   // rows [0, nr) (nr <= ld: ld for a whole multiply incl. padding, less for a row chunk)
   const uint64_t pol = l2_policy(l2ef);
   const int64_t nq = (nr + 3) >> 2;
@@ -580,7 +596,7 @@ __global__ void __launch_bounds__(256) k_ell(const int32_t *__restrict__ ecol, c
 #pragma unroll
       for (int t = 0; t < 4; ++t) acc[t] += (double)part[t];
     }
-    store4<VT>(y, i0, N, acc);
+    out4<FUSED, VT>(y, po, i0, N, acc);
   }
 }
 
@@ -594,12 +610,13 @@ __global__ void __launch_bounds__(256) k_ell(const int32_t *__restrict__ ecol, c
 // resident warps matter more than per-thread bytes in flight.  (U and DS stay
 // template parameters fixed at 1: the loop below is written for them.)
 constexpr int kDiaSmemOffs = 12288;
-template <typename VT, bool GOFF, int U = 1, int DS = 1>  // GOFF: offsets read through L1 (D > kDiaSmemOffs)
+template <typename VT, bool GOFF, bool FUSED = false, int U = 1, int DS = 1>  // GOFF: offsets read through L1 (D > kDiaSmemOffs)
 __global__ void __launch_bounds__(256, sizeof(VT) == 4 ? 8 : 1)  // fp32: <= 32 regs, full occupancy
     k_dia(const int32_t *__restrict__ offs, const VT *__restrict__ dval,
                                              const VT *__restrict__ x, VT *__restrict__ y, int64_t N, int64_t M,
                                              int64_t D, int64_t ld, int64_t nr, int64_t row0, int64_t off_min,
-                                             int64_t off_max, bool x_aligned, bool l2ef, int pf, bool pfh) {
+                                             int64_t off_max, bool x_aligned, bool l2ef, int pf, bool pfh,
+                                             const PeerOut po = PeerOut{}) {
   constexpr int64_t RB = 1024 / DS;  // rows per block iteration
   const uint64_t pol = l2_policy(l2ef);
   extern __shared__ int s_off[];
@@ -697,7 +714,7 @@ __global__ void __launch_bounds__(256, sizeof(VT) == 4 ? 8 : 1)  // fp32: <= 32 
     for (int o = 1; o < DS; o <<= 1)
 #pragma unroll
       for (int t = 0; t < 4; ++t) acc[t] += __shfl_xor_sync(kFull, acc[t], o);
-    if (active && q == 0) store4<VT>(y, i0, N, acc);
+    if (active && q == 0) out4<FUSED, VT>(y, po, i0, N, acc);
   }
 }
 
@@ -826,16 +843,17 @@ __global__ void __launch_bounds__(256) k_hyb_tail_ls(const int32_t *__restrict__
 // row-oriented K6 wastes lane groups on empty and short rows and serialises
 // hub rows; here every warp takes a fixed chunk of 32*EP nonzeros (EP = 8
 // fp32 / 4 fp64 consecutive entries per lane, 128-bit loads), so the work is
-// balanced by nnz.  The row of each entry is found from rowptr: the chunk's
-// rows [chunk_row[c], chunk_row[c+1]] are walked in windows of 32 row starts
-// held one per lane, and each entry binary-searches the window by shuffles
-// (5 steps, starts rebased to the chunk as 32-bit values).  Products are
-// formed and summed in fp64 (R2), lane-sequentially per row, with one
-// segmented scan across lanes (as K9b).  Rows wholly inside a chunk are
-// written directly; a chunk's first and last rows go to two carry slots that
-// k_hyb_fixup_seg<.., false> sums per row in slot order and STORES; empty
-// rows between a chunk's rows are zeroed by that chunk (rows before the first
-// nonempty row by chunk 0).  No atomics; deterministic.
+// balanced by nnz.  The row of each entry is found from rowptr: the starts
+// of the chunk's rows (chunk_row[c], chunk_row[c+1]] are counted at their
+// chunk positions in shared memory (windows of 32 rows, one per lane) and a
+// prefix sum over the positions gives every entry's row.  Products are formed
+// and summed in fp64 (R2), lane-sequentially per row, with one segmented scan
+// across lanes (as K9b).  Rows wholly inside a chunk are written directly; a
+// chunk's first and last rows go to two carry slots that k_hyb_fixup_seg<..,
+// false> sums per row in slot order and STORES; empty rows between a chunk's
+// rows are zeroed by that chunk (rows before the first nonempty row by chunk
+// 0).  No global atomics (the shared-memory counts are integers):
+// deterministic.
 template <typename IT, typename VT, int EP>
 __global__ void __launch_bounds__(256) k_csr_stream(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
                                                     const VT *__restrict__ val, const VT *__restrict__ x,
@@ -845,6 +863,7 @@ __global__ void __launch_bounds__(256) k_csr_stream(const IT *__restrict__ rowpt
                                                     bool vec, bool l2ef) {
   static_assert(EP == 4 || EP == 8, "EP");
   constexpr int64_t CH = 32 * EP;
+  __shared__ __align__(16) int s_cnt[8][CH];  // per warp: row starts per chunk position
   const uint64_t pol = l2_policy(l2ef);
   const int lane = threadIdx.x & 31;
   const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
@@ -853,12 +872,12 @@ __global__ void __launch_bounds__(256) k_csr_stream(const IT *__restrict__ rowpt
     const int r0 = nch > 0 ? chunk_row[0] : (int)N;
     for (int r = lane; r < r0; r += 32) y[r] = (VT)0;
   }
-  for (int64_t ch = warp; ch < nch; ch += nw) {
+  // software pipeline over the warp's chunks: the next chunk's (col, val) and
+  // row range are loaded while the current chunk's gathers and row work run
+  auto load = [&](int64_t ch, int (&c)[EP], VT (&v)[EP], int &rlo, int &rnx) {
     const int64_t c0 = ch * CH, cend = c0 + CH < Z ? c0 + CH : Z;
     const int64_t e0 = c0 + (int64_t)lane * EP;
     const int nv = e0 >= cend ? 0 : (cend - e0 < EP ? (int)(cend - e0) : EP);
-    int c[EP];
-    VT v[EP];
     if (nv == EP && vec) {
 #pragma unroll
       for (int k = 0; k < EP; k += 4) {
@@ -872,40 +891,74 @@ __global__ void __launch_bounds__(256) k_csr_stream(const IT *__restrict__ rowpt
 #pragma unroll
       for (int k = 0; k < EP; ++k) {
         const bool ok = k < nv;
-        c[k] = ok ? ld_stream_i(col + e0 + k, pol) : 0;
+        c[k] = ok ? ld_stream_i(col + e0 + k, pol) : -1;
         v[k] = ok ? ld_stream(val + e0 + k, pol) : (VT)0;
       }
     }
+    rlo = chunk_row[ch];
+    rnx = chunk_row[ch + 1];
+  };
+  int cn[EP], rlo_n = 0, rnx_n = 0;
+  VT vn[EP];
+  if (warp < nch) load(warp, cn, vn, rlo_n, rnx_n);
+  for (int64_t ch = warp; ch < nch; ch += nw) {
+    const int64_t c0 = ch * CH, cend = c0 + CH < Z ? c0 + CH : Z;
+    const int64_t e0 = c0 + (int64_t)lane * EP;
+    const int nv = e0 >= cend ? 0 : (cend - e0 < EP ? (int)(cend - e0) : EP);
+    VT v[EP], xv[EP];
+#pragma unroll
+    for (int k = 0; k < EP; ++k) {
+      v[k] = vn[k];
+      xv[k] = k < nv ? __ldg(x + cn[k]) : (VT)0;
+    }
+    const int r_lo = rlo_n, r_nx = rnx_n;
+    if (ch + nw < nch) load(ch + nw, cn, vn, rlo_n, rnx_n);
     double p[EP];
 #pragma unroll
-    for (int k = 0; k < EP; ++k) p[k] = k < nv ? (double)v[k] * (double)__ldg(x + c[k]) : 0.0;
-    // rows of the entries: windows of 32 row starts over [r_lo, r_hi]
-    const int r_lo = chunk_row[ch], r_nx = chunk_row[ch + 1];
+    for (int k = 0; k < EP; ++k) p[k] = (double)v[k] * (double)xv[k];
+    // rows of the entries: row(e) = r_lo + #{rows r in (r_lo, r_hi] starting at
+    // or before chunk position e}.  The rows' starts are counted into a per-warp
+    // shared array over the chunk's positions (windows of 32 rows, one per
+    // lane, smem atomics), then each lane prefix-sums its EP positions and one
+    // warp scan adds the lanes before it.
     const int r_hi = r_nx < (int)N ? r_nx : (int)N - 1;
-    int r[EP];
+    int *cnt = s_cnt[threadIdx.x >> 5];
+    {
+      int4 *c4 = reinterpret_cast<int4 *>(cnt + lane * EP);
 #pragma unroll
-    for (int k = 0; k < EP; ++k) r[k] = k < nv ? r_lo : -2;
-    for (int w0 = r_lo; w0 <= r_hi; w0 += 32) {  // warp-uniform
+      for (int k = 0; k < EP; k += 4) c4[k / 4] = make_int4(0, 0, 0, 0);
+    }
+    __syncwarp();
+    for (int w0 = r_lo + 1; w0 <= r_hi; w0 += 32) {  // warp-uniform
       const int rr = w0 + lane;
-      int rel = CH;  // row start rebased to the chunk, clamped to [-1, CH]
       if (rr <= r_hi) {
         const int64_t rs = (int64_t)rowptr[rr];
-        rel = rs < c0 ? -1 : (rs - c0 > CH ? (int)CH : (int)(rs - c0));
+        if (rs - c0 < CH) atomicAdd(cnt + (int)(rs - c0), 1);  // rs > c0 for every row after r_lo
         // an empty row strictly inside the chunk's row range: nobody else writes it
-        if (rr > r_lo && rr < r_nx && (int64_t)rowptr[rr + 1] == rs) y[rr] = (VT)0;
+        if (rr < r_nx && (int64_t)rowptr[rr + 1] == rs) y[rr] = (VT)0;
       }
-      const int ws0 = __shfl_sync(kFull, rel, 0);
+    }
+    __syncwarp();
+    int r[EP];
+    {
+      int inc[EP];
+      const int4 *c4 = reinterpret_cast<const int4 *>(cnt + lane * EP);
 #pragma unroll
-      for (int k = 0; k < EP; ++k) {
-        const int e = (int)(e0 - c0) + k;  // < CH
-        int pos = 0;
-#pragma unroll
-        for (int step = 16; step > 0; step >>= 1) {
-          const int t = __shfl_sync(kFull, rel, pos + step);
-          if (t <= e) pos += step;
-        }
-        if (k < nv && ws0 <= e) r[k] = w0 + pos;
+      for (int k = 0; k < EP; k += 4) {
+        const int4 t = c4[k / 4];
+        inc[k] = t.x; inc[k + 1] = t.y; inc[k + 2] = t.z; inc[k + 3] = t.w;
       }
+#pragma unroll
+      for (int k = 1; k < EP; ++k) inc[k] += inc[k - 1];
+      int ex = inc[EP - 1];  // lane total -> exclusive prefix over lanes
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int t = __shfl_up_sync(kFull, ex, o);
+        if (lane >= o) ex += t;
+      }
+      ex -= inc[EP - 1];
+#pragma unroll
+      for (int k = 0; k < EP; ++k) r[k] = k < nv ? r_lo + ex + inc[k] : -2;
     }
     const int first_row = r_lo;
     const int lastl = (int)((cend - 1 - c0) / EP), lastk = (int)((cend - 1 - c0) % EP);
@@ -1389,6 +1442,72 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
 }
 
 }  // namespace
+
+namespace {
+// whole-multiply launches of the row-separable variants with the f3 (ii)
+// peer-store epilogue (same kernels, FUSED instantiation: identical
+// arithmetic, so y and the peer copies are bit-identical to launch_spmv's y)
+template <typename IT, typename VT>
+nitro_status_t run_fused_t(nitro_spmv *A, int variant, const VT *x, VT *y, const PeerOut &po, cudaStream_t s) {
+  const int64_t N = A->N;
+  if (N == 0) return NITRO_OK;
+  const IT *rp = (const IT *)A->rowptr;
+  const VT *val = (const VT *)A->val;
+  switch (variant) {
+    case NITRO_CSR_SCALAR: {
+      const unsigned g = grid_cap((N + 255) / 256, 16);
+      switch (csrs_head(A)) {
+        case 4: k_csr_scalar<4, IT, VT, true><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, po); break;
+        case 16: k_csr_scalar<16, IT, VT, true><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, po); break;
+        default: k_csr_scalar<8, IT, VT, true><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, po); break;
+      }
+      break;
+    }
+    case NITRO_ELL: {
+      const bool local = diag_local(A);
+      const int64_t K = A->ell.K, ld = A->ell.ld;
+      const int pf = local ? ell_prefetch() : 0;
+      const unsigned g = grid_cap(((ld + 3) / 4 + 255) / 256, 16);
+      const bool small = (double)K * (double)ld * (double)(sizeof(VT) + 4) <= 2.0 * 1073741824.0;
+      if (ell_batch(sizeof(VT), local && small) == 1)
+        k_ell<VT, 1, true><<<g, 256, 0, s>>>(A->ell.col.as<int32_t>(), A->ell.val.as<VT>(), x, y, N, K, ld, ld,
+                                             l2_evict_first(), pf, prefetch_hint(), po);
+      else
+        k_ell<VT, 2, true><<<g, 256, 0, s>>>(A->ell.col.as<int32_t>(), A->ell.val.as<VT>(), x, y, N, K, ld, ld,
+                                             l2_evict_first(), pf, prefetch_hint(), po);
+      break;
+    }
+    case NITRO_DIA: {
+      const int64_t nr = A->dia.ld, row0 = A->row0;
+      const bool x_al = ((reinterpret_cast<uintptr_t>(x) & 15) == 0) && (row0 % 4 == 0);
+      const unsigned g = grid_cap((nr + 1023) / 1024, dia_blocks_per_sm());
+      if (A->dia.D <= kDiaSmemOffs)
+        k_dia<VT, false, true><<<g, 256, (size_t)std::max<int64_t>(A->dia.D, 1) * 4, s>>>(
+            A->dia.off.as<int32_t>(), A->dia.val.as<VT>(), x, y, N, A->M, A->dia.D, A->dia.ld, nr, row0,
+            A->dia.off_min, A->dia.off_max, x_al, l2_evict_first(), dia_prefetch(), prefetch_hint(), po);
+      else
+        k_dia<VT, true, true><<<g, 256, 0, s>>>(A->dia.off.as<int32_t>(), A->dia.val.as<VT>(), x, y, N, A->M,
+                                                A->dia.D, A->dia.ld, nr, row0, A->dia.off_min, A->dia.off_max, x_al,
+                                                l2_evict_first(), dia_prefetch(), prefetch_hint(), po);
+      break;
+    }
+    default:
+      return fail(NITRO_E_UNSUPPORTED, "fused peer-store epilogue: CSR-scalar, ELL and DIA only");
+  }
+  NITRO_CUDA(cudaGetLastError());
+  return NITRO_OK;
+}
+}  // namespace
+
+nitro_status_t launch_spmv_fused(nitro_spmv *A, int variant, const void *x, void *y, const PeerOut &po,
+                                 cudaStream_t s) {
+  if (A->rp64) {
+    if (A->fp64) return run_fused_t<int64_t, double>(A, variant, (const double *)x, (double *)y, po, s);
+    return run_fused_t<int64_t, float>(A, variant, (const float *)x, (float *)y, po, s);
+  }
+  if (A->fp64) return run_fused_t<int32_t, double>(A, variant, (const double *)x, (double *)y, po, s);
+  return run_fused_t<int32_t, float>(A, variant, (const float *)x, (float *)y, po, s);
+}
 
 nitro_status_t launch_spmv(nitro_spmv *A, int variant, const void *x, void *y, cudaStream_t s) {
   if (A->rp64) {

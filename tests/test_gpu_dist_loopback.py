@@ -150,3 +150,96 @@ def test_loopback_empty_rank_and_uneven_blocks(cuda):
         res = run_group(A, x, 4, exchange, [n.CSR_SCALAR, n.CSR_VECTOR, n.HYB], cuda, bounds=bounds)
         for v, y in res["y"].items():
             assert np.all(np.abs(y.astype(np.float64) - y_ref) <= 1e-5 * r + 1e-30), (exchange, v)
+
+
+# ------------------------------------------------------------------ f3 (ii): fused y -> x epilogue (solver loop)
+def _loop_ref(A, x0, steps):
+    """x_{k+1} = A x_k with the oracle (fp64); integer data keeps it exact."""
+    xs, x = [], np.asarray(x0, np.float64)
+    for _ in range(steps):
+        x, _ = oracle.spmv(A, x)
+        xs.append(x)
+    return xs
+
+
+def run_loop_group(A, x0, P, variant, steps, cuda):
+    import torch
+    n = nitro()
+    bounds = n.dist_partition(np.asarray(A.rowptr, np.int64), P)
+    group = n.Loopback(P, 0)
+    ys = [[None] * P for _ in range(steps)]
+    xnext = [None] * P
+    err = []
+
+    def rank(q):
+        try:
+            torch.cuda.set_device(0)
+            with torch.cuda.stream(torch.cuda.Stream()):
+                D = n.Dist.loopback(group, q)
+                blk = synth.to_device(block(A, bounds[q], bounds[q + 1]), cuda)
+                M = D.spmv(A.rows, bounds, blk.rowptr, blk.colidx, blk.vals, exchange=0)
+                L = D.loop(M)
+                L.x().copy_(torch.from_numpy(np.ascontiguousarray(x0[bounds[q]:bounds[q + 1]])).to(cuda))
+                L.start()
+                for k in range(steps):
+                    y = torch.full((M.rows,), float("nan"), dtype=M.dtype, device=cuda)
+                    L.step(variant, y)
+                    torch.cuda.current_stream().synchronize()
+                    ys[k][q] = y.cpu().numpy()
+                xnext[q] = L.x().cpu().numpy()           # the fused epilogue's copy of my block
+                L.close()
+                M.close()
+                D.close()
+        except Exception as e:
+            err.append((q, repr(e)))
+
+    th = [threading.Thread(target=rank, args=(q,)) for q in range(P)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join(timeout=300)
+    assert not any(t.is_alive() for t in th), "loop ranks hung"
+    assert not err, err
+    group.close()
+    return [np.concatenate(ys[k]) for k in range(steps)], np.concatenate(xnext)
+
+
+@pytest.mark.parametrize("P", [2, 4])
+@pytest.mark.parametrize("variant", [0, 1, 2, 3, 4], ids=["csr_scalar", "csr_vector", "ell", "dia", "hyb"])
+def test_solver_loop_fused_epilogue(cuda, variant, P):
+    """Three multiplies x_{k+1} = A x_k on P loopback ranks: every rank's y
+    block equals the oracle's (integer stencil, exact), and the next x each
+    rank holds (written by the fused epilogue of every rank: CSR-scalar, ELL,
+    DIA; the push fallback for CSR-vector, HYB) equals the last y."""
+    A = synth.stencil("2d5", 48)                    # values 4, -1: |row sum| <= 8 -> exact after 3 steps
+    x0 = synth.vector(A.cols, seed=3, mode=1)
+    ref = _loop_ref(A, x0, 3)
+    ys, xlast = run_loop_group(A, x0, P, variant, 3, cuda)
+    for k in range(3):
+        assert np.array_equal(ys[k].astype(np.float64), ref[k]), (variant, P, k)
+    assert np.array_equal(xlast.astype(np.float64), ref[-1])
+
+
+def test_solver_loop_nccl_single_rank(cuda):
+    """The NCCL path of the loop (symmetric windows, device-API peer pointers,
+    LSA barrier kernel) with one rank: same results as the oracle."""
+    import torch
+    n = nitro()
+    A = synth.stencil("2d5", 40)
+    x0 = synth.vector(A.cols, seed=5, mode=1)
+    ref = _loop_ref(A, x0, 3)
+    D = n.Dist(n.dist_unique_id(), 0, 1, 0)
+    Ad = synth.to_device(A, cuda)
+    M = D.spmv(A.rows, np.array([0, A.rows], np.int64), Ad.rowptr, Ad.colidx, Ad.vals, exchange=0)
+    for v in (n.DIA, n.CSR_SCALAR, n.CSR_VECTOR):
+        L = D.loop(M)
+        L.x().copy_(torch.from_numpy(x0).to(cuda))
+        L.start()
+        for k in range(3):
+            y = torch.full((A.rows,), float("nan"), device=cuda)
+            L.step(v, y)
+            torch.cuda.synchronize()
+            assert np.array_equal(y.cpu().numpy().astype(np.float64), ref[k]), (v, k)
+        L.close()
+    M.close()
+    D.close()
