@@ -51,8 +51,8 @@ def load(path):
 
 
 def short(name):
-    for k in ("k_features_long", "k_features", "k_csr_scalar", "k_csr_vector", "k_hyb_tail", "k_hyb_fixup", "k_ell",
-              "k_dia"):
+    for k in ("k_features_long", "k_features", "k_csr_scalar", "k_csr_vector", "k_csr_stream", "k_hyb_tail",
+              "k_hyb_fixup", "k_ell", "k_dia"):
         if k in name:
             return k
     return name[:40]
@@ -65,7 +65,7 @@ def main():
     summary = json.load(open(summ_path)) if os.path.exists(summ_path) else {}
     md = [f"# ncu --set full summary ({tag})", "",
           "Cold-cache replays (ncu default cache control), one row per captured launch.", ""]
-    for cfg in ("c1", "c2a", "c2b"):
+    for cfg in ("c1", "c2a", "c2b", "c4"):
         p = os.path.join(src, f"prof_{cfg}_raw.csv")
         if not os.path.exists(p):
             continue
@@ -77,7 +77,7 @@ def main():
         for i, r in enumerate(recs):
             k = short(r["kernel"])
             var = {"k_features": "features", "k_features_long": "features_long", "k_csr_scalar": "csr_scalar",
-                   "k_csr_vector": "csr_vector", "k_dia": "dia", "k_hyb_tail": "hyb",
+                   "k_csr_vector": "csr_vector", "k_csr_stream": "csr_vector", "k_dia": "dia", "k_hyb_tail": "hyb",
                    "k_hyb_fixup": "hyb_fixup"}.get(k)
             if k == "k_ell":
                 var = "ell" if seen_ell < 2 and cfg != "c2b" else "hyb_ell"

@@ -18,6 +18,8 @@ def make(cfg, dev):
         return synth.stencil("2d5", 64, device=dev)
     if cfg == "c1":
         return synth.stencil("3d27", 128, mode=1, seed=1, device=dev)
+    if cfg == "c4":      # BASELINE configs[4]: 3D 27-pt 512^3 (int64 rowptr), the bench workload
+        return synth.stencil("3d27", 512, mode=1, seed=1, device=dev)
     if cfg == "c1big":   # 3D 27-pt 256^3: the asymptotic (ramp-free) DIA/ELL rate
         return synth.stencil("3d27", 256, mode=1, seed=1, device=dev)
     if cfg == "c2a":
@@ -45,13 +47,14 @@ def main():
     timing = "--time" in args
     csr_ab = "--csr-ab" in args   # also time the CSR variants with the direct kernels
     args = [a for a in args if a not in ("--time", "--csr-ab")]
-    cfgs = [a for a in args if a in ("c0", "c1", "c1big", "c2a", "c2b", "short", "band01", "uvar3", "band48", "band96h")] or ["c1"]
+    cfgs = [a for a in args if a in ("c0", "c1", "c1big", "c2a", "c2b", "c4", "short", "band01", "uvar3", "band48", "band96h")] or ["c1"]
     want = [] if "none" in args else ([nitro.VARIANT_NAMES.index(v) for v in args if v in nitro.VARIANT_NAMES] or list(range(5)))
     dev = torch.device("cuda:0")
     table = {}
     for cfg in cfgs:
         A = make(cfg, dev)
-        A.rowptr = A.rowptr.to(torch.int32)
+        if A.nnz < 2 ** 31:
+            A.rowptr = A.rowptr.to(torch.int32)
         M = nitro.SpMV.from_csr(A)
         s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         M.features()                    # allocates the feature buffers
@@ -69,7 +72,8 @@ def main():
         x = synth.vector(A.cols, seed=2, fp64=A.fp64, device=dev)
         y = torch.empty(A.rows, dtype=x.dtype, device=dev)
         row = {"rows": A.rows, "nnz": A.nnz, "feature_ms": feat_ms,
-               "feature_GBps": ((A.rows + 1) * 4 + A.nnz * 4) / (feat_ms * 1e-3) / 1e9, "variants": {}}
+               "feature_GBps": ((A.rows + 1) * A.rowptr.element_size() + A.nnz * 4) / (feat_ms * 1e-3) / 1e9,
+               "variants": {}}
         for v in want:
             if not M.allowed(v):
                 continue
