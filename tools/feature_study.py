@@ -41,7 +41,7 @@ LEVELS = [("L0", ["nnz", "rows"]), ("L0m", ["nnz", "rows", "mean"]),
           ("L2", ["nnz", "rows", "mean", "sd", "max_dev", "dia_fill", "ell_fill"])]
 
 
-def ablation(table, nitro):
+def ablation(table, nitro, ext=False):
     names = list(nitro.FEATURE_NAMES)
     Ftr = np.array([r["features"] for r in table["train"]], np.float64)
     Ctr = np.array([r["cost"] for r in table["train"]], np.float64)
@@ -55,7 +55,8 @@ def ablation(table, nitro):
         for f in feats:
             cv.add_feature(f, lambda i: 0.0)
         cv.set_default(nitro.CSR_VECTOR)
-        cv.set_feature_transform((1 << len(cols)) - 1, True)   # as nitro_spmv_register (R11)
+        if ext:
+            cv.set_feature_transform((1 << len(cols)) - 1, True)   # R11x extension (log1p + clip)
         cv.train_from_table(Ftr[:, cols], Ctr)
         ratios = []
         for r in table["test"]:
@@ -152,7 +153,8 @@ def main():
     args = ap.parse_args()
     import paper_conf_ipps_muralidharanshgc14_b200 as nitro
     table = json.load(open(args.table))
-    res = {"ablation": ablation(table, nitro)}
+    res = {"ablation": ablation(table, nitro), "scaling": "paper: [-1, 1] min-max (P:L179)",
+           "ablation_r11x": ablation(table, nitro, ext=True)}
     if args.gpu:
         rows, summ = gpu_overheads(table, nitro, args.model)
         res["per_matrix"] = rows
