@@ -855,7 +855,7 @@ __global__ void __launch_bounds__(256) k_hyb_tail_ls(const int32_t *__restrict__
 // 0).  No global atomics (the shared-memory counts are integers):
 // deterministic.
 template <typename IT, typename VT, int EP>
-__global__ void __launch_bounds__(256) k_csr_stream(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
+__global__ void __launch_bounds__(256, EP == 4 ? 8 : 4) k_csr_stream(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
                                                     const VT *__restrict__ val, const VT *__restrict__ x,
                                                     VT *__restrict__ y, int64_t N, int64_t Z, int64_t nch,
                                                     const int32_t *__restrict__ chunk_row,
