@@ -355,8 +355,14 @@ def run_nitro(args):
         sys.exit(2)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+    use_dist = world > 1 or args.dist   # --dist: the multi-rank code path with one rank (NCCL communicator of 1)
+    if use_dist:
+        if world == 1:
+            os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+            os.environ.setdefault("MASTER_PORT", str(_free_port()))
+            dist.init_process_group("nccl", device_id=dev, rank=0, world_size=1)
+        else:
+            dist.init_process_group("nccl", device_id=dev)
     stream = torch.cuda.current_stream(dev)
     models = load_models(nitro)
     deployed = args.model if args.model in models else next(iter(models), None)
@@ -365,7 +371,7 @@ def run_nitro(args):
     t_start = time.time()
 
     # ---- this rank's rows (N = 1: the whole matrix)
-    if world == 1:
+    if not use_dist:
         A = make(cfg, dev)
         bounds = None
     else:
@@ -380,11 +386,11 @@ def run_nitro(args):
     torch.cuda.synchronize()
     log(f"generated {cfg} rows {A.rows} nnz {A.nnz} in {time.time() - t_start:.1f}s")
     Ng = A.cols                               # global rows = cols (square)
-    row0 = int(bounds[rank]) if world > 1 else 0
+    row0 = int(bounds[rank]) if use_dist else 0
     xfull_seed = 2
     y = torch.empty(A.rows, dtype=A.vals.dtype, device=dev)
 
-    if world == 1:
+    if not use_dist:
         M = nitro.SpMV.from_csr(A)
         x = synth.vector(Ng, seed=xfull_seed, fp64=A.fp64, device=dev)
         D = None
@@ -440,7 +446,7 @@ def run_nitro(args):
         for _ in range(2):
             run(v, xx, yy)
         torch.cuda.synchronize()
-        if world > 1:
+        if use_dist:
             dist.barrier()
         ts = []
         for _ in range(reps):
@@ -453,7 +459,7 @@ def run_nitro(args):
             e1.synchronize()
             ts.append(e0.elapsed_time(e1))
         med = statistics.median(ts)
-        if world > 1:
+        if use_dist:
             tt = torch.tensor([med], device=dev)
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             med = float(tt.item())
@@ -475,7 +481,7 @@ def run_nitro(args):
         info = fmt_info(v)
         ms = timed(v, args.ex_reps)
         nb = info["compulsory_bytes"]
-        if world > 1:
+        if use_dist:
             tb = torch.tensor([nb], dtype=torch.float64, device=dev)
             dist.all_reduce(tb)
             nb = float(tb.item())
@@ -493,13 +499,13 @@ def run_nitro(args):
     for _ in range(args.warmup):
         run(sel, x, y)
     torch.cuda.synchronize()
-    if world > 1:
+    if use_dist:
         dist.barrier()
     starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
     ends = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
     with Clocks(local) as clk:
         torch.cuda.synchronize()
-        if world > 1:
+        if use_dist:
             dist.barrier()
         for i in range(args.steps):
             M.flush_l2()
@@ -507,12 +513,12 @@ def run_nitro(args):
             run(sel, x, y)
             ends[i].record(stream)
         torch.cuda.synchronize()
-        if world > 1:
+        if use_dist:
             dist.barrier()
     times = [s.elapsed_time(e) for s, e in zip(starts, ends)]
     ms = sum(times) / len(times)
     tot_bytes = nbytes
-    if world > 1:
+    if use_dist:
         tt = torch.tensor([ms], device=dev)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         ms = float(tt.item())
@@ -573,7 +579,7 @@ def run_nitro(args):
             if i >= 2:
                 et.append(e0.elapsed_time(e1))
     e2e_ms = sum(et) / len(et)
-    if world > 1:
+    if use_dist:
         tt = torch.tensor([e2e_ms], device=dev)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         e2e_ms = float(tt.item())
@@ -598,7 +604,7 @@ def run_nitro(args):
         selection = selection_leg(nitro, dev, models, args.selection_per_class, 10, log)
 
     if rank != 0:
-        if world > 1:
+        if use_dist:
             dist.destroy_process_group()
         return
     pk, pk_kind = peaks()
@@ -610,7 +616,7 @@ def run_nitro(args):
             traffic = rec.get("dram_bytes_per_launch")
     except Exception:
         pass
-    par = "single GPU" if world == 1 else \
+    par = "single GPU" if not use_dist else \
         f"row-partitioned x{world} (nnz-balanced blocks), NCCL in-place x all-gather per multiply (A13), " \
         f"interior rows overlap the exchange"
     line = {
@@ -648,7 +654,7 @@ def run_nitro(args):
     }
     if halo:
         line["halo_exchange"] = halo
-    if world > 1:
+    if use_dist:
         line["nccl_all_gather_floor_ms"] = (world - 1) / world * Ng * sv / 900e9 * 1e3
     if extra:
         line["configs"] = extra
@@ -658,17 +664,22 @@ def run_nitro(args):
         line["cpu_baseline"] = cpu_baseline(bytes_per_row)
     line["bench_wall_s"] = time.time() - t_start
     print(json.dumps(line), flush=True)
-    if world > 1:
+    if use_dist:
         dist.destroy_process_group()
 
 
-def relaunch(args):
-    """--gpus N > 1 without torchrun: start N ranks with torch.distributed.run."""
+def _free_port():
     import socket
     s = socket.socket()
     s.bind(("127.0.0.1", 0))
     port = s.getsockname()[1]
     s.close()
+    return port
+
+
+def relaunch(args):
+    """--gpus N > 1 without torchrun: start N ranks with torch.distributed.run."""
+    port = _free_port()
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
            "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
     return subprocess.call(cmd)
@@ -686,6 +697,8 @@ def main():
     ap.add_argument("--selection-per-class", type=int, default=10, help="held-out configs[3] matrices per class")
     ap.add_argument("--quick", action="store_true", help="primary workload only (no extra configs/selection leg)")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--dist", action="store_true",
+                    help="the multi-rank (nitro_dist_*, NCCL) code path even with one rank")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     if args.gpus > 1 and "WORLD_SIZE" not in os.environ:

@@ -177,7 +177,7 @@ template <typename IT>
 __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
                                                         int64_t N, int64_t M, int64_t Z, int64_t row0, int64_t G,
                                                         FeatAcc *__restrict__ acc, uint32_t *__restrict__ bitmap,
-                                                        int2 *__restrict__ tasks, int64_t cap_tasks, bool tbs) {
+                                                        int2 *__restrict__ tasks, int64_t cap_tasks) {
   __shared__ int s_stage[kWarps][kStage + kStage / 32];
   __shared__ int8_t s_slot[kWarps][32];
   __shared__ uint32_t s_seen[kCache];
@@ -200,12 +200,10 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
   // fills: full), then a fire-and-forget global OR (no returned value, so no
   // dependent L2 round trip)
   auto lane_far = [&](uint32_t idx, bool full) {
-    if (full) {
-      // tbs: skip the OR when an L1-cached read already shows the bit (bits only
-      // go 0 -> 1, so a stale line can only cost a redundant OR)
-      if (!tbs || !(__ldca(bitmap + (idx >> 5)) & (1u << (idx & 31)))) atomicOr(bitmap + (idx >> 5), 1u << (idx & 31));
-      return;
-    }
+    // (testing the bit with an L1-cached read before the OR was measured: no
+    // gain on configs[2] uniform — 1.529 vs 1.546 ms, the random sector access
+    // costs the same as the fire-and-forget OR — and 1.8x slower on short random rows)
+    if (full) { atomicOr(bitmap + (idx >> 5), 1u << (idx & 31)); return; }
     bool hit = false;
     int free_slot = -1;
     const uint32_t h = idx * 0x9E3779B1u >> 22;
@@ -518,15 +516,6 @@ __global__ void __launch_bounds__(256) k_popc(const uint32_t *__restrict__ bm, i
 
 }  // namespace
 
-// A/B knob of the far-offset test-before-set (NITRO_FEAT_TBS=1)
-bool feat_tbs() {
-  static bool v = [] {
-    const char *e = getenv("NITRO_FEAT_TBS");
-    return e ? atoi(e) != 0 : false;
-  }();
-  return v;
-}
-
 void finish_features(int64_t N, int64_t M, int64_t Z, uint64_t s1, uint64_t s2, int64_t lmax, int64_t D,
                      nitro_spmv_feat *f) {
   // DESIGN.md R4 — fixed fp64 expression (compiled with -ffp-contract=off)
@@ -571,13 +560,13 @@ nitro_status_t features_launch(nitro_spmv *A) {
                                                                            (A->Z / kChunk + kWarps - 1) / kWarps));
   if (A->rp64) {
     k_features<int64_t><<<(unsigned)grid, kThreads, 0, s>>>((const int64_t *)A->rowptr, A->col, A->N, A->M, A->Z,
-                                                            A->row0, G, acc, A->bitmap.as<uint32_t>(), tasks, cap_tasks, feat_tbs());
+                                                            A->row0, G, acc, A->bitmap.as<uint32_t>(), tasks, cap_tasks);
     if (A->Z > kLong)
       k_features_long<int64_t><<<glong, kThreads, 0, s>>>((const int64_t *)A->rowptr, A->col, A->M, A->row0, G, acc,
                                                           A->bitmap.as<uint32_t>(), tasks, cap_tasks);
   } else {
     k_features<int32_t><<<(unsigned)grid, kThreads, 0, s>>>((const int32_t *)A->rowptr, A->col, A->N, A->M, A->Z,
-                                                            A->row0, G, acc, A->bitmap.as<uint32_t>(), tasks, cap_tasks, feat_tbs());
+                                                            A->row0, G, acc, A->bitmap.as<uint32_t>(), tasks, cap_tasks);
     if (A->Z > kLong)
       k_features_long<int32_t><<<glong, kThreads, 0, s>>>((const int32_t *)A->rowptr, A->col, A->M, A->row0, G, acc,
                                                           A->bitmap.as<uint32_t>(), tasks, cap_tasks);

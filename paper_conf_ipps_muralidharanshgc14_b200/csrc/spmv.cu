@@ -855,7 +855,7 @@ __global__ void __launch_bounds__(256) k_hyb_tail_ls(const int32_t *__restrict__
 // 0).  No global atomics (the shared-memory counts are integers):
 // deterministic.
 template <typename IT, typename VT, int EP>
-__global__ void __launch_bounds__(256, EP == 4 ? 8 : 4) k_csr_stream(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
+__global__ void __launch_bounds__(256) k_csr_stream(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
                                                     const VT *__restrict__ val, const VT *__restrict__ x,
                                                     VT *__restrict__ y, int64_t N, int64_t Z, int64_t nch,
                                                     const int32_t *__restrict__ chunk_row,
@@ -874,7 +874,8 @@ __global__ void __launch_bounds__(256, EP == 4 ? 8 : 4) k_csr_stream(const IT *_
   }
   // (a one-chunk software pipeline — the next chunk's col / val / row range
   // loaded before the current chunk's row work — measured slower: 53 vs 40
-  // registers, c2b 0.741 vs 0.716 ms)
+  // registers, c2b 0.741 vs 0.716 ms; so did full occupancy by launch bounds,
+  // 32 registers + spills: 0.753 ms)
   for (int64_t ch = warp; ch < nch; ch += nw) {
     const int64_t c0 = ch * CH, cend = c0 + CH < Z ? c0 + CH : Z;
     const int64_t e0 = c0 + (int64_t)lane * EP;
