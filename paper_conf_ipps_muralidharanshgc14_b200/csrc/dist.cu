@@ -236,11 +236,11 @@ __global__ void k_interior(const IT *__restrict__ rowptr, const int32_t *__restr
   }
 }
 
-template <typename IT>
-__global__ void k_rebase(const IT *__restrict__ rowptr, int64_t s, int64_t cnt, int32_t *__restrict__ out) {
+template <typename IT, typename OT>
+__global__ void k_rebase(const IT *__restrict__ rowptr, int64_t s, int64_t cnt, OT *__restrict__ out) {
   const int64_t base = (int64_t)rowptr[s];
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i <= cnt; i += (int64_t)gridDim.x * blockDim.x)
-    out[i] = (int32_t)((int64_t)rowptr[s + i] - base);
+    out[i] = (OT)((int64_t)rowptr[s + i] - base);
 }
 
 __global__ void k_to_local(int32_t *__restrict__ ids, int64_t n, int64_t lo) {
@@ -524,15 +524,17 @@ nitro_status_t nitro_dist_spmv_create_ex(nitro_dist *D, int64_t global_rows, con
         ab[0] = t[0]; ab[1] = t[1];
       }
       const int64_t pz = ab[1] - ab[0];
-      if (pz > 2147483647LL) return bail(fail(NITRO_E_UNSUPPORTED, "a rank part needs < 2^31 nonzeros"));
-      if ((rc = st->rp_part[k].alloc((cnt + 1) * 4))) return bail(rc);
-      if (rowptr_is_64)
-        k_rebase<int64_t><<<grid_n(cnt + 1), 256>>>((const int64_t *)d_rowptr, beg[k], cnt, st->rp_part[k].as<int32_t>());
-      else
-        k_rebase<int32_t><<<grid_n(cnt + 1), 256>>>((const int32_t *)d_rowptr, beg[k], cnt, st->rp_part[k].as<int32_t>());
+      const bool p64 = pz > 2147483647LL;  // parts of >= 2^31 nonzeros keep 64-bit row pointers
+      if ((rc = st->rp_part[k].alloc((cnt + 1) * (p64 ? 8 : 4)))) return bail(rc);
+      if (rowptr_is_64) {
+        if (p64) k_rebase<int64_t, int64_t><<<grid_n(cnt + 1), 256>>>((const int64_t *)d_rowptr, beg[k], cnt, st->rp_part[k].as<int64_t>());
+        else k_rebase<int64_t, int32_t><<<grid_n(cnt + 1), 256>>>((const int64_t *)d_rowptr, beg[k], cnt, st->rp_part[k].as<int32_t>());
+      } else {
+        k_rebase<int32_t, int32_t><<<grid_n(cnt + 1), 256>>>((const int32_t *)d_rowptr, beg[k], cnt, st->rp_part[k].as<int32_t>());
+      }
       NITRO_CUDA(cudaGetLastError());
-      rc = nitro_spmv_create(D->device, nullptr, cnt, Mx, pz, st->rp_part[k].p, 0, st->colmap.as<int32_t>() + ab[0],
-                             (const char *)d_vals + ab[0] * sv, is_fp64, &st->part[k]);
+      rc = nitro_spmv_create(D->device, nullptr, cnt, Mx, pz, st->rp_part[k].p, p64 ? 1 : 0,
+                             st->colmap.as<int32_t>() + ab[0], (const char *)d_vals + ab[0] * sv, is_fp64, &st->part[k]);
       if (rc) return bail(rc);
       st->part[k]->row0 = xoff + beg[k];  // local row i sits at layout index xoff + i: diagonal offsets kept
     }
