@@ -230,25 +230,13 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
   // it is set.  The bound checks sit outside the loop: the pass is issue-bound
   // on stencils (ncu: SM throughput 74 %, IPC 3.2), so instructions per entry
   // are what the loop is tuned for.
-  // The window bits of consecutive entries of a row (columns ascend) mostly
-  // share a 32-bit word (a stencil row's 27 offsets fall in 9 runs of 3): the
-  // bits are collected per word in registers and the shared word is tested /
-  // ORed once per run, through 32-bit shared addresses (the generic form
-  // re-derived the window's shared address on every entry).  ncu on configs[1]
-  // (round 1): ~22 instructions per entry in this loop, issue-bound.
-  const uint32_t win_sa = (uint32_t)__cvta_generic_to_shared(s_win);
-  auto win_flush = [&](uint32_t w, uint32_t b) {
-    if (w == kEmpty) return;
-    const uint32_t a = win_sa + 4u * w;
-    uint32_t cur;
-    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(cur) : "r"(a));
-    if ((cur & b) != b) asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(a), "r"(b) : "memory");
-  };
+  // (Collecting a row's window bits per 32-bit word in registers and testing /
+  // ORing the shared word once per run, through 32-bit shared addresses, was
+  // measured slower: configs[1] 0.131 -> 0.140 ms, configs[4] 5.75 -> 6.18 ms.)
   auto lane_walk_core = [&](auto ld, int L, uint32_t myrow, bool full) {
     const uint32_t rbase = myrow - (kWin >> 1);
     int prev = -1;
     bool inc = true;
-    uint32_t cw = kEmpty, cb = 0;  // pending window word and its bits
 #pragma unroll 4
     for (int k = 0; k < L; ++k) {
       const int c = ld(k);
@@ -256,19 +244,12 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
       prev = c;
       const uint32_t rel = (uint32_t)c - rbase;
       if (rel < kWin) {
-        const uint32_t w = rel >> 5, bit = 1u << (rel & 31);
-        if (w == cw) {
-          cb |= bit;
-        } else {
-          win_flush(cw, cb);
-          cw = w;
-          cb = bit;
-        }
+        const uint32_t bit = 1u << (rel & 31);
+        if (!(s_win[rel >> 5] & bit)) atomicOr(&s_win[rel >> 5], bit);
       } else if ((uint32_t)c < M32) {
         lane_far((uint32_t)c - myrow + G32, full);
       }
     }
-    win_flush(cw, cb);
     const int first = ld(0);
     if (first < 0 || (uint32_t)prev >= M32) bad |= 4;
     else if (!inc) bad |= 2;

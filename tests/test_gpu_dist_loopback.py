@@ -243,3 +243,45 @@ def test_solver_loop_nccl_single_rank(cuda):
         L.close()
     M.close()
     D.close()
+
+
+def test_dist_format_info_sums_the_rank_parts(cuda):
+    """nitro_dist_format_info: a rank's compulsory bytes = its parts' matrix +
+    y bytes + the exchanged x layout read once.  Summed over the ranks of a
+    CSR-scalar multiply that is the single-GPU CSR bytes minus the single
+    x read plus P layout reads (+ (#parts - 1) extra rowptr entries per rank)."""
+    import torch
+    n = nitro()
+    A = synth.stencil("3d27", 24, mode=1, seed=8)
+    P = 4
+    bounds = n.dist_partition(np.asarray(A.rowptr, np.int64), P)
+    group = n.Loopback(P, 0)
+    got = [None] * P
+    err = []
+
+    def rank(q):
+        try:
+            torch.cuda.set_device(0)
+            with torch.cuda.stream(torch.cuda.Stream()):
+                D = n.Dist.loopback(group, q)
+                blk = synth.to_device(block(A, bounds[q], bounds[q + 1]), cuda)
+                M = D.spmv(A.rows, bounds, blk.rowptr, blk.colidx, blk.vals, exchange=0)
+                got[q] = (n.Dist.format_info(M, n.CSR_SCALAR), n.Dist.exchange_info(M), n.Dist.layout(M))
+                M.close()
+                D.close()
+        except Exception as e:
+            err.append(repr(e))
+
+    th = [threading.Thread(target=rank, args=(q,)) for q in range(P)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join(timeout=300)
+    assert not err, err
+    group.close()
+    N, Z = A.rows, A.nnz
+    nparts = [sum(1 for lo, hi in ((0, l[1]), (l[1], l[2]), (l[2], hi_q - lo_q)) if hi > lo)
+              for l, lo_q, hi_q in ((g[2], bounds[q], bounds[q + 1]) for q, g in enumerate(got))]
+    want = Z * 8 + N * 4 + sum(p + 0 for p in nparts) * 4 + sum(g[1]["layout_len"] * 4 for g in got) + N * 4
+    tot = sum(g[0]["compulsory_bytes"] for g in got)
+    assert abs(tot - want) < 1e-6 * want, (tot, want, nparts)
