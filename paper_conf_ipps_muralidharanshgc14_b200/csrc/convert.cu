@@ -501,6 +501,8 @@ nitro_status_t prepare_csrv(nitro_spmv *A) {
   A->csrv.V = V;
   A->csrv.stream = csrv_stream_mode(A);
   if (A->csrv.stream && A->Z > 0) {
+    // entries per lane: B200 A/B on c2b (fp64) EP 4 vs 8: 0.716 vs 0.753 ms; on
+    // fp32 (c2a) 8 beats 4: 1.297 vs 1.462 ms
     const int EP = A->fp64 ? 4 : 8;
     const int64_t CH = 32LL * EP, nch = (A->Z + CH - 1) / CH, nslot = 2 * nch;
     A->csrv.EP = EP;

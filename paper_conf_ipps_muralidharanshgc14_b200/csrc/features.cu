@@ -508,6 +508,160 @@ __global__ void __launch_bounds__(256) k_rowstats(const IT *__restrict__ rowptr,
   }
 }
 
+// K1s — nnz-split feature pass (the K6s decomposition applied to K1).  Each
+// warp walks a contiguous range of 256-entry chunks (8 consecutive entries per
+// lane, 128-bit loads); it finds the row of its first entry once (a 32-ary
+// cooperative search of rowptr) and then derives every entry's row from the
+// row starts falling inside each chunk (counted per chunk position in shared
+// memory, prefix-summed), carrying the row and the last column from chunk to
+// chunk.  Per entry: the canonical checks (column in [0, cols), strictly above
+// the previous entry of the same row) and the occupied-diagonal bit (per-block
+// shared window for |offset| < 2^15, else the per-block offset set / global
+// OR, as K1).  The row-length moments and the rowptr checks come from
+// k_rowstats (one pass over rowptr), launched before it.  The work per warp is
+// fixed by nnz, independent of the row-length distribution, and the per-entry
+// path has no staging copy.
+template <typename IT>
+__global__ void __launch_bounds__(kThreads) k_feat_stream(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
+                                                           int64_t N, int64_t M, int64_t Z, int64_t row0, int64_t G,
+                                                           int64_t nch, int64_t q, FeatAcc *__restrict__ acc,
+                                                           uint32_t *__restrict__ bitmap) {
+  constexpr int EP = 8;
+  constexpr int64_t CH = 32 * EP;
+  __shared__ __align__(16) int s_cnt[kWarps][CH];
+  __shared__ uint32_t s_seen[kCache];
+  __shared__ uint32_t s_win[kWin / 32];
+  __shared__ unsigned s_bad, s_full;
+  for (int i = threadIdx.x; i < kCache; i += kThreads) s_seen[i] = kEmpty;
+  for (int i = threadIdx.x; i < (int)(kWin / 32); i += kThreads) s_win[i] = 0u;
+  if (threadIdx.x == 0) { s_bad = 0; s_full = 0; }
+  __syncthreads();
+  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const uint32_t G32 = (uint32_t)G, M32 = (uint32_t)M;
+  const uint32_t win_lo = G32 - (kWin >> 1);
+  unsigned bad = 0;
+  auto far = [&](uint32_t idx) {  // as K1's lane_far
+    const bool full = *(volatile unsigned *)&s_full != 0;
+    if (full) { atomicOr(bitmap + (idx >> 5), 1u << (idx & 31)); return; }
+    bool hit = false;
+    int free_slot = -1;
+    const uint32_t h = idx * 0x9E3779B1u >> 22;
+    for (int p = 0; p < kProbe; ++p) {
+      const int slot = (int)((h + p) & (kCache - 1));
+      const uint32_t cur = s_seen[slot];
+      if (cur == idx) { hit = true; break; }
+      if (cur == kEmpty) { free_slot = slot; break; }
+    }
+    if (!hit) {
+      atomicOr(bitmap + (idx >> 5), 1u << (idx & 31));
+      if (free_slot >= 0) atomicCAS(&s_seen[free_slot], kEmpty, idx);
+      else s_full = 1;
+    }
+  };
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t ch0 = gw * q, ch1 = ch0 + q < nch ? ch0 + q : nch;
+  if (ch0 < ch1) {
+    // row of entry ch0 * CH: last r with rowptr[r] <= e (32-ary search)
+    const int64_t e = ch0 * CH;
+    int64_t lo = 0, hi = N;
+    while (hi - lo > 1) {
+      const int64_t step = (hi - lo + 31) / 32;
+      const int64_t pr = lo + (int64_t)lane * step;
+      const int64_t v = pr < hi ? (int64_t)rowptr[pr] : INT64_MAX;
+      const unsigned m = __ballot_sync(kFull, v <= e);
+      const int j = m ? 31 - __clz(m) : 0;
+      lo = lo + (int64_t)j * step;
+      hi = lo + step < hi ? lo + step : hi;
+    }
+    int64_t r_lo = lo;
+    int last_c = -1;
+    int64_t last_r = -1;
+    int *cnt = s_cnt[wib];
+    for (int64_t ch = ch0; ch < ch1; ++ch) {
+      const int64_t c0 = ch * CH, cend = c0 + CH < Z ? c0 + CH : Z;
+      const int64_t e0 = c0 + (int64_t)lane * EP;
+      const int nv = e0 >= cend ? 0 : (cend - e0 < EP ? (int)(cend - e0) : EP);
+      int c[EP];
+      if (nv == EP && ((reinterpret_cast<uintptr_t>(col + e0) & 15) == 0)) {
+        const int4 a = ld_stream_i4(reinterpret_cast<const int4 *>(col + e0));
+        const int4 b = ld_stream_i4(reinterpret_cast<const int4 *>(col + e0) + 1);
+        c[0] = a.x; c[1] = a.y; c[2] = a.z; c[3] = a.w; c[4] = b.x; c[5] = b.y; c[6] = b.z; c[7] = b.w;
+      } else {
+#pragma unroll
+        for (int k = 0; k < EP; ++k) c[k] = k < nv ? ld_stream_i(col + e0 + k) : 0;
+      }
+      reinterpret_cast<int4 *>(cnt + lane * EP)[0] = make_int4(0, 0, 0, 0);
+      reinterpret_cast<int4 *>(cnt + lane * EP)[1] = make_int4(0, 0, 0, 0);
+      __syncwarp();
+      // row starts inside (c0, cend): counted at their chunk position; r_next =
+      // the last row starting at or before cend (the next chunk's first row)
+      int64_t r_next = r_lo;
+      for (int64_t w0 = r_lo + 1; w0 < N; w0 += 32) {
+        const int64_t rr = w0 + lane;
+        const int64_t rs = rr < N ? (int64_t)rowptr[rr] : INT64_MAX;
+        if (rs > c0 && rs < cend) atomicAdd(cnt + (int)(rs - c0), 1);
+        const unsigned le = __ballot_sync(kFull, rs <= cend);
+        if (le) r_next = w0 + 31 - __clz(le);
+        if (le != kFull) break;
+      }
+      __syncwarp();
+      int64_t row[EP];
+      {
+        const int4 a = reinterpret_cast<const int4 *>(cnt + lane * EP)[0];
+        const int4 b = reinterpret_cast<const int4 *>(cnt + lane * EP)[1];
+        int inc[EP] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
+#pragma unroll
+        for (int k = 1; k < EP; ++k) inc[k] += inc[k - 1];
+        int ex = inc[EP - 1];
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const int t = __shfl_up_sync(kFull, ex, o);
+          if (lane >= o) ex += t;
+        }
+        ex -= inc[EP - 1];
+#pragma unroll
+        for (int k = 0; k < EP; ++k) row[k] = r_lo + ex + inc[k];
+      }
+      // the previous entry of each lane's first entry: the previous lane's last
+      // valid one, or (lane 0) the previous chunk's last entry
+      int pc = __shfl_up_sync(kFull, c[EP - 1], 1);
+      int64_t pr = __shfl_up_sync(kFull, row[EP - 1], 1);
+      if (lane == 0) { pc = last_c; pr = last_r; }
+#pragma unroll
+      for (int k = 0; k < EP; ++k) {
+        if (k < nv) {
+          const int cc = c[k];
+          const int64_t rk = row[k];
+          if ((uint32_t)cc >= M32) {
+            bad |= 4;
+          } else {
+            if (rk == pr && cc <= pc) bad |= 2;
+            const uint32_t myrow = (uint32_t)(row0 + rk);
+            const uint32_t rel = (uint32_t)cc - myrow + (kWin >> 1);
+            if (rel < kWin) {
+              const uint32_t bit = 1u << (rel & 31);
+              if (!(s_win[rel >> 5] & bit)) atomicOr(&s_win[rel >> 5], bit);
+            } else {
+              far((uint32_t)cc - myrow + G32);
+            }
+          }
+          pc = cc;
+          pr = rk;
+        }
+      }
+      const int lastl = (int)((cend - 1 - c0) / EP);
+      last_c = __shfl_sync(kFull, pc, lastl);
+      last_r = __shfl_sync(kFull, pr, lastl);
+      r_lo = r_next;
+    }
+  }
+  bad = __reduce_or_sync(kFull, bad);
+  if (lane == 0 && bad) atomicOr(&s_bad, bad);
+  __syncthreads();
+  merge_window(s_win, win_lo, G + M, bitmap);
+  if (threadIdx.x == 0 && s_bad) atomicOr(&acc->bad, s_bad);
+}
+
 __global__ void __launch_bounds__(256) k_popc(const uint32_t *__restrict__ bm, int64_t nwords, FeatAcc *acc) {
   unsigned long long s = 0;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nwords; i += (int64_t)gridDim.x * blockDim.x)
@@ -518,6 +672,15 @@ __global__ void __launch_bounds__(256) k_popc(const uint32_t *__restrict__ bm, i
 }
 
 }  // namespace
+
+// K1s (nnz-split feature pass) on/off: NITRO_FEAT_STREAM=1 (A/B)
+bool feat_stream_on() {
+  static bool v = [] {
+    const char *e = getenv("NITRO_FEAT_STREAM");
+    return e ? atoi(e) != 0 : false;
+  }();
+  return v;
+}
 
 void finish_features(int64_t N, int64_t M, int64_t Z, uint64_t s1, uint64_t s2, int64_t lmax, int64_t D,
                      nitro_spmv_feat *f) {
@@ -561,7 +724,24 @@ nitro_status_t features_launch(nitro_spmv *A) {
   int2 *tasks = A->feat_long.as<int2>();
   const unsigned glong = (unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)num_sms() * 4,
                                                                            (A->Z / kChunk + kWarps - 1) / kWarps));
-  if (A->rp64) {
+  if (feat_stream_on()) {  // K1s: rowptr moments (k_rowstats) + the nnz-split pass
+    if (A->N > 0) {
+      const unsigned gr = (unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)num_sms() * 8, (A->N + 255) / 256));
+      if (A->rp64) k_rowstats<int64_t><<<gr, 256, 0, s>>>((const int64_t *)A->rowptr, A->N, A->Z, acc);
+      else k_rowstats<int32_t><<<gr, 256, 0, s>>>((const int32_t *)A->rowptr, A->N, A->Z, acc);
+    }
+    const int64_t nch = (A->Z + 255) / 256;
+    if (nch > 0) {
+      const int64_t gs = std::max<int64_t>(1, std::min<int64_t>((int64_t)num_sms() * 8, (nch + kWarps - 1) / kWarps));
+      const int64_t q = (nch + gs * kWarps - 1) / (gs * kWarps);
+      if (A->rp64)
+        k_feat_stream<int64_t><<<(unsigned)gs, kThreads, 0, s>>>((const int64_t *)A->rowptr, A->col, A->N, A->M, A->Z,
+                                                                 A->row0, G, nch, q, acc, A->bitmap.as<uint32_t>());
+      else
+        k_feat_stream<int32_t><<<(unsigned)gs, kThreads, 0, s>>>((const int32_t *)A->rowptr, A->col, A->N, A->M, A->Z,
+                                                                 A->row0, G, nch, q, acc, A->bitmap.as<uint32_t>());
+    }
+  } else if (A->rp64) {
     k_features<int64_t><<<(unsigned)grid, kThreads, 0, s>>>((const int64_t *)A->rowptr, A->col, A->N, A->M, A->Z,
                                                             A->row0, G, acc, A->bitmap.as<uint32_t>(), tasks, cap_tasks);
     if (A->Z > kLong)
