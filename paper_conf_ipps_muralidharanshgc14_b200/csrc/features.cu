@@ -521,12 +521,12 @@ __global__ void __launch_bounds__(256) k_rowstats(const IT *__restrict__ rowptr,
 // k_rowstats (one pass over rowptr), launched before it.  The work per warp is
 // fixed by nnz, independent of the row-length distribution, and the per-entry
 // path has no staging copy.
-template <typename IT>
+template <typename IT, int EP>
 __global__ void __launch_bounds__(kThreads) k_feat_stream(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
                                                            int64_t N, int64_t M, int64_t Z, int64_t row0, int64_t G,
                                                            int64_t nch, int64_t q, FeatAcc *__restrict__ acc,
                                                            uint32_t *__restrict__ bitmap) {
-  constexpr int EP = 8;
+  static_assert(EP % 4 == 0 && EP <= 16, "EP");
   constexpr int64_t CH = 32 * EP;
   __shared__ __align__(16) int s_cnt[kWarps][CH];
   __shared__ uint32_t s_seen[kCache];
@@ -581,35 +581,41 @@ __global__ void __launch_bounds__(kThreads) k_feat_stream(const IT *__restrict__
       const int64_t c0 = ch * CH, cend = c0 + CH < Z ? c0 + CH : Z;
       const int64_t e0 = c0 + (int64_t)lane * EP;
       const int nv = e0 >= cend ? 0 : (cend - e0 < EP ? (int)(cend - e0) : EP);
+      // the chunk's column loads and its first row-start window are issued together
       int c[EP];
       if (nv == EP && ((reinterpret_cast<uintptr_t>(col + e0) & 15) == 0)) {
-        const int4 a = ld_stream_i4(reinterpret_cast<const int4 *>(col + e0));
-        const int4 b = ld_stream_i4(reinterpret_cast<const int4 *>(col + e0) + 1);
-        c[0] = a.x; c[1] = a.y; c[2] = a.z; c[3] = a.w; c[4] = b.x; c[5] = b.y; c[6] = b.z; c[7] = b.w;
+#pragma unroll
+        for (int k = 0; k < EP; k += 4) {
+          const int4 a = ld_stream_i4(reinterpret_cast<const int4 *>(col + e0 + k));
+          c[k] = a.x; c[k + 1] = a.y; c[k + 2] = a.z; c[k + 3] = a.w;
+        }
       } else {
 #pragma unroll
         for (int k = 0; k < EP; ++k) c[k] = k < nv ? ld_stream_i(col + e0 + k) : 0;
       }
-      reinterpret_cast<int4 *>(cnt + lane * EP)[0] = make_int4(0, 0, 0, 0);
-      reinterpret_cast<int4 *>(cnt + lane * EP)[1] = make_int4(0, 0, 0, 0);
+      int64_t rs = r_lo + 1 + lane < N ? (int64_t)rowptr[r_lo + 1 + lane] : INT64_MAX;
+#pragma unroll
+      for (int k = 0; k < EP; k += 4) reinterpret_cast<int4 *>(cnt + lane * EP)[k / 4] = make_int4(0, 0, 0, 0);
       __syncwarp();
       // row starts inside (c0, cend): counted at their chunk position; r_next =
       // the last row starting at or before cend (the next chunk's first row)
       int64_t r_next = r_lo;
       for (int64_t w0 = r_lo + 1; w0 < N; w0 += 32) {
-        const int64_t rr = w0 + lane;
-        const int64_t rs = rr < N ? (int64_t)rowptr[rr] : INT64_MAX;
+        if (w0 != r_lo + 1) rs = w0 + lane < N ? (int64_t)rowptr[w0 + lane] : INT64_MAX;
         if (rs > c0 && rs < cend) atomicAdd(cnt + (int)(rs - c0), 1);
         const unsigned le = __ballot_sync(kFull, rs <= cend);
         if (le) r_next = w0 + 31 - __clz(le);
         if (le != kFull) break;
       }
       __syncwarp();
-      int64_t row[EP];
+      int row[EP];  // relative to r_lo
       {
-        const int4 a = reinterpret_cast<const int4 *>(cnt + lane * EP)[0];
-        const int4 b = reinterpret_cast<const int4 *>(cnt + lane * EP)[1];
-        int inc[EP] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
+        int inc[EP];
+#pragma unroll
+        for (int k = 0; k < EP; k += 4) {
+          const int4 a = reinterpret_cast<const int4 *>(cnt + lane * EP)[k / 4];
+          inc[k] = a.x; inc[k + 1] = a.y; inc[k + 2] = a.z; inc[k + 3] = a.w;
+        }
 #pragma unroll
         for (int k = 1; k < EP; ++k) inc[k] += inc[k - 1];
         int ex = inc[EP - 1];
@@ -620,23 +626,24 @@ __global__ void __launch_bounds__(kThreads) k_feat_stream(const IT *__restrict__
         }
         ex -= inc[EP - 1];
 #pragma unroll
-        for (int k = 0; k < EP; ++k) row[k] = r_lo + ex + inc[k];
+        for (int k = 0; k < EP; ++k) row[k] = ex + inc[k];
       }
       // the previous entry of each lane's first entry: the previous lane's last
       // valid one, or (lane 0) the previous chunk's last entry
       int pc = __shfl_up_sync(kFull, c[EP - 1], 1);
-      int64_t pr = __shfl_up_sync(kFull, row[EP - 1], 1);
+      int64_t pr = r_lo + __shfl_up_sync(kFull, row[EP - 1], 1);
       if (lane == 0) { pc = last_c; pr = last_r; }
+      const uint32_t rbase = (uint32_t)(row0 + r_lo);
 #pragma unroll
       for (int k = 0; k < EP; ++k) {
         if (k < nv) {
           const int cc = c[k];
-          const int64_t rk = row[k];
+          const int64_t rk = r_lo + row[k];
           if ((uint32_t)cc >= M32) {
             bad |= 4;
           } else {
             if (rk == pr && cc <= pc) bad |= 2;
-            const uint32_t myrow = (uint32_t)(row0 + rk);
+            const uint32_t myrow = rbase + (uint32_t)row[k];
             const uint32_t rel = (uint32_t)cc - myrow + (kWin >> 1);
             if (rel < kWin) {
               const uint32_t bit = 1u << (rel & 31);
@@ -680,6 +687,14 @@ bool feat_stream_on() {
     return e ? atoi(e) != 0 : false;
   }();
   return v;
+}
+
+int feat_stream_ep() {
+  static int v = [] {
+    const char *e = getenv("NITRO_FEAT_EP");
+    return e ? atoi(e) : 16;
+  }();
+  return v == 8 ? 8 : 16;
 }
 
 void finish_features(int64_t N, int64_t M, int64_t Z, uint64_t s1, uint64_t s2, int64_t lmax, int64_t D,
@@ -730,16 +745,17 @@ nitro_status_t features_launch(nitro_spmv *A) {
       if (A->rp64) k_rowstats<int64_t><<<gr, 256, 0, s>>>((const int64_t *)A->rowptr, A->N, A->Z, acc);
       else k_rowstats<int32_t><<<gr, 256, 0, s>>>((const int32_t *)A->rowptr, A->N, A->Z, acc);
     }
-    const int64_t nch = (A->Z + 255) / 256;
+    const int ep = feat_stream_ep();
+    const int64_t nch = (A->Z + 32 * ep - 1) / (32 * ep);
     if (nch > 0) {
       const int64_t gs = std::max<int64_t>(1, std::min<int64_t>((int64_t)num_sms() * 8, (nch + kWarps - 1) / kWarps));
       const int64_t q = (nch + gs * kWarps - 1) / (gs * kWarps);
-      if (A->rp64)
-        k_feat_stream<int64_t><<<(unsigned)gs, kThreads, 0, s>>>((const int64_t *)A->rowptr, A->col, A->N, A->M, A->Z,
-                                                                 A->row0, G, nch, q, acc, A->bitmap.as<uint32_t>());
-      else
-        k_feat_stream<int32_t><<<(unsigned)gs, kThreads, 0, s>>>((const int32_t *)A->rowptr, A->col, A->N, A->M, A->Z,
-                                                                 A->row0, G, nch, q, acc, A->bitmap.as<uint32_t>());
+#define NITRO_K1S(IT, EPV)                                                                                   \
+  k_feat_stream<IT, EPV><<<(unsigned)gs, kThreads, 0, s>>>((const IT *)A->rowptr, A->col, A->N, A->M, A->Z, \
+                                                           A->row0, G, nch, q, acc, A->bitmap.as<uint32_t>())
+      if (A->rp64) { if (ep == 16) NITRO_K1S(int64_t, 16); else NITRO_K1S(int64_t, 8); }
+      else { if (ep == 16) NITRO_K1S(int32_t, 16); else NITRO_K1S(int32_t, 8); }
+#undef NITRO_K1S
     }
   } else if (A->rp64) {
     k_features<int64_t><<<(unsigned)grid, kThreads, 0, s>>>((const int64_t *)A->rowptr, A->col, A->N, A->M, A->Z,
