@@ -680,22 +680,14 @@ __global__ void __launch_bounds__(256) k_popc(const uint32_t *__restrict__ bm, i
 
 }  // namespace
 
-// K1s (nnz-split feature pass) on/off: NITRO_FEAT_STREAM=1 (A/B)
-bool feat_stream_on() {
-  static bool v = [] {
-    const char *e = getenv("NITRO_FEAT_STREAM");
-    return e ? atoi(e) != 0 : false;
-  }();
-  return v;
-}
-
-int feat_stream_ep() {
-  static int v = [] {
-    const char *e = getenv("NITRO_FEAT_EP");
-    return e ? atoi(e) : 16;
-  }();
-  return v == 8 ? 8 : 16;
-}
+// K1s (nnz-split feature pass) for matrices whose mean row length exceeds
+// kRowCap (K1 walks those rows warp-wide; B200, dense band b = 48, 97 entries
+// per row: K1 0.964 ms -> K1s 0.470 ms).  K1 stays for shorter rows: configs[1]
+// 0.131 vs 0.175 ms, configs[4] 5.8 vs 12.0 ms, 1D 3-pt 0.118 vs 0.139 ms.  K1s
+// is also ahead on skewed rows (configs[2] R-MAT 0.943 -> 0.804 ms) and sparse
+// bands (0.275 -> 0.200 ms), but telling those apart needs the row-length SD,
+// i.e. a pass before the launch; the rule uses what is known at create time.
+bool feat_stream_on(const nitro_spmv *A) { return A->N > 0 && A->Z > (int64_t)kRowCap * A->N; }
 
 void finish_features(int64_t N, int64_t M, int64_t Z, uint64_t s1, uint64_t s2, int64_t lmax, int64_t D,
                      nitro_spmv_feat *f) {
@@ -739,13 +731,13 @@ nitro_status_t features_launch(nitro_spmv *A) {
   int2 *tasks = A->feat_long.as<int2>();
   const unsigned glong = (unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)num_sms() * 4,
                                                                            (A->Z / kChunk + kWarps - 1) / kWarps));
-  if (feat_stream_on()) {  // K1s: rowptr moments (k_rowstats) + the nnz-split pass
+  if (feat_stream_on(A)) {  // K1s: rowptr moments (k_rowstats) + the nnz-split pass
     if (A->N > 0) {
       const unsigned gr = (unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)num_sms() * 8, (A->N + 255) / 256));
       if (A->rp64) k_rowstats<int64_t><<<gr, 256, 0, s>>>((const int64_t *)A->rowptr, A->N, A->Z, acc);
       else k_rowstats<int32_t><<<gr, 256, 0, s>>>((const int32_t *)A->rowptr, A->N, A->Z, acc);
     }
-    const int ep = feat_stream_ep();
+    constexpr int ep = 8;  // entries per lane (16: configs[1] 0.188 vs 0.175 ms, dense band 0.476 vs 0.470)
     const int64_t nch = (A->Z + 32 * ep - 1) / (32 * ep);
     if (nch > 0) {
       const int64_t gs = std::max<int64_t>(1, std::min<int64_t>((int64_t)num_sms() * 8, (nch + kWarps - 1) / kWarps));
@@ -753,8 +745,8 @@ nitro_status_t features_launch(nitro_spmv *A) {
 #define NITRO_K1S(IT, EPV)                                                                                   \
   k_feat_stream<IT, EPV><<<(unsigned)gs, kThreads, 0, s>>>((const IT *)A->rowptr, A->col, A->N, A->M, A->Z, \
                                                            A->row0, G, nch, q, acc, A->bitmap.as<uint32_t>())
-      if (A->rp64) { if (ep == 16) NITRO_K1S(int64_t, 16); else NITRO_K1S(int64_t, 8); }
-      else { if (ep == 16) NITRO_K1S(int32_t, 16); else NITRO_K1S(int32_t, 8); }
+      if (A->rp64) NITRO_K1S(int64_t, ep);
+      else NITRO_K1S(int32_t, ep);
 #undef NITRO_K1S
     }
   } else if (A->rp64) {

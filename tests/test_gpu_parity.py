@@ -47,6 +47,9 @@ def small_mats():
     yield "empty_rows", Csr(70, 70, np.array([0] * 35 + [2] * 36, np.int64), np.array([3, 69], np.int32),
                             np.array([1.0, 2.0], np.float32), False)
     yield "nnz0", Csr(40, 33, np.zeros(41, np.int64), np.zeros(0, np.int32), np.zeros(0, np.float32), False)
+    # mean row length > 64: the nnz-split feature pass K1s
+    yield "uniform_k100_rect", synth.uniform(3000, 100, seed=14, M=9000)
+    yield "banded_b70_half", synth.banded(4001, 70, 0.5, seed=15)
 
 
 def long_row_matrix(L=150_000, N=5000, fp64=False, seed=21):
