@@ -887,7 +887,8 @@ __global__ void __launch_bounds__(256) k_csr_stream(const IT *__restrict__ rowpt
   // (a one-chunk software pipeline — the next chunk's col / val / row range
   // loaded before the current chunk's row work — measured slower: 53 vs 40
   // registers, c2b 0.741 vs 0.716 ms; so did full occupancy by launch bounds,
-  // 32 registers + spills: 0.753 ms)
+  // 32 registers + spills: 0.753 ms; and a per-warp two-stage TMA ring for the
+  // col / val streams, leaving L1TEX to the gathers: 1.056 vs 0.718 ms)
   const int64_t nfull = Z / CH;  // chunks [0, nfull) are full
   auto tma_issue = [&](int64_t chn, int st) {  // lane 0
     const int64_t cn = chn * CH;
