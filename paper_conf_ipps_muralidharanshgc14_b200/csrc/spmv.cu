@@ -854,13 +854,7 @@ __global__ void __launch_bounds__(256) k_hyb_tail_ls(const int32_t *__restrict__
 // rows are zeroed by that chunk (rows before the first nonempty row by chunk
 // 0).  No global atomics (the shared-memory counts are integers):
 // deterministic.
-// TMA: the chunk's column and value arrays are brought into a per-warp
-// two-stage shared-memory ring by cp.async.bulk (one elected lane, mbarrier
-// completion), the next chunk's copy issued before the current chunk is
-// processed, so the L1TEX pipeline serves only the x gathers (ncu, c2b: L1TEX
-// 79 % busy with streams + gathers).  Full chunks only; the last partial
-// chunk (and unaligned arrays: vec false) are read from global memory.
-template <typename IT, typename VT, int EP, bool TMA = false>
+template <typename IT, typename VT, int EP>
 __global__ void __launch_bounds__(256) k_csr_stream(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
                                                     const VT *__restrict__ val, const VT *__restrict__ x,
                                                     VT *__restrict__ y, int64_t N, int64_t Z, int64_t nch,
@@ -870,14 +864,8 @@ __global__ void __launch_bounds__(256) k_csr_stream(const IT *__restrict__ rowpt
   static_assert(EP == 4 || EP == 8, "EP");
   constexpr int64_t CH = 32 * EP;
   __shared__ __align__(16) int s_cnt[8][CH];  // per warp: row starts per chunk position
-  constexpr int RING = TMA ? 2 : 1;
-  constexpr int RC = TMA ? (int)CH : 4;
-  __shared__ __align__(128) int32_t s_col[8][RING][RC];
-  __shared__ __align__(128) VT s_val[8][RING][RC];
-  __shared__ __align__(8) uint64_t s_bar[8][RING];
   const uint64_t pol = l2_policy(l2ef);
   const int lane = threadIdx.x & 31;
-  const int wib = threadIdx.x >> 5;
   const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   if (warp == 0) {  // rows before the first nonempty row (chunk_row[0] = last row starting at 0)
@@ -889,50 +877,13 @@ __global__ void __launch_bounds__(256) k_csr_stream(const IT *__restrict__ rowpt
   // registers, c2b 0.741 vs 0.716 ms; so did full occupancy by launch bounds,
   // 32 registers + spills: 0.753 ms; and a per-warp two-stage TMA ring for the
   // col / val streams, leaving L1TEX to the gathers: 1.056 vs 0.718 ms)
-  const int64_t nfull = Z / CH;  // chunks [0, nfull) are full
-  auto tma_issue = [&](int64_t chn, int st) {  // lane 0
-    const int64_t cn = chn * CH;
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // earlier generic reads of the stage
-    mbar_arrive_expect_tx(&s_bar[wib][st], (uint32_t)(CH * (4 + sizeof(VT))));
-    bulk_g2s_evict_first(&s_col[wib][st][0], col + cn, (uint32_t)(CH * 4), &s_bar[wib][st], pol);
-    bulk_g2s_evict_first(&s_val[wib][st][0], val + cn, (uint32_t)(CH * sizeof(VT)), &s_bar[wib][st], pol);
-  };
-  const bool use_tma = TMA && vec;
-  if constexpr (TMA) {
-    if (lane == 0) {
-      for (int st = 0; st < RING; ++st) mbar_init(&s_bar[wib][st], 1);
-      fence_mbar_init();
-    }
-    __syncwarp();
-    if (use_tma && lane == 0 && warp < nfull) tma_issue(warp, 0);
-  }
-  int it = 0;  // this warp's chunk count (ring stage / parity)
-  for (int64_t ch = warp; ch < nch; ch += nw, ++it) {
+  for (int64_t ch = warp; ch < nch; ch += nw) {
     const int64_t c0 = ch * CH, cend = c0 + CH < Z ? c0 + CH : Z;
     const int64_t e0 = c0 + (int64_t)lane * EP;
     const int nv = e0 >= cend ? 0 : (cend - e0 < EP ? (int)(cend - e0) : EP);
     int c[EP];
     VT v[EP];
-    if (use_tma && ch < nfull) {
-      if (lane == 0 && ch + nw < nfull) tma_issue(ch + nw, (it + 1) & 1);
-      mbar_wait(&s_bar[wib][it & 1], (uint32_t)((it >> 1) & 1));
-      const int4 *sc = reinterpret_cast<const int4 *>(&s_col[wib][it & 1][lane * EP]);
-      const VT *sv = &s_val[wib][it & 1][lane * EP];
-#pragma unroll
-      for (int k = 0; k < EP; k += 4) {
-        const int4 cc = sc[k / 4];
-        c[k] = cc.x; c[k + 1] = cc.y; c[k + 2] = cc.z; c[k + 3] = cc.w;
-        if constexpr (sizeof(VT) == 4) {
-          const float4 t = *reinterpret_cast<const float4 *>(sv + k);
-          v[k] = t.x; v[k + 1] = t.y; v[k + 2] = t.z; v[k + 3] = t.w;
-        } else {
-          const double2 a = *reinterpret_cast<const double2 *>(sv + k);
-          const double2 b = *reinterpret_cast<const double2 *>(sv + k + 2);
-          v[k] = a.x; v[k + 1] = a.y; v[k + 2] = b.x; v[k + 3] = b.y;
-        }
-      }
-      __syncwarp();  // every lane has read the stage before it is refilled
-    } else if (nv == EP && vec) {
+    if (nv == EP && vec) {
 #pragma unroll
       for (int k = 0; k < EP; k += 4) {
         const int4 cc = ld_stream_i4(reinterpret_cast<const int4 *>(col + e0 + k), pol);
@@ -1360,22 +1311,14 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
         const int64_t nch = A->csrv.nch;
         const bool vec = ((reinterpret_cast<uintptr_t>(A->col) | reinterpret_cast<uintptr_t>(val)) & 15) == 0;
         const unsigned gs = grid_cap(std::max<int64_t>((nch + 7) / 8, 1), 16);
-        static const bool tma = [] {
-          const char *e = getenv("NITRO_CSRV_TMA");
-          return e ? atoi(e) != 0 : false;
-        }();
-#define NITRO_K6S(EPV, TM)                                                                                          \
-  k_csr_stream<IT, VT, EPV, TM><<<gs, 256, 0, s>>>(rp, A->col, val, x, y, N, A->Z, nch, A->csrv.chunk_row.as<int32_t>(), \
-                                                  A->csrv.carry_row.as<int32_t>(), A->csrv.carry_val.as<double>(), vec,  \
-                                                  l2_evict_first())
-        if (A->csrv.EP == 4) {
-          if (tma) NITRO_K6S(4, true); else NITRO_K6S(4, false);
-        } else if constexpr (sizeof(VT) == 4) {  // (EP = 8 is the fp32 width only)
-          if (tma) NITRO_K6S(8, true); else NITRO_K6S(8, false);
-        } else {
-          NITRO_K6S(8, false);
-        }
-#undef NITRO_K6S
+        if (A->csrv.EP == 4)
+          k_csr_stream<IT, VT, 4><<<gs, 256, 0, s>>>(rp, A->col, val, x, y, N, A->Z, nch,
+                                                     A->csrv.chunk_row.as<int32_t>(), A->csrv.carry_row.as<int32_t>(),
+                                                     A->csrv.carry_val.as<double>(), vec, l2_evict_first());
+        else
+          k_csr_stream<IT, VT, 8><<<gs, 256, 0, s>>>(rp, A->col, val, x, y, N, A->Z, nch,
+                                                     A->csrv.chunk_row.as<int32_t>(), A->csrv.carry_row.as<int32_t>(),
+                                                     A->csrv.carry_val.as<double>(), vec, l2_evict_first());
         if (nch > 0) {
           const unsigned nshort = grid_cap((A->csrv.fix_S + 255) / 256, 8);
           const unsigned nlong_blk = A->csrv.fix_nlong > 0
