@@ -274,11 +274,14 @@ int run_host_chunks(const nitro_spmv *A, int variant) {
     return e ? atoi(e) : 0;
   }();
   if (variant != NITRO_CSR_SCALAR && variant != NITRO_ELL && variant != NITRO_DIA) return 1;
-  // 4: B200 host wall time of the configs[1] DIA call, pinned buffers (ms):
-  // 1 chunk 0.372, 2 0.320, 4 0.313, 8 0.340, 16 0.410 (smaller copies lose
-  // more to per-copy setup than the finer overlap gains); a CUDA-graph
-  // capture of the enqueue made no difference (the copies, not the host, bound it)
-  const int want = env > 0 ? env : 4;
+  // about one chunk per 32 MB of x, 4 to 16: B200, pinned buffers, DIA —
+  // configs[1] (x 8 MB, ms per call) 1 chunk 0.372, 2 0.320, 4 0.313, 8 0.340,
+  // 16 0.410 (smaller copies lose more to per-copy setup than the finer overlap
+  // gains); configs[4] (x 537 MB) 1: 21.5, 4: 15.1, 8: 13.6, 16: 13.3, 32: 13.4
+  // (81 GB/s of H2D + D2H, the PCIe limit with both directions busy).  A
+  // CUDA-graph capture of the enqueue made no difference (copies, not the host, bound it)
+  const double xmb = (double)A->M * (A->fp64 ? 8 : 4) / (32.0 * 1048576.0);
+  const int want = env > 0 ? env : (int)std::max(4.0, std::min(16.0, std::ceil(xmb)));
   if (want <= 1 || A->N < (int64_t)want * 32768) return 1;
   return want;
 }
