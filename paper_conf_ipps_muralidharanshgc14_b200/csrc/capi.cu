@@ -237,7 +237,9 @@ nitro_status_t nitro_spmv_format_info(nitro_spmv *A, int variant, nitro_format_i
       out->width = A->csrv.stream ? 0 : A->csrv.V;  // 0: nnz-split stream mode (K6s)
       out->tail = A->csrv.stream ? A->csrv.nch : A->csrv.n_long;
       out->bytes = (int64_t)(A->csrv.long_rows.bytes + A->csrv.chunk_row.bytes + A->csrv.carry_row.bytes +
-                             A->csrv.carry_val.bytes + A->csrv.fix_seg.bytes + A->csrv.fix_long.bytes);
+                             A->csrv.carry_val.bytes + A->csrv.fix_seg.bytes + A->csrv.fix_long.bytes +
+                             A->csrv.hot_cols.bytes + A->csrv.hcol.bytes);
+      out->ld = A->csrv.nhot;  // stream mode: hot x values staged in shared memory (0 = none)
       break;
     case NITRO_ELL: out->ld = A->ell.ld; out->width = A->ell.K; out->bytes = (int64_t)(A->ell.col.bytes + A->ell.val.bytes); break;
     case NITRO_DIA: out->ld = A->dia.ld; out->width = A->dia.D; out->bytes = (int64_t)(A->dia.off.bytes + A->dia.val.bytes); break;
@@ -477,6 +479,7 @@ nitro_status_t nitro_spmv_release(nitro_spmv *A, int variant) {
     A->csrv.long_rows.release();
     A->csrv.chunk_row.release(); A->csrv.carry_row.release(); A->csrv.carry_val.release();
     A->csrv.fix_seg.release(); A->csrv.fix_long.release();
+    A->csrv.hot_cols.release(); A->csrv.hcol.release(); A->csrv.nhot = 0;
     A->csrv.ready = false;
   }
   return NITRO_OK;

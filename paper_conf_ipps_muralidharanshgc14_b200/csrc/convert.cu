@@ -449,6 +449,15 @@ bool csrv_stream_mode(const nitro_spmv *A) {
   return A->feat_ready && A->feat.sd > A->feat.mean;
 }
 
+// NITRO_CSRV_HOT=0 disables the hot-x staging of K6s
+bool csrv_hot_on() {
+  static int env = [] {
+    const char *e = getenv("NITRO_CSRV_HOT");
+    return e ? atoi(e) : 1;
+  }();
+  return env != 0;
+}
+
 // ------------------------------------------------------------------ CSR-vector stream mode (K6s)
 // chunk_row[c] = the row holding entry c*CH (the last row whose start <= c*CH),
 // chunk_row[nch] = N; eff[2c] / eff[2c+1] = rows of the chunk's first / last
@@ -472,6 +481,104 @@ __global__ void k_stream_rows(const IT *__restrict__ rowptr, int64_t N, int64_t 
     eff[2 * c] = r0;
     eff[2 * c + 1] = row_of(e1);
   }
+}
+
+// ------------------------------------------------------------------ K6s hot-x staging
+__global__ void k_col_deg(const int32_t *__restrict__ col, int64_t Z, unsigned *__restrict__ deg) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < Z; e += (int64_t)gridDim.x * blockDim.x)
+    atomicAdd(deg + col[e], 1u);
+}
+// bins[b] = #columns with floor(log2(deg)) == b (deg >= 1), b < 32
+__global__ void k_deg_hist(const unsigned *__restrict__ deg, int64_t M, unsigned long long *__restrict__ bins) {
+  __shared__ unsigned long long sb[32];
+  if (threadIdx.x < 32) sb[threadIdx.x] = 0;
+  __syncthreads();
+  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < M; c += (int64_t)gridDim.x * blockDim.x)
+    if (deg[c]) atomicAdd(&sb[31 - __clz(deg[c])], 1ull);
+  __syncthreads();
+  if (threadIdx.x < 32 && sb[threadIdx.x]) atomicAdd(bins + threadIdx.x, sb[threadIdx.x]);
+}
+__global__ void k_hot_flags(const unsigned *__restrict__ deg, int64_t M, unsigned thr, int64_t *__restrict__ f,
+                            unsigned long long *__restrict__ covered) {
+  unsigned long long cv = 0;
+  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < M; c += (int64_t)gridDim.x * blockDim.x) {
+    const bool h = deg[c] >= thr;
+    f[c] = h ? 1 : 0;
+    if (h) cv += deg[c];
+  }
+  for (int o = 16; o > 0; o >>= 1) cv += __shfl_xor_sync(0xffffffffu, cv, o);
+  if ((threadIdx.x & 31) == 0 && cv) atomicAdd(covered, cv);
+}
+// hot column c -> slot pos[c]: hot_cols[slot] = c, and slot_of[c] = slot (else -1)
+__global__ void k_hot_emit(const int64_t *__restrict__ f, const int64_t *__restrict__ pos, int64_t M,
+                           int32_t *__restrict__ hot_cols, int32_t *__restrict__ slot_of) {
+  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < M; c += (int64_t)gridDim.x * blockDim.x) {
+    if (f[c]) { hot_cols[pos[c]] = (int32_t)c; slot_of[c] = (int32_t)pos[c]; }
+    else slot_of[c] = -1;
+  }
+}
+__global__ void k_hot_remap(const int32_t *__restrict__ col, int64_t Z, const int32_t *__restrict__ slot_of,
+                            int32_t *__restrict__ hcol) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < Z; e += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t c = col[e], sl = slot_of[c];
+    hcol[e] = sl >= 0 ? ~sl : c;
+  }
+}
+
+// The hot set: the columns of degree >= 2^b for the smallest b that keeps at
+// most cap of them (whole log2 degree classes), at least kHotMinDeg
+// references each; used when they cover >= kHotMinShare of the nonzeros.
+constexpr unsigned kHotMinDeg = 16;
+constexpr double kHotMinShare = 0.10;
+nitro_status_t prepare_hot(nitro_spmv *A, int64_t cap) {
+  cudaStream_t s = A->stream;
+  const int64_t M = A->M, Z = A->Z;
+  A->csrv.nhot = 0;
+  A->csrv.hot_share = 0.0;
+  if (M <= 0 || Z <= 0 || cap <= 0) return NITRO_OK;
+  DevBuf deg, aux;
+  NITRO_TRY(deg.alloc((size_t)M * 4));
+  NITRO_TRY(aux.alloc(34 * 8));
+  unsigned long long *bins = aux.as<unsigned long long>(), *covered = bins + 32;
+  NITRO_CUDA(cudaMemsetAsync(deg.p, 0, (size_t)M * 4, s));
+  NITRO_CUDA(cudaMemsetAsync(aux.p, 0, 34 * 8, s));
+  k_col_deg<<<grid_of(Z), 256, 0, s>>>(A->col, Z, deg.as<unsigned>());
+  k_deg_hist<<<grid_of(M), 256, 0, s>>>(deg.as<unsigned>(), M, bins);
+  unsigned long long hb[32];
+  NITRO_CUDA(cudaMemcpyAsync(hb, bins, sizeof(hb), cudaMemcpyDeviceToHost, s));
+  NITRO_CUDA(cudaStreamSynchronize(s));
+  int bsel = -1;  // whole log2 degree classes from the top, >= kHotMinDeg, at most cap columns
+  int64_t n = 0;
+  for (int k = 31; k >= 0 && (1u << k) >= kHotMinDeg; --k) {
+    if (n + (int64_t)hb[k] > cap) break;
+    n += (int64_t)hb[k];
+    bsel = k;
+  }
+  if (bsel < 0 || n == 0) return NITRO_OK;
+  const unsigned thr = 1u << bsel;
+  DevBuf fl;
+  NITRO_TRY(fl.alloc((size_t)(2 * M + 2) * 8));
+  int64_t *f = fl.as<int64_t>(), *pos = f + M + 1;
+  k_hot_flags<<<grid_of(M), 256, 0, s>>>(deg.as<unsigned>(), M, thr, f, covered);
+  NITRO_TRY(exclusive_scan_i64(f, pos, M, A->scratch, s));
+  int64_t nh = 0;
+  unsigned long long cov = 0;
+  NITRO_CUDA(cudaMemcpyAsync(&nh, pos + M, 8, cudaMemcpyDeviceToHost, s));
+  NITRO_CUDA(cudaMemcpyAsync(&cov, covered, 8, cudaMemcpyDeviceToHost, s));
+  NITRO_CUDA(cudaStreamSynchronize(s));
+  const double share = (double)cov / (double)Z;
+  if (nh == 0 || nh > cap || share < kHotMinShare) return NITRO_OK;
+  NITRO_TRY(A->csrv.hot_cols.alloc((size_t)nh * 4));
+  NITRO_TRY(A->csrv.hcol.alloc((size_t)Z * 4));
+  DevBuf slot;
+  NITRO_TRY(slot.alloc((size_t)M * 4));
+  k_hot_emit<<<grid_of(M), 256, 0, s>>>(f, pos, M, A->csrv.hot_cols.as<int32_t>(), slot.as<int32_t>());
+  k_hot_remap<<<grid_of(Z), 256, 0, s>>>(A->col, Z, slot.as<int32_t>(), A->csrv.hcol.as<int32_t>());
+  NITRO_CUDA(cudaGetLastError());
+  NITRO_CUDA(cudaStreamSynchronize(s));  // deg / fl / slot are freed on return
+  A->csrv.nhot = nh;
+  A->csrv.hot_share = share;
+  return NITRO_OK;
 }
 
 // ------------------------------------------------------------------ CSR-vector (C8)
@@ -536,6 +643,9 @@ nitro_status_t prepare_csrv(nitro_spmv *A) {
     A->csrv.fix_S = S;
     A->csrv.fix_nlong = (int64_t)nl;
     A->csrv.n_long = 0;
+    // hot-x staging: up to 64 KB of x values per CTA (8192 fp64 / 16384 fp32)
+    if (csrv_hot_on()) NITRO_TRY(prepare_hot(A, (int64_t)(65536 / (A->fp64 ? 8 : 4))));
+    else A->csrv.nhot = 0;
     A->csrv.ready = true;
     return NITRO_OK;
   }

@@ -85,6 +85,12 @@ struct CsrvFmt {
   int64_t nch = 0;
   DevBuf chunk_row, carry_row, carry_val, fix_seg, fix_long;
   int64_t fix_S = 0, fix_nlong = 0;
+  // hot-x staging (x-locality, the modern "-Tx"): the nhot most referenced
+  // columns (power-law matrices) are copied into shared memory per CTA; hcol
+  // = the column ids with a hot column c replaced by ~slot (negative)
+  int64_t nhot = 0;
+  double hot_share = 0.0;  // fraction of the nonzeros whose column is hot
+  DevBuf hot_cols, hcol;
 };
 
 }  // namespace nitro
@@ -188,6 +194,7 @@ int hyb_windows(size_t sv);
 // CSR-vector mode: the nnz-split stream kernel (K6s) for skewed row lengths
 // (row-length SD above the mean); NITRO_CSRV_STREAM=0/1 forces it off/on.
 bool csrv_stream_mode(const nitro_spmv *A);
+bool csrv_hot_on();
 // bitmap index of diagonal offset d is d + G; the bitmap spans G + M bits
 inline int64_t diag_shift(const nitro_spmv *A) { return A->feat_G >= 0 ? A->feat_G : A->row0 + A->N - 1; }
 int num_sms();

@@ -854,16 +854,30 @@ __global__ void __launch_bounds__(256) k_hyb_tail_ls(const int32_t *__restrict__
 // rows are zeroed by that chunk (rows before the first nonempty row by chunk
 // 0).  No global atomics (the shared-memory counts are integers):
 // deterministic.
-template <typename IT, typename VT, int EP>
-__global__ void __launch_bounds__(256) k_csr_stream(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
+// HOT (x-locality, the modern analogue of the paper's texture-cached "-Tx"
+// variants): the nhot most referenced columns of a power-law
+// matrix are staged in shared memory once per CTA (persistent CTAs, one per
+// SM, 1024 threads); `col` is then the remapped column array whose hot entries
+// hold ~slot, and their x value comes from shared memory instead of an L1TEX
+// gather (the resource that binds this kernel, §9.0).
+template <typename IT, typename VT, int EP, bool HOT = false>
+__global__ void __launch_bounds__(HOT ? 1024 : 256) k_csr_stream(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
                                                     const VT *__restrict__ val, const VT *__restrict__ x,
                                                     VT *__restrict__ y, int64_t N, int64_t Z, int64_t nch,
                                                     const int32_t *__restrict__ chunk_row,
                                                     int32_t *__restrict__ carry_row, double *__restrict__ carry_val,
-                                                    bool vec, bool l2ef) {
+                                                    bool vec, bool l2ef, const int32_t *__restrict__ hot_cols = nullptr,
+                                                    int nhot = 0) {
   static_assert(EP == 4 || EP == 8, "EP");
   constexpr int64_t CH = 32 * EP;
-  __shared__ __align__(16) int s_cnt[8][CH];  // per warp: row starts per chunk position
+  constexpr int NW = HOT ? 32 : 8;
+  __shared__ __align__(16) int s_cnt[NW][CH];  // per warp: row starts per chunk position
+  extern __shared__ __align__(16) unsigned char s_dyn[];
+  VT *s_hot = reinterpret_cast<VT *>(s_dyn);
+  if constexpr (HOT) {
+    for (int j = threadIdx.x; j < nhot; j += blockDim.x) s_hot[j] = __ldg(x + hot_cols[j]);
+    __syncthreads();
+  }
   const uint64_t pol = l2_policy(l2ef);
   const int lane = threadIdx.x & 31;
   const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
@@ -903,7 +917,14 @@ __global__ void __launch_bounds__(256) k_csr_stream(const IT *__restrict__ rowpt
     const int r_lo = chunk_row[ch], r_nx = chunk_row[ch + 1];
     double p[EP];
 #pragma unroll
-    for (int k = 0; k < EP; ++k) p[k] = k < nv ? (double)v[k] * (double)__ldg(x + c[k]) : 0.0;
+    for (int k = 0; k < EP; ++k) {
+      VT xv = (VT)0;
+      if (k < nv) {
+        if constexpr (HOT) xv = c[k] >= 0 ? __ldg(x + c[k]) : s_hot[~c[k]];
+        else xv = __ldg(x + c[k]);
+      }
+      p[k] = (double)v[k] * (double)xv;
+    }
     // rows of the entries: row(e) = r_lo + #{rows r in (r_lo, r_hi] starting at
     // or before chunk position e}.  The rows' starts are counted into a per-warp
     // shared array over the chunk's positions (windows of 32 rows, one per
@@ -1310,6 +1331,28 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
       if (A->csrv.stream) {  // K6s: nnz-split chunks + carry fixup
         const int64_t nch = A->csrv.nch;
         const bool vec = ((reinterpret_cast<uintptr_t>(A->col) | reinterpret_cast<uintptr_t>(val)) & 15) == 0;
+        if (A->csrv.nhot > 0) {  // hot-x staging: one persistent 1024-thread CTA per SM
+          const size_t hs = (size_t)A->csrv.nhot * sizeof(VT);
+          const unsigned gh = (unsigned)std::max<int64_t>(1, std::min<int64_t>(num_sms(), (nch + 31) / 32));
+          const int32_t *hc = A->csrv.hcol.as<int32_t>();
+#define NITRO_K6H(EPV)                                                                                            \
+  do {                                                                                                            \
+    static bool attr_ = false;                                                                                    \
+    if (!attr_) {                                                                                                 \
+      NITRO_CUDA(cudaFuncSetAttribute(k_csr_stream<IT, VT, EPV, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, \
+                                      65536));                                                                    \
+      attr_ = true;                                                                                               \
+    }                                                                                                             \
+    k_csr_stream<IT, VT, EPV, true><<<gh, 1024, hs, s>>>(rp, hc, val, x, y, N, A->Z, nch,                          \
+                                                         A->csrv.chunk_row.as<int32_t>(),                          \
+                                                         A->csrv.carry_row.as<int32_t>(),                          \
+                                                         A->csrv.carry_val.as<double>(), vec, l2_evict_first(),    \
+                                                         A->csrv.hot_cols.as<int32_t>(), (int)A->csrv.nhot);       \
+  } while (0)
+          if (A->csrv.EP == 4) NITRO_K6H(4);
+          else NITRO_K6H(8);
+#undef NITRO_K6H
+        } else {
         const unsigned gs = grid_cap(std::max<int64_t>((nch + 7) / 8, 1), 16);
         if (A->csrv.EP == 4)
           k_csr_stream<IT, VT, 4><<<gs, 256, 0, s>>>(rp, A->col, val, x, y, N, A->Z, nch,
@@ -1319,6 +1362,7 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
           k_csr_stream<IT, VT, 8><<<gs, 256, 0, s>>>(rp, A->col, val, x, y, N, A->Z, nch,
                                                      A->csrv.chunk_row.as<int32_t>(), A->csrv.carry_row.as<int32_t>(),
                                                      A->csrv.carry_val.as<double>(), vec, l2_evict_first());
+        }
         if (nch > 0) {
           const unsigned nshort = grid_cap((A->csrv.fix_S + 255) / 256, 8);
           const unsigned nlong_blk = A->csrv.fix_nlong > 0
