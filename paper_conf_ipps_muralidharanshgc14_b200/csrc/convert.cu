@@ -498,6 +498,14 @@ __global__ void k_deg_hist(const unsigned *__restrict__ deg, int64_t M, unsigned
   __syncthreads();
   if (threadIdx.x < 32 && sb[threadIdx.x]) atomicAdd(bins + threadIdx.x, sb[threadIdx.x]);
 }
+__global__ void k_deg_count(const unsigned *__restrict__ deg, int64_t M, unsigned t,
+                            unsigned long long *__restrict__ out) {
+  unsigned long long c = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < M; i += (int64_t)gridDim.x * blockDim.x)
+    c += deg[i] >= t;
+  for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+  if ((threadIdx.x & 31) == 0 && c) atomicAdd(out, c);
+}
 __global__ void k_hot_flags(const unsigned *__restrict__ deg, int64_t M, unsigned thr, int64_t *__restrict__ f,
                             unsigned long long *__restrict__ covered) {
   unsigned long long cv = 0;
@@ -525,9 +533,9 @@ __global__ void k_hot_remap(const int32_t *__restrict__ col, int64_t Z, const in
   }
 }
 
-// The hot set: the columns of degree >= 2^b for the smallest b that keeps at
-// most cap of them (whole log2 degree classes), at least kHotMinDeg
-// references each; used when they cover >= kHotMinShare of the nonzeros.
+// The hot set: the columns of degree >= T for the smallest T >= kHotMinDeg
+// that keeps at most cap of them; used when they cover >= kHotMinShare of the
+// nonzeros.
 constexpr unsigned kHotMinDeg = 16;
 constexpr double kHotMinShare = 0.10;
 nitro_status_t prepare_hot(nitro_spmv *A, int64_t cap) {
@@ -547,15 +555,35 @@ nitro_status_t prepare_hot(nitro_spmv *A, int64_t cap) {
   unsigned long long hb[32];
   NITRO_CUDA(cudaMemcpyAsync(hb, bins, sizeof(hb), cudaMemcpyDeviceToHost, s));
   NITRO_CUDA(cudaStreamSynchronize(s));
-  int bsel = -1;  // whole log2 degree classes from the top, >= kHotMinDeg, at most cap columns
-  int64_t n = 0;
-  for (int k = 31; k >= 0 && (1u << k) >= kHotMinDeg; --k) {
-    if (n + (int64_t)hb[k] > cap) break;
-    n += (int64_t)hb[k];
-    bsel = k;
+  // the smallest degree threshold T >= kHotMinDeg with #{c : deg(c) >= T} <= cap
+  // (bisection over T, one counting pass per step; the log2 histogram bounds it)
+  int top = 31;
+  while (top > 0 && hb[top] == 0) --top;
+  unsigned lo = kHotMinDeg, hi = top >= 31 ? 0xffffffffu : (2u << top);  // count(hi) == 0
+  if (hi <= lo) return NITRO_OK;
+  DevBuf cntb;
+  NITRO_TRY(cntb.alloc(8));
+  auto count_ge = [&](unsigned t, int64_t &out) -> nitro_status_t {
+    NITRO_CUDA(cudaMemsetAsync(cntb.p, 0, 8, s));
+    k_deg_count<<<grid_of(M), 256, 0, s>>>(deg.as<unsigned>(), M, t, cntb.as<unsigned long long>());
+    unsigned long long h = 0;
+    NITRO_CUDA(cudaMemcpyAsync(&h, cntb.p, 8, cudaMemcpyDeviceToHost, s));
+    NITRO_CUDA(cudaStreamSynchronize(s));
+    out = (int64_t)h;
+    return NITRO_OK;
+  };
+  int64_t c_lo = 0;
+  NITRO_TRY(count_ge(lo, c_lo));
+  unsigned thr = lo;
+  if (c_lo > cap) {  // bisection: count(lo) > cap >= count(hi)
+    while (hi - lo > 1) {
+      const unsigned mid = lo + (hi - lo) / 2;
+      int64_t cm = 0;
+      NITRO_TRY(count_ge(mid, cm));
+      if (cm > cap) lo = mid; else hi = mid;
+    }
+    thr = hi;
   }
-  if (bsel < 0 || n == 0) return NITRO_OK;
-  const unsigned thr = 1u << bsel;
   DevBuf fl;
   NITRO_TRY(fl.alloc((size_t)(2 * M + 2) * 8));
   int64_t *f = fl.as<int64_t>(), *pos = f + M + 1;

@@ -856,12 +856,12 @@ __global__ void __launch_bounds__(256) k_hyb_tail_ls(const int32_t *__restrict__
 // deterministic.
 // HOT (x-locality, the modern analogue of the paper's texture-cached "-Tx"
 // variants): the nhot most referenced columns of a power-law
-// matrix are staged in shared memory once per CTA (persistent CTAs, one per
-// SM, 1024 threads); `col` is then the remapped column array whose hot entries
+// matrix are staged in shared memory once per CTA (persistent CTAs, two per
+// SM, 768 threads); `col` is then the remapped column array whose hot entries
 // hold ~slot, and their x value comes from shared memory instead of an L1TEX
 // gather (the resource that binds this kernel, §9.0).
 template <typename IT, typename VT, int EP, bool HOT = false>
-__global__ void __launch_bounds__(HOT ? 1024 : 256) k_csr_stream(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
+__global__ void __launch_bounds__(HOT ? 768 : 256, HOT ? 2 : 1) k_csr_stream(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
                                                     const VT *__restrict__ val, const VT *__restrict__ x,
                                                     VT *__restrict__ y, int64_t N, int64_t Z, int64_t nch,
                                                     const int32_t *__restrict__ chunk_row,
@@ -870,7 +870,7 @@ __global__ void __launch_bounds__(HOT ? 1024 : 256) k_csr_stream(const IT *__res
                                                     int nhot = 0) {
   static_assert(EP == 4 || EP == 8, "EP");
   constexpr int64_t CH = 32 * EP;
-  constexpr int NW = HOT ? 32 : 8;
+  constexpr int NW = HOT ? 24 : 8;
   __shared__ __align__(16) int s_cnt[NW][CH];  // per warp: row starts per chunk position
   extern __shared__ __align__(16) unsigned char s_dyn[];
   VT *s_hot = reinterpret_cast<VT *>(s_dyn);
@@ -1331,9 +1331,9 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
       if (A->csrv.stream) {  // K6s: nnz-split chunks + carry fixup
         const int64_t nch = A->csrv.nch;
         const bool vec = ((reinterpret_cast<uintptr_t>(A->col) | reinterpret_cast<uintptr_t>(val)) & 15) == 0;
-        if (A->csrv.nhot > 0) {  // hot-x staging: one persistent 1024-thread CTA per SM
+        if (A->csrv.nhot > 0) {  // hot-x staging: two persistent 768-thread CTAs per SM
           const size_t hs = (size_t)A->csrv.nhot * sizeof(VT);
-          const unsigned gh = (unsigned)std::max<int64_t>(1, std::min<int64_t>(num_sms(), (nch + 31) / 32));
+          const unsigned gh = (unsigned)std::max<int64_t>(1, std::min<int64_t>(2 * num_sms(), (nch + 23) / 24));
           const int32_t *hc = A->csrv.hcol.as<int32_t>();
 #define NITRO_K6H(EPV)                                                                                            \
   do {                                                                                                            \
@@ -1343,7 +1343,7 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
                                       65536));                                                                    \
       attr_ = true;                                                                                               \
     }                                                                                                             \
-    k_csr_stream<IT, VT, EPV, true><<<gh, 1024, hs, s>>>(rp, hc, val, x, y, N, A->Z, nch,                          \
+    k_csr_stream<IT, VT, EPV, true><<<gh, 768, hs, s>>>(rp, hc, val, x, y, N, A->Z, nch,                           \
                                                          A->csrv.chunk_row.as<int32_t>(),                          \
                                                          A->csrv.carry_row.as<int32_t>(),                          \
                                                          A->csrv.carry_val.as<double>(), vec, l2_evict_first(),    \
