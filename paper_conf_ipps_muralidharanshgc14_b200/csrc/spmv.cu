@@ -861,7 +861,7 @@ __global__ void __launch_bounds__(256) k_hyb_tail_ls(const int32_t *__restrict__
 // hold ~slot, and their x value comes from shared memory instead of an L1TEX
 // gather (the resource that binds this kernel, §9.0).
 template <typename IT, typename VT, int EP, bool HOT = false>
-__global__ void __launch_bounds__(HOT ? 768 : 256, HOT ? 2 : 1) k_csr_stream(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
+__global__ void __launch_bounds__(HOT ? 768 : 256, HOT ? (EP == 4 ? 2 : 1) : (EP == 4 ? 6 : 4)) k_csr_stream(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
                                                     const VT *__restrict__ val, const VT *__restrict__ x,
                                                     VT *__restrict__ y, int64_t N, int64_t Z, int64_t nch,
                                                     const int32_t *__restrict__ chunk_row,
@@ -916,14 +916,13 @@ __global__ void __launch_bounds__(HOT ? 768 : 256, HOT ? 2 : 1) k_csr_stream(con
     }
     const int r_lo = chunk_row[ch], r_nx = chunk_row[ch + 1];
     double p[EP];
+    if constexpr (HOT) {
 #pragma unroll
-    for (int k = 0; k < EP; ++k) {
-      VT xv = (VT)0;
-      if (k < nv) {
-        if constexpr (HOT) xv = c[k] >= 0 ? __ldg(x + c[k]) : s_hot[~c[k]];
-        else xv = __ldg(x + c[k]);
-      }
-      p[k] = (double)v[k] * (double)xv;
+      for (int k = 0; k < EP; ++k)
+        p[k] = k < nv ? (double)v[k] * (double)(c[k] >= 0 ? __ldg(x + c[k]) : s_hot[~c[k]]) : 0.0;
+    } else {
+#pragma unroll
+      for (int k = 0; k < EP; ++k) p[k] = k < nv ? (double)v[k] * (double)__ldg(x + c[k]) : 0.0;
     }
     // rows of the entries: row(e) = r_lo + #{rows r in (r_lo, r_hi] starting at
     // or before chunk position e}.  The rows' starts are counted into a per-warp
@@ -1333,7 +1332,8 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
         const bool vec = ((reinterpret_cast<uintptr_t>(A->col) | reinterpret_cast<uintptr_t>(val)) & 15) == 0;
         if (A->csrv.nhot > 0) {  // hot-x staging: two persistent 768-thread CTAs per SM
           const size_t hs = (size_t)A->csrv.nhot * sizeof(VT);
-          const unsigned gh = (unsigned)std::max<int64_t>(1, std::min<int64_t>(2 * num_sms(), (nch + 23) / 24));
+          const int per_sm = A->csrv.EP == 4 ? 2 : 1;  // resident 768-thread CTAs (registers)
+          const unsigned gh = (unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)per_sm * num_sms(), (nch + 23) / 24));
           const int32_t *hc = A->csrv.hcol.as<int32_t>();
 #define NITRO_K6H(EPV)                                                                                            \
   do {                                                                                                            \

@@ -719,7 +719,10 @@ def test_csr_stream_mode(cuda, name, A):
         M.run(n.CSR_VECTOR, xd, y)
         torch.cuda.synchronize()
         ys.append(y.cpu().numpy())
-    assert M.format_info(n.CSR_VECTOR)["width"] == 0          # stream mode active
+    fi = M.format_info(n.CSR_VECTOR)
+    assert fi["width"] == 0                                    # stream mode active
+    if name.startswith("rmat"):
+        assert fi["ld"] > 0                                    # hot-x staging engaged (power-law columns)
     assert np.all(np.isfinite(ys[0]))                          # every row written (empty rows = 0)
     if exact:
         assert np.array_equal(ys[0].astype(np.float64), y_ref)
