@@ -173,7 +173,7 @@ __device__ __forceinline__ void merge_window(const uint32_t *s_win, uint32_t win
 
 // Offset index idx = col - row + G is < 2^32 (rows, cols < 2^31), so all
 // per-entry arithmetic is 32-bit.
-template <typename IT, bool MATCH = false>
+template <typename IT>
 __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
                                                         int64_t N, int64_t M, int64_t Z, int64_t row0, int64_t G,
                                                         FeatAcc *__restrict__ acc, uint32_t *__restrict__ bitmap,
@@ -244,18 +244,8 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
       prev = c;
       const uint32_t rel = (uint32_t)c - rbase;
       if (rel < kWin) {
-        if (MATCH) {
-          // rows of a stencil / band block share their offsets: one lane per
-          // distinct offset among the converged lanes tests / sets the bit
-          const unsigned grp = __match_any_sync(__activemask(), rel);
-          if ((unsigned)(__ffs(grp) - 1) == (unsigned)lane) {
-            const uint32_t bit = 1u << (rel & 31);
-            if (!(s_win[rel >> 5] & bit)) atomicOr(&s_win[rel >> 5], bit);
-          }
-        } else {
-          const uint32_t bit = 1u << (rel & 31);
-          if (!(s_win[rel >> 5] & bit)) atomicOr(&s_win[rel >> 5], bit);
-        }
+        const uint32_t bit = 1u << (rel & 31);
+        if (!(s_win[rel >> 5] & bit)) atomicOr(&s_win[rel >> 5], bit);
       } else if ((uint32_t)c < M32) {
         lane_far((uint32_t)c - myrow + G32, full);
       }
@@ -697,14 +687,6 @@ __global__ void __launch_bounds__(256) k_popc(const uint32_t *__restrict__ bm, i
 // is also ahead on skewed rows (configs[2] R-MAT 0.943 -> 0.804 ms) and sparse
 // bands (0.275 -> 0.200 ms), but telling those apart needs the row-length SD,
 // i.e. a pass before the launch; the rule uses what is known at create time.
-bool feat_match_on() {  // A/B: NITRO_FEAT_MATCH=1
-  static bool v = [] {
-    const char *e = getenv("NITRO_FEAT_MATCH");
-    return e ? atoi(e) != 0 : false;
-  }();
-  return v;
-}
-
 bool feat_stream_on(const nitro_spmv *A) { return A->N > 0 && A->Z > (int64_t)kRowCap * A->N; }
 
 void finish_features(int64_t N, int64_t M, int64_t Z, uint64_t s1, uint64_t s2, int64_t lmax, int64_t D,
@@ -768,22 +750,12 @@ nitro_status_t features_launch(nitro_spmv *A) {
 #undef NITRO_K1S
     }
   } else if (A->rp64) {
-    if (feat_match_on())
-      k_features<int64_t, true><<<(unsigned)grid, kThreads, 0, s>>>((const int64_t *)A->rowptr, A->col, A->N, A->M,
-                                                                    A->Z, A->row0, G, acc, A->bitmap.as<uint32_t>(),
-                                                                    tasks, cap_tasks);
-    else
     k_features<int64_t><<<(unsigned)grid, kThreads, 0, s>>>((const int64_t *)A->rowptr, A->col, A->N, A->M, A->Z,
                                                             A->row0, G, acc, A->bitmap.as<uint32_t>(), tasks, cap_tasks);
     if (A->Z > kLong)
       k_features_long<int64_t><<<glong, kThreads, 0, s>>>((const int64_t *)A->rowptr, A->col, A->M, A->row0, G, acc,
                                                           A->bitmap.as<uint32_t>(), tasks, cap_tasks);
   } else {
-    if (feat_match_on())
-      k_features<int32_t, true><<<(unsigned)grid, kThreads, 0, s>>>((const int32_t *)A->rowptr, A->col, A->N, A->M,
-                                                                    A->Z, A->row0, G, acc, A->bitmap.as<uint32_t>(),
-                                                                    tasks, cap_tasks);
-    else
     k_features<int32_t><<<(unsigned)grid, kThreads, 0, s>>>((const int32_t *)A->rowptr, A->col, A->N, A->M, A->Z,
                                                             A->row0, G, acc, A->bitmap.as<uint32_t>(), tasks, cap_tasks);
     if (A->Z > kLong)
