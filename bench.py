@@ -59,6 +59,21 @@ MODELS = {"paper": os.path.join(ROOT, "artifacts", "spmv_model.txt"),
 MODEL_DOC = {"paper": "plain [-1,1] min-max scaling (P:L179)",
              "r11x": "EXTENSION R11x: log1p of the 7 features + clip (DESIGN.md; not from the paper)"}
 NCU_SUMMARY = os.path.join(ROOT, "profiles", "ncu_summary.json")
+GATHER_PROBE = os.path.join(ROOT, "profiles", "r02", "l2_gather_probe.jsonl")
+
+
+def gather_rate():
+    """Measured random-gather ceiling (gathers/s) of this part: the best
+    'gathers only' case of tools/probes/l2_gather_probe.cu (profiles/r02)."""
+    try:
+        best = 0.0
+        for line in open(GATHER_PROBE):
+            d = json.loads(line)
+            if str(d.get("case", "")).startswith("A_gather_only"):
+                best = max(best, float(d["gathers_per_s"]))
+        return best or None
+    except Exception:
+        return None
 
 WORKLOADS = {
     "c4": ("3d27pt_stencil_512^3_fp32 (BASELINE configs[4])", "stencil", ("3d27", 512, False)),
@@ -294,12 +309,17 @@ def measure_config(nitro, cfg, dev, models, reps, log):
                                       "bytes": info["compulsory_bytes"], "conversion_ms": a.elapsed_time(b)}
         M.release(v)
     best = min(ex, key=lambda k: ex[k]["ms"])
+    A_nnz = A.nnz
     out = {"workload": WORKLOADS[cfg][0], "rows": A.rows, "nnz": A.nnz, "generate_s": gen_s,
            "feature_ms": statistics.median(fts), "features": {k: f[k] for k in nitro.FEATURE_NAMES},
            "allowed": [nitro.VARIANT_NAMES[v] for v in range(nitro.NUM_VARIANTS) if allowed[v]],
            "picks": picks, "exhaustive_best": best, "exhaustive": ex}
     for k, name in picks.items():
         out[f"pct_of_exhaustive_best_{k}"] = ex[best]["ms"] / ex[name]["ms"]
+    g = gather_rate()
+    if g:  # random-column classes: one x gather per nonzero bounds the multiply
+        out["gather_bound_ms"] = A_nnz / g * 1e3
+        out["best_frac_of_gather_bound"] = out["gather_bound_ms"] / ex[best]["ms"]
     M.close()
     del A, x, y, M
     torch.cuda.empty_cache()
