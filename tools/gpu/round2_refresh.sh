@@ -4,6 +4,7 @@ nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv,noheader
 timeout 1800 python tools/train_select.py > gpurun_out/c3_train_select.log 2>&1; echo "c3 rc=$?"; tail -30 gpurun_out/c3_train_select.log
 timeout 900 python tools/itune_c3.py > gpurun_out/c3_itune.log 2>&1; echo "itune rc=$?"; tail -3 gpurun_out/c3_itune.log
 timeout 1200 python tools/feature_study.py --gpu > gpurun_out/feature_study.log 2>&1; echo "fstudy rc=$?"; tail -4 gpurun_out/feature_study.log
+timeout 600 python tools/profile_variants.py --time c1 c2a c2b short band01 uvar3 band48 c4 > gpurun_out/variant_table_r02.json 2>/dev/null; echo "table rc=$?"
 cp artifacts/* gpurun_out/artifacts/
 timeout 900 python bench.py > gpurun_out/bench_r02.json 2> gpurun_out/bench_r02.err; echo "bench rc=$?"; tail -20 gpurun_out/bench_r02.err
 timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none --csv -c 600 \
