@@ -285,3 +285,17 @@ def test_dist_format_info_sums_the_rank_parts(cuda):
     want = Z * 8 + N * 4 + sum(p + 0 for p in nparts) * 4 + sum(g[1]["layout_len"] * 4 for g in got) + N * 4
     tot = sum(g[0]["compulsory_bytes"] for g in got)
     assert abs(tot - want) < 1e-6 * want, (tot, want, nparts)
+
+
+def test_solver_loop_needs_the_allgather_layout(cuda):
+    """nitro_dist_loop_create on a halo-exchange handle: NITRO_E_UNSUPPORTED (9)."""
+    n = nitro()
+    A = synth.stencil("2d5", 32)
+    D = n.Dist(n.dist_unique_id(), 0, 1, 0)
+    Ad = synth.to_device(A, cuda)
+    M = D.spmv(A.rows, np.array([0, A.rows], np.int64), Ad.rowptr, Ad.colidx, Ad.vals, exchange=1)
+    with pytest.raises(n.NitroError) as e:
+        D.loop(M)
+    assert e.value.code == 9
+    M.close()
+    D.close()
