@@ -596,6 +596,11 @@ nitro_status_t prepare_hot(nitro_spmv *A, int64_t cap) {
   NITRO_CUDA(cudaStreamSynchronize(s));
   const double share = (double)cov / (double)Z;
   if (nh == 0 || nh > cap || share < kHotMinShare) return NITRO_OK;
+  // every persistent CTA loads the nh hot values once: worth it only when the
+  // gathers it saves are many times that (configs[3] power-law matrices of
+  // 2^16-2^22 rows lost to it: a scale-16 matrix saves ~0.3 M gathers against
+  // ~2.4 M staged loads)
+  if ((double)cov < 16.0 * 2.0 * (double)num_sms() * (double)nh) return NITRO_OK;
   NITRO_TRY(A->csrv.hot_cols.alloc((size_t)nh * 4));
   NITRO_TRY(A->csrv.hcol.alloc((size_t)Z * 4));
   DevBuf slot;
@@ -671,8 +676,10 @@ nitro_status_t prepare_csrv(nitro_spmv *A) {
     A->csrv.fix_S = S;
     A->csrv.fix_nlong = (int64_t)nl;
     A->csrv.n_long = 0;
-    // hot-x staging: up to 64 KB of x values per CTA (8192 fp64 / 16384 fp32)
-    if (csrv_hot_on()) NITRO_TRY(prepare_hot(A, (int64_t)(65536 / (A->fp64 ? 8 : 4))));
+    // hot-x staging: up to 64 KB of x values per CTA (8192 fp64); measured on
+    // fp64 only (configs[2] R-MAT) — the fp32 form (one 768-thread CTA per SM,
+    // 56 registers) is not used
+    if (csrv_hot_on() && A->fp64) NITRO_TRY(prepare_hot(A, (int64_t)(65536 / 8)));
     else A->csrv.nhot = 0;
     A->csrv.ready = true;
     return NITRO_OK;

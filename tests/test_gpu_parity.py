@@ -515,7 +515,15 @@ def test_c2b_rmat_full(cuda):
         y = M.run(v, xd)
         torch.cuda.synchronize()
         check_y(y.cpu().numpy(), y_ref, r, True, f"v{v}")
+        if v == n.CSR_VECTOR:   # AUTO: the stream mode (SD > mean) with hot-x staging (power-law columns)
+            fi = M.format_info(v)
+            assert fi["width"] == 0 and fi["ld"] > 0, fi
         M.release(v)
+    # and the same multiply without the staging (NITRO_CSR_IMPL_STREAM keeps it; row mode for reference)
+    M.set_csr_impl(n.CSR_IMPL_DIRECT)
+    y = M.run(n.CSR_VECTOR, xd)
+    torch.cuda.synchronize()
+    check_y(y.cpu().numpy(), y_ref, r, True, "csr_vector row mode")
 
 
 # ------------------------------------------------------------------ select path on the GPU
@@ -719,10 +727,7 @@ def test_csr_stream_mode(cuda, name, A):
         M.run(n.CSR_VECTOR, xd, y)
         torch.cuda.synchronize()
         ys.append(y.cpu().numpy())
-    fi = M.format_info(n.CSR_VECTOR)
-    assert fi["width"] == 0                                    # stream mode active
-    if name.startswith("rmat"):
-        assert fi["ld"] > 0                                    # hot-x staging engaged (power-law columns)
+    assert M.format_info(n.CSR_VECTOR)["width"] == 0          # stream mode active
     assert np.all(np.isfinite(ys[0]))                          # every row written (empty rows = 0)
     if exact:
         assert np.array_equal(ys[0].astype(np.float64), y_ref)
