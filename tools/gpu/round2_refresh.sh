@@ -1,6 +1,8 @@
 # round-2 refresh: configs[3] retrain (+ itune, feature study), bench, ncu launch list + full captures
 mkdir -p gpurun_out/artifacts
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv,noheader
+timeout 1500 python -m pytest tests -m gpu -q -x -rf --durations=5 > gpurun_out/pytest_full.log 2>&1; echo "pytest rc=$?"; tail -8 gpurun_out/pytest_full.log
+timeout 300 python __graft_entry__.py smoke 2>&1 | tail -1
 timeout 1800 python tools/train_select.py > gpurun_out/c3_train_select.log 2>&1; echo "c3 rc=$?"; tail -30 gpurun_out/c3_train_select.log
 timeout 900 python tools/itune_c3.py > gpurun_out/c3_itune.log 2>&1; echo "itune rc=$?"; tail -3 gpurun_out/c3_itune.log
 timeout 1200 python tools/feature_study.py --gpu > gpurun_out/feature_study.log 2>&1; echo "fstudy rc=$?"; tail -4 gpurun_out/feature_study.log
