@@ -89,3 +89,20 @@ def test_grid_tie_break_smaller_C_larger_gamma():
     (acc, lc, lg), table = S.grid_search(Xs, y, log2c=(-1, 3), log2g=(1, -3))
     assert acc == 1.0
     assert lc == -1 and lg == 1
+
+
+def test_decided_marks_only_near_boundary_points():
+    """C12 helper: with two mirror-symmetric classes the decision value on the
+    mirror plane is 0 (within solver tolerance): not decided; points near the
+    class centres are decided.  A 3-class problem: a point whose only
+    near-zero pair cannot change the vote winner stays decided."""
+    import numpy as np
+    from oracle import select as S
+    F = np.array([[-1.0, 0.0], [-0.8, 0.1], [-0.9, -0.1], [1.0, 0.0], [0.8, -0.1], [0.9, 0.1]])
+    m = S.train(F, [0, 0, 0, 1, 1, 1], log2c=(1,), log2g=(1,))
+    assert list(S.decided(m, np.array([[0.0, 0.0], [-0.9, 0.0], [0.9, 0.0]]))) == [False, True, True]
+    # three classes on a line: a point deep inside class 0 is decided even if
+    # the (1, 2) pair is exactly balanced there
+    F3 = np.array([[-2.0, 0], [-2.1, 0.1], [0.0, 1.0], [0.1, 1.1], [0.0, -1.0], [0.1, -1.1]])
+    m3 = S.train(F3, [0, 0, 1, 1, 2, 2], log2c=(1,), log2g=(-1,))
+    assert bool(S.decided(m3, np.array([[-2.05, 0.0]]))[0])
