@@ -597,10 +597,9 @@ nitro_status_t prepare_hot(nitro_spmv *A, int64_t cap) {
   const double share = (double)cov / (double)Z;
   if (nh == 0 || nh > cap || share < kHotMinShare) return NITRO_OK;
   // every persistent CTA loads the nh hot values once: worth it only when the
-  // gathers it saves are many times that (configs[3] power-law matrices of
-  // 2^16-2^22 rows lost to it: a scale-16 matrix saves ~0.3 M gathers against
-  // ~2.4 M staged loads)
-  if ((double)cov < 16.0 * 2.0 * (double)num_sms() * (double)nh) return NITRO_OK;
+  // gathers it saves are several times that (small power-law matrices lost to
+  // it: a 2^16-row one saves ~0.3 M gathers against ~2.4 M staged loads)
+  if ((double)cov < 4.0 * 2.0 * (double)num_sms() * (double)nh) return NITRO_OK;
   NITRO_TRY(A->csrv.hot_cols.alloc((size_t)nh * 4));
   NITRO_TRY(A->csrv.hcol.alloc((size_t)Z * 4));
   DevBuf slot;

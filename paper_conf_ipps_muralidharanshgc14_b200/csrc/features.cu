@@ -233,6 +233,9 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
   // (Collecting a row's window bits per 32-bit word in registers and testing /
   // ORing the shared word once per run, through 32-bit shared addresses, was
   // measured slower: configs[1] 0.131 -> 0.140 ms, configs[4] 5.75 -> 6.18 ms.)
+  // the window through 32-bit shared addresses computed once (the generic
+  // form re-derived the window's shared address on every entry: S2R + 4 ops)
+  const uint32_t win_sa = (uint32_t)__cvta_generic_to_shared(s_win);
   auto lane_walk_core = [&](auto ld, int L, uint32_t myrow, bool full) {
     const uint32_t rbase = myrow - (kWin >> 1);
     int prev = -1;
@@ -244,8 +247,10 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
       prev = c;
       const uint32_t rel = (uint32_t)c - rbase;
       if (rel < kWin) {
-        const uint32_t bit = 1u << (rel & 31);
-        if (!(s_win[rel >> 5] & bit)) atomicOr(&s_win[rel >> 5], bit);
+        const uint32_t bit = 1u << (rel & 31), a = win_sa + ((rel >> 5) << 2);
+        uint32_t w;
+        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(w) : "r"(a));
+        if (!(w & bit)) asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(a), "r"(bit) : "memory");
       } else if ((uint32_t)c < M32) {
         lane_far((uint32_t)c - myrow + G32, full);
       }
