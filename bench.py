@@ -369,10 +369,13 @@ def run_nitro(args):
     rank, world, local = dist_env()
     log = (lambda m: print(f"[bench] {m}", file=sys.stderr, flush=True)) if rank == 0 else (lambda m: None)
     if world > 1 and torch.cuda.device_count() < world:
+        # rank 0 reports and fails the job; the other ranks leave quietly (a
+        # failing rank would make torchrun stop rank 0 before it prints)
         if rank == 0:
             print(json.dumps({"error": f"--gpus {world} needs {world} GPUs, this node has "
                                        f"{torch.cuda.device_count()}", "n_gpus": world}), flush=True)
-        sys.exit(2)
+            sys.exit(2)
+        sys.exit(0)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     use_dist = world > 1 or args.dist   # --dist: the multi-rank code path with one rank (NCCL communicator of 1)
