@@ -14,7 +14,10 @@
  *     a borrowed device CSR, the GPU feature pass, the CSR->ELL/DIA/HYB
  *     converters, the five SpMV variants, timing, and a registration helper
  *     that plugs the five variants + features + constraints into layer 1.
- *  3. the multi-GPU row-partitioned SpMV (x all-gathered with NCCL).
+ *  3. the multi-GPU row-partitioned SpMV (x all-gathered or halo-exchanged
+ *     with NCCL, or over the single-GPU loopback transport; the solver-loop
+ *     mode with the exchange fused into the SpMV epilogue).
+ *  4. the histogram code-variant family (a second workload).
  *
  * Conventions (all functions):
  *  - extern "C"; return nitro_status_t (NITRO_OK = 0); never throw or abort.
@@ -226,9 +229,10 @@ typedef struct {
 
 /* Format facts after prepare. */
 typedef struct {
-  int64_t ld;         /* padded row pitch of ELL/DIA/HYB-ELL (multiple of 32) */
-  int64_t width;      /* ELL: K = Lmax; DIA: ndiag; HYB: K_hyb; CSR-vector: lanes per row */
-  int64_t tail;       /* HYB: COO tail entries; CSR-vector: number of long rows */
+  int64_t ld;         /* padded row pitch of ELL/DIA/HYB-ELL (multiple of 32);
+                         CSR-vector stream mode: hot x values staged in shared memory (0 = none) */
+  int64_t width;      /* ELL: K = Lmax; DIA: ndiag; HYB: K_hyb; CSR-vector: lanes per row (0 = stream mode) */
+  int64_t tail;       /* HYB: COO tail entries; CSR-vector: long-row segments (row mode) or chunks (stream mode) */
   int64_t bytes;      /* device bytes owned for this format */
   double compulsory_bytes; /* algorithmic bytes of one multiply */
 } nitro_format_info;
