@@ -449,14 +449,17 @@ bool csrv_stream_mode(const nitro_spmv *A) {
   return A->feat_ready && A->feat.sd > A->feat.mean;
 }
 
-// NITRO_CSRV_HOT=0 disables the hot-x staging of K6s
-bool csrv_hot_on() {
+// NITRO_CSRV_HOT=0 disables the hot-x staging of K6s; =2 skips its benefit
+// test (small matrices: tools/sanitize_run.py exercises the kernel that way)
+int csrv_hot_env() {
   static int env = [] {
     const char *e = getenv("NITRO_CSRV_HOT");
     return e ? atoi(e) : 1;
   }();
-  return env != 0;
+  return env;
 }
+bool csrv_hot_on() { return csrv_hot_env() != 0; }
+bool csrv_hot_forced() { return csrv_hot_env() == 2; }
 
 // ------------------------------------------------------------------ CSR-vector stream mode (K6s)
 // chunk_row[c] = the row holding entry c*CH (the last row whose start <= c*CH),
@@ -599,7 +602,7 @@ nitro_status_t prepare_hot(nitro_spmv *A, int64_t cap) {
   // every persistent CTA loads the nh hot values once: worth it only when the
   // gathers it saves are several times that (small power-law matrices lost to
   // it: a 2^16-row one saves ~0.3 M gathers against ~2.4 M staged loads)
-  if ((double)cov < 4.0 * 2.0 * (double)num_sms() * (double)nh) return NITRO_OK;
+  if ((double)cov < 4.0 * 2.0 * (double)num_sms() * (double)nh && !csrv_hot_forced()) return NITRO_OK;
   NITRO_TRY(A->csrv.hot_cols.alloc((size_t)nh * 4));
   NITRO_TRY(A->csrv.hcol.alloc((size_t)Z * 4));
   DevBuf slot;

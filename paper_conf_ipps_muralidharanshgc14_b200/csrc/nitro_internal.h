@@ -195,6 +195,7 @@ int hyb_windows(size_t sv);
 // (row-length SD above the mean); NITRO_CSRV_STREAM=0/1 forces it off/on.
 bool csrv_stream_mode(const nitro_spmv *A);
 bool csrv_hot_on();
+bool csrv_hot_forced();
 // bitmap index of diagonal offset d is d + G; the bitmap spans G + M bits
 inline int64_t diag_shift(const nitro_spmv *A) { return A->feat_G >= 0 ? A->feat_G : A->row0 + A->N - 1; }
 int num_sms();
