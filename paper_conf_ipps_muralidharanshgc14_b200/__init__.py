@@ -16,7 +16,8 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libnitro.so")
+# NITRO_LIB: another build of the library (A/B timing of two builds on one box)
+LIB_PATH = os.environ.get("NITRO_LIB") or os.path.join(_HERE, "libnitro.so")
 
 CSR_SCALAR, CSR_VECTOR, ELL, DIA, HYB = range(5)
 NUM_VARIANTS = 5

@@ -32,7 +32,7 @@ namespace {
 
 constexpr int kThreads = 256;
 constexpr int kWarps = kThreads / 32;
-constexpr int kCache = 1024;            // per-block open-addressing offset set (u32 keys, 4 KB)
+constexpr int kCache = 512;             // per-block open-addressing offset set (u32 keys, 2 KB)
 constexpr int kProbe = 4;               // linear-probe length
 constexpr uint32_t kWin = 1u << 16;     // per-block bitmap of offsets in [-2^15, 2^15) (8 KB)
 constexpr uint32_t kEmpty = 0xffffffffu;
@@ -41,10 +41,36 @@ constexpr int kRowCap = 64;             // lane-per-row walk only for rows up to
 constexpr int kQ = 4;                   // 32-row blocks per super-block (one staging round trip for short rows)
 constexpr int64_t kLong = 4096;         // rows longer than this go to k_features_long
 constexpr int64_t kChunk = 4096;        // entries per task of k_features_long
+constexpr int kPatMin = 8;              // shifted-row test for lane-walked blocks with rows of >= this many entries
+constexpr int kPatRows = 8;             // ... taken when at most this many of the 32 rows fail the quick test
 
-// staging slot of span entry e: one pad word per 32 entries, so lanes walking
-// rows of 32 (or 16, 8 ...) entries hit distinct banks
-__device__ __forceinline__ int skew(int e) { return e + (e >> 5); }
+// staging slot of span entry e (relative to a 16-byte aligned base): four pad
+// words per 32 entries, so 16-byte chunks stay aligned (cp.async of 16 bytes)
+// and lanes walking rows of 32 entries meet at most 4 to a bank (odd lengths:
+// none)
+__device__ __forceinline__ int skew(int e) { return e + ((e >> 5) << 2); }
+
+// cp.async of the colidx span [E0, E1) into buf at slots skew(e - E0a), E0a =
+// E0 rounded down to a 16-byte boundary of the column array: aligned 16-byte
+// chunks, the partial chunks at both ends entry by entry (no read outside
+// [E0, E1)).  Returns E0a; the caller waits (cp.async.wait_group 0).
+__device__ __forceinline__ int64_t stage_span(int *buf, const int32_t *__restrict__ col, int64_t E0, int64_t E1,
+                                              int lane) {
+  const int h = (int)((reinterpret_cast<uintptr_t>(col + E0) >> 2) & 3);
+  const int64_t E0a = E0 - h;
+  const int span = (int)(E1 - E0a);
+  const int lo = h ? 4 : 0, hi = span & ~3;
+  const uint32_t sb = (uint32_t)__cvta_generic_to_shared(buf);
+  const int32_t *g = col + E0a;
+  for (int q = lo + 4 * lane; q < hi; q += 128)
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 16;" ::"r"(sb + 4u * (uint32_t)skew(q)), "l"(g + q) : "memory");
+  // head [h, min(lo, span)) and tail [max(hi, lo), span): at most 3 + 3 entries
+  const int e = lane < 3 ? h + lane : (hi > lo ? hi : lo) + lane - 3;
+  if ((lane < 3 && e < lo && e < span) || (lane >= 3 && lane < 6 && e < span))
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(sb + 4u * (uint32_t)skew(e)), "l"(g + e) : "memory");
+  asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
+  return E0a;
+}
 
 // The offset bits of one 32-entry window held one per lane (key = bitmap word
 // or kEmpty, bits = its bit): a segmented inclusive OR scan merges runs of
@@ -178,7 +204,7 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
                                                         int64_t N, int64_t M, int64_t Z, int64_t row0, int64_t G,
                                                         FeatAcc *__restrict__ acc, uint32_t *__restrict__ bitmap,
                                                         int2 *__restrict__ tasks, int64_t cap_tasks) {
-  __shared__ int s_stage[kWarps][kStage + kStage / 32];
+  __shared__ __align__(16) int s_stage[kWarps][kStage + 4 + (kStage + 4) / 8];  // skew(kStage + 3) < this
   __shared__ int8_t s_slot[kWarps][32];
   __shared__ uint32_t s_seen[kCache];
   __shared__ uint32_t s_win[kWin / 32];
@@ -265,7 +291,70 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
   auto lane_walk_global = [&](int64_t a, int L, uint32_t myrow, bool full) {
     lane_walk_core([&](int k) { return __ldg(col + a + k); }, L, myrow, full);
   };
+  // Whole-warp walk of one staged row (lane = entry; L <= kRowCap: two steps):
+  // canonical checks and the offsets of that row, as lane_walk_core.
+  auto row_walk_lanes = [&](auto ld, int L, uint32_t row, bool full) {
+    const uint32_t rbase = row - (kWin >> 1);
+    int lastc = -1;
+    for (int k0 = 0; k0 < L; k0 += 32) {
+      const int k = k0 + lane;
+      const int c = k < L ? ld(k) : 0;
+      int prevc = __shfl_up_sync(kFull, c, 1);
+      if (lane == 0) prevc = lastc;
+      if (k < L) {
+        if ((uint32_t)c >= M32) bad |= 4;  // also catches c < 0
+        else {
+          if (c <= prevc) bad |= 2;
+          const uint32_t rel = (uint32_t)c - rbase;
+          if (rel < kWin) {
+            const uint32_t bit = 1u << (rel & 31), a = win_sa + ((rel >> 5) << 2);
+            uint32_t w;
+            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(w) : "r"(a));
+            if (!(w & bit)) asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(a), "r"(bit) : "memory");
+          } else {
+            lane_far((uint32_t)c - row + G32, full);
+          }
+        }
+      }
+      lastc = __shfl_sync(kFull, c, 31);
+    }
+  };
+  // Shifted rows (stencils, bands): row j whose entries are row j-1's plus one,
+  // entry by entry (same length), has row j-1's offsets c - row, so only the
+  // rows that are not such a shift of their predecessor are walked (lane =
+  // entry, above); a shifted row adds one check: its last column < M (strictly
+  // increasing and >= 0 follow from row j-1).  A first test on the lengths and
+  // the first and last entries; when more than kPatRows rows of the 32 fail it
+  // (random columns) the warp returns false and walks lane per row instead.
+  // Warp-collective; L = this lane's row length, rel0 its staged start.
+  auto pattern_walk = [&](const int *buf, int rel0, int L, uint32_t myrow, bool full) -> bool {
+    const int relp = __shfl_up_sync(kFull, rel0, 1);
+    const int Lp = __shfl_up_sync(kFull, L, 1);
+    bool shifted = lane > 0 && L > 1 && L == Lp;
+    if (shifted)
+      shifted = buf[skew(rel0)] == buf[skew(relp)] + 1 && buf[skew(rel0 + L - 1)] == buf[skew(relp + L - 1)] + 1;
+    if (__popc(__ballot_sync(kFull, L > 0 && !shifted)) > kPatRows) return false;
+    // entries 1 .. L-2 against the predecessor's through a shuffle (a shifted
+    // lane's predecessor has the same length, so it loads the same k)
+    const int Lw = __reduce_max_sync(kFull, (unsigned)L);
+#pragma unroll 4
+    for (int k = 1; k < Lw - 1; ++k) {
+      const int c = k < L ? buf[skew(rel0 + k)] : 0;
+      const int cp = __shfl_up_sync(kFull, c, 1);
+      shifted &= k >= L - 1 || c == cp + 1;
+    }
+    if (shifted && (uint32_t)buf[skew(rel0 + L - 1)] >= M32) bad |= 4;
+    unsigned todo = __ballot_sync(kFull, L > 0 && !shifted);
+    while (todo) {
+      const int j = __ffs(todo) - 1;
+      todo &= todo - 1;
+      const int rj = __shfl_sync(kFull, rel0, j);
+      row_walk_lanes([&](int k) { return buf[skew(rj + k)]; }, __shfl_sync(kFull, L, j), myrow - lane + j, full);
+    }
+    return true;
+  };
 
+  int pat_skip = 0;  // warp-uniform
   // One block of 32 rows (lane j <-> row rb*32 + j) with its row bounds a, b.
   auto process_block = [&](int64_t rb, int64_t a, int64_t b) {
     const int64_t r = rb * 32 + lane;
@@ -294,15 +383,11 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
     const unsigned long_mask = __ballot_sync(kFull, is_long);
     const bool staged = E1 - E0 <= kStage;  // implies no long row
     int *buf = s_stage[wib];
+    int64_t E0a = E0;
     if (staged) {
       // cp.async (LDGSTS): the whole span is in flight at once, no registers,
       // one memory round trip per block of rows
-      const int span = (int)(E1 - E0);
-      for (int e = lane; e < span; e += 32)
-        asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"((uint32_t)__cvta_generic_to_shared(buf + skew(e))),
-                     "l"(col + E0 + e)
-                     : "memory");
-      asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
+      E0a = stage_span(buf, col, E0, E1, lane);
       __syncwarp();
     }
     // lane per row when the rows are short and of similar length (stencils,
@@ -311,13 +396,19 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
     const unsigned maxL = __reduce_max_sync(kFull, (unsigned)(Ln > kRowCap ? kRowCap + 1 : Ln));
     const unsigned sumL = __reduce_add_sync(kFull, (unsigned)(Ln > kRowCap ? kRowCap + 1 : Ln));
     if (maxL <= (unsigned)kRowCap && maxL * 32u <= 2u * sumL) {
-      if (Ln > 0) {
-        const bool full = *(volatile unsigned *)&s_full != 0;
-        if (staged) lane_walk_staged(buf, (int)(a - E0), (int)Ln, myrow, full);
+      const bool full = *(volatile unsigned *)&s_full != 0;
+      bool done = false;
+      if (staged && maxL >= (unsigned)kPatMin && maxL * 32u <= sumL + 32u) {  // near-equal lengths
+        if (pat_skip > 0) --pat_skip;  // the test failed on a recent block of this warp: random rows
+        else if (!(done = pattern_walk(buf, (int)(a - E0a), (int)Ln, myrow, full))) pat_skip = 16;
+      }
+      if (done) {
+      } else if (Ln > 0) {
+        if (staged) lane_walk_staged(buf, (int)(a - E0a), (int)Ln, myrow, full);
         else lane_walk_global(a, (int)Ln, myrow, full);
       }
     } else if (staged) {
-      walk_span_warp<true>(buf, E0, E1, E0, a, L > 0, rowbase, G32, M32, win_lo, s_win, s_slot[wib], bitmap, lane,
+      walk_span_warp<true>(buf, E0, E1, E0a, a, L > 0, rowbase, G32, M32, win_lo, s_win, s_slot[wib], bitmap, lane,
                            bad);
     } else {
       // runs of consecutive non-long rows between the long ones
@@ -388,23 +479,16 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
         const int64_t rb = sb * kQ + j;
         if (rb >= nblk) break;
         const int64_t r = rb * 32 + lane;
-        int64_t aa = pick(a, j), bb = pick(b, j);
-        if (r >= N) aa = bb = (int64_t)rowptr[N];
+        // reloaded (L1 hits) rather than kept live across process_block: registers
+        const int64_t aa = (int64_t)rowptr[r < N ? r : N], bb = (int64_t)rowptr[r < N ? r + 1 : N];
         process_block(rb, aa, bb);
       }
       continue;
     }
     const int64_t E0 = __shfl_sync(kFull, a[0], 0), E1 = __shfl_sync(kFull, b[kQ - 1], 31);
     int *buf = s_stage[wib];
-    {
-      const int span = (int)(E1 - E0);
-      for (int e = lane; e < span; e += 32)
-        asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"((uint32_t)__cvta_generic_to_shared(buf + skew(e))),
-                     "l"(col + E0 + e)
-                     : "memory");
-      asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;" ::: "memory");
-      __syncwarp();
-    }
+    const int64_t E0a = stage_span(buf, col, E0, E1, lane);
+    __syncwarp();
     const bool full = *(volatile unsigned *)&s_full != 0;
 #pragma unroll 1
     for (int j = 0; j < kQ; ++j) {
@@ -414,7 +498,7 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
         s2 += (unsigned long long)L * (unsigned long long)L;
         if ((unsigned long long)L > lmax) lmax = (unsigned long long)L;
         const uint32_t myrow = (uint32_t)(row0 + (sb * kQ + j) * 32 + lane);
-        lane_walk_staged(buf, (int)(aj - E0), (int)L, myrow, full);
+        lane_walk_staged(buf, (int)(aj - E0a), (int)L, myrow, full);
       }
     }
     __syncwarp();  // the staging buffer is reused by the next iteration

@@ -163,6 +163,78 @@ def test_features_mixed_walks(cuda, rp32):
         assert f[k] == f_ref[k], k
 
 
+def _shift_rows_case(kind, n, changes):
+    """A stencil with edits that break the one-column shift between consecutive
+    rows (K1's shifted-row path, rows of >= 8 entries): ("last", r) moves row
+    r's last column right, ("mid", r) its middle column, ("first", r) its first
+    column left — each where the row stays strictly increasing and in range."""
+    A = synth.stencil(kind, n)
+    rp = np.asarray(A.rowptr, np.int64)
+    ci = A.colidx.copy()
+    for how, r in changes:
+        a, b = int(rp[r]), int(rp[r + 1])
+        if how == "last" and ci[b - 1] + 1 < A.cols:
+            ci[b - 1] += 1
+        elif how == "first" and ci[a] > 0:
+            ci[a] -= 1
+        else:  # "mid" (or a blocked edge): the first middle entry with a gap after it
+            for e in range(a + 1, b - 1):
+                if ci[e] + 1 < ci[e + 1]:
+                    ci[e] += 1
+                    break
+    return Csr(A.rows, A.cols, rp, ci, A.vals, A.fp64)
+
+
+@pytest.mark.parametrize("kind,n,changes", [
+    ("3d27", 16, []),
+    ("3d27", 16, [("mid", 1000)]),                                 # one middle entry of an interior row
+    ("3d27", 16, [("last", 1024)]),                                # lane 0 of a block
+    ("3d27", 16, [("first", 1055)]),                               # lane 31
+    ("3d27", 16, [("mid", 1030), ("mid", 1033)]),                 # a few unshifted rows: shifted path
+    ("3d27", 16, [("mid", r) for r in range(1030, 1040)]),         # many: the warp walks lane per row
+    ("3d27", 16, [("mid", r) for r in range(1030, 1062, 2)] + [("last", 4095)]),
+    ("3d27", (40, 12, 6), [("mid", 2000), ("first", 2001)]),       # x-lines longer than a block
+    ("2d9", 48, [("mid", 900), ("last", 901)]),
+])
+def test_features_shifted_rows(cuda, kind, n, changes):
+    """K1's shifted-row path (a row equal to its predecessor plus one column is
+    not walked): every edit that breaks the shift brings its own diagonals,
+    counted bit-exactly against the oracle."""
+    if kind not in synth.STENCIL_KINDS:
+        pytest.skip(kind)
+    B = _shift_rows_case(kind, n, changes)
+    assert oracle.is_canonical(B)
+    f_ref = oracle.features(B)
+    for rp32 in (True, False):
+        M, _ = handle(B, cuda, rowptr32=rp32)
+        f = M.features()
+        for k in FEAT_KEYS:
+            assert f[k] == f_ref[k], (k, rp32, f[k], f_ref[k])
+
+
+@pytest.mark.parametrize("last_ok", [True, False])
+def test_features_shifted_rows_column_range(cuda, last_ok):
+    """Rows [i, i + 9) of a matrix with M columns: every row is a shift of the
+    previous one, so the only check a shifted row adds is its last column < M —
+    one past it is rejected (NITRO_E_BAD_MATRIX), exactly at M - 1 is accepted."""
+    n = nitro()
+    N, L = 256, 9
+    M = N + L - 1 if last_ok else N + L - 2
+    rp = np.arange(N + 1, dtype=np.int64) * L
+    ci = (np.arange(N)[:, None] + np.arange(L)[None, :]).astype(np.int32).ravel()
+    B = Csr(N, M, rp, ci, np.ones(N * L, np.float32), False)
+    assert oracle.is_canonical(B) == last_ok
+    Md, _ = handle(B, cuda)
+    if last_ok:
+        f, f_ref = Md.features(), oracle.features(B)
+        for k in FEAT_KEYS:
+            assert f[k] == f_ref[k], k
+    else:
+        with pytest.raises(n.NitroError) as e:
+            Md.features()
+        assert e.value.code == 2
+
+
 @pytest.mark.parametrize("rows", [[1000], [1024], [1055], [1023, 1024], [2000, 2001, 2002], [64 * 64 - 1]])
 def test_features_single_row_pattern_change(cuda, rows):
     """The feature pass skips rows whose offset pattern equals the previous
