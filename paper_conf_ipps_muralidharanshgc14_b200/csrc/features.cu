@@ -354,6 +354,21 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
     return true;
   };
 
+  // 32 rows of one length L (interior stencil rows): the shift is checked
+  // position-parallel over the staged span — entry e == entry e - L, plus 1,
+  // for e >= L (lane = position: coalesced, conflict-free, ~10 instructions per
+  // 32 entries) — then only row 0 is walked.  False: some row is not a shift
+  // (pattern_walk finds which).
+  auto uniform_walk = [&](const int *buf, int h, int L, uint32_t rowbase, bool full) -> bool {
+    const int span = 32 * L;
+    bool ok = true;
+#pragma unroll 4
+    for (int e = L + lane; e < span; e += 32) ok &= buf[skew(h + e)] == buf[skew(h + e - L)] + 1;
+    if (!__all_sync(kFull, ok)) return false;
+    row_walk_lanes([&](int k) { return buf[skew(h + k)]; }, L, rowbase, full);
+    if (lane == 0 && (uint32_t)buf[skew(h + span - 1)] >= M32) bad |= 4;  // row 31's last column
+    return true;
+  };
   int pat_skip = 0;  // warp-uniform
   // One block of 32 rows (lane j <-> row rb*32 + j) with its row bounds a, b.
   auto process_block = [&](int64_t rb, int64_t a, int64_t b) {
@@ -400,7 +415,10 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
       bool done = false;
       if (staged && maxL >= (unsigned)kPatMin && maxL * 32u <= sumL + 32u) {  // near-equal lengths
         if (pat_skip > 0) --pat_skip;  // the test failed on a recent block of this warp: random rows
-        else if (!(done = pattern_walk(buf, (int)(a - E0a), (int)Ln, myrow, full))) pat_skip = 16;
+        else {
+          if (maxL * 32u == sumL) done = uniform_walk(buf, (int)(E0 - E0a), (int)maxL, rowbase, full);
+          if (!done && !(done = pattern_walk(buf, (int)(a - E0a), (int)Ln, myrow, full))) pat_skip = 16;
+        }
       }
       if (done) {
       } else if (Ln > 0) {
