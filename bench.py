@@ -174,6 +174,24 @@ def load_models(nitro):
     return out
 
 
+def feature_gpu_times(M, stream, reps=3):
+    """Device time of the feature pass (A1): the launches enqueued asynchronously
+    (features_async), CUDA events on the launching stream around them."""
+    import torch
+    out = []
+    for _ in range(reps):
+        M.invalidate()
+        M.flush_l2()
+        a, b = ev_pair()
+        a.record(stream) if stream is not None else a.record()
+        M.features_async()
+        b.record(stream) if stream is not None else b.record()
+        torch.cuda.synchronize()
+        M.features()
+        out.append(a.elapsed_time(b))
+    return out
+
+
 def ev_pair():
     import torch
     return torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -291,6 +309,7 @@ def measure_config(nitro, cfg, dev, models, reps, log):
         b.record()
         torch.cuda.synchronize()
         fts.append(a.elapsed_time(b))
+    fgs = feature_gpu_times(M, None)
     allowed = M.allowed_mask()
     fvec = [f[k] for k in nitro.FEATURE_NAMES]
     picks = {k: nitro.VARIANT_NAMES[cv.predict(fvec, allowed)] for k, (_, cv) in models.items()}
@@ -311,7 +330,8 @@ def measure_config(nitro, cfg, dev, models, reps, log):
     best = min(ex, key=lambda k: ex[k]["ms"])
     A_nnz = A.nnz
     out = {"workload": WORKLOADS[cfg][0], "rows": A.rows, "nnz": A.nnz, "generate_s": gen_s,
-           "feature_ms": statistics.median(fts), "features": {k: f[k] for k in nitro.FEATURE_NAMES},
+           "feature_ms": statistics.median(fts), "feature_gpu_ms": statistics.median(fgs),
+           "features": {k: f[k] for k in nitro.FEATURE_NAMES},
            "allowed": [nitro.VARIANT_NAMES[v] for v in range(nitro.NUM_VARIANTS) if allowed[v]],
            "picks": picks, "exhaustive_best": best, "exhaustive": ex}
     for k, name in picks.items():
@@ -441,6 +461,7 @@ def run_nitro(args):
             b.record(stream)
             torch.cuda.synchronize()
             fts.append(a.elapsed_time(b))
+    fgs = feature_gpu_times(M, stream) if D is None else []
     fvec = [feats[k] for k in nitro.FEATURE_NAMES]
     allowed = M.allowed_mask() if D is None else [True] * nitro.NUM_VARIANTS   # dist parts check their own
     picks, select_us = {}, {}
@@ -662,7 +683,12 @@ def run_nitro(args):
         "exhaustive_best": best, "exhaustive": exhaustive,
         "gflops": 2.0 * (feats["nnz"]) / (ms * 1e-3) / 1e9,
         "pct_of_hbm_peak": per_gpu / peak,
-        "feature_ms": statistics.median(fts) if fts else None, "feature_first_call_ms": feature_first_ms,
+        "feature_ms": statistics.median(fts) if fts else None,
+        "feature_gpu_ms": statistics.median(fgs) if fgs else None,
+        "feature_ms_note": "feature_ms: the blocking features() call (launches, device time, D2H of the sums, host "
+                           "wake-up); feature_gpu_ms: the same launches enqueued asynchronously, stream events around "
+                           "them (device time of the pass incl. its small launches and the D2H)",
+        "feature_first_call_ms": feature_first_ms,
         "features": {k: feats[k] for k in nitro.FEATURE_NAMES},
         "roofline": {"bound": "hbm", "achieved": per_gpu, "peak": peak, "unit": "GB/s", "frac": per_gpu / peak,
                      "traffic": traffic, "peak_kind": f"{pk_kind} hbm_gbs (device copy, read+write)",

@@ -776,13 +776,32 @@ __global__ void __launch_bounds__(kThreads) k_feat_stream(const IT *__restrict__
   if (threadIdx.x == 0 && s_bad) atomicOr(&acc->bad, s_bad);
 }
 
-__global__ void __launch_bounds__(256) k_popc(const uint32_t *__restrict__ bm, int64_t nwords, FeatAcc *acc) {
+// D = popcount of the bitmap; the last block to finish copies the sums into
+// the caller's mapped pinned FeatAcc (no separate device-to-host copy).
+__global__ void __launch_bounds__(256) k_popc(const uint32_t *__restrict__ bm, int64_t nwords, FeatAcc *acc,
+                                              FeatAcc *host_out) {
   unsigned long long s = 0;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nwords; i += (int64_t)gridDim.x * blockDim.x)
     s += __popc(bm[i]);
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(kFull, s, o);
   if ((threadIdx.x & 31) == 0 && s) atomicAdd(&acc->ndiag, s);
+  __syncthreads();
+  __shared__ bool last;
+  if (threadIdx.x == 0) {
+    __threadfence();
+    last = atomicAdd(&acc->popc_done, 1u) == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (last && threadIdx.x == 0) {
+    __threadfence();
+    const volatile FeatAcc *v = acc;
+    FeatAcc h;
+    h.s1 = v->s1; h.s2 = v->s2; h.lmax = v->lmax; h.bad = v->bad; h.nlong = v->nlong; h.ndiag = v->ndiag;
+    h.popc_done = gridDim.x; h.pad_ = 0;
+    *host_out = h;
+    __threadfence_system();
+  }
 }
 
 }  // namespace
@@ -821,7 +840,10 @@ nitro_status_t features_launch(nitro_spmv *A) {
   const int64_t nwords = (span + 31) / 32;
   NITRO_TRY(A->feat_acc.alloc(sizeof(FeatAcc)));
   NITRO_TRY(A->bitmap.alloc((size_t)(nwords > 0 ? nwords : 1) * 4));
-  if (!A->h_acc) NITRO_CUDA(cudaMallocHost(&A->h_acc, sizeof(FeatAcc)));
+  if (!A->h_acc) {
+    NITRO_CUDA(cudaHostAlloc(&A->h_acc, sizeof(FeatAcc), cudaHostAllocMapped));
+    NITRO_CUDA(cudaHostGetDevicePointer(&A->h_acc_dev, A->h_acc, 0));
+  }
   if (!A->feat_done) NITRO_CUDA(cudaEventCreateWithFlags(&A->feat_done, cudaEventDisableTiming));
   FeatAcc *acc = A->feat_acc.as<FeatAcc>();
   NITRO_CUDA(cudaMemsetAsync(acc, 0, sizeof(FeatAcc), s));
@@ -869,13 +891,13 @@ nitro_status_t features_launch(nitro_spmv *A) {
       k_features_long<int32_t><<<glong, kThreads, 0, s>>>((const int32_t *)A->rowptr, A->col, A->M, A->row0, G, acc,
                                                           A->bitmap.as<uint32_t>(), tasks, cap_tasks);
   }
-  if (nwords) {
+  {
     int64_t g2 = (nwords + 255) / 256;
     if (g2 > (int64_t)num_sms() * 8) g2 = (int64_t)num_sms() * 8;
-    k_popc<<<(unsigned)g2, 256, 0, s>>>(A->bitmap.as<uint32_t>(), nwords, acc);
+    if (g2 < 1) g2 = 1;
+    k_popc<<<(unsigned)g2, 256, 0, s>>>(A->bitmap.as<uint32_t>(), nwords, acc, A->h_acc_dev);
   }
   NITRO_CUDA(cudaGetLastError());
-  NITRO_CUDA(cudaMemcpyAsync(A->h_acc, acc, sizeof(FeatAcc), cudaMemcpyDeviceToHost, s));
   NITRO_CUDA(cudaEventRecord(A->feat_done, s));
   A->feat_pending = true;
   return NITRO_OK;

@@ -47,6 +47,8 @@ struct FeatAcc {
   unsigned int bad;      // bit0 rowptr not monotone / wrong ends, bit1 unsorted/dup col, bit2 col out of range
   unsigned int nlong;    // rows deferred to the long-row pass (k_features_long)
   unsigned long long ndiag;
+  unsigned int popc_done;  // k_popc blocks finished (the last one copies the sums to the host)
+  unsigned int pad_;
 };
 
 // ------------------------------------------------------------------ formats
@@ -114,7 +116,8 @@ struct nitro_spmv {
   nitro::DevBuf feat_long;  // int32 row ids of the rows longer than the feature pass's kLong
   nitro::DevBuf offsets;    // int32 [ndiag] ascending
   nitro::DevBuf scratch;    // scan scratch
-  nitro::FeatAcc *h_acc = nullptr;  // pinned
+  nitro::FeatAcc *h_acc = nullptr;  // pinned, mapped: written by k_popc's last block (no D2H copy)
+  nitro::FeatAcc *h_acc_dev = nullptr;  // its device address
   cudaEvent_t feat_done = nullptr;
 
   double budget = -1.0;
