@@ -459,6 +459,19 @@ int csrv_hot_env() {
   return env;
 }
 bool csrv_hot_on() { return csrv_hot_env() != 0; }
+// NITRO_CSRV_HOT_KB: shared memory for the hot x values per CTA (KB, 8-96).
+// Default 48 (6144 fp64): two CTAs then fit the 132 KB shared carveout and
+// keep 124 KB of L1 for the other gathers; B200, configs[2] R-MAT: 16 KB 0.671,
+// 32 KB 0.663, 48 KB 0.654, 56 KB 0.695 (the 164 KB carveout), 64 KB 0.688,
+// 80 KB 0.861 ms; forcing the max-shared carveout: 1.73 ms (L1 starved)
+int csrv_hot_kb() {
+  static int kb = [] {
+    const char *e = getenv("NITRO_CSRV_HOT_KB");
+    const int v = e ? atoi(e) : 48;
+    return v < 8 ? 8 : v > 96 ? 96 : v;
+  }();
+  return kb;
+}
 bool csrv_hot_forced() { return csrv_hot_env() == 2; }
 
 // ------------------------------------------------------------------ CSR-vector stream mode (K6s)
@@ -678,10 +691,10 @@ nitro_status_t prepare_csrv(nitro_spmv *A) {
     A->csrv.fix_S = S;
     A->csrv.fix_nlong = (int64_t)nl;
     A->csrv.n_long = 0;
-    // hot-x staging: up to 64 KB of x values per CTA (8192 fp64); measured on
-    // fp64 only (configs[2] R-MAT) — the fp32 form (one 768-thread CTA per SM,
-    // 56 registers) is not used
-    if (csrv_hot_on() && A->fp64) NITRO_TRY(prepare_hot(A, (int64_t)(65536 / 8)));
+    // hot-x staging: up to 48 KB of x values per CTA (6144 fp64, csrv_hot_kb);
+    // measured on fp64 only (configs[2] R-MAT) — the fp32 form (one 768-thread
+    // CTA per SM, 56 registers) is not used
+    if (csrv_hot_on() && A->fp64) NITRO_TRY(prepare_hot(A, (int64_t)csrv_hot_kb() * 1024 / 8));
     else A->csrv.nhot = 0;
     A->csrv.ready = true;
     return NITRO_OK;

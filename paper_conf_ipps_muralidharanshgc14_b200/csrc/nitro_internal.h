@@ -199,6 +199,7 @@ int hyb_windows(size_t sv);
 bool csrv_stream_mode(const nitro_spmv *A);
 bool csrv_hot_on();
 bool csrv_hot_forced();
+int csrv_hot_kb();
 // bitmap index of diagonal offset d is d + G; the bitmap spans G + M bits
 inline int64_t diag_shift(const nitro_spmv *A) { return A->feat_G >= 0 ? A->feat_G : A->row0 + A->N - 1; }
 int num_sms();

@@ -1340,7 +1340,7 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
     static bool attr_ = false;                                                                                    \
     if (!attr_) {                                                                                                 \
       NITRO_CUDA(cudaFuncSetAttribute(k_csr_stream<IT, VT, EPV, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, \
-                                      65536));                                                                    \
+                                      96 * 1024));                                                                \
       attr_ = true;                                                                                               \
     }                                                                                                             \
     k_csr_stream<IT, VT, EPV, true><<<gh, 768, hs, s>>>(rp, hc, val, x, y, N, A->Z, nch,                           \
