@@ -776,6 +776,14 @@ __global__ void __launch_bounds__(kThreads) k_feat_stream(const IT *__restrict__
   if (threadIdx.x == 0 && s_bad) atomicOr(&acc->bad, s_bad);
 }
 
+__global__ void __launch_bounds__(256) k_feat_zero(FeatAcc *acc, uint32_t *__restrict__ bm, int64_t nwords) {
+  const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x, nt = (int64_t)gridDim.x * blockDim.x;
+  if (t == 0) *acc = FeatAcc{};
+  const int64_t n4 = (reinterpret_cast<uintptr_t>(bm) & 15) == 0 ? nwords / 4 : 0;
+  for (int64_t i = t; i < n4; i += nt) reinterpret_cast<uint4 *>(bm)[i] = make_uint4(0, 0, 0, 0);
+  for (int64_t i = n4 * 4 + t; i < nwords; i += nt) bm[i] = 0;
+}
+
 // D = popcount of the bitmap; the last block to finish copies the sums into
 // the caller's mapped pinned FeatAcc (no separate device-to-host copy).
 __global__ void __launch_bounds__(256) k_popc(const uint32_t *__restrict__ bm, int64_t nwords, FeatAcc *acc,
@@ -846,8 +854,11 @@ nitro_status_t features_launch(nitro_spmv *A) {
   }
   if (!A->feat_done) NITRO_CUDA(cudaEventCreateWithFlags(&A->feat_done, cudaEventDisableTiming));
   FeatAcc *acc = A->feat_acc.as<FeatAcc>();
-  NITRO_CUDA(cudaMemsetAsync(acc, 0, sizeof(FeatAcc), s));
-  if (nwords) NITRO_CUDA(cudaMemsetAsync(A->bitmap.p, 0, (size_t)nwords * 4, s));
+  {  // FeatAcc and the bitmap zeroed by one launch
+    int64_t gz = (nwords / 4 + 255) / 256;
+    gz = gz < 1 ? 1 : gz > (int64_t)num_sms() * 4 ? (int64_t)num_sms() * 4 : gz;
+    k_feat_zero<<<(unsigned)gz, 256, 0, s>>>(acc, A->bitmap.as<uint32_t>(), nwords);
+  }
 
   const int64_t nblk = (A->N + 31) / 32;
   int64_t grid = (nblk + kWarps - 1) / kWarps;
@@ -858,6 +869,7 @@ nitro_status_t features_launch(nitro_spmv *A) {
   const int64_t cap_tasks = A->Z / kChunk + A->Z / kLong + 1;
   NITRO_TRY(A->feat_long.alloc((size_t)cap_tasks * sizeof(int2)));
   int2 *tasks = A->feat_long.as<int2>();
+  // (one 1024-thread CTA per SM instead: configs[1] -1 %, R-MAT +1 %: kept)
   const unsigned glong = (unsigned)std::max<int64_t>(1, std::min<int64_t>((int64_t)num_sms() * 4,
                                                                            (A->Z / kChunk + kWarps - 1) / kWarps));
   if (feat_stream_on(A)) {  // K1s: rowptr moments (k_rowstats) + the nnz-split pass
