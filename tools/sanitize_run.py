@@ -21,9 +21,13 @@ def main():
     import paper_conf_ipps_muralidharanshgc14_b200 as nitro
     import synth
     dev = torch.device("cuda:0")
-    mats = [synth.stencil("2d5", 64), synth.stencil("3d27", 12, mode=1, seed=2),
-            synth.uniform(3000, 9, variable=True, seed=3, M=4000), synth.rmat(11, 8, seed=4, fp64=True),
-            synth.banded(2000, 5, 0.5, seed=5), synth.uniform(1500, 90, seed=6, M=5000)]   # last: K1s
+    if os.environ.get("SANITIZE_PARTS", "all") == "loopback":
+        mats = []
+    else:
+        mats = [synth.stencil("2d5", 64), synth.stencil("3d27", 12, mode=1, seed=2),
+                synth.uniform(3000, 9, variable=True, seed=3, M=4000), synth.rmat(11, 8, seed=4, fp64=True),
+                synth.banded(2000, 5, 0.5, seed=5), synth.uniform(1500, 90, seed=6, M=5000),   # K1s
+                synth.stencil("3d27", (40, 12, 6), mode=1, seed=7), synth.stencil("2d9", 48)]  # K1 shifted-row paths
     for A in mats:
         Ad = synth.to_device(A, dev)
         M = nitro.SpMV.from_csr(Ad)
@@ -56,6 +60,9 @@ def main():
             for v in range(nitro.NUM_VARIANTS):
                 D.run_gathered(Mq, v, xg, yq)
             torch.cuda.synchronize()
+    if os.environ.get("SANITIZE_PARTS", "all") == "single":
+        print("sanitize run complete (single-thread part)")
+        return
     # 2 loopback ranks: the all-gather and halo exchanges, features, the fused solver loop
     import threading
     A = synth.stencil("2d5", 40)
