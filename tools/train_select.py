@@ -33,9 +33,12 @@ CLASSES = ("stencil", "banded", "uniform", "powerlaw")
 R11X_LOG_MASK = 0x7F   # DESIGN.md R11x: log1p of all seven SpMV features (extension, not the paper's reading)
 
 
+WIDE = False   # --wide: sizes up to 2^26 rows / R-MAT scale 24, half the power-law matrices fp64 (experiment)
+
+
 def params_for(cls: str, seed: int) -> dict:
     rnd = random.Random(seed)
-    logN = rnd.uniform(18, 23)
+    logN = rnd.uniform(18, 26 if WIDE else 23)
     if cls == "stencil":
         kind = rnd.choice(["1d3", "2d5", "2d9", "3d7", "3d27"])
         d = int(kind[0])
@@ -49,7 +52,10 @@ def params_for(cls: str, seed: int) -> dict:
                 "variable": rnd.random() < 0.5}
     a = rnd.uniform(0.45, 0.60)
     bc = (1.0 - a - 0.05) / 2
-    return {"class": cls, "scale": rnd.randint(16, 22), "ef": rnd.randint(4, 32), "a": a, "b": bc, "c": bc}
+    p = {"class": cls, "scale": rnd.randint(16, 24 if WIDE else 22), "ef": rnd.randint(4, 32), "a": a, "b": bc, "c": bc}
+    if WIDE:
+        p["fp64"] = rnd.random() < 0.5
+    return p
 
 
 def generate(p: dict, seed: int, dev):
@@ -61,7 +67,7 @@ def generate(p: dict, seed: int, dev):
         return synth.banded(p["N"], p["b"], p["density"], seed=seed, device=dev)
     if c == "uniform":
         return synth.uniform(p["N"], p["k"], variable=p["variable"], seed=seed, device=dev)
-    return synth.rmat(p["scale"], p["ef"], p["a"], p["b"], p["c"], seed=seed, fp64=False, device=dev)
+    return synth.rmat(p["scale"], p["ef"], p["a"], p["b"], p["c"], seed=seed, fp64=p.get("fp64", False), device=dev)
 
 
 def measure(p, seed, dev, reps):
@@ -74,8 +80,8 @@ def measure(p, seed, dev, reps):
     M = nitro.SpMV.from_csr(A)
     f = M.features()
     allowed = M.allowed_mask()
-    x = synth.vector(A.cols, seed=seed + 7, device=dev)
-    y = torch.empty(A.rows, dtype=torch.float32, device=dev)
+    x = synth.vector(A.cols, seed=seed + 7, fp64=A.fp64, device=dev)
+    y = torch.empty(A.rows, dtype=x.dtype, device=dev)
     cost, gbps = [], []
     for v in range(nitro.NUM_VARIANTS):
         if not allowed[v]:
@@ -100,9 +106,12 @@ def main():
     ap.add_argument("--test", type=int, default=10, help="held-out matrices per class")
     ap.add_argument("--reps", type=int, default=20)
     ap.add_argument("--out", default=os.path.join(ROOT, "artifacts"))
+    ap.add_argument("--wide", action="store_true", help="experiment: wider size range (see WIDE)")
     ap.add_argument("--from-table", default=None,
                     help="retrain / reselect from a measured c3_table.json (no GPU) instead of measuring")
     args = ap.parse_args()
+    global WIDE
+    WIDE = args.wide
     import numpy as np
     import paper_conf_ipps_muralidharanshgc14_b200 as nitro
 
