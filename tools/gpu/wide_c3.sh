@@ -1,7 +1,7 @@
 # experiment: configs[3] with a wider size range (train_select --wide), then the picks of both models on
 # the bench's configs[4] / c2a / c2b feature vectors
 mkdir -p gpurun_out/wide
-timeout 3000 python tools/train_select.py --wide --out gpurun_out/wide > gpurun_out/wide/train.log 2>&1; echo "rc=$?"
+timeout 3000 python tools/train_select.py --wide --wide-log2 ${WL:-26} --out gpurun_out/wide > gpurun_out/wide/train.log 2>&1; echo "rc=$?"
 tail -28 gpurun_out/wide/train.log
 python - <<'PY'
 import json, sys

@@ -33,27 +33,38 @@ CLASSES = ("stencil", "banded", "uniform", "powerlaw")
 R11X_LOG_MASK = 0x7F   # DESIGN.md R11x: log1p of all seven SpMV features (extension, not the paper's reading)
 
 
-WIDE = False   # --wide: sizes up to 2^26 rows / R-MAT scale 24, half the power-law matrices fp64 (experiment)
+# configs[3] recipe: row counts log-uniform in [2^18, 2^27.2] — the range spans every matrix the
+# bench deploys on (configs[1], [2], [4]: 2^21-2^27 rows), so the [-1, 1] scaling of P:L179 sees them inside
+# the training range; at most 2^32 nonzeros per matrix; R-MAT scale 16-24, half of them fp64 (configs[2]'s
+# R-MAT is fp64).  --narrow: the round-1 recipe (2^18-2^23 rows, R-MAT scale 16-22, fp32), kept for reference.
+NARROW = False
+MAX_LOG2_ROWS = 27.2
+MAX_NNZ = 2 ** 32
 
 
 def params_for(cls: str, seed: int) -> dict:
     rnd = random.Random(seed)
-    logN = rnd.uniform(18, 26 if WIDE else 23)
+    logN = rnd.uniform(18, 23 if NARROW else MAX_LOG2_ROWS)
     if cls == "stencil":
         kind = rnd.choice(["1d3", "2d5", "2d9", "3d7", "3d27"])
         d = int(kind[0])
         n = int(round(2 ** (logN / d)))
         return {"class": cls, "kind": kind, "n": n}
     if cls == "banded":
-        return {"class": cls, "N": int(2 ** logN), "b": int(round(math.exp(rnd.uniform(0, math.log(48))))),
-                "density": rnd.choice([1.0, 0.5, 0.1])}
+        p = {"class": cls, "N": int(2 ** logN), "b": int(round(math.exp(rnd.uniform(0, math.log(48))))),
+             "density": rnd.choice([1.0, 0.5, 0.1])}
+        p["b"] = max(1, min(p["b"], int(MAX_NNZ / p["N"] / p["density"] / 2)))
+        return p
     if cls == "uniform":
-        return {"class": cls, "N": int(2 ** logN), "k": max(1, int(round(math.exp(rnd.uniform(0, math.log(64)))))),
-                "variable": rnd.random() < 0.5}
+        p = {"class": cls, "N": int(2 ** logN), "k": max(1, int(round(math.exp(rnd.uniform(0, math.log(64)))))),
+             "variable": rnd.random() < 0.5}
+        p["k"] = max(1, min(p["k"], int(MAX_NNZ / p["N"] / (1.5 if p["variable"] else 1.0))))
+        return p
     a = rnd.uniform(0.45, 0.60)
     bc = (1.0 - a - 0.05) / 2
-    p = {"class": cls, "scale": rnd.randint(16, 24 if WIDE else 22), "ef": rnd.randint(4, 32), "a": a, "b": bc, "c": bc}
-    if WIDE:
+    p = {"class": cls, "scale": rnd.randint(16, 22 if NARROW else 24), "ef": rnd.randint(4, 32), "a": a, "b": bc,
+         "c": bc}
+    if not NARROW:
         p["fp64"] = rnd.random() < 0.5
     return p
 
@@ -106,12 +117,12 @@ def main():
     ap.add_argument("--test", type=int, default=10, help="held-out matrices per class")
     ap.add_argument("--reps", type=int, default=20)
     ap.add_argument("--out", default=os.path.join(ROOT, "artifacts"))
-    ap.add_argument("--wide", action="store_true", help="experiment: wider size range (see WIDE)")
+    ap.add_argument("--narrow", action="store_true", help="the round-1 recipe (see NARROW)")
     ap.add_argument("--from-table", default=None,
                     help="retrain / reselect from a measured c3_table.json (no GPU) instead of measuring")
     args = ap.parse_args()
-    global WIDE
-    WIDE = args.wide
+    global NARROW
+    NARROW = args.narrow
     import numpy as np
     import paper_conf_ipps_muralidharanshgc14_b200 as nitro
 
