@@ -19,8 +19,8 @@ every timed step, outside the per-step CUDA events.
 Selection: two models trained on configs[3] (tools/train_select.py):
 artifacts/spmv_model.txt = the paper's plain [-1, 1] scaling and
 artifacts/spmv_model_r11x.txt = the R11x extension (log1p + clip).
---model picks the deployed one (default r11x: configs[4] lies 16x beyond the
-training range in rows, where the plain-scaled RBF model extrapolates); both
+--model picks the deployed one (default paper: the configs[3] recipe spans
+2^18-2^27.2 rows, so every bench matrix lies inside its training range); both
 picks and their % of the exhaustive best are always reported.
 
 N = 1 adds (unless --quick): the same measurement on configs[1], configs[2]
@@ -741,7 +741,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="nitro", choices=["nitro", "reference"])
     ap.add_argument("--workload", default="c4", choices=["c4", "c1"])
-    ap.add_argument("--model", default="r11x", choices=["paper", "r11x"], help="deployed selection model")
+    ap.add_argument("--model", default="paper", choices=["paper", "r11x"], help="deployed selection model")
     ap.add_argument("--ex-reps", type=int, default=7, help="timed reps per variant in the exhaustive reference")
     ap.add_argument("--selection-per-class", type=int, default=10, help="held-out configs[3] matrices per class")
     ap.add_argument("--quick", action="store_true", help="primary workload only (no extra configs/selection leg)")
