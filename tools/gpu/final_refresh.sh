@@ -13,7 +13,7 @@ timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__byte
 echo "ncu launches rc=$?"
 for cfg in c1 c2a c2b c4; do
   case $cfg in
-    c4) rx='regex:k_(features|dia)'; n=6 ;;
+    c4) rx='regex:k_(features|dia)'; n=8 ;;
     *) rx='regex:k_(features|csr_scalar|csr_vector|csr_stream|ell|dia|hyb_tail|hyb_fixup)'; n=24 ;;
   esac
   timeout 1200 ncu --set full --clock-control none --import-source on -k "$rx" -c $n \

@@ -70,7 +70,7 @@ def main():
             fts.append(s.elapsed_time(e))
         feat_ms = sorted(fts)[len(fts) // 2]
         fgs = []
-        for _ in range(7 if timing else 1):   # device time of the pass: async launches, events around them
+        for _ in range(7 if timing else 0):   # device time of the pass: async launches, events around them
             M.invalidate()
             M.flush_l2()
             torch.cuda.synchronize()
@@ -80,7 +80,7 @@ def main():
             torch.cuda.synchronize()
             M.features()
             fgs.append(s.elapsed_time(e))
-        feat_gpu_ms = sorted(fgs)[len(fgs) // 2]
+        feat_gpu_ms = sorted(fgs)[len(fgs) // 2] if fgs else None
         x = synth.vector(A.cols, seed=2, fp64=A.fp64, device=dev)
         y = torch.empty(A.rows, dtype=x.dtype, device=dev)
         row = {"rows": A.rows, "nnz": A.nnz, "feature_ms": feat_ms, "feature_gpu_ms": feat_gpu_ms,
