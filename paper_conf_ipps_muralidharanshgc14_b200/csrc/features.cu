@@ -354,19 +354,43 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
     return true;
   };
 
-  // 32 rows of one length L (interior stencil rows): the shift is checked
-  // position-parallel over the staged span — entry e == entry e - L, plus 1,
-  // for e >= L (lane = position: coalesced, conflict-free, ~10 instructions per
-  // 32 entries) — then only row 0 is walked.  False: some row is not a shift
+  // A run of consecutive rows j0..j1 of the block all of the maximum length L
+  // (interior stencil rows: the whole block; a block holding a grid-line
+  // boundary row: all but one or two rows): the shift of each row j0 < j <= j1
+  // against row j - 1 is checked position-parallel over the run's staged span
+  // — entry e == entry e - L, plus 1 (lane = position: coalesced,
+  // conflict-free) — then only row j0 and the rows outside the run are walked
+  // (lane = entry).  skew(e + 32) = skew(e) + 36, so both shared addresses
+  // advance by a constant (no per-entry skew arithmetic).  False: the rows at
+  // the maximum length are not one run, or some row is not a shift
   // (pattern_walk finds which).
-  auto uniform_walk = [&](const int *buf, int h, int L, uint32_t rowbase, bool full) -> bool {
-    const int span = 32 * L;
+  auto run_walk = [&](const int *buf, int rel0, int L, int Lmax, uint32_t rowbase, bool full) -> bool {
+    const unsigned m = __ballot_sync(kFull, L == Lmax);
+    const int j0 = __ffs(m) - 1, j1 = 31 - __clz(m);
+    if (j1 - j0 < 15 || m != ((kFull >> (31 - j1)) & (kFull << j0))) return false;
+    const int h = __shfl_sync(kFull, rel0, j0);
+    const int span = (j1 - j0 + 1) * Lmax;
+    const uint32_t sb = (uint32_t)__cvta_generic_to_shared(buf);
+    uint32_t a1 = sb + 4u * (uint32_t)skew(h + Lmax + lane);
+    const uint32_t d = a1 - (sb + 4u * (uint32_t)skew(h + lane));
     bool ok = true;
 #pragma unroll 4
-    for (int e = L + lane; e < span; e += 32) ok &= buf[skew(h + e)] == buf[skew(h + e - L)] + 1;
+    for (int e = Lmax + lane; e < span; e += 32, a1 += 36u * 4u) {
+      int v1, v0;
+      asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v1) : "r"(a1));
+      asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v0) : "r"(a1 - d));
+      ok &= v1 == v0 + 1;
+    }
     if (!__all_sync(kFull, ok)) return false;
-    row_walk_lanes([&](int k) { return buf[skew(h + k)]; }, L, rowbase, full);
-    if (lane == 0 && (uint32_t)buf[skew(h + span - 1)] >= M32) bad |= 4;  // row 31's last column
+    row_walk_lanes([&](int k) { return buf[skew(h + k)]; }, Lmax, rowbase + (uint32_t)j0, full);
+    if (lane == 0 && (uint32_t)buf[skew(h + span - 1)] >= M32) bad |= 4;  // row j1's last column
+    unsigned todo = __ballot_sync(kFull, L > 0) & ~m;
+    while (todo) {
+      const int j = __ffs(todo) - 1;
+      todo &= todo - 1;
+      const int rj = __shfl_sync(kFull, rel0, j);
+      row_walk_lanes([&](int k) { return buf[skew(rj + k)]; }, __shfl_sync(kFull, L, j), rowbase + (uint32_t)j, full);
+    }
     return true;
   };
   int pat_skip = 0;  // warp-uniform
@@ -416,7 +440,7 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
       if (staged && maxL >= (unsigned)kPatMin && maxL * 32u <= sumL + 32u) {  // near-equal lengths
         if (pat_skip > 0) --pat_skip;  // the test failed on a recent block of this warp: random rows
         else {
-          if (maxL * 32u == sumL) done = uniform_walk(buf, (int)(E0 - E0a), (int)maxL, rowbase, full);
+          done = run_walk(buf, (int)(a - E0a), (int)Ln, (int)maxL, rowbase, full);
           if (!done && !(done = pattern_walk(buf, (int)(a - E0a), (int)Ln, myrow, full))) pat_skip = 16;
         }
       }
@@ -470,7 +494,8 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
       else { a[j] = b[j] = -1; }
     }
     const bool full_sb = (sb + 1) * kQ <= nblk;
-    bool fast = full_sb;
+    // the joint span first (one pair of shuffles): longer rows skip the per-block tests
+    bool fast = full_sb && __shfl_sync(kFull, b[kQ - 1], 31) - __shfl_sync(kFull, a[0], 0) <= kStage / 2;
     unsigned mx[kQ];
     if (fast) {
 #pragma unroll
