@@ -36,7 +36,13 @@ constexpr int kCache = 512;             // per-block open-addressing offset set 
 constexpr int kProbe = 4;               // linear-probe length
 constexpr uint32_t kWin = 1u << 16;     // per-block bitmap of offsets in [-2^15, 2^15) (8 KB)
 constexpr uint32_t kEmpty = 0xffffffffu;
-constexpr int kStage = 1024;            // per-warp staging buffer (entries)
+#ifndef NITRO_K1_STAGE
+#define NITRO_K1_STAGE 1024
+#endif
+#ifndef NITRO_K1_MINB
+#define NITRO_K1_MINB 4  // 4 resident CTAs per SM: <= 64 registers (at 66 the pass lost 10 %)
+#endif
+constexpr int kStage = NITRO_K1_STAGE;  // per-warp staging buffer (entries)
 constexpr int kRowCap = 64;             // lane-per-row walk only for rows up to this length
 constexpr int kQ = 4;                   // 32-row blocks per super-block (one staging round trip for short rows)
 constexpr int64_t kLong = 4096;         // rows longer than this go to k_features_long
@@ -62,8 +68,12 @@ __device__ __forceinline__ int64_t stage_span(int *buf, const int32_t *__restric
   const int lo = h ? 4 : 0, hi = span & ~3;
   const uint32_t sb = (uint32_t)__cvta_generic_to_shared(buf);
   const int32_t *g = col + E0a;
-  for (int q = lo + 4 * lane; q < hi; q += 128)
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 16;" ::"r"(sb + 4u * (uint32_t)skew(q)), "l"(g + q) : "memory");
+  {  // skew(q + 128) = skew(q) + 144: both addresses advance by constants
+    const int32_t *gq = g + lo + 4 * lane;
+    uint32_t sq = sb + 4u * (uint32_t)skew(lo + 4 * lane);
+    for (int q = lo + 4 * lane; q < hi; q += 128, gq += 128, sq += 144u * 4u)
+      asm volatile("cp.async.ca.shared.global [%0], [%1], 16;" ::"r"(sq), "l"(gq) : "memory");
+  }
   // head [h, min(lo, span)) and tail [max(hi, lo), span): at most 3 + 3 entries
   const int e = lane < 3 ? h + lane : (hi > lo ? hi : lo) + lane - 3;
   if ((lane < 3 && e < lo && e < span) || (lane >= 3 && lane < 6 && e < span))
@@ -200,7 +210,7 @@ __device__ __forceinline__ void merge_window(const uint32_t *s_win, uint32_t win
 // Offset index idx = col - row + G is < 2^32 (rows, cols < 2^31), so all
 // per-entry arithmetic is 32-bit.
 template <typename IT>
-__global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
+__global__ void __launch_bounds__(kThreads, NITRO_K1_MINB) k_features(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
                                                         int64_t N, int64_t M, int64_t Z, int64_t row0, int64_t G,
                                                         FeatAcc *__restrict__ acc, uint32_t *__restrict__ bitmap,
                                                         int2 *__restrict__ tasks, int64_t cap_tasks) {
@@ -213,6 +223,8 @@ __global__ void __launch_bounds__(kThreads) k_features(const IT *__restrict__ ro
   for (int i = threadIdx.x; i < kCache; i += kThreads) s_seen[i] = kEmpty;
   for (int i = threadIdx.x; i < (int)(kWin / 32); i += kThreads) s_win[i] = 0u;
   if (threadIdx.x == 0) { s_bad = 0; s_full = 0; }
+  pdl_trigger();  // k_features_long may be scheduled as CTAs of this grid retire
+  pdl_wait();     // the bitmap / FeatAcc zeroing (k_feat_zero) is complete
   __syncthreads();
 
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
@@ -582,6 +594,8 @@ __global__ void __launch_bounds__(kThreads) k_features_long(const IT *__restrict
                                                              int64_t G, FeatAcc *__restrict__ acc,
                                                              uint32_t *__restrict__ bitmap,
                                                              const int2 *__restrict__ tasks, int64_t cap_tasks) {
+  pdl_trigger();
+  pdl_wait();  // k_features has listed every long-row task
   const int64_t n0 = (int64_t)*(volatile unsigned *)&acc->nlong;
   const int64_t n = n0 < cap_tasks ? n0 : cap_tasks;  // more = malformed rowptr (flagged by k_features)
   const int lane = threadIdx.x & 31;
@@ -803,6 +817,7 @@ __global__ void __launch_bounds__(kThreads) k_feat_stream(const IT *__restrict__
 
 __global__ void __launch_bounds__(256) k_feat_zero(FeatAcc *acc, uint32_t *__restrict__ bm, int64_t nwords) {
   const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x, nt = (int64_t)gridDim.x * blockDim.x;
+  pdl_trigger();
   if (t == 0) *acc = FeatAcc{};
   const int64_t n4 = (reinterpret_cast<uintptr_t>(bm) & 15) == 0 ? nwords / 4 : 0;
   for (int64_t i = t; i < n4; i += nt) reinterpret_cast<uint4 *>(bm)[i] = make_uint4(0, 0, 0, 0);
@@ -813,6 +828,7 @@ __global__ void __launch_bounds__(256) k_feat_zero(FeatAcc *acc, uint32_t *__res
 // the caller's mapped pinned FeatAcc (no separate device-to-host copy).
 __global__ void __launch_bounds__(256) k_popc(const uint32_t *__restrict__ bm, int64_t nwords, FeatAcc *acc,
                                               FeatAcc *host_out) {
+  pdl_wait();  // every OR of the feature pass has landed
   unsigned long long s = 0;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nwords; i += (int64_t)gridDim.x * blockDim.x)
     s += __popc(bm[i]);
@@ -887,7 +903,16 @@ nitro_status_t features_launch(nitro_spmv *A) {
 
   const int64_t nblk = (A->N + 31) / 32;
   int64_t grid = (nblk + kWarps - 1) / kWarps;
+#ifdef NITRO_K1_PERSIST
+  static const int occ = [] {  // resident CTAs per SM: the grid is one full wave
+    int b = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_features<int32_t>, kThreads, 0) != cudaSuccess || b < 1) b = 1;
+    return b;
+  }();
+  const int64_t cap = (int64_t)num_sms() * occ;
+#else
   const int64_t cap = (int64_t)num_sms() * 8;
+#endif
   if (grid > cap) grid = cap;
   if (grid < 1) grid = 1;
   // long-row chunk tasks: at most Z / kChunk + (number of long rows <= Z / kLong) entries
@@ -915,24 +940,28 @@ nitro_status_t features_launch(nitro_spmv *A) {
       else NITRO_K1S(int32_t, ep);
 #undef NITRO_K1S
     }
-  } else if (A->rp64) {
-    k_features<int64_t><<<(unsigned)grid, kThreads, 0, s>>>((const int64_t *)A->rowptr, A->col, A->N, A->M, A->Z,
-                                                            A->row0, G, acc, A->bitmap.as<uint32_t>(), tasks, cap_tasks);
-    if (A->Z > kLong)
-      k_features_long<int64_t><<<glong, kThreads, 0, s>>>((const int64_t *)A->rowptr, A->col, A->M, A->row0, G, acc,
-                                                          A->bitmap.as<uint32_t>(), tasks, cap_tasks);
   } else {
-    k_features<int32_t><<<(unsigned)grid, kThreads, 0, s>>>((const int32_t *)A->rowptr, A->col, A->N, A->M, A->Z,
-                                                            A->row0, G, acc, A->bitmap.as<uint32_t>(), tasks, cap_tasks);
-    if (A->Z > kLong)
-      k_features_long<int32_t><<<glong, kThreads, 0, s>>>((const int32_t *)A->rowptr, A->col, A->M, A->row0, G, acc,
-                                                          A->bitmap.as<uint32_t>(), tasks, cap_tasks);
+    // the K1 chain zero -> k_features -> k_features_long -> k_popc by
+    // programmatic dependent launch: each kernel's launch overlaps the tail of
+    // its predecessor and waits (griddepcontrol.wait) before touching its output
+#define NITRO_K1(IT)                                                                                               \
+  do {                                                                                                             \
+    NITRO_CUDA(launch_pdl(k_features<IT>, (unsigned)grid, kThreads, 0, s, (const IT *)A->rowptr, A->col, A->N, A->M,  \
+                          A->Z, A->row0, G, acc, A->bitmap.as<uint32_t>(), tasks, cap_tasks));                     \
+    if (A->Z > kLong)                                                                                              \
+      NITRO_CUDA(launch_pdl(k_features_long<IT>, glong, kThreads, 0, s, (const IT *)A->rowptr, A->col, A->M,       \
+                            A->row0, G, acc, A->bitmap.as<uint32_t>(), (const int2 *)tasks, cap_tasks));           \
+  } while (0)
+    if (A->rp64) NITRO_K1(int64_t);
+    else NITRO_K1(int32_t);
+#undef NITRO_K1
   }
   {
     int64_t g2 = (nwords + 255) / 256;
     if (g2 > (int64_t)num_sms() * 8) g2 = (int64_t)num_sms() * 8;
     if (g2 < 1) g2 = 1;
-    k_popc<<<(unsigned)g2, 256, 0, s>>>(A->bitmap.as<uint32_t>(), nwords, acc, A->h_acc_dev);
+    NITRO_CUDA(launch_pdl(k_popc, (unsigned)g2, 256u, 0, s, (const uint32_t *)A->bitmap.as<uint32_t>(), nwords, acc,
+                          A->h_acc_dev));
   }
   NITRO_CUDA(cudaGetLastError());
   NITRO_CUDA(cudaEventRecord(A->feat_done, s));
