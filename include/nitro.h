@@ -230,7 +230,8 @@ typedef struct {
 /* Format facts after prepare. */
 typedef struct {
   int64_t ld;         /* padded row pitch of ELL/DIA/HYB-ELL (multiple of 32);
-                         CSR-vector stream mode: hot x values staged in shared memory (0 = none) */
+                         CSR-vector stream mode: hot x values staged in shared memory (0 = none);
+                         CSR-vector row mode: 1 = the vector-load kernel K6v, 0 = K6 */
   int64_t width;      /* ELL: K = Lmax; DIA: ndiag; HYB: K_hyb; CSR-vector: lanes per row (0 = stream mode) */
   int64_t tail;       /* HYB: COO tail entries; CSR-vector: long-row segments (row mode) or chunks (stream mode) */
   int64_t bytes;      /* device bytes owned for this format */
@@ -276,12 +277,17 @@ nitro_status_t nitro_spmv_set_budget(nitro_spmv *A, double bytes);
  * the TMA row-tile pipeline for every matrix (tiles that do not fit the
  * shared-memory stage are computed from global memory); _STREAM = the
  * nnz-split stream kernel for CSR-vector (CSR-scalar keeps the direct
- * kernel).  Within a mode the result is deterministic; the row-oriented
+ * kernel); _VEC4 = the vector-load CSR-vector kernel (K6v: V lanes per row,
+ * 4 consecutive entries per lane per step by 128-bit loads; needs 16-byte
+ * aligned col / val, else the direct kernel runs), which AUTO also picks for
+ * rows of similar length when the build's default says so.
+ * Within a mode the result is deterministic; the row-oriented
  * implementations are bit-identical to each other, the stream mode sums each
  * row in fp64 in a different association (within the R2 tolerance).
  * Returns NITRO_E_INVALID_ARG for any other value.  Takes effect at the next
  * run (the CSR-vector format is rebuilt if its mode changes). */
-enum { NITRO_CSR_IMPL_AUTO = 0, NITRO_CSR_IMPL_DIRECT = 1, NITRO_CSR_IMPL_STAGED = 2, NITRO_CSR_IMPL_STREAM = 3 };
+enum { NITRO_CSR_IMPL_AUTO = 0, NITRO_CSR_IMPL_DIRECT = 1, NITRO_CSR_IMPL_STAGED = 2, NITRO_CSR_IMPL_STREAM = 3,
+       NITRO_CSR_IMPL_VEC4 = 4 };
 nitro_status_t nitro_spmv_set_csr_impl(nitro_spmv *A, int impl);
 /* Build the variant's format (cached; conversions are amortised). */
 nitro_status_t nitro_spmv_prepare(nitro_spmv *A, int variant);

@@ -21,7 +21,7 @@ LIB_PATH = os.environ.get("NITRO_LIB") or os.path.join(_HERE, "libnitro.so")
 
 CSR_SCALAR, CSR_VECTOR, ELL, DIA, HYB = range(5)
 NUM_VARIANTS = 5
-CSR_IMPL_AUTO, CSR_IMPL_DIRECT, CSR_IMPL_STAGED, CSR_IMPL_STREAM = range(4)
+CSR_IMPL_AUTO, CSR_IMPL_DIRECT, CSR_IMPL_STAGED, CSR_IMPL_STREAM, CSR_IMPL_VEC4 = range(5)
 VARIANT_NAMES = ("csr_scalar", "csr_vector", "ell", "dia", "hyb")
 FEATURE_NAMES = ("nnz", "rows", "mean", "sd", "max_dev", "dia_fill", "ell_fill")
 
@@ -314,7 +314,7 @@ class SpMV:
         _check(_L.nitro_spmv_set_budget(self.h, float(nbytes)))
 
     def set_csr_impl(self, impl: int):
-        """CSR_IMPL_AUTO / _DIRECT / _STAGED / _STREAM (nitro_spmv_set_csr_impl)."""
+        """CSR_IMPL_AUTO / _DIRECT / _STAGED / _STREAM / _VEC4 (nitro_spmv_set_csr_impl)."""
         _check(_L.nitro_spmv_set_csr_impl(self.h, int(impl)))
 
     def prepare(self, v: int):

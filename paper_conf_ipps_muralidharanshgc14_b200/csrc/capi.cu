@@ -209,7 +209,7 @@ nitro_status_t nitro_spmv_set_budget(nitro_spmv *A, double bytes) {
 }
 
 nitro_status_t nitro_spmv_set_csr_impl(nitro_spmv *A, int impl) {
-  if (!A || impl < NITRO_CSR_IMPL_AUTO || impl > NITRO_CSR_IMPL_STREAM) return fail(NITRO_E_INVALID_ARG, "bad argument");
+  if (!A || impl < NITRO_CSR_IMPL_AUTO || impl > NITRO_CSR_IMPL_VEC4) return fail(NITRO_E_INVALID_ARG, "bad argument");
   A->csr_impl = impl;
   // the CSR-vector format depends on the mode (stream chunks vs long-row segments)
   if (A->csrv.ready && A->csrv.stream != csrv_stream_mode(A)) A->csrv.ready = false;
@@ -239,7 +239,9 @@ nitro_status_t nitro_spmv_format_info(nitro_spmv *A, int variant, nitro_format_i
       out->bytes = (int64_t)(A->csrv.long_rows.bytes + A->csrv.chunk_row.bytes + A->csrv.carry_row.bytes +
                              A->csrv.carry_val.bytes + A->csrv.fix_seg.bytes + A->csrv.fix_long.bytes +
                              A->csrv.hot_cols.bytes + A->csrv.hcol.bytes);
-      out->ld = A->csrv.nhot;  // stream mode: hot x values staged in shared memory (0 = none)
+      // stream mode: hot x values staged in shared memory (0 = none); row
+      // mode: 1 when the vector-load kernel K6v runs, else 0
+      out->ld = A->csrv.stream ? A->csrv.nhot : (csrv_vec_mode(A) ? 1 : 0);
       break;
     case NITRO_ELL: out->ld = A->ell.ld; out->width = A->ell.K; out->bytes = (int64_t)(A->ell.col.bytes + A->ell.val.bytes); break;
     case NITRO_DIA: out->ld = A->dia.ld; out->width = A->dia.D; out->bytes = (int64_t)(A->dia.off.bytes + A->dia.val.bytes); break;

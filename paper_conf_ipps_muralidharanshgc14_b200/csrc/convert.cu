@@ -449,6 +449,23 @@ bool csrv_stream_mode(const nitro_spmv *A) {
   return A->feat_ready && A->feat.sd > A->feat.mean;
 }
 
+// K6v (vector-load CSR-vector) for regular rows: explicit NITRO_CSR_IMPL_VEC4,
+// or AUTO when not in stream mode, the longest row is at most 16 steps of 4V
+// entries, and col / val are 16-byte aligned (NITRO_CSRV_VEC=0 / 1 overrides
+// the AUTO choice)
+bool csrv_vec_mode(const nitro_spmv *A) {
+  static int env = [] {
+    const char *e = getenv("NITRO_CSRV_VEC");
+    return e ? atoi(e) : -1;
+  }();
+  const bool aligned = ((reinterpret_cast<uintptr_t>(A->col) | reinterpret_cast<uintptr_t>(A->val)) & 15) == 0;
+  if (!aligned || !A->csrv.ready || A->csrv.stream) return false;
+  if (A->csr_impl == NITRO_CSR_IMPL_VEC4) return true;
+  if (A->csr_impl != NITRO_CSR_IMPL_AUTO || env == 0) return false;
+  const bool bounded = A->feat_ready && A->feat.max_row <= 16LL * 4 * A->csrv.V;
+  return bounded && (env == 1 || kCsrvVecDefault);
+}
+
 // NITRO_CSRV_HOT=0 disables the hot-x staging of K6s; =2 skips its benefit
 // test (small matrices: tools/sanitize_run.py exercises the kernel that way)
 int csrv_hot_env() {

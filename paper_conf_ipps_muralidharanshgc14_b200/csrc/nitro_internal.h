@@ -197,6 +197,8 @@ int hyb_windows(size_t sv);
 // CSR-vector mode: the nnz-split stream kernel (K6s) for skewed row lengths
 // (row-length SD above the mean); NITRO_CSRV_STREAM=0/1 forces it off/on.
 bool csrv_stream_mode(const nitro_spmv *A);
+bool csrv_vec_mode(const nitro_spmv *A);   // K6v (convert.cu)
+constexpr bool kCsrvVecDefault = true;      // AUTO picks K6v (B200 A/B)
 bool csrv_hot_on();
 bool csrv_hot_forced();
 int csrv_hot_kb();

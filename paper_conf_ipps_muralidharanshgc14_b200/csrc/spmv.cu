@@ -361,6 +361,107 @@ __global__ void __launch_bounds__(256, csrv_min_blocks<V, R, kB, VT>()) k_csr_ve
   }
 }
 
+// ------------------------------------------------------------------ K6v CSR-vector, vector-load mode
+// Rows of similar length (row-length SD <= mean, so no stream mode) and a
+// bounded longest row: V lanes per row (V = mean / 4 rounded to a power of
+// two, as K6), each lane taking 4 CONSECUTIVE entries per step with one
+// 128-bit column load and one 4-wide value load from the row's 16-byte
+// aligned base (entries of the neighbouring rows in the first and last chunk
+// masked: their x gathers are predicated off and their values zeroed), so a
+// row of L entries costs ceil(((a mod 4) + L) / 4V) steps — one for the
+// interior rows of a 27-point stencil at V = 8.  Two rows per lane group in
+// flight (R = 2: both rows' loads issued before either's gathers).  Sums in
+// VT by fma in entry order per lane, then a butterfly over the V lanes.
+// The last partial chunk of the arrays (Z not a multiple of 4) is read entry
+// by entry (no read past nnz).
+template <int V, typename IT, typename VT>
+__global__ void __launch_bounds__(256) k_csr_vec4(const IT *__restrict__ rowptr, const int32_t *__restrict__ col,
+                                                  const VT *__restrict__ val, const VT *__restrict__ x,
+                                                  VT *__restrict__ y, int64_t N, int64_t Z, bool l2ef) {
+  constexpr int G = 32 / V;
+#ifndef NITRO_K6V_R
+#define NITRO_K6V_R 2
+#endif
+  constexpr int R = (sizeof(VT) == 4 && V >= NITRO_K6V_R) ? NITRO_K6V_R : 2;
+  static_assert(V >= 2 && V <= 32 && V % R == 0, "V");
+  const uint64_t pol = l2_policy(l2ef);
+  const int lane = threadIdx.x & 31, g = lane / V, li = lane % V;
+  const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarp = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t t0 = warp * 32; t0 < N; t0 += nwarp * 32) {
+    const int64_t r = t0 + lane;
+    int64_t ra = 0, rb = 0;
+    if (r < N) { ra = (int64_t)rowptr[r]; rb = (int64_t)rowptr[r + 1]; }
+    const int64_t base = __shfl_sync(kFull, ra, 0) & ~(int64_t)3;  // 16-byte aligned tile base
+    const int rel_a = (int)(ra - base), rel_b = (int)(rb - base);   // < 2^31: bounded rows (launch rule)
+    const int32_t *cb = col + base;
+    const VT *vb = val + base;
+    const int zrel = Z - base < (int64_t)INT32_MAX ? (int)(Z - base) : INT32_MAX;
+#pragma unroll 1
+    for (int q = 0; q < V; q += R) {
+      int sa[R], sb[R], e0[R];
+      int nst = 0;
+#pragma unroll
+      for (int u = 0; u < R; ++u) {
+        const int src = g + G * (q + u);
+        sa[u] = __shfl_sync(kFull, rel_a, src);
+        sb[u] = __shfl_sync(kFull, rel_b, src);
+        e0[u] = (sa[u] & ~3) + 4 * li;
+        const int steps = sb[u] > (sa[u] & ~3) ? (sb[u] - (sa[u] & ~3) + 4 * V - 1) / (4 * V) : 0;
+        nst = steps > nst ? steps : nst;
+      }
+      VT part[R];
+#pragma unroll
+      for (int u = 0; u < R; ++u) part[u] = (VT)0;
+      for (int s = 0; s < nst; ++s) {  // uniform per lane group
+        int c[R][4];
+        VT v[R][4];
+#pragma unroll
+        for (int u = 0; u < R; ++u) {
+          const int e = e0[u] + s * 4 * V;
+          if (e < sb[u] && e + 4 <= zrel) {
+            const int4 cc = ld_stream_i4(reinterpret_cast<const int4 *>(cb + e), pol);
+            c[u][0] = cc.x; c[u][1] = cc.y; c[u][2] = cc.z; c[u][3] = cc.w;
+            V4<VT> vv;
+            vv.load(vb + e, pol);
+#pragma unroll
+            for (int j = 0; j < 4; ++j) v[u][j] = vv.v[j];
+          } else {
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+              const bool ok = e + j < sb[u] && e + j < zrel;
+              c[u][j] = ok ? ld_stream_i(cb + e + j, pol) : 0;
+              v[u][j] = ok ? ld_stream(vb + e + j, pol) : (VT)0;
+            }
+          }
+        }
+        VT xv[R][4];
+#pragma unroll
+        for (int u = 0; u < R; ++u) {
+          const int e = e0[u] + s * 4 * V;
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {
+            const bool in = e + j >= sa[u] && e + j < sb[u];
+            xv[u][j] = in ? __ldg(x + c[u][j]) : (VT)0;
+            if (!in) v[u][j] = (VT)0;
+          }
+        }
+#pragma unroll
+        for (int u = 0; u < R; ++u)
+#pragma unroll
+          for (int j = 0; j < 4; ++j) part[u] = fma(v[u][j], xv[u][j], part[u]);
+      }
+#pragma unroll
+      for (int u = 0; u < R; ++u) {
+#pragma unroll
+        for (int o = V / 2; o > 0; o >>= 1) part[u] += __shfl_xor_sync(kFull, part[u], o);
+        const int64_t row = t0 + g + G * (q + u);
+        if (li == 0 && row < N) y[row] = part[u];
+      }
+    }
+  }
+}
+
 // ------------------------------------------------------------------ K5/K6 staged: TMA row-tile pipeline
 // Persistent CTAs walk row tiles of TR rows round-robin.  For each tile one
 // elected thread issues three 1D bulk copies (cp.async.bulk, evict-first) of
@@ -1327,6 +1428,18 @@ nitro_status_t run_t(nitro_spmv *A, int variant, const VT *x, VT *y, cudaStream_
     case NITRO_CSR_VECTOR: {
       if (part) return fail(NITRO_E_INVALID_ARG, "CSR-vector has no row-range launch");
       if (N == 0) break;
+      if (csrv_vec_mode(A)) {  // K6v: 128-bit loads, V lanes per row
+        const unsigned g = grid_cap((N + 255) / 256, 8);
+        const bool ef = l2_evict_first();
+        switch (A->csrv.V) {
+          case 2: k_csr_vec4<2, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, A->Z, ef); break;
+          case 4: k_csr_vec4<4, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, A->Z, ef); break;
+          case 8: k_csr_vec4<8, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, A->Z, ef); break;
+          case 16: k_csr_vec4<16, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, A->Z, ef); break;
+          default: k_csr_vec4<32, IT, VT><<<g, 256, 0, s>>>(rp, A->col, val, x, y, N, A->Z, ef); break;
+        }
+        break;
+      }
       if (A->csrv.stream) {  // K6s: nnz-split chunks + carry fixup
         const int64_t nch = A->csrv.nch;
         const bool vec = ((reinterpret_cast<uintptr_t>(A->col) | reinterpret_cast<uintptr_t>(val)) & 15) == 0;

@@ -73,10 +73,12 @@ def test_emulated_ranks_match_single_gpu(cuda, name, A, P):
         yd, y1 = yd.cpu().numpy(), y1.cpu().numpy()
         err = np.abs(yd.astype(np.float64) - y_ref)
         assert np.all(err <= tol * r + 1e-30), (name, P, v)
-        if v == n.CSR_SCALAR or (v == n.CSR_VECTOR and name.startswith("3d27")):
-            # row-local summation order is partition independent for CSR-scalar;
-            # CSR-vector too when every part picks the same lane count V (it
-            # follows each part's own mean row length)
+        if v == n.CSR_SCALAR:
+            # row-local summation order is partition independent for CSR-scalar.
+            # (CSR-vector's is not: K6v's lanes take 16-byte-aligned chunks of
+            # the arrays, so the association follows each row start's phase
+            # modulo 4 within its part, and a part whose slices are misaligned
+            # runs K6 — within the tolerance above, not bit-identical.)
             assert np.array_equal(yd, y1), (name, P, v)
 
 

@@ -416,12 +416,17 @@ def _csr_impls(A, x, cuda, rowptr32=None, shift=(0, 0, 0)):
     xd = torch.from_numpy(x).to(cuda)
     out = {}
     for v in (n.CSR_SCALAR, n.CSR_VECTOR):
-        for impl in (n.CSR_IMPL_AUTO, n.CSR_IMPL_DIRECT, n.CSR_IMPL_STAGED, n.CSR_IMPL_STREAM):
+        for impl in (n.CSR_IMPL_AUTO, n.CSR_IMPL_DIRECT, n.CSR_IMPL_STAGED, n.CSR_IMPL_STREAM, n.CSR_IMPL_VEC4):
             M.set_csr_impl(impl)
             y = torch.full((A.rows,), float("nan"), dtype=xd.dtype, device=cuda)
             M.run(v, xd, y)
+            y2 = M.run(v, xd)
             torch.cuda.synchronize()
             out[(v, impl)] = y.cpu().numpy()
+            assert np.array_equal(out[(v, impl)], y2.cpu().numpy()), (v, impl)   # deterministic
+            if v == n.CSR_VECTOR:   # which row-mode kernel ran (format_info ld: 1 = K6v)
+                info = M.format_info(v)
+                out[("vec", impl)] = info["width"] > 0 and info["ld"] == 1
     M.close()
     return out
 
@@ -441,18 +446,26 @@ def test_csr_impls_bit_identical(cuda, name, A):
     global memory when their span overflows a stage) and the direct kernels run
     the same per-row arithmetic: y bit-identical, and within the oracle bound.
     The nnz-split stream mode of CSR-vector (K6s; AUTO picks it when the
-    row-length SD exceeds the mean) sums in another association: within the
-    bound, deterministic, and AUTO equals it exactly when it is picked."""
+    row-length SD exceeds the mean) and the vector-load mode (K6v) sum in other
+    associations: within the bound, deterministic, and AUTO equals the one it
+    picks exactly."""
     n = nitro()
     x = synth.vector(A.cols, seed=41, mode=0, fp64=A.fp64)
     y_ref, r = oracle.spmv(A, x)
     skewed = oracle.features(A)["sd"] > oracle.features(A)["mean"]
     for rp32 in ((True, False) if A.nnz < 2**31 else (False,)):
         out = _csr_impls(A, x, cuda, rowptr32=rp32)
+        assert out[("vec", n.CSR_IMPL_VEC4)], name   # arrays from torch: 16-byte aligned
+        assert not out[("vec", n.CSR_IMPL_DIRECT)]
         for (v, impl), y in out.items():
+            if v == "vec":
+                continue
             check_y(y, y_ref, r, A.fp64, f"{name} v{v} impl{impl} rp32={rp32}")
-            stream = v == n.CSR_VECTOR and (impl == n.CSR_IMPL_STREAM or (impl == n.CSR_IMPL_AUTO and skewed))
-            want = out[(v, n.CSR_IMPL_STREAM)] if stream else out[(v, n.CSR_IMPL_DIRECT)]
+            auto = impl == n.CSR_IMPL_AUTO
+            stream = v == n.CSR_VECTOR and (impl == n.CSR_IMPL_STREAM or (auto and skewed))
+            vec = v == n.CSR_VECTOR and not stream and (impl == n.CSR_IMPL_VEC4 or (auto and out[("vec", impl)]))
+            want = out[(v, n.CSR_IMPL_STREAM)] if stream else out[(v, n.CSR_IMPL_VEC4)] if vec \
+                else out[(v, n.CSR_IMPL_DIRECT)]
             assert np.array_equal(y, want), (name, v, impl, rp32)
 
 
@@ -463,7 +476,10 @@ def test_csr_staged_misaligned_spans(cuda, shift):
     y_ref, r = oracle.spmv(A, x)
     out = _csr_impls(A, x, cuda, rowptr32=True, shift=shift)
     n = nitro()
+    assert not out[("vec", n.CSR_IMPL_VEC4)]   # misaligned col / val: K6v falls back to K6
     for (v, impl), y in out.items():
+        if v == "vec":
+            continue
         check_y(y, y_ref, r, False, f"shift {shift} v{v} impl{impl}")
         if not (v == n.CSR_VECTOR and impl == n.CSR_IMPL_STREAM):   # misaligned arrays: the scalar-load path of K6s
             assert np.array_equal(y, out[(v, 1)]), (shift, v, impl)
