@@ -14,7 +14,7 @@ echo "ncu launches rc=$?"
 for cfg in c1 c2a c2b c4; do
   case $cfg in
     c4) rx='regex:k_(features|dia)'; n=8 ;;
-    *) rx='regex:k_(features|csr_scalar|csr_vector|csr_stream|ell|dia|hyb_tail|hyb_fixup)'; n=24 ;;
+    *) rx='regex:k_(features|csr_scalar|csr_vector|csr_vec4|csr_stream|ell|dia|hyb_tail|hyb_fixup)'; n=24 ;;
   esac
   timeout 1200 ncu --set full --clock-control none --import-source on -k "$rx" -c $n \
       -o /tmp/prof_$cfg -f python tools/profile_variants.py $cfg > gpurun_out/prof_$cfg.log 2>&1

@@ -51,7 +51,7 @@ def load(path):
 
 
 def short(name):
-    for k in ("k_features_long", "k_features", "k_csr_scalar", "k_csr_vector", "k_csr_stream", "k_hyb_tail",
+    for k in ("k_features_long", "k_features", "k_csr_scalar", "k_csr_vector", "k_csr_vec4", "k_csr_stream", "k_hyb_tail",
               "k_hyb_fixup", "k_ell", "k_dia"):
         if k in name:
             return k
@@ -77,7 +77,7 @@ def main():
         for i, r in enumerate(recs):
             k = short(r["kernel"])
             var = {"k_features": "features", "k_features_long": "features_long", "k_csr_scalar": "csr_scalar",
-                   "k_csr_vector": "csr_vector", "k_csr_stream": "csr_vector", "k_dia": "dia", "k_hyb_tail": "hyb",
+                   "k_csr_vector": "csr_vector", "k_csr_vec4": "csr_vector", "k_csr_stream": "csr_vector", "k_dia": "dia", "k_hyb_tail": "hyb",
                    "k_hyb_fixup": "hyb_fixup"}.get(k)
             if k == "k_ell":
                 var = "ell" if seen_ell < 2 and cfg != "c2b" else "hyb_ell"
