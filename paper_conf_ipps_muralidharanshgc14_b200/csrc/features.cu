@@ -903,16 +903,7 @@ nitro_status_t features_launch(nitro_spmv *A) {
 
   const int64_t nblk = (A->N + 31) / 32;
   int64_t grid = (nblk + kWarps - 1) / kWarps;
-#ifdef NITRO_K1_PERSIST
-  static const int occ = [] {  // resident CTAs per SM: the grid is one full wave
-    int b = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_features<int32_t>, kThreads, 0) != cudaSuccess || b < 1) b = 1;
-    return b;
-  }();
-  const int64_t cap = (int64_t)num_sms() * occ;
-#else
-  const int64_t cap = (int64_t)num_sms() * 8;
-#endif
+  const int64_t cap = (int64_t)num_sms() * 8;  // (one persistent wave measured: -5 % configs[4], +11 % uniform)
   if (grid > cap) grid = cap;
   if (grid < 1) grid = 1;
   // long-row chunk tasks: at most Z / kChunk + (number of long rows <= Z / kLong) entries
