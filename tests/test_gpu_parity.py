@@ -438,6 +438,8 @@ def _impl_mats():
     yield "banded_b33_d01", synth.banded(40_000, 33, 0.1, seed=23)   # CSR-scalar's class in configs[3]
     yield "uniform_var_k3", synth.uniform(50_001, 3, variable=True, seed=24)
     yield "3d27_n40_fp64", synth.stencil("3d27", 40, mode=1, seed=25, fp64=True)
+    yield "banded_b40_dense", synth.banded(30_001, 40, 1.0, seed=27)        # consecutive-column runs (K6v x runs)
+    yield "banded_b40_dense_fp64", synth.banded(20_003, 40, 1.0, seed=28, fp64=True)
 
 
 @pytest.mark.parametrize("name,A", list(_impl_mats()))
