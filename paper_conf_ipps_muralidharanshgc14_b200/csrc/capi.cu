@@ -169,6 +169,7 @@ nitro_status_t nitro_spmv_set_stream(nitro_spmv *A, void *stream) {
 }
 
 nitro_status_t nitro_spmv_features(nitro_spmv *A, nitro_spmv_feat *out) {
+  NITRO_NVTX("nitro_spmv_features");
   NITRO_GUARD_BEGIN
   if (!A || !out) return fail(NITRO_E_INVALID_ARG, "NULL argument");
   DeviceGuard g(A->device);
@@ -187,6 +188,7 @@ nitro_status_t nitro_spmv_row_features(nitro_spmv *A, nitro_spmv_feat *out) {
 }
 
 nitro_status_t nitro_spmv_features_async(nitro_spmv *A) {
+  NITRO_NVTX("nitro_spmv_features_async");
   NITRO_GUARD_BEGIN
   if (!A) return fail(NITRO_E_INVALID_ARG, "NULL handle");
   DeviceGuard g(A->device);
@@ -217,6 +219,7 @@ nitro_status_t nitro_spmv_set_csr_impl(nitro_spmv *A, int impl) {
 }
 
 nitro_status_t nitro_spmv_prepare(nitro_spmv *A, int variant) {
+  NITRO_NVTX("nitro_spmv_prepare");
   NITRO_GUARD_BEGIN
   if (!A || !valid_variant(variant)) return fail(NITRO_E_INVALID_ARG, "bad argument");
   DeviceGuard g(A->device);
@@ -257,6 +260,7 @@ nitro_status_t nitro_spmv_format_info(nitro_spmv *A, int variant, nitro_format_i
 }
 
 nitro_status_t nitro_spmv_run(nitro_spmv *A, int variant, const void *d_x, void *d_y) {
+  NITRO_NVTX("nitro_spmv_run");
   NITRO_GUARD_BEGIN
   if (!A || !valid_variant(variant)) return fail(NITRO_E_INVALID_ARG, "bad argument");
   if ((A->M > 0 && !d_x) || (A->N > 0 && !d_y)) return fail(NITRO_E_INVALID_ARG, "x or y is NULL");
@@ -358,6 +362,7 @@ nitro_status_t run_host_pipelined(nitro_spmv *A, int variant, const void *h_x, v
 extern "C" {
 
 nitro_status_t nitro_spmv_run_host(nitro_spmv *A, int variant, const void *h_x, void *h_y) {
+  NITRO_NVTX("nitro_spmv_run_host");
   NITRO_GUARD_BEGIN
   if (!A || !valid_variant(variant)) return fail(NITRO_E_INVALID_ARG, "bad argument");
   if ((A->M > 0 && !h_x) || (A->N > 0 && !h_y)) return fail(NITRO_E_INVALID_ARG, "x or y is NULL");
@@ -386,6 +391,7 @@ nitro_status_t nitro_spmv_flush_l2(nitro_spmv *A) {
 
 nitro_status_t nitro_spmv_time(nitro_spmv *A, int variant, const void *d_x, void *d_y, int warmup, int reps,
                                int flush_l2, double *out_median_s, double *out_all) {
+  NITRO_NVTX("nitro_spmv_time");
   NITRO_GUARD_BEGIN
   if (!A || !valid_variant(variant) || reps < 1 || warmup < 0 || !out_median_s)
     return fail(NITRO_E_INVALID_ARG, "bad argument");

@@ -299,6 +299,7 @@ nitro_status_t nitro_cv_add_training_input(nitro_cv *cv, void *input) {
 }
 
 nitro_status_t nitro_cv_train(nitro_cv *cv, const nitro_train_opts *opts) {
+  NITRO_NVTX("nitro_cv_train");
   GUARD_BEGIN
   if (!cv) return fail(NITRO_E_INVALID_ARG, "NULL cv");
   if (cv->variants.empty() || cv->n_feat == 0 || cv->inputs.empty())
@@ -375,6 +376,7 @@ void nitro_itune_opts_default(nitro_itune_opts *o) {
 }
 
 nitro_status_t nitro_cv_itune(nitro_cv *cv, const nitro_train_opts *topts, const nitro_itune_opts *iopts) {
+  NITRO_NVTX("nitro_cv_itune");
   GUARD_BEGIN
   if (!cv) return fail(NITRO_E_INVALID_ARG, "NULL cv");
   if (cv->variants.empty() || cv->n_feat == 0 || cv->inputs.empty())
@@ -677,6 +679,7 @@ nitro_status_t nitro_cv_predict(nitro_cv *cv, const double *feat, const int *all
 }
 
 nitro_status_t nitro_cv_select(nitro_cv *cv, const void *input, int *out_variant, double *out_feat) {
+  NITRO_NVTX("nitro_cv_select");
   GUARD_BEGIN
   if (!cv || !out_variant) return fail(NITRO_E_INVALID_ARG, "NULL argument");
   if (!cv->trained) return fail(NITRO_E_STATE, "select before train/load");
@@ -691,6 +694,7 @@ nitro_status_t nitro_cv_select(nitro_cv *cv, const void *input, int *out_variant
 }
 
 nitro_status_t nitro_cv_call(nitro_cv *cv, void *input, int *out_variant, double *out_cost) {
+  NITRO_NVTX("nitro_cv_call");
   GUARD_BEGIN
   int v = 0;
   NITRO_TRY(nitro_cv_select(cv, input, &v, nullptr));

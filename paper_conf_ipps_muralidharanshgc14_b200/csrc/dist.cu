@@ -567,6 +567,7 @@ nitro_status_t nitro_dist_spmv_create(nitro_dist *D, int64_t global_rows, const 
 }
 
 nitro_status_t nitro_dist_spmv_run(nitro_dist *D, nitro_spmv *A, int variant, const void *d_x_local, void *d_y_local) {
+  NITRO_NVTX("nitro_dist_spmv_run");
   if (!D || !A || !A->dist_state || variant < 0 || variant >= NITRO_NUM_VARIANTS)
     return fail(NITRO_E_INVALID_ARG, "bad argument");
   if (!D->has_transport() && D->nranks > 1) return fail(NITRO_E_STATE, "communicator-less handle: use run_gathered");
@@ -677,6 +678,7 @@ nitro_status_t nitro_dist_x_local(nitro_spmv *A, void **ptr) {
 }
 
 nitro_status_t nitro_dist_features(nitro_dist *D, nitro_spmv *A, nitro_spmv_feat *out) {
+  NITRO_NVTX("nitro_dist_features");
   if (!D || !A || !A->dist_state || !out) return fail(NITRO_E_INVALID_ARG, "bad argument");
   if (!D->has_transport() && D->nranks > 1) return fail(NITRO_E_STATE, "communicator-less handle");
   DistState *st = (DistState *)A->dist_state;

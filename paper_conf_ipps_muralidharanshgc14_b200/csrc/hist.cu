@@ -476,6 +476,7 @@ nitro_status_t nitro_hist_allowed(nitro_hist *H, int variant, int *out_allowed) 
 }
 
 nitro_status_t nitro_hist_run(nitro_hist *H, int variant, uint32_t *d_hist) {
+  NITRO_NVTX("nitro_hist_run");
   HIST_GUARD_BEGIN
   if (!H || !d_hist || !hist_valid(variant)) return fail(NITRO_E_INVALID_ARG, "bad argument");
   DevGuard g(H->device);

@@ -8,8 +8,19 @@
 #include <string>
 
 #include "../../include/nitro.h"
+#include <nvtx3/nvToolsExt.h>   // header-only NVTX v3: ranges cost nothing without an attached tool
 
 namespace nitro {
+
+// NVTX range over one C-ABI call (nsys / ncu --nvtx timelines name the phases:
+// features, select, train, conversion, multiply, exchange)
+struct NvtxRange {
+  explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+  NvtxRange(const NvtxRange &) = delete;
+  NvtxRange &operator=(const NvtxRange &) = delete;
+};
+#define NITRO_NVTX(name) ::nitro::NvtxRange nitro_nvtx_range_(name)
 
 // ------------------------------------------------------------------ errors
 void set_error(const std::string &msg);
