@@ -69,6 +69,21 @@ def long_row_matrix(L=150_000, N=5000, fp64=False, seed=21):
     return Csr(N, M, rp, ci, v.astype(np.float64 if fp64 else np.float32), fp64)
 
 
+def outlier_row_matrix(N=40_000, k=32, L=3000, seed=29):
+    """Uniform random rows of k entries plus one row of L: row-length SD stays
+    below the mean (no stream mode) while the longest row exceeds 16 steps of
+    4V entries, so AUTO keeps K6 for CSR-vector instead of K6v."""
+    rng = np.random.default_rng(seed)
+    lens = np.full(N, k)
+    lens[123] = L
+    rp = np.zeros(N + 1, np.int64)
+    rp[1:] = np.cumsum(lens)
+    ci = np.concatenate([np.sort(rng.choice(N, l, replace=False)) for l in lens]).astype(np.int32)
+    v = rng.uniform(-1, 1, rp[-1])
+    v[v == 0] = 0.5
+    return Csr(N, N, rp, ci, v.astype(np.float32), False)
+
+
 def check_y(y, y_ref, r, fp64, what=""):
     tol = (1e-12 if fp64 else 1e-5) * r + 1e-30
     err = np.abs(np.asarray(y, np.float64) - y_ref)
@@ -440,6 +455,7 @@ def _impl_mats():
     yield "3d27_n40_fp64", synth.stencil("3d27", 40, mode=1, seed=25, fp64=True)
     yield "banded_b40_dense", synth.banded(30_001, 40, 1.0, seed=27)        # consecutive-column runs (K6v x runs)
     yield "banded_b40_dense_fp64", synth.banded(20_003, 40, 1.0, seed=28, fp64=True)
+    yield "uniform_k32_outlier_row", outlier_row_matrix()      # AUTO: K6 (longest row beyond the K6v bound)
 
 
 @pytest.mark.parametrize("name,A", list(_impl_mats()))
@@ -459,6 +475,10 @@ def test_csr_impls_bit_identical(cuda, name, A):
         out = _csr_impls(A, x, cuda, rowptr32=rp32)
         assert out[("vec", n.CSR_IMPL_VEC4)], name   # arrays from torch: 16-byte aligned
         assert not out[("vec", n.CSR_IMPL_DIRECT)]
+        if name == "uniform_k32_outlier_row":
+            assert not skewed and not out[("vec", n.CSR_IMPL_AUTO)]   # the K6v row bound sends AUTO to K6
+        if name.startswith("banded_b40_dense"):
+            assert out[("vec", n.CSR_IMPL_AUTO)]                      # regular rows: AUTO picks K6v
         for (v, impl), y in out.items():
             if v == "vec":
                 continue
